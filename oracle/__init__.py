@@ -1,0 +1,180 @@
+"""ctypes wrapper of the CPU oracle (oracle/igk_oracle.c).
+
+TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+cpu_baseline / --impl reference legs of bench.py may import this module.
+The product package (paper_conf_dac_leejlczcshh25_b200) never imports it.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libigk_oracle.so")
+
+STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in",
+         "evicted", "rounds", "moves_applied", "moves_deferred", "cut", "cap",
+         "max_part_weight", "imbalanced"]
+
+OK, EINVAL, ENOMEM, WIMBALANCED = 0, 1, 2, 6
+
+
+def build(force: bool = False) -> str:
+    src = os.path.join(_HERE, "igk_oracle.c")
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
+        subprocess.check_call(["gcc", "-O2", "-Wall", "-fPIC", "-shared", src, "-o", _SO])
+    return _SO
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = C.CDLL(_SO)
+        P = C.c_void_p
+        i64p = C.POINTER(C.c_int64)
+        i32p = C.POINTER(C.c_int32)
+        L.ora_create.restype = P
+        L.ora_create.argtypes = [C.c_int64, i64p, i32p, i32p, i32p, C.c_int32, C.c_double, i32p, C.POINTER(C.c_int)]
+        L.ora_destroy.argtypes = [P]
+        L.ora_last_error.restype = C.c_char_p
+        L.ora_last_error.argtypes = [P]
+        L.ora_apply.argtypes = [P, i32p, C.c_int64, i64p, i64p]
+        L.ora_refine.argtypes = [P, i64p]
+        L.ora_n_total.restype = C.c_int64
+        L.ora_n_total.argtypes = [P]
+        L.ora_n_active.restype = C.c_int64
+        L.ora_n_active.argtypes = [P]
+        L.ora_partition.argtypes = [P, i32p]
+        L.ora_cut.restype = C.c_int64
+        L.ora_cut.argtypes = [P]
+        L.ora_part_weights.argtypes = [P, i64p]
+        L.ora_total_weight.restype = C.c_int64
+        L.ora_total_weight.argtypes = [P]
+        L.ora_cap_value.restype = C.c_int64
+        L.ora_cap_value.argtypes = [P]
+        L.ora_num_slots.restype = C.c_int64
+        L.ora_num_slots.argtypes = [P]
+        L.ora_export_csr.argtypes = [P, i64p, i32p, i32p]
+        L.ora_check_invariants.argtypes = [P, C.c_char_p, C.c_int]
+        L.ora_cap.restype = C.c_int64
+        L.ora_cap.argtypes = [C.c_int64, C.c_double, C.c_int32]
+        L.ora_trace_rounds.restype = C.c_int64
+        L.ora_trace_rounds.argtypes = [P, i64p, i64p, C.c_int64]
+        L.ora_trace_moves.restype = C.c_int64
+        L.ora_trace_moves.argtypes = [P, i64p, C.c_int64]
+        L.ora_trace_sets.argtypes = [P, C.c_void_p, C.c_void_p, C.c_void_p]
+        _lib = L
+    return _lib
+
+
+def _p(a, ct):
+    return None if a is None else a.ctypes.data_as(C.POINTER(ct))
+
+
+def cap(W: int, eps: float, k: int) -> int:
+    return int(lib().ora_cap(W, eps, k))
+
+
+class Oracle:
+    """One oracle graph (IGK-SEM v1)."""
+
+    def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None):
+        L = lib()
+        xadj = np.ascontiguousarray(xadj, dtype=np.int64)
+        adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
+        part = np.ascontiguousarray(part, dtype=np.int32)
+        vwgt = None if vwgt is None else np.ascontiguousarray(vwgt, dtype=np.int32)
+        adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
+        st = C.c_int(0)
+        n = len(xadj) - 1
+        self.k = int(k)
+        self.h = L.ora_create(n, _p(xadj, C.c_int64), _p(adjncy, C.c_int32), _p(vwgt, C.c_int32),
+                              _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(st))
+        if not self.h:
+            raise ValueError(f"ora_create rejected the input (status {st.value})")
+
+    def __del__(self):
+        h = getattr(self, "h", None)
+        if h:
+            lib().ora_destroy(h)
+            self.h = None
+
+    def apply(self, mods):
+        """mods: int32 array of shape (B, 4) = {kind, u, v, w}. Returns (status, first_new_id, bad_index)."""
+        m = np.ascontiguousarray(mods, dtype=np.int32).reshape(-1, 4)
+        fid = C.c_int64(0)
+        bad = C.c_int64(-1)
+        s = lib().ora_apply(self.h, _p(m, C.c_int32), len(m), C.byref(fid), C.byref(bad))
+        return int(s), int(fid.value), int(bad.value)
+
+    def refine(self):
+        st = np.zeros(len(STATS), dtype=np.int64)
+        s = lib().ora_refine(self.h, _p(st, C.c_int64))
+        return int(s), dict(zip(STATS, (int(x) for x in st)))
+
+    @property
+    def n_total(self):
+        return int(lib().ora_n_total(self.h))
+
+    @property
+    def n_active(self):
+        return int(lib().ora_n_active(self.h))
+
+    def partition(self):
+        out = np.empty(self.n_total, dtype=np.int32)
+        lib().ora_partition(self.h, _p(out, C.c_int32))
+        return out
+
+    def cut(self):
+        return int(lib().ora_cut(self.h))
+
+    def part_weights(self):
+        out = np.empty(self.k, dtype=np.int64)
+        lib().ora_part_weights(self.h, _p(out, C.c_int64))
+        return out
+
+    def total_weight(self):
+        return int(lib().ora_total_weight(self.h))
+
+    def cap(self):
+        return int(lib().ora_cap_value(self.h))
+
+    def export_csr(self):
+        n = self.n_total
+        m = int(lib().ora_num_slots(self.h))
+        xadj = np.empty(n + 1, dtype=np.int64)
+        adj = np.empty(max(m, 1), dtype=np.int32)
+        w = np.empty(max(m, 1), dtype=np.int32)
+        lib().ora_export_csr(self.h, _p(xadj, C.c_int64), _p(adj, C.c_int32), _p(w, C.c_int32))
+        return xadj, adj[:m], w[:m]
+
+    def check_invariants(self):
+        buf = C.create_string_buffer(256)
+        r = lib().ora_check_invariants(self.h, buf, 256)
+        return None if r == 0 else buf.value.decode()
+
+    def trace_rounds(self, maxr=1 << 16):
+        S = np.zeros(maxr, dtype=np.int64)
+        Lr = np.zeros(maxr, dtype=np.int64)
+        r = int(lib().ora_trace_rounds(self.h, _p(S, C.c_int64), _p(Lr, C.c_int64), maxr))
+        return S[:r], Lr[:r]
+
+    def trace_moves(self, maxm=1 << 20):
+        out = np.zeros(3 * maxm, dtype=np.int64)
+        m = int(lib().ora_trace_moves(self.h, _p(out, C.c_int64), 3 * maxm))
+        return out[: 3 * m].reshape(m, 3)
+
+    def trace_sets(self):
+        n = self.n_total
+        a = np.zeros(n, dtype=np.uint8)
+        b = np.zeros(n, dtype=np.uint8)
+        c = np.zeros(n, dtype=np.uint8)
+        lib().ora_trace_sets(self.h, a.ctypes.data, b.ctypes.data, c.ctypes.data)
+        return a.astype(bool), b.astype(bool), c.astype(bool)

@@ -1,0 +1,92 @@
+/*
+ * igk_oracle.h -- CPU oracle for the iG-kway incremental refinement step.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load this library.
+ * The product path (paper_conf_dac_leejlczcshh25_b200/) never includes,
+ * links or calls anything under oracle/, and this file shares no header,
+ * constant or helper with include/igk.h.
+ *
+ * Semantics: IGK-SEM v1, i.e. the paper's
+ * Alg. 1-4 (PAPER.md P:94-P:270) read under the fixed readings listed in
+ * DESIGN.md section 4.  A plain, single-threaded, slow implementation on
+ * flat arrays; every function cites the passage it follows.
+ *
+ * Modifiers are passed as int32 quadruples {kind, u, v, w}:
+ *   kind 0 = edge deletion  M-(u,v)
+ *   kind 1 = vertex deletion M-u      (Alg. 2)
+ *   kind 2 = vertex insertion M+u     (Alg. 2); w = vertex weight
+ *   kind 3 = edge insertion  M+(u,v)  (Alg. 1); w = edge weight
+ */
+#ifndef IGK_ORACLE_H
+#define IGK_ORACLE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct ora_graph ora_graph;
+
+/* return codes (numerically equal to the product's, by specification) */
+#define ORA_OK 0
+#define ORA_EINVAL 1
+#define ORA_ENOMEM 2
+#define ORA_WIMBALANCED 6
+
+/* stats vector layout (ORA_NSTATS int64 entries) */
+enum {
+  ORA_ST_AFFECTED = 0,   /* |A u Psi0|: directly affected (A) + pending inserted */
+  ORA_ST_INSERTED,       /* |Psi0|: pending pseudo vertices at refine start      */
+  ORA_ST_EXPANDED,       /* |N|: non-pseudo neighbours of Psi examined in R2     */
+  ORA_ST_FILTERED_IN,    /* |C1|                                                  */
+  ORA_ST_EXPANDED_IN,    /* |C2|                                                  */
+  ORA_ST_EVICTED,        /* |R3 evictions|                                        */
+  ORA_ST_ROUNDS,         /* R                                                     */
+  ORA_ST_MOVES_APPLIED,  /* sum L_r                                               */
+  ORA_ST_MOVES_DEFERRED, /* sum (|S_r| - L_r)                                     */
+  ORA_ST_CUT,            /* cut after refine                                      */
+  ORA_ST_CAP,            /* c = cap(W)                                            */
+  ORA_ST_MAX_PART_WEIGHT,
+  ORA_ST_IMBALANCED,     /* 1 if the weighted fallback fired                      */
+  ORA_NSTATS
+};
+
+ora_graph* ora_create(int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                      const int32_t* vwgt, const int32_t* adjwgt, int32_t k,
+                      double epsilon, const int32_t* init_part, int* status);
+void ora_destroy(ora_graph* g);
+const char* ora_last_error(const ora_graph* g);
+
+int ora_apply(ora_graph* g, const int32_t* mods, int64_t count,
+              int64_t* first_new_id, int64_t* bad_index);
+int ora_refine(ora_graph* g, int64_t* stats /* ORA_NSTATS, nullable */);
+
+int64_t ora_n_total(const ora_graph* g);
+int64_t ora_n_active(const ora_graph* g);
+/* out[v] = part, -1 = deleted, -2 = pending (pseudo) */
+void ora_partition(const ora_graph* g, int32_t* out);
+int64_t ora_cut(const ora_graph* g);             /* recount from scratch */
+void ora_part_weights(const ora_graph* g, int64_t* out_k);
+int64_t ora_total_weight(const ora_graph* g);
+int64_t ora_cap_value(const ora_graph* g);
+/* symmetric CSR of the current graph over all IDs, rows sorted ascending */
+int64_t ora_num_slots(const ora_graph* g);
+void ora_export_csr(const ora_graph* g, int64_t* xadj, int32_t* adjncy, int32_t* adjwgt);
+/* invariants I1-I6; returns 0 if all hold, else writes msg */
+int ora_check_invariants(const ora_graph* g, char* msg, int msglen);
+
+/* step-level hooks used by the pinning tests (tests/test_oracle_*.py) */
+int64_t ora_cap(int64_t W, double epsilon, int32_t k);
+/* last refine trace: per round |S_r| and L_r (up to maxr rounds) */
+int64_t ora_trace_rounds(const ora_graph* g, int64_t* S, int64_t* L, int64_t maxr);
+/* last refine: the sorted move list of every round, (u, p*, g) triples
+ * concatenated in round order; returns the number of moves */
+int64_t ora_trace_moves(const ora_graph* g, int64_t* out, int64_t cap3);
+/* last refine sets: which vertices entered Psi in R1, R2, R3 (flags per ID) */
+void ora_trace_sets(const ora_graph* g, uint8_t* c1, uint8_t* c2, uint8_t* r3);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
