@@ -1,0 +1,154 @@
+/*
+ * igk.h -- C ABI of the B200-native iG-kway incremental refinement library
+ *          (libigk.so, hand-written CUDA for sm_100a).
+ *
+ * The operation is the incremental step of iG-kway (Lee et al., DAC'25;
+ * "P:N" = line N of the paper text): apply a batch of graph modifiers to a
+ * GPU-resident graph (Sec. V.B, Alg. 1-2), then refine the k-way
+ * partition over the affected vertices only (Sec. V.C, Alg. 3-4) until
+ * every part weight is <= W_pmax with a low cut.  The exact,
+ * deterministic semantics (IGK-SEM v1) and every reading of a garbled or
+ * silent passage are in DESIGN.md sections 3-4; results are bit-identical
+ * to the CPU oracle under oracle/ (which shares no code with this library).
+ *
+ * Conventions (all functions):
+ *  - Host pointers are read (or written) before the call returns and are
+ *    never retained; the caller owns them.  Device pointers (only in the
+ *    *_device variants) must stay valid until the call returns.
+ *  - Calls are synchronous with respect to host buffers; device work runs
+ *    on igk_options.stream (NULL = the legacy default stream).
+ *  - Errors: IGK_EINVAL leaves the handle unchanged.  A CUDA error poisons
+ *    the handle: every later call returns IGK_ESTATE.  No C++ exception
+ *    crosses this boundary.  igk_last_error() describes the last failure.
+ *  - One handle per host thread at a time.
+ */
+#ifndef IGK_H
+#define IGK_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct igk_graph igk_graph; /* opaque; owns all device memory */
+
+typedef enum {
+  IGK_OK = 0,
+  IGK_EINVAL = 1,       /* invalid argument or invalid modifier batch (state unchanged) */
+  IGK_ENOMEM = 2,       /* vertex or adjacency capacity exhausted / allocation failed   */
+  IGK_ECUDA = 3,        /* CUDA error; the handle is poisoned                            */
+  IGK_ENCCL = 4,        /* reserved for the sharded build                                */
+  IGK_ESTATE = 5,       /* handle poisoned by an earlier CUDA error, or NULL handle      */
+  IGK_WIMBALANCED = 6   /* result valid, but a weighted corner case left W_p > cap (Q8)  */
+} igk_status;
+
+/* modifier kinds: M-(u,v), M-u, M+u, M+(u,v) */
+enum {
+  IGK_EDGE_DELETE = 0,
+  IGK_VERTEX_DELETE = 1,
+  IGK_VERTEX_INSERT = 2,
+  IGK_EDGE_INSERT = 3
+};
+
+/* One modifier, 16 bytes.  Edges are undirected: one modifier per edge; the
+ * store keeps both directions (the paper lists both, Fig. 4 caption P:90).
+ * w = edge weight (EDGE_INSERT) or vertex weight (VERTEX_INSERT); ignored
+ * otherwise.  On a handle created without vwgt (resp. adjwgt) the vertex
+ * (resp. edge) weight of an insertion must be 1. */
+typedef struct {
+  int32_t kind, u, v, w;
+} igk_modifier;
+
+typedef struct {
+  int device;              /* CUDA device ordinal                                         */
+  void* stream;            /* cudaStream_t; NULL = default stream                          */
+  int64_t max_vertices;    /* vertex-ID capacity (0 = 2 n + 65536)                        */
+  int64_t max_slots;       /* adjacency slab capacity in entries (0 = 4 x initial + 2^22)  */
+  int32_t slack_min;       /* minimum spare slots per vertex (0 = 2), cf. gamma      */
+  int32_t validate;        /* reserved: batches are always validated                       */
+  int32_t check_invariants;/* 1 = recount cut/W_p after every refine and compare (slow)    */
+  int32_t blocks_per_sm;   /* persistent-kernel CTAs per SM (0 = auto)                     */
+} igk_options;
+
+typedef struct {
+  int64_t affected;        /* |A u Psi0|: directly affected vertices + pending inserts */
+  int64_t inserted;        /* |Psi0|: pending pseudo vertices at refine start (Alg. 3 L2-5)  */
+  int64_t expanded;        /* |N|: neighbours of pseudo vertices examined in R2      */
+  int64_t filtered_in;     /* |C1|: affected vertices moved to the pseudo-partition (R1)     */
+  int64_t expanded_in;     /* |C2| (R2)                                                      */
+  int64_t evicted;         /* R3 balance-restoration evictions                               */
+  int64_t rounds;          /* R: Alg. 4 rounds until the pseudo-partition is empty   */
+  int64_t moves_applied;   /* sum of the balanced prefixes L_r                                */
+  int64_t moves_deferred;  /* sum of |S_r| - L_r                                              */
+  int64_t cut;             /* cut size after the refine                                */
+  int64_t cap;             /* c = cap(W) used by this refine (reading Q4)               */
+  int64_t max_part_weight;
+  int64_t imbalanced;      /* 1 iff the weighted fallback fired (IGK_WIMBALANCED)             */
+  int64_t adj_entries_scanned; /* adjacency entries read by the refine kernels               */
+} igk_refine_stats;
+
+/* Create a handle from a symmetric CSR graph.  n vertices with IDs
+ * 0..n-1; xadj[n+1] (int64), adjncy[xadj[n]] (no self loops, no duplicate
+ * neighbours, symmetric), vwgt[n] in [1,65535] or NULL (unit), adjwgt
+ * [xadj[n]] in [1,255] and symmetric, or NULL (unit); 2 <= k <= 254;
+ * 0 < epsilon <= 1 (imbalance ratio); init_part[n] in [0,k) (need not
+ * be balanced: the first igk_refine restores balance).  opt may be NULL.
+ * Returns IGK_EINVAL (no handle) on invalid input. */
+igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj,
+                      const int32_t* adjncy, const int32_t* vwgt, const int32_t* adjwgt,
+                      int32_t k, double epsilon, const int32_t* init_part, igk_graph** out);
+
+/* Apply one batch of modifiers (S1, Alg. 1-2; Alg. 3 L1-7 marking).
+ * The whole batch is validated on the device first; any invalid modifier ->
+ * IGK_EINVAL, nothing changes, and *bad_index (nullable) = the lowest
+ * invalid index.  Validity (against the pre-batch graph): no self loops; an
+ * undirected edge appears at most once among the batch's edge modifiers;
+ * EDGE_DELETE needs an existing edge whose endpoints are not deleted in the
+ * batch; VERTEX_DELETE needs an active vertex, at most once; EDGE_INSERT
+ * needs an absent edge whose endpoints are active and not deleted in the
+ * batch, or inserted in this batch (the j-th VERTEX_INSERT gets ID
+ * n_total + j); weights in range.  Phase order: edge deletions, vertex
+ * deletions, vertex insertions, edge insertions; inside a phase the batch
+ * order is irrelevant.  *first_new_id (nullable) = ID of the 1st insertion.
+ * mods is a HOST array. */
+igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count,
+                               int64_t* first_new_id, int64_t* bad_index);
+/* Same, with mods in DEVICE memory (count entries on the handle's device). */
+igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, int64_t count,
+                                      int64_t* first_new_id, int64_t* bad_index);
+
+/* Incremental refinement (Sec. V.C; R1 filter, R2 expansion, R3 balance
+ * restoration, R4 rounds of Alg. 4).  stats may be NULL.  Returns IGK_OK, or
+ * IGK_WIMBALANCED in the weighted corner case (result still valid). */
+igk_status igk_refine(igk_graph* g, igk_refine_stats* stats);
+
+/* out[v] for v < n_total: part in [0,k), -1 = deleted, -2 = pending (in the
+ * pseudo-partition between apply and refine).  cap_len too small ->
+ * IGK_EINVAL with *n_total still set. */
+igk_status igk_partition(const igk_graph* g, int32_t* out, int64_t cap_len, int64_t* n_total);
+/* cut size, maintained incrementally; edges with a pending endpoint
+ * are not counted. */
+igk_status igk_cut_size(const igk_graph* g, int64_t* out);
+/* part weights W_p, k entries */
+igk_status igk_part_weights(const igk_graph* g, int64_t* out_k);
+igk_status igk_num_vertices(const igk_graph* g, int64_t* n_total, int64_t* n_active);
+/* Recount cut and W_p from scratch with the cut/weight reduction kernel
+ * (S9, HBM-bound full store scan).  out_wp may be NULL. */
+igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp);
+/* Debug/test: current graph as a symmetric CSR over all IDs (deleted rows
+ * empty; row order unspecified).  Size query: call with xadj == NULL to get
+ * *n_total and *n_slots. */
+igk_status igk_export_csr(const igk_graph* g, int64_t* xadj, int64_t xadj_len, int32_t* adjncy,
+                          int32_t* adjwgt, int64_t adj_len, int64_t* n_total, int64_t* n_slots);
+/* number of kernels this handle has launched so far (instrumentation) */
+int64_t igk_kernel_launches(const igk_graph* g);
+/* device-side duration (ms) of the last igk_refine / apply / recount kernel,
+ * measured with CUDA events on the handle's stream */
+igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms);
+const char* igk_last_error(const igk_graph* g);
+void igk_destroy(igk_graph* g);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

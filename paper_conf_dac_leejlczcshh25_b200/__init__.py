@@ -1,0 +1,210 @@
+"""B200-native iG-kway incremental refinement (libigk.so, sm_100a).
+
+Thin ctypes binding of the C ABI in include/igk.h: argument marshalling only;
+every step of apply/refine runs in the CUDA kernels of csrc/.  There is no
+CPU fallback: if libigk.so is missing the import fails loudly.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libigk.so")
+
+OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE, WIMBALANCED = 0, 1, 2, 3, 4, 5, 6
+EDGE_DELETE, VERTEX_DELETE, VERTEX_INSERT, EDGE_INSERT = 0, 1, 2, 3
+
+STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evicted", "rounds",
+         "moves_applied", "moves_deferred", "cut", "cap", "max_part_weight", "imbalanced",
+         "adj_entries_scanned"]
+
+# every symbol include/igk.h declares (checked by tests/test_abi.py)
+SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine",
+           "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
+           "igk_export_csr", "igk_kernel_launches", "igk_last_kernel_ms", "igk_last_error", "igk_destroy"]
+
+
+class Options(C.Structure):
+    _fields_ = [("device", C.c_int), ("stream", C.c_void_p), ("max_vertices", C.c_int64),
+                ("max_slots", C.c_int64), ("slack_min", C.c_int32), ("validate", C.c_int32),
+                ("check_invariants", C.c_int32), ("blocks_per_sm", C.c_int32)]
+
+
+class Stats(C.Structure):
+    _fields_ = [(s, C.c_int64) for s in STATS]
+
+
+class IGKError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"igk status {status}: {msg}")
+        self.status = status
+
+
+_lib = None
+
+
+def lib():
+    """Load libigk.so (fails loudly if it was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_SO):
+            raise ImportError(f"{_SO} is missing: build it with `python -m "
+                              "paper_conf_dac_leejlczcshh25_b200.build` (no CPU fallback exists)")
+        L = C.CDLL(_SO)
+        P, i64, i32 = C.c_void_p, C.c_int64, C.c_int32
+        i64p, i32p = C.POINTER(C.c_int64), C.POINTER(C.c_int32)
+        L.igk_create.restype = C.c_int
+        L.igk_create.argtypes = [C.POINTER(Options), i64, i64p, i32p, i32p, i32p, i32, C.c_double, i32p,
+                                 C.POINTER(P)]
+        L.igk_apply_modifiers.restype = C.c_int
+        L.igk_apply_modifiers.argtypes = [P, P, i64, i64p, i64p]
+        L.igk_apply_modifiers_device.restype = C.c_int
+        L.igk_apply_modifiers_device.argtypes = [P, P, i64, i64p, i64p]
+        L.igk_refine.restype = C.c_int
+        L.igk_refine.argtypes = [P, C.POINTER(Stats)]
+        L.igk_partition.restype = C.c_int
+        L.igk_partition.argtypes = [P, i32p, i64, i64p]
+        L.igk_cut_size.restype = C.c_int
+        L.igk_cut_size.argtypes = [P, i64p]
+        L.igk_part_weights.restype = C.c_int
+        L.igk_part_weights.argtypes = [P, i64p]
+        L.igk_num_vertices.restype = C.c_int
+        L.igk_num_vertices.argtypes = [P, i64p, i64p]
+        L.igk_recount.restype = C.c_int
+        L.igk_recount.argtypes = [P, i64p, i64p]
+        L.igk_export_csr.restype = C.c_int
+        L.igk_export_csr.argtypes = [P, i64p, i64, i32p, i32p, i64, i64p, i64p]
+        L.igk_kernel_launches.restype = i64
+        L.igk_kernel_launches.argtypes = [P]
+        L.igk_last_kernel_ms.restype = C.c_int
+        L.igk_last_kernel_ms.argtypes = [P, C.POINTER(C.c_float), C.POINTER(C.c_float), C.POINTER(C.c_float)]
+        L.igk_last_error.restype = C.c_char_p
+        L.igk_last_error.argtypes = [P]
+        L.igk_destroy.restype = None
+        L.igk_destroy.argtypes = [P]
+        _lib = L
+    return _lib
+
+
+def _p(a, ct):
+    return None if a is None else a.ctypes.data_as(C.POINTER(ct))
+
+
+class IGKGraph:
+    """One GPU-resident graph + k-way partition (igk_create)."""
+
+    def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, device=0, stream=None,
+                 max_vertices=0, max_slots=0, slack_min=0, check=False, blocks_per_sm=0):
+        L = lib()
+        xadj = np.ascontiguousarray(xadj, dtype=np.int64)
+        adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
+        part = np.ascontiguousarray(part, dtype=np.int32)
+        vwgt = None if vwgt is None else np.ascontiguousarray(vwgt, dtype=np.int32)
+        adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
+        o = Options(device, stream or None, max_vertices, max_slots, slack_min, 1, int(check), blocks_per_sm)
+        h = C.c_void_p()
+        s = L.igk_create(C.byref(o), len(xadj) - 1, _p(xadj, C.c_int64), _p(adjncy, C.c_int32),
+                         _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(h))
+        if s != OK:
+            raise IGKError(s, "igk_create failed")
+        self.h = h
+        self.k = int(k)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().igk_destroy(self.h)
+            self.h = None
+
+    __del__ = close
+
+    def _err(self):
+        return lib().igk_last_error(self.h).decode()
+
+    def apply(self, mods):
+        m = np.ascontiguousarray(mods, dtype=np.int32).reshape(-1, 4)
+        fid, bad = C.c_int64(0), C.c_int64(-1)
+        s = lib().igk_apply_modifiers(self.h, m.ctypes.data, len(m), C.byref(fid), C.byref(bad))
+        return s, fid.value, bad.value
+
+    def apply_device(self, ptr: int, count: int):
+        """mods already in device memory (e.g. torch int32 (B,4) tensor .data_ptr())."""
+        fid, bad = C.c_int64(0), C.c_int64(-1)
+        s = lib().igk_apply_modifiers_device(self.h, C.c_void_p(ptr), count, C.byref(fid), C.byref(bad))
+        return s, fid.value, bad.value
+
+    def refine(self):
+        st = Stats()
+        s = lib().igk_refine(self.h, C.byref(st))
+        if s not in (OK, WIMBALANCED):
+            raise IGKError(s, self._err())
+        return s, {f: int(getattr(st, f)) for f in STATS}
+
+    def num_vertices(self):
+        nt, na = C.c_int64(0), C.c_int64(0)
+        s = lib().igk_num_vertices(self.h, C.byref(nt), C.byref(na))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return nt.value, na.value
+
+    def partition(self):
+        nt = C.c_int64(0)
+        lib().igk_partition(self.h, None, 0, C.byref(nt))
+        out = np.empty(max(nt.value, 1), dtype=np.int32)
+        s = lib().igk_partition(self.h, _p(out, C.c_int32), len(out), C.byref(nt))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return out[: nt.value]
+
+    def cut(self):
+        c = C.c_int64(0)
+        s = lib().igk_cut_size(self.h, C.byref(c))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return c.value
+
+    def part_weights(self):
+        out = np.zeros(self.k, dtype=np.int64)
+        s = lib().igk_part_weights(self.h, _p(out, C.c_int64))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return out
+
+    def recount(self):
+        c = C.c_int64(0)
+        wp = np.zeros(self.k, dtype=np.int64)
+        s = lib().igk_recount(self.h, C.byref(c), _p(wp, C.c_int64))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return c.value, wp
+
+    def export_csr(self, sort_rows=True):
+        nt, ns = C.c_int64(0), C.c_int64(0)
+        L = lib()
+        L.igk_export_csr(self.h, None, 0, None, None, 0, C.byref(nt), C.byref(ns))
+        xadj = np.empty(nt.value + 1, dtype=np.int64)
+        adj = np.empty(max(ns.value, 1), dtype=np.int32)
+        w = np.empty(max(ns.value, 1), dtype=np.int32)
+        s = L.igk_export_csr(self.h, _p(xadj, C.c_int64), len(xadj), _p(adj, C.c_int32), _p(w, C.c_int32),
+                             len(adj), C.byref(nt), C.byref(ns))
+        if s != OK:
+            raise IGKError(s, self._err())
+        adj, w = adj[: ns.value], w[: ns.value]
+        if sort_rows:
+            for u in range(nt.value):
+                a, b = xadj[u], xadj[u + 1]
+                if b - a > 1:
+                    o = np.argsort(adj[a:b], kind="stable")
+                    adj[a:b] = adj[a:b][o]
+                    w[a:b] = w[a:b][o]
+        return xadj, adj, w
+
+    def kernel_launches(self):
+        return int(lib().igk_kernel_launches(self.h))
+
+    def last_ms(self):
+        r, a, c = C.c_float(0), C.c_float(0), C.c_float(0)
+        lib().igk_last_kernel_ms(self.h, C.byref(r), C.byref(a), C.byref(c))
+        return {"refine": r.value, "apply": a.value, "recount": c.value}

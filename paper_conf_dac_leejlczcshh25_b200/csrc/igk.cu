@@ -1,0 +1,643 @@
+// igk.cu -- libigk: C ABI (include/igk.h) + create-time / query kernels.
+//
+// Hot path: k_apply (apply.cuh) and k_refine (refine.cuh), each ONE
+// persistent cooperative launch per call.  This file holds the handle, the
+// store build (S0), the cut/weight reduction (S9) and the exports.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/igk.h"
+#include "apply.cuh"
+#include "common.cuh"
+#include "refine.cuh"
+
+using namespace igk;
+
+// ---------------------------------------------------------------------------
+// create-time store build: copy every CSR row into its slab prefix
+// ---------------------------------------------------------------------------
+__global__ void k_build(Dev d, const int64_t* xadj, const int32_t* adjncy, const int32_t* adjwgt, int64_t n) {
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long u = gw; u < n; u += nw) {
+    const long long s = xadj[u], e = xadj[u + 1], o = d.off[u];
+    for (long long j = s + lane_id(); j < e; j += 32) {
+      d.adj[o + j - s] = adjncy[j];
+      if (d.adjw) d.adjw[o + j - s] = adjwgt[j];
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// S9: cut / part-weight reduction.  Each warp owns 32 consecutive
+// vertices and walks their concatenated adjacency 32 entries at a time
+// (owner lane found by a shuffle binary search), so slab reads stay
+// coalesced; the 1-byte label gather hits L2.  Edges counted once (u < x).
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp) {
+  __shared__ long long s_wp[256];
+  __shared__ long long s_red[32];
+  for (int p = threadIdx.x; p < 256; p += blockDim.x) s_wp[p] = 0;
+  __syncthreads();
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  const int lane = lane_id();
+  long long cut = 0;
+  for (long long base = gw * 32; base < n; base += nw * 32) {
+    long long v = base + lane;
+    bool act = v < n && __ldg(d.active + v);
+    uint8_t pv = act ? __ldg(d.part + v) : kPsi;
+    int dg = act ? __ldg(d.deg + v) : 0;
+    long long o = act ? __ldg(d.off + v) : 0;
+    if (act && pv != kPsi) atomicAdd((unsigned long long*)&s_wp[pv], (unsigned long long)vert_w(d.vw, v));
+    if (pv == kPsi) dg = 0;  // pending vertices own no cut edges
+    int pre = dg;
+#pragma unroll
+    for (int s = 1; s < 32; s <<= 1) {
+      int y = __shfl_up_sync(0xffffffffu, pre, s);
+      if (lane >= s) pre += y;
+    }
+    const int total = __shfl_sync(0xffffffffu, pre, 31);
+    pre -= dg;  // exclusive
+    for (int e0 = 0; e0 < total; e0 += 32) {
+      int e = e0 + lane;
+      int lo = 0;
+#pragma unroll
+      for (int st = 16; st > 0; st >>= 1) {
+        int cand = lo + st;
+        int pc = __shfl_sync(0xffffffffu, pre, cand & 31);
+        if (cand < 32 && pc <= e) lo = cand;
+      }
+      long long oo = __shfl_sync(0xffffffffu, o, lo);
+      int po = __shfl_sync(0xffffffffu, pre, lo);
+      int pp = __shfl_sync(0xffffffffu, (int)pv, lo);
+      if (e < total) {
+        long long j = oo + (e - po);
+        int x = __ldg(d.adj + j);
+        long long owner = base + lo;
+        uint8_t px = __ldg(d.part + x);
+        if (x > owner && px != kPsi && px != (uint8_t)pp) cut += edge_w(d.adjw, j);
+      }
+    }
+  }
+  block_atomic_add(out_cut, cut, s_red);
+  for (int p = threadIdx.x; p < d.k; p += blockDim.x)
+    if (s_wp[p]) atomicAdd((unsigned long long*)&out_wp[p], (unsigned long long)s_wp[p]);
+}
+
+__global__ void k_export_part(Dev d, long long n, int32_t* out) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
+    uint8_t p = d.part[v];
+    out[v] = !d.active[v] ? -1 : (p == kPsi ? -2 : (int)p);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// handle
+// ---------------------------------------------------------------------------
+struct igk_graph {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool poisoned = false;
+  std::string err;
+  Dev d{};
+  long long e_ppm = 0;
+  int vw_unit = 1, ew_unit = 1;
+  uint32_t epoch = 1;   // last stamp value handed out
+  uint32_t epochA = 0;  // stamp of the current affected set
+  int grid_apply = 0, grid_refine = 0;
+  size_t smem_refine = 0;
+  long long launches = 0;
+  igk_modifier* h_stage = nullptr;  // pinned staging for host batches
+  long long h_stage_cap = 0;
+  int4* d_mods = nullptr;
+  long long d_mods_cap = 0;
+  long long newid_cap = 0;
+  int check = 0;
+  long long hash_cap = 0;
+  int32_t* d_out = nullptr;  // export buffer
+  long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp
+  Ctl* h_ctl = nullptr;        // pinned mirror of the control block
+  cudaEvent_t ev[6] = {};
+  float ms_refine = 0, ms_apply = 0, ms_recount = 0;
+  std::vector<void*> allocs;
+};
+
+namespace {
+
+igk_status fail(igk_graph* g, igk_status s, const std::string& msg) {
+  if (g) g->err = msg;
+  return s;
+}
+
+bool cuda_ok(igk_graph* g, cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return true;
+  if (g) {
+    g->poisoned = true;
+    g->err = std::string(what) + ": " + cudaGetErrorString(e);
+  }
+  return false;
+}
+
+#define CK(call)                                            \
+  do {                                                      \
+    if (!cuda_ok(g, (call), #call)) return IGK_ECUDA;       \
+  } while (0)
+
+template <class T>
+bool dalloc(igk_graph* g, T** p, size_t count) {
+  void* q = nullptr;
+  if (cudaMalloc(&q, std::max<size_t>(count, 1) * sizeof(T)) != cudaSuccess) return false;
+  g->allocs.push_back(q);
+  *p = (T*)q;
+  return true;
+}
+
+uint32_t next_epoch(igk_graph* g) { return ++g->epoch; }
+
+int coop_grid(const void* fn, size_t smem, int want_per_sm) {
+  int dev = 0, sms = 0, occ = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kThreads, smem);
+  if (occ < 1) occ = 1;
+  int per = want_per_sm > 0 ? std::min(want_per_sm, occ) : 1;
+  return sms * per;
+}
+
+igk_status launch_recount(igk_graph* g) {
+  CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 257, g->stream));
+  int sms = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device));
+  long long n = g->h_ctl->n_total;
+  CK(cudaEventRecord(g->ev[4], g->stream));
+  k_recount<<<sms * 4, 512, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1);
+  g->launches++;
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(g->ev[5], g->stream));
+  return IGK_OK;
+}
+
+igk_status sync_ctl(igk_graph* g) {
+  CK(cudaMemcpyAsync(g->h_ctl, g->d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  return IGK_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                      const int32_t* vwgt, const int32_t* adjwgt, int32_t k, double epsilon,
+                      const int32_t* init_part, igk_graph** out) {
+  if (!out) return IGK_EINVAL;
+  *out = nullptr;
+  if (n < 0 || n > kNMax || k < 2 || k > kMaxK || !(epsilon > 0.0) || !(epsilon <= 1.0)) return IGK_EINVAL;
+  if (n > 0 && (!xadj || !init_part || (xadj[n] > 0 && !adjncy))) return IGK_EINVAL;
+  igk_options o{};
+  if (opt) o = *opt;
+  // ---- host-side validation of the CSR (create-time plumbing) ----
+  const long long m2 = n > 0 ? xadj[n] : 0;
+  if (n > 0 && xadj[0] != 0) return IGK_EINVAL;
+  for (int64_t u = 0; u < n; u++) {
+    if (xadj[u + 1] < xadj[u] || xadj[u + 1] - xadj[u] > kDegMax) return IGK_EINVAL;
+    if (init_part[u] < 0 || init_part[u] >= k) return IGK_EINVAL;
+    if (vwgt && (vwgt[u] < 1 || vwgt[u] > kVwMax)) return IGK_EINVAL;
+  }
+  {
+    std::vector<std::pair<int32_t, int32_t>> rows((size_t)m2);
+    for (int64_t u = 0; u < n; u++) {
+      for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+        int32_t x = adjncy[j], w = adjwgt ? adjwgt[j] : 1;
+        if (x < 0 || x >= n || x == u || w < 1 || w > kEwMax) return IGK_EINVAL;
+        rows[j] = {x, w};
+      }
+      std::sort(rows.begin() + xadj[u], rows.begin() + xadj[u + 1]);
+      for (int64_t j = xadj[u] + 1; j < xadj[u + 1]; j++)
+        if (rows[j].first == rows[j - 1].first) return IGK_EINVAL;
+    }
+    for (int64_t u = 0; u < n; u++) {
+      for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+        int32_t x = rows[j].first;
+        auto b = rows.begin() + xadj[x], e = rows.begin() + xadj[x + 1];
+        auto it = std::lower_bound(b, e, std::make_pair((int32_t)u, INT32_MIN));
+        if (it == e || it->first != u || it->second != rows[j].second) return IGK_EINVAL;
+      }
+    }
+  }
+  igk_graph* g = new igk_graph();
+  g->device = o.device;
+  g->stream = (cudaStream_t)o.stream;
+  g->e_ppm = llround(epsilon * 1e6);
+  g->vw_unit = vwgt == nullptr;
+  g->ew_unit = adjwgt == nullptr;
+  g->check = o.check_invariants;
+  if (cudaSetDevice(g->device) != cudaSuccess) {
+    delete g;
+    return IGK_ECUDA;
+  }
+  Dev& d = g->d;
+  d.k = k;
+  d.n_cap = o.max_vertices > 0 ? o.max_vertices : 2 * n + 65536;
+  if (d.n_cap < n || d.n_cap > kNMax) {
+    delete g;
+    return IGK_EINVAL;
+  }
+  d.slack_min = o.slack_min > 0 ? o.slack_min : 2;
+  int ib = 1;
+  while ((1ll << ib) < d.n_cap) ib++;
+  d.idbits = ib;
+  // slack capacities and offsets (prefix sum on the host at create time)
+  std::vector<int64_t> off((size_t)std::max<int64_t>(n, 1));
+  std::vector<int32_t> deg((size_t)std::max<int64_t>(n, 1)), capv((size_t)std::max<int64_t>(n, 1));
+  long long used = 0;
+  for (int64_t u = 0; u < n; u++) {
+    long long dg = xadj[u + 1] - xadj[u];
+    long long c = dg + std::max<long long>(d.slack_min, dg / 4);
+    c = (c + 3) & ~3ll;
+    off[u] = used;
+    deg[u] = (int32_t)dg;
+    capv[u] = (int32_t)c;
+    used += c;
+  }
+  d.slot_cap = o.max_slots > 0 ? o.max_slots : 4 * used + (1ll << 22);
+  if (d.slot_cap < used) {
+    delete g;
+    return IGK_EINVAL;
+  }
+  const size_t N = (size_t)d.n_cap;
+  bool ok = dalloc(g, &d.off, N) && dalloc(g, &d.deg, N) && dalloc(g, &d.capv, N) &&
+            dalloc(g, &d.adj, (size_t)d.slot_cap) && (g->ew_unit || dalloc(g, &d.adjw, (size_t)d.slot_cap)) &&
+            dalloc(g, &d.active, N) && (g->vw_unit || dalloc(g, &d.vw, N)) && dalloc(g, &d.part, N) &&
+            dalloc(g, &d.markA, N) && dalloc(g, &d.markT, N) && dalloc(g, &d.markD, N) &&
+            dalloc(g, &d.markG, N) && dalloc(g, &d.vcnt, N) && dalloc(g, &d.icnt, N) &&
+            dalloc(g, &d.Alist, N) && dalloc(g, &d.psi[0], N) && dalloc(g, &d.psi[1], N) &&
+            dalloc(g, &d.cand, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
+            dalloc(g, &d.dlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
+            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) &&
+            dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
+            dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
+            dalloc(g, &g->d_red, 257);
+  if (!ok) {
+    igk_destroy(g);
+    return IGK_ENOMEM;
+  }
+  if (cudaMallocHost(&g->h_ctl, sizeof(Ctl)) != cudaSuccess) {
+    igk_destroy(g);
+    return IGK_ENOMEM;
+  }
+  for (auto& e : g->ev) cudaEventCreate(&e);
+  // zero-init
+  cudaStream_t s = g->stream;
+  cudaMemsetAsync(d.active, 0, N, s);
+  cudaMemsetAsync(d.part, kDel, N, s);
+  cudaMemsetAsync(d.deg, 0, N * 4, s);
+  cudaMemsetAsync(d.capv, 0, N * 4, s);
+  cudaMemsetAsync(d.off, 0, N * 8, s);
+  cudaMemsetAsync(d.markA, 0, N * 4, s);
+  cudaMemsetAsync(d.markT, 0, N * 4, s);
+  cudaMemsetAsync(d.markD, 0, N * 4, s);
+  cudaMemsetAsync(d.markG, 0, N * 4, s);
+  cudaMemsetAsync(d.vcnt, 0, N * 4, s);
+  cudaMemsetAsync(d.icnt, 0, N * 4, s);
+  cudaMemsetAsync(d.hist0, 0, 256 * kDigits * 8, s);
+  cudaMemsetAsync(d.histR, 0, 3 * 256 * kDigits * 8, s);
+  cudaMemsetAsync(d.ctl, 0, sizeof(Ctl), s);
+  // upload
+  int64_t* d_xadj = nullptr;
+  int32_t *d_adjncy = nullptr, *d_adjwgt = nullptr;
+  if (cudaMalloc(&d_xadj, (n + 1) * 8) != cudaSuccess || cudaMalloc(&d_adjncy, std::max<long long>(m2, 1) * 4) != cudaSuccess ||
+      (!g->ew_unit && cudaMalloc(&d_adjwgt, std::max<long long>(m2, 1) * 4) != cudaSuccess)) {
+    cudaFree(d_xadj);
+    cudaFree(d_adjncy);
+    igk_destroy(g);
+    return IGK_ENOMEM;
+  }
+  std::vector<uint8_t> part8((size_t)std::max<int64_t>(n, 1)), act((size_t)std::max<int64_t>(n, 1), 1);
+  for (int64_t u = 0; u < n; u++) part8[u] = (uint8_t)init_part[u];
+  cudaError_t e = cudaSuccess;
+  if (n > 0) {
+    e = cudaMemcpy(d_xadj, xadj, (n + 1) * 8, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && m2) e = cudaMemcpy(d_adjncy, adjncy, m2 * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && m2 && d_adjwgt) e = cudaMemcpy(d_adjwgt, adjwgt, m2 * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d.off, off.data(), n * 8, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d.deg, deg.data(), n * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d.capv, capv.data(), n * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d.part, part8.data(), n, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d.active, act.data(), n, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && d.vw) e = cudaMemcpy(d.vw, vwgt, n * 4, cudaMemcpyHostToDevice);
+  }
+  if (e == cudaSuccess && n > 0) {
+    k_build<<<1184, 256, 0, s>>>(d, d_xadj, d_adjncy, d_adjwgt, n);
+    g->launches++;
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaFree(d_xadj);
+  cudaFree(d_adjncy);
+  cudaFree(d_adjwgt);
+  if (e != cudaSuccess) {
+    igk_destroy(g);
+    return IGK_ECUDA;
+  }
+  // control block: n_total, slab top, W, W_p, cut (from the reduction kernel)
+  long long W = 0;
+  for (int64_t u = 0; u < n; u++) W += vwgt ? vwgt[u] : 1;
+  std::memset(g->h_ctl, 0, sizeof(Ctl));
+  g->h_ctl->n_total = n;
+  g->h_ctl->slab_top = used;
+  g->h_ctl->W = W;
+  g->h_ctl->err_idx = kNoErr;
+  if (launch_recount(g) != IGK_OK) {
+    igk_destroy(g);
+    return IGK_ECUDA;
+  }
+  long long red[257];
+  if (cudaMemcpy(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost) != cudaSuccess) {
+    igk_destroy(g);
+    return IGK_ECUDA;
+  }
+  g->h_ctl->cut = red[0];
+  for (int p = 0; p < k; p++) g->h_ctl->Wp[p] = red[1 + p];
+  if (cudaMemcpy(d.ctl, g->h_ctl, sizeof(Ctl), cudaMemcpyHostToDevice) != cudaSuccess) {
+    igk_destroy(g);
+    return IGK_ECUDA;
+  }
+  // persistent grids
+  g->smem_refine = sizeof(RefSmem);
+  cudaFuncSetAttribute(k_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
+  g->grid_apply = coop_grid((const void*)k_apply, 0, o.blocks_per_sm);
+  g->grid_refine = coop_grid((const void*)k_refine, g->smem_refine, o.blocks_per_sm);
+  if (g->grid_apply > 4096) g->grid_apply = 4096;
+  g->epochA = next_epoch(g);
+  *out = g;
+  return IGK_OK;
+}
+
+static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t* first_new_id, int64_t* bad_index) {
+  if (bad_index) *bad_index = -1;
+  if (first_new_id) *first_new_id = g->h_ctl->n_total;
+  if (count == 0) return IGK_OK;
+  // duplicate-detection hash: >= 2 * count slots, power of two
+  long long need = 64;
+  while (need < 2 * count + 2) need <<= 1;
+  if (need > g->hash_cap) {
+    if (g->d.hkeys) cudaFree(g->d.hkeys);
+    if (g->d.hcnt) cudaFree(g->d.hcnt);
+    g->d.hkeys = nullptr;
+    g->d.hcnt = nullptr;
+    if (cudaMalloc(&g->d.hkeys, need * 8) != cudaSuccess || cudaMalloc(&g->d.hcnt, need * 4) != cudaSuccess)
+      return fail(g, IGK_ENOMEM, "hash allocation failed");
+    g->hash_cap = need;
+  }
+  if (count > g->newid_cap) {
+    if (g->d.newid) cudaFree(g->d.newid);
+    g->d.newid = nullptr;
+    g->newid_cap = 0;
+    if (cudaMalloc(&g->d.newid, count * 4) != cudaSuccess) return fail(g, IGK_ENOMEM, "newid allocation failed");
+    g->newid_cap = count;
+  }
+  g->d.hmask = g->hash_cap - 1;
+  ApplyArgs a;
+  a.mods = dm;
+  a.B = count;
+  a.n0 = g->h_ctl->n_total;
+  a.epD = next_epoch(g);
+  a.epT = next_epoch(g);
+  a.epG = next_epoch(g);
+  a.epA = g->epochA;
+  a.vw_unit = g->vw_unit;
+  a.ew_unit = g->ew_unit;
+  void* args[] = {(void*)&g->d, (void*)&a};
+  CK(cudaEventRecord(g->ev[2], g->stream));
+  CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply, kThreads, args, 0, g->stream));
+  g->launches++;
+  CK(cudaEventRecord(g->ev[3], g->stream));
+  igk_status st = sync_ctl(g);
+  if (st != IGK_OK) return st;
+  cudaEventElapsedTime(&g->ms_apply, g->ev[2], g->ev[3]);
+  if (g->h_ctl->err_idx != kNoErr) {
+    if (bad_index) *bad_index = g->h_ctl->err_idx;
+    char buf[128];
+    snprintf(buf, sizeof buf, "invalid modifier at index %lld", g->h_ctl->err_idx);
+    return fail(g, IGK_EINVAL, buf);
+  }
+  if (g->h_ctl->err_nomem) return fail(g, IGK_ENOMEM, "vertex or slot capacity exhausted");
+  return IGK_OK;
+}
+
+igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count, int64_t* first_new_id,
+                               int64_t* bad_index) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
+  if (count == 0) return apply_dev(g, nullptr, 0, first_new_id, bad_index);
+  if (count > g->h_stage_cap) {
+    if (g->h_stage) cudaFreeHost(g->h_stage);
+    g->h_stage = nullptr;
+    if (cudaMallocHost(&g->h_stage, count * sizeof(igk_modifier)) != cudaSuccess)
+      return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
+    g->h_stage_cap = count;
+  }
+  if (count > g->d_mods_cap) {
+    if (g->d_mods) cudaFree(g->d_mods);
+    g->d_mods = nullptr;
+    g->d_mods_cap = 0;
+    if (cudaMalloc(&g->d_mods, count * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
+    g->d_mods_cap = count;
+  }
+  std::memcpy(g->h_stage, mods, count * sizeof(igk_modifier));
+  CK(cudaMemcpyAsync(g->d_mods, g->h_stage, count * 16, cudaMemcpyHostToDevice, g->stream));
+  return apply_dev(g, g->d_mods, count, first_new_id, bad_index);
+}
+
+igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, int64_t count,
+                                      int64_t* first_new_id, int64_t* bad_index) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (count < 0 || (count > 0 && !d_mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
+  return apply_dev(g, (const int4*)d_mods, count, first_new_id, bad_index);
+}
+
+igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  RefineArgs a;
+  a.e_ppm = g->e_ppm;
+  a.epC1 = next_epoch(g);
+  a.epN = next_epoch(g);
+  a.epC2 = next_epoch(g);
+  a.epE = next_epoch(g);
+  void* args[] = {(void*)&g->d, (void*)&a};
+  CK(cudaEventRecord(g->ev[0], g->stream));
+  CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
+  g->launches++;
+  CK(cudaEventRecord(g->ev[1], g->stream));
+  igk_status st = sync_ctl(g);
+  if (st != IGK_OK) return st;
+  cudaEventElapsedTime(&g->ms_refine, g->ev[0], g->ev[1]);
+  g->epochA = next_epoch(g);
+  const long long* so = g->h_ctl->st_out;
+  if (stats) {
+    stats->affected = so[ST_AFFECTED];
+    stats->inserted = so[ST_INSERTED];
+    stats->expanded = so[ST_EXPANDED];
+    stats->filtered_in = so[ST_FILTERED_IN];
+    stats->expanded_in = so[ST_EXPANDED_IN];
+    stats->evicted = so[ST_EVICTED];
+    stats->rounds = so[ST_ROUNDS];
+    stats->moves_applied = so[ST_MOVES_APPLIED];
+    stats->moves_deferred = so[ST_MOVES_DEFERRED];
+    stats->cut = so[ST_CUT];
+    stats->cap = so[ST_CAP];
+    stats->max_part_weight = so[ST_MAXW];
+    stats->imbalanced = so[ST_IMBAL];
+    stats->adj_entries_scanned = so[ST_SCANNED];
+  }
+  const bool imbal = so[ST_IMBAL] != 0;
+  if (g->check) {  // invariant I1/I2: maintained cut and W_p equal a recount
+    int64_t cut = 0;
+    int64_t wp[256];
+    st = igk_recount(g, &cut, wp);
+    if (st != IGK_OK) return st;
+    bool bad = cut != g->h_ctl->cut;
+    for (int p = 0; p < g->d.k; p++) bad |= wp[p] != g->h_ctl->Wp[p];
+    if (bad) {
+      g->poisoned = true;
+      return fail(g, IGK_ESTATE, "invariant check failed: maintained cut/W_p differ from the recount");
+    }
+  }
+  return imbal ? IGK_WIMBALANCED : IGK_OK;
+}
+
+igk_status igk_partition(const igk_graph* gc, int32_t* out, int64_t cap_len, int64_t* n_total) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return IGK_ESTATE;
+  long long n = g->h_ctl->n_total;
+  if (n_total) *n_total = n;
+  if (!out || cap_len < n) return fail(g, IGK_EINVAL, "output buffer too small");
+  if (n == 0) return IGK_OK;
+  k_export_part<<<592, 256, 0, g->stream>>>(g->d, n, g->d_out);
+  g->launches++;
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(out, g->d_out, n * 4, cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  return IGK_OK;
+}
+
+igk_status igk_cut_size(const igk_graph* gc, int64_t* out) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (!out) return IGK_EINVAL;
+  CK(cudaMemcpyAsync(&g->h_ctl->cut, &g->d.ctl->cut, 8, cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  *out = g->h_ctl->cut;
+  return IGK_OK;
+}
+
+igk_status igk_part_weights(const igk_graph* gc, int64_t* out_k) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (!out_k) return IGK_EINVAL;
+  CK(cudaMemcpyAsync(g->h_ctl->Wp, g->d.ctl->Wp, 8 * g->d.k, cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  for (int p = 0; p < g->d.k; p++) out_k[p] = g->h_ctl->Wp[p];
+  return IGK_OK;
+}
+
+igk_status igk_num_vertices(const igk_graph* gc, int64_t* n_total, int64_t* n_active) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (n_total) *n_total = g->h_ctl->n_total;
+  if (n_active) {
+    long long n = g->h_ctl->n_total;
+    std::vector<uint8_t> act((size_t)std::max<long long>(n, 1));
+    if (n) CK(cudaMemcpy(act.data(), g->d.active, n, cudaMemcpyDeviceToHost));
+    long long c = 0;
+    for (long long v = 0; v < n; v++) c += act[v];
+    *n_active = c;
+  }
+  return IGK_OK;
+}
+
+igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  igk_status st = launch_recount(g);
+  if (st != IGK_OK) return st;
+  long long red[257];
+  CK(cudaMemcpyAsync(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  cudaEventElapsedTime(&g->ms_recount, g->ev[4], g->ev[5]);
+  if (out_cut) *out_cut = red[0];
+  if (out_wp)
+    for (int p = 0; p < g->d.k; p++) out_wp[p] = red[1 + p];
+  return IGK_OK;
+}
+
+igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, int32_t* adjncy, int32_t* adjwgt,
+                          int64_t adj_len, int64_t* n_total, int64_t* n_slots) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return IGK_ESTATE;
+  long long n = g->h_ctl->n_total;
+  std::vector<int64_t> off((size_t)std::max<long long>(n, 1));
+  std::vector<int32_t> deg((size_t)std::max<long long>(n, 1));
+  if (n) {
+    CK(cudaMemcpy(off.data(), g->d.off, n * 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(deg.data(), g->d.deg, n * 4, cudaMemcpyDeviceToHost));
+  }
+  long long tot = 0;
+  for (long long v = 0; v < n; v++) tot += deg[v];
+  if (n_total) *n_total = n;
+  if (n_slots) *n_slots = tot;
+  if (!xadj) return IGK_OK;
+  if (xadj_len < n + 1 || adj_len < tot || !adjncy) return fail(g, IGK_EINVAL, "export buffers too small");
+  xadj[0] = 0;
+  long long pos = 0;
+  for (long long v = 0; v < n; v++) {
+    if (deg[v]) {
+      CK(cudaMemcpy(adjncy + pos, g->d.adj + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
+      if (adjwgt) {
+        if (g->d.adjw) {
+          CK(cudaMemcpy(adjwgt + pos, g->d.adjw + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
+        } else {
+          for (int i = 0; i < deg[v]; i++) adjwgt[pos + i] = 1;
+        }
+      }
+    }
+    pos += deg[v];
+    xadj[v + 1] = pos;
+  }
+  return IGK_OK;
+}
+
+int64_t igk_kernel_launches(const igk_graph* g) { return g ? g->launches : 0; }
+
+igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms) {
+  if (!g) return IGK_ESTATE;
+  if (refine_ms) *refine_ms = g->ms_refine;
+  if (apply_ms) *apply_ms = g->ms_apply;
+  if (recount_ms) *recount_ms = g->ms_recount;
+  return IGK_OK;
+}
+
+const char* igk_last_error(const igk_graph* g) { return g ? g->err.c_str() : "null handle"; }
+
+void igk_destroy(igk_graph* g) {
+  if (!g) return;
+  cudaStreamSynchronize(g->stream);
+  for (void* p : g->allocs) cudaFree(p);
+  if (g->d.hkeys) cudaFree(g->d.hkeys);
+  if (g->d.hcnt) cudaFree(g->d.hcnt);
+  if (g->d.newid) cudaFree(g->d.newid);
+  if (g->d_mods) cudaFree(g->d_mods);
+  if (g->h_stage) cudaFreeHost(g->h_stage);
+  if (g->h_ctl) cudaFreeHost(g->h_ctl);
+  for (auto& e : g->ev)
+    if (e) cudaEventDestroy(e);
+  delete g;
+}
+
+}  // extern "C"

@@ -1,0 +1,64 @@
+"""Side-by-side driver: CUDA path (through the C ABI) vs the CPU oracle on the
+same seeded inputs; every comparison is bit-exact (integer-only method)."""
+from __future__ import annotations
+
+import numpy as np
+
+import oracle
+import paper_conf_dac_leejlczcshh25_b200 as igk
+
+COMMON = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evicted", "rounds",
+          "moves_applied", "moves_deferred", "cut", "cap", "max_part_weight", "imbalanced"]
+
+
+class Pair:
+    def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, check=True, **kw):
+        self.O = oracle.Oracle(xadj, adjncy, k, eps, part, vwgt, adjwgt)
+        self.G = igk.IGKGraph(xadj, adjncy, k, eps, part, vwgt, adjwgt, check=check, **kw)
+        self.k = k
+
+    def compare_state(self, where="", full_csr=False):
+        po, pg = self.O.partition(), self.G.partition()
+        assert len(po) == len(pg), where
+        if not np.array_equal(po, pg):
+            bad = np.nonzero(po != pg)[0]
+            raise AssertionError(f"{where}: {len(bad)} partition entries differ, first {bad[:8]} "
+                                 f"oracle {po[bad[:8]]} gpu {pg[bad[:8]]}")
+        assert self.O.cut() == self.G.cut(), where
+        assert np.array_equal(self.O.part_weights(), self.G.part_weights()), where
+        rc, rwp = self.G.recount()
+        assert rc == self.G.cut(), f"{where}: maintained cut != recount"
+        if full_csr:
+            xo, ao, wo = self.O.export_csr()
+            xg, ag, wg = self.G.export_csr()
+            assert np.array_equal(xo, xg) and np.array_equal(ao, ag) and np.array_equal(wo, wg), where
+
+    def apply(self, batch, where=""):
+        so = self.O.apply(batch)
+        sg = self.G.apply(batch)
+        assert so[0] == sg[0], f"{where}: status oracle {so} gpu {sg}"
+        assert so[1] == sg[1], where
+        if so[0] != 0:
+            assert so[2] == sg[2], f"{where}: bad index oracle {so[2]} gpu {sg[2]}"
+        return so[0]
+
+    def refine(self, where=""):
+        so, sto = self.O.refine()
+        sg, stg = self.G.refine()
+        assert so == sg, where
+        diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
+        assert not diff, f"{where}: stats differ (oracle, gpu): {diff}"
+        return sto, stg
+
+
+def run_stream(pair: Pair, batches, full_csr_every=0, tag=""):
+    stats = []
+    for it, b in enumerate(batches):
+        st = pair.apply(b, f"{tag} it{it} apply")
+        assert st == 0
+        pair.compare_state(f"{tag} it{it} after apply",
+                           full_csr=bool(full_csr_every) and it % full_csr_every == 0)
+        sto, stg = pair.refine(f"{tag} it{it} refine")
+        pair.compare_state(f"{tag} it{it} after refine")
+        stats.append(stg)
+    return stats

@@ -1,0 +1,70 @@
+"""CPU-only checks of the boundary: libigk.so loads and exports every entry
+point include/igk.h declares; the product and the oracle share no code."""
+import os
+import re
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HDR = os.path.join(ROOT, "include", "igk.h")
+PKG = os.path.join(ROOT, "paper_conf_dac_leejlczcshh25_b200")
+SO = os.path.join(PKG, "libigk.so")
+
+
+def _declared():
+    txt = open(HDR).read()
+    return sorted(set(re.findall(r"\b(igk_[a-z_]+)\s*\(", txt)))
+
+
+def _ensure_built():
+    if not os.path.exists(SO):
+        from paper_conf_dac_leejlczcshh25_b200 import build
+        build.build()
+
+
+def test_header_declares_the_boundary():
+    names = _declared()
+    for req in ["igk_create", "igk_apply_modifiers", "igk_refine", "igk_partition", "igk_cut_size"]:
+        assert req in names
+
+
+def test_library_exports_every_declared_symbol():
+    _ensure_built()
+    out = subprocess.run(["nm", "-D", "--defined-only", SO], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (igk_[a-z_]+)\b", out))
+    missing = [s for s in _declared() if s not in exported]
+    assert not missing, missing
+    import paper_conf_dac_leejlczcshh25_b200 as igk
+    L = igk.lib()
+    for s in _declared():
+        assert hasattr(L, s)
+    assert sorted(igk.SYMBOLS) == _declared()
+
+
+def test_library_is_sm100a_and_has_no_oracle_code():
+    _ensure_built()
+    out = subprocess.run(["nm", "-D", SO], capture_output=True, text=True).stdout
+    assert "ora_" not in out
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", SO], capture_output=True, text=True).stdout
+    assert "sm_100a" in sass
+
+
+def test_product_sources_do_not_touch_the_oracle():
+    bad = re.compile(r"import\s+oracle|from\s+oracle|igk_oracle|\bora_[a-z]|liboracle|oracle/igk")
+    for dirpath, _, files in os.walk(PKG):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                assert not bad.search(open(os.path.join(dirpath, f)).read()), f
+    bad2 = re.compile(r"#include\s+\"[^\"]*igk\.h\"|import\s+paper_conf|from\s+paper_conf|csrc/")
+    for f in os.listdir(os.path.join(ROOT, "oracle")):
+        if f.endswith((".c", ".h", ".py")):
+            assert not bad2.search(open(os.path.join(ROOT, "oracle", f)).read()), f
+
+
+def test_gpu_free_import_fails_loudly_without_library(tmp_path, monkeypatch):
+    import paper_conf_dac_leejlczcshh25_b200 as igk
+    monkeypatch.setattr(igk, "_SO", str(tmp_path / "missing.so"))
+    monkeypatch.setattr(igk, "_lib", None)
+    with pytest.raises(ImportError):
+        igk.lib()

@@ -1,0 +1,242 @@
+"""GPU parity: the CUDA path (C ABI) vs the CPU oracle, bit-exact.
+
+Covers the worked examples, tiny random graphs (weighted and unit), invalid
+batches (atomic rejection with the same first index), the BASELINE configs C1
+(all 20 iterations), C2 (1M vertices, full-size, 100 iterations; 1000 under
+the `slow` marker), C3-style k / batch sweeps, C5-style forced restoration,
+batch-order invariance, multi-apply accumulation and edge cases.
+"""
+import json
+import os
+import random
+
+import numpy as np
+import pytest
+
+import igk_inputs as gi
+from tests.parity import Pair, run_stream
+from tests.tinycases import random_batch, random_graph
+
+pytestmark = pytest.mark.gpu
+GOLD = os.path.join(os.path.dirname(__file__), "golden", "examples.json")
+
+
+def _csr(n, edges):
+    adj = {u: set() for u in range(n)}
+    for u, v in edges:
+        adj[u].add(v)
+        adj[v].add(u)
+    xadj, a = [0], []
+    for u in range(n):
+        a += sorted(adj[u])
+        xadj.append(len(a))
+    return np.array(xadj, np.int64), np.array(a, np.int32)
+
+
+@pytest.mark.parametrize("ex", json.load(open(GOLD))["examples"], ids=lambda e: e["name"])
+def test_worked_examples(ex):
+    xadj, adj = _csr(ex["n"], ex["edges"])
+    P = Pair(xadj, adj, ex["k"], ex["eps"], np.array(ex["part0"], np.int32))
+    assert P.apply(np.array(ex["batch"], np.int32)) == 0
+    P.compare_state("after apply", full_csr=True)
+    sto, stg = P.refine()
+    assert list(P.G.partition()) == ex["final_part"]
+    assert stg["cut"] == ex["final_cut"] and stg["rounds"] == ex["rounds"]
+    P.compare_state("after refine", full_csr=True)
+
+
+def _tiny(seed):
+    rng = random.Random(seed)
+    n = rng.randint(3, 40)
+    k = rng.choice([2, 3, 4, 7])
+    weighted = rng.random() < 0.4
+    eps = rng.choice([0.03, 0.1, 0.5, 1.0])
+    xadj, adjncy, adjwgt, vwgt, adj = random_graph(rng, n, rng.choice([0.1, 0.2, 0.4]), weighted)
+    part0 = np.array([rng.randrange(k) for _ in range(n)], np.int32)
+    P = Pair(xadj, adjncy, k, eps, part0, vwgt if weighted else None, adjwgt if weighted else None)
+    P.refine("settle")
+    P.compare_state("settle", full_csr=True)
+    for it in range(4):
+        xa, aj, aw = P.O.export_csr()
+        part = P.O.partition()
+        cur = {u: {int(aj[j]): int(aw[j]) for j in range(xa[u], xa[u + 1])} for u in range(len(part))}
+        active = {u: part[u] != -1 for u in range(len(part))}
+        b = random_batch(rng, cur, active, weighted, max_ops=10)
+        assert P.apply(b, f"seed{seed} it{it}") == 0
+        P.compare_state(f"seed{seed} it{it} apply", full_csr=True)
+        P.refine(f"seed{seed} it{it}")
+        P.compare_state(f"seed{seed} it{it} refine", full_csr=True)
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_tiny_random(seed):
+    _tiny(seed)
+
+
+def test_invalid_batches_atomic():
+    xadj, adj = _csr(6, [(0, 1), (1, 2), (3, 4), (4, 5)])
+    part0 = np.array([0, 0, 0, 1, 1, 1], np.int32)
+    bad = [[[0, 0, 2, 0]], [[3, 0, 1, 1]], [[3, 2, 2, 1]], [[1, 7, 0, 0]], [[1, 2, 0, 0], [1, 2, 0, 0]],
+           [[3, 0, 3, 1], [3, 3, 0, 1]], [[3, 0, 3, 1], [0, 3, 0, 0]], [[1, 1, 0, 0], [0, 0, 1, 0]],
+           [[1, 4, 0, 0], [3, 0, 4, 1]], [[3, 0, 6, 1]], [[2, 0, 0, 1], [3, 0, 7, 1]], [[2, 0, 0, 2]],
+           [[3, 0, 3, 2]], [[9, 0, 1, 1]], [[3, 0, 3, 1], [0, 0, 5, 0]], [[3, -1, 3, 1]]]
+    P = Pair(xadj, adj, 2, 0.1, part0)
+    for b in bad:
+        before = (P.G.partition().tobytes(), P.G.export_csr()[1].tobytes())
+        st = P.apply(np.array(b, np.int32), str(b))
+        assert st == 1, b
+        assert (P.G.partition().tobytes(), P.G.export_csr()[1].tobytes()) == before
+    # a valid batch still works afterwards
+    assert P.apply(np.array([[2, 0, 0, 1], [3, 6, 0, 1], [0, 3, 4, 0]], np.int32)) == 0
+    P.refine()
+    P.compare_state("after", full_csr=True)
+
+
+def _cfg_pair(name, idx, n=None, k=None, weighted=False, check=True):
+    cfg = dict(gi.CONFIGS[name])
+    n = n or cfg["n"]
+    k = k or (cfg["k"] if isinstance(cfg["k"], int) else cfg["k"][0])
+    g = gi.make_graph(n, cfg["fmax"], gi.graph_seed(idx), weighted=weighted)
+    part, _ = gi.metis_partition(g, k)
+    P = Pair(g.xadj, g.adjncy, k, cfg["eps"], part, g.vwgt, g.adjwgt, check=check)
+    return cfg, g, part, P
+
+
+def test_c1_all_iterations():
+    cfg, g, part, P = _cfg_pair("C1", 1)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(1)))
+    batches = [gi.next_batch(S, cfg) for _ in range(cfg["iters"])]
+    run_stream(P, batches, full_csr_every=5, tag="C1")
+
+
+def _c2(iters):
+    cfg, g, part, P = _cfg_pair("C2", 2, check=False)
+    P.refine("settle")
+    P.compare_state("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(2)))
+    for it in range(iters):
+        b = gi.next_batch(S, cfg)
+        assert P.apply(b, f"C2 it{it}") == 0
+        P.refine(f"C2 it{it}")
+        if it % 10 == 0 or it == iters - 1:
+            P.compare_state(f"C2 it{it}")
+    P.compare_state("C2 end", full_csr=True)
+
+
+def test_c2_full_size_100_iterations():
+    _c2(100)
+
+
+@pytest.mark.slow
+def test_c2_full_size_1000_iterations():
+    _c2(1000)
+
+
+@pytest.mark.parametrize("k", [2, 8, 32, 64])
+def test_c3_k_sweep_large_frontier(k):
+    cfg, g, part, P = _cfg_pair("C3", 3, n=200_000, k=k, check=False)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(3)) + k)
+    for it, frac in enumerate([0.001, 0.01, 0.1, 0.1, 0.03]):
+        b = S.next(gi.MODE_MIX, frac)
+        assert P.apply(b, f"k{k} it{it}") == 0
+        P.refine(f"k{k} it{it}")
+        P.compare_state(f"k{k} it{it}")
+
+
+def test_weighted_mixed_stream():
+    cfg, g, part, P = _cfg_pair("C1", 6, n=20_000, k=8, weighted=True)
+    P.refine("settle")
+    P.compare_state("settle")
+    S = gi.Stream(g, 99, weighted=True)
+    for it in range(10):
+        b = S.next(gi.MODE_MIX, 0.02)
+        assert P.apply(b, f"w it{it}") == 0
+        P.refine(f"w it{it}")
+        P.compare_state(f"w it{it}", full_csr=(it % 3 == 0))
+
+
+def test_adversarial_restoration():
+    n, k = 40_000, 8
+    g = gi.make_graph(n, 1000, gi.graph_seed(5))
+    part, _ = gi.metis_partition(g, k)
+    P = Pair(g.xadj, g.adjncy, k, 0.03, part)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(5)), region0=(part == 0).astype(np.int32))
+    ev = 0
+    for it in range(12):
+        b = S.next(gi.MODE_ADVERSARIAL, 0.0, n // 100, n // 200, 0, 0)
+        assert P.apply(b, f"adv it{it}") == 0
+        sto, stg = P.refine(f"adv it{it}")
+        ev += stg["evicted"]
+        P.compare_state(f"adv it{it}")
+    assert ev > 0
+
+
+def test_batch_permutation_invariance():
+    g = gi.make_graph(5000, 64, 17)
+    part = gi.block_partition(g.n, 4)
+    S = gi.Stream(g, 3)
+    b = S.next(gi.MODE_MIX, 0.05)
+    res = []
+    for perm in range(3):
+        bb = b.copy()
+        if perm:
+            vi = bb[:, 0] == 2
+            others = np.nonzero(~vi)[0]
+            rng = np.random.default_rng(perm)
+            idx = np.arange(len(bb))
+            idx[others] = rng.permutation(others)   # vertex insertions keep their order
+            bb = bb[idx]
+        P = Pair(g.xadj, g.adjncy, 4, 0.03, part)
+        assert P.apply(bb) == 0
+        P.refine()
+        res.append((P.G.partition().tobytes(), P.G.cut()))
+    assert res[0] == res[1] == res[2]
+
+
+def test_multiple_applies_then_one_refine():
+    g = gi.make_graph(20_000, 64, 23)
+    part, _ = gi.metis_partition(g, 4)
+    P = Pair(g.xadj, g.adjncy, 4, 0.03, part)
+    P.refine()
+    S = gi.Stream(g, 5)
+    for it in range(3):
+        for j in range(3):
+            assert P.apply(S.next(gi.MODE_MIX, 0.01), f"it{it}.{j}") == 0
+            P.compare_state(f"it{it}.{j}")
+        P.refine(f"it{it}")
+        P.compare_state(f"it{it}", full_csr=True)
+
+
+def test_edge_cases():
+    # empty batch, refine without modifiers, imbalanced start, k=254, growth from n=3
+    xadj, adj = _csr(3, [(0, 1)])
+    P = Pair(xadj, adj, 2, 0.5, np.array([0, 0, 0], np.int32))
+    P.refine("imbalanced start")
+    P.compare_state("imbalanced start", full_csr=True)
+    assert P.apply(np.zeros((0, 4), np.int32)) == 0
+    P.refine("empty")
+    P.compare_state("empty")
+    batch = [[2, 0, 0, 1]] * 50 + [[3, 3 + i, 3 + (i * 7 + 1) % 50, 1] for i in range(50) if i != (i * 7 + 1) % 50]
+    seen = set()
+    bb = []
+    for m in batch:
+        key = (min(m[1], m[2]), max(m[1], m[2]))
+        if m[0] == 3 and key in seen:
+            continue
+        seen.add(key)
+        bb.append(m)
+    assert P.apply(np.array(bb, np.int32)) == 0
+    P.refine("growth")
+    P.compare_state("growth", full_csr=True)
+    g = gi.make_graph(3000, 64, 31)
+    part = (np.arange(g.n) % 254).astype(np.int32)
+    Q = Pair(g.xadj, g.adjncy, 254, 0.03, part)
+    Q.refine("k254")
+    S = gi.Stream(g, 1)
+    for it in range(3):
+        assert Q.apply(S.next(gi.MODE_MIX, 0.05)) == 0
+        Q.refine(f"k254 it{it}")
+        Q.compare_state(f"k254 it{it}")
