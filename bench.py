@@ -1,0 +1,323 @@
+#!/usr/bin/env python
+"""bench.py -- iG-kway incremental refinement on B200 (BASELINE.json metric).
+
+One step = one incremental iteration = igk_apply_modifiers + igk_refine over one
+seeded synthetic modifier batch (all SURVEY 8(a) rows: S1 apply/mark, S2-S4
+filter/expansion, S5 restoration when a part is overweight, S6-S8 rounds).
+Default workload = BASELINE configs[1] (C2): 1M-vertex circuit-shaped graph,
+k=4, eps=3%, 1% modified vertices per iteration.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
+
+value       = affected vertices/s (whole job), device-resident batches, CUDA events
+ms_per_step = device ms per incremental iteration (apply + refine)
+e2e         = same metric through the public C ABI with HOST batches (H2D of the
+              batch + D2H of the cut inside the timed region)
+--impl reference = the CPU oracle (oracle/) timed on this host (the slow arm).
+Multi-GPU: "replicas" -- each rank refines its own independent graph instance
+(no data-path collective), weak scaling, max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import igk_inputs as gi  # noqa: E402
+
+METRIC = "ms per incremental iteration & affected vertices/s; cut vs full repartition"
+UNIT = "affected vertices/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--k", type=int, default=0)
+    ap.add_argument("--frac", type=float, default=0.0)
+    ap.add_argument("--n", type=int, default=0)
+    ap.add_argument("--cpu-iters", type=int, default=150, help="oracle sample size (iterations)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
+    return ap.parse_args()
+
+
+def workload(args, rank):
+    idx = int(args.config[1:])
+    cfg = dict(gi.CONFIGS[args.config])
+    n = args.n or cfg["n"]
+    k = args.k or (cfg["k"] if isinstance(cfg["k"], int) else cfg["k"][0])
+    frac = args.frac or (cfg.get("frac") if not isinstance(cfg.get("frac"), tuple) else cfg["frac"][2])
+    gseed = gi.graph_seed(idx) + 1000 * rank  # rank 0 = the canonical instance
+    g = gi.make_graph(n, cfg["fmax"], gseed)
+    part, metis_cut = gi.metis_partition(g, k)
+    region0 = (part == 0).astype(np.int32) if cfg["mode"] == gi.MODE_ADVERSARIAL else None
+    S = gi.Stream(g, gi.stream_seed(gseed), region0=region0)
+    cfg = dict(cfg, frac=frac)
+    desc = (f"{args.config}: {n}-vertex circuit-shaped graph (avg deg ~4, fanout <= {cfg['fmax']}), "
+            f"k={k}, eps={cfg['eps']}, " +
+            (f"{frac * 100:g}% modified vertices per iteration" if cfg["mode"] == gi.MODE_MIX else "literal batch mix"))
+    return g, part, metis_cut, S, cfg, k, desc
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self._stop = False
+
+    def start(self):
+        def run():
+            while not self._stop:
+                try:
+                    out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                         timeout=5).stdout.strip()
+                    if out:
+                        self.samples.append([x.strip() for x in out.split(",")])
+                except Exception:
+                    pass
+                time.sleep(0.1)
+        self.t = threading.Thread(target=run, daemon=True)
+        self.t.start()
+
+    def stop(self):
+        self._stop = True
+        self.t.join(timeout=10)
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[3 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"], "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def refine_bytes(st, weighted=False):
+    """Algorithmic bytes of one k_refine launch: every scanned
+    adjacency entry = 4 B neighbour ID + 1 B label gather (+4 B weight), every
+    touched vertex = 16 B of per-vertex state (offset, degree, label, flags,
+    list entry)."""
+    per_entry = 5 + (4 if weighted else 0)
+    touched = st["affected"] + st["expanded"] + st["moves_applied"] + st["moves_deferred"] + st["evicted"]
+    return st["adj_entries_scanned"] * per_entry + touched * 16
+
+
+def cpu_baseline(g, part, k, eps, batches, gpu_cuts, iters):
+    import oracle
+    n_it = min(iters, len(batches))
+    t0 = time.perf_counter()
+    O = oracle.Oracle(g.xadj, g.adjncy, k, eps, part)
+    O.refine()
+    t_setup = time.perf_counter() - t0
+    aff, tt, cut_ok = 0, 0.0, True
+    for i in range(n_it):
+        t = time.perf_counter()
+        O.apply(batches[i])
+        _, st = O.refine()
+        tt += time.perf_counter() - t
+        aff += st["affected"]
+        if i < len(gpu_cuts) and gpu_cuts[i] != st["cut"]:
+            cut_ok = False
+    return {"value": aff / tt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"first {n_it} iterations of the same workload (apply+refine, single-threaded, "
+                      f"{tt:.1f}s; setup {t_setup:.1f}s excluded)",
+            "ms_per_iteration": 1e3 * tt / n_it,
+            "parity_cut_checked_iters": min(n_it, len(gpu_cuts)), "parity_cut_match": cut_ok}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    g, part, metis_cut, S, cfg, k, desc = workload(args, 0)
+    import oracle
+    batches = [gi.next_batch(S, cfg) for _ in range(args.warmup + args.steps)]
+    O = oracle.Oracle(g.xadj, g.adjncy, k, cfg["eps"], part)
+    O.refine()
+    for i in range(args.warmup):
+        O.apply(batches[i])
+        O.refine()
+    aff, tt = 0, 0.0
+    for i in range(args.warmup, args.warmup + args.steps):
+        t = time.perf_counter()
+        O.apply(batches[i])
+        _, st = O.refine()
+        tt += time.perf_counter() - t
+        aff += st["affected"]
+    v = aff / tt
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tt / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic", "config": {"workload": desc, "n": g.n, "k": k},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} timed iterations after {args.warmup} warm-up"},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import torch
+    import paper_conf_dac_leejlczcshh25_b200 as igk
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    g, part, metis_cut, S, cfg, k, desc = workload(args, rank)
+    W, K = args.warmup, args.steps
+    e2e_steps = 0 if args.profile else K
+    batches = [gi.next_batch(S, cfg) for _ in range(W + K + e2e_steps)]
+    stream = torch.cuda.current_stream()
+    G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part, device=local, stream=stream.cuda_stream)
+    G.refine()  # settle the METIS partition (untimed)
+    dev_batches = [torch.from_numpy(b).cuda() for b in batches[: W + K]]
+    flush = None if args.no_flush else torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    gpu_cuts = []
+    for i in range(W):
+        G.apply_device(dev_batches[i].data_ptr(), len(batches[i]))
+        _, st = G.refine()
+        gpu_cuts.append(st["cut"])
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    l0 = G.kernel_launches()
+    clk = ClockSampler(local)
+    clk.start()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    aff, refine_ms, apply_ms, rbytes, stats = 0, 0.0, 0.0, 0, []
+    for i in range(K):
+        b = batches[W + i]
+        if flush is not None:
+            flush.zero_()  # L2 flush (256 MiB > 126 MB L2), outside the timed events
+        ev[i][0].record(stream)
+        s, fid, bad = G.apply_device(dev_batches[W + i].data_ptr(), len(b))
+        _, st = G.refine()
+        ev[i][1].record(stream)
+        ms = G.last_ms()
+        refine_ms += ms["refine"]
+        apply_ms += ms["apply"]
+        aff += st["affected"]
+        rbytes += refine_bytes(st)
+        stats.append(st)
+        gpu_cuts.append(st["cut"])
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    clocks = clk.stop()
+    launches = G.kernel_launches() - l0
+    t_ms = sum(a.elapsed_time(b) for a, b in ev)
+    if dist:
+        tt = torch.tensor([t_ms], device="cuda", dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ta = torch.tensor([float(aff)], device="cuda", dtype=torch.float64)
+        dist.all_reduce(ta, op=dist.ReduceOp.SUM)
+        t_ms, aff_all = tt.item(), ta.item()
+    else:
+        aff_all = aff
+    value = aff_all / (t_ms / 1e3)
+
+    # ---- e2e: public C ABI with HOST batches; H2D + D2H inside the timed region
+    e2e = None
+    if e2e_steps:
+        h_batches = batches[W + K:]
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        aff_e = 0
+        e0.record(stream)
+        for b in h_batches:
+            G.apply(b)          # pinned staging + H2D copy inside
+            _, st = G.refine()
+            G.cut()             # D2H read of the step's result
+            aff_e += st["affected"]
+        e1.record(stream)
+        torch.cuda.synchronize()
+        te = e0.elapsed_time(e1)
+        if dist:
+            tt = torch.tensor([te], device="cuda", dtype=torch.float64)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ta = torch.tensor([float(aff_e)], device="cuda", dtype=torch.float64)
+            dist.all_reduce(ta, op=dist.ReduceOp.SUM)
+            te, aff_e = tt.item(), ta.item()
+        e2e = {"value": aff_e / (te / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(np.mean([b.nbytes for b in h_batches])),
+               "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches)}
+
+    if rank != 0:
+        if dist:
+            dist.destroy_process_group()
+        return
+    peak, peak_kind = peaks()
+    achieved = rbytes / (refine_ms / 1e3) / 1e9 if refine_ms > 0 else 0.0
+    traffic = None
+    try:
+        tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        traffic = tj.get(args.config, {}).get("k_refine")
+    except Exception:
+        pass
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": W,
+        "ms_per_step": t_ms / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "int32", "data": "synthetic",
+        "config": {"workload": desc, "n": g.n, "k": k, "parallelism": "replicas" if world > 1 else "single",
+                   "l2": "flushed between iterations (256 MiB write)" if flush is not None else "not flushed",
+                   "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]]))},
+        "gpu_launches": launches,
+        "roofline": {"kernel": "k_refine", "bound": "hbm", "achieved": achieved, "peak": peak,
+                     "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                     "bytes_per_launch": rbytes / K, "launch_ms": refine_ms / K,
+                     "share_of_step": refine_ms / t_ms if t_ms else None},
+        "kernel_ms": {"k_apply": apply_ms / K, "k_refine": refine_ms / K},
+        "iteration": {"affected": aff / K, "rounds": float(np.mean([s["rounds"] for s in stats])),
+                      "moves": float(np.mean([s["moves_applied"] for s in stats])),
+                      "evicted": float(np.mean([s["evicted"] for s in stats])),
+                      "cut_last": stats[-1]["cut"], "cap": stats[-1]["cap"],
+                      "max_part_weight_last": stats[-1]["max_part_weight"], "metis_initial_cut": metis_cut,
+                      "ms_p50": float(np.median([a.elapsed_time(b) for a, b in ev])),
+                      "ms_p90": float(np.percentile([a.elapsed_time(b) for a, b in ev], 90))},
+        "clocks": clocks,
+    }
+    if e2e:
+        line["e2e"] = e2e
+    if not args.no_cpu_baseline and not args.profile:
+        line["cpu_baseline"] = cpu_baseline(g, part, k, cfg["eps"], batches, gpu_cuts, args.cpu_iters)
+    print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
