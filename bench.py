@@ -207,10 +207,10 @@ def main():
     dev_batches = [torch.from_numpy(b).cuda() for b in batches[: W + K]]
     flush = None if args.no_flush else torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     gpu_cuts = []
+    st_buf = igk.Stats()
     for i in range(W):
-        G.apply_device(dev_batches[i].data_ptr(), len(batches[i]))
-        _, st = G.refine()
-        gpu_cuts.append(st["cut"])
+        G.step_device(dev_batches[i].data_ptr(), len(batches[i]), st_buf)
+        gpu_cuts.append(st_buf.cut)
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
@@ -224,9 +224,9 @@ def main():
         if flush is not None:
             flush.zero_()  # L2 flush (256 MiB > 126 MB L2), outside the timed events
         ev[i][0].record(stream)
-        s, fid, bad = G.apply_device(dev_batches[W + i].data_ptr(), len(b))
-        _, st = G.refine()
+        s, _ = G.step_device(dev_batches[W + i].data_ptr(), len(b), st_buf)  # igk_step_device: apply + refine
         ev[i][1].record(stream)
+        st = {f: int(getattr(st_buf, f)) for f in igk.STATS}
         ms = G.last_ms()
         refine_ms += ms["refine"]
         apply_ms += ms["apply"]
@@ -259,9 +259,8 @@ def main():
         aff_e = 0
         e0.record(stream)
         for b in h_batches:
-            G.apply(b)          # pinned staging + H2D copy inside
-            _, st = G.refine()
-            G.cut()             # D2H read of the step's result
+            _, st, _ = G.step(b)  # igk_step: pinned staging + H2D copy, apply + refine
+            G.cut()               # D2H read of the step's result
             aff_e += st["affected"]
         e1.record(stream)
         torch.cuda.synchronize()

@@ -122,6 +122,16 @@ igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, 
  * IGK_WIMBALANCED in the weighted corner case (result still valid). */
 igk_status igk_refine(igk_graph* g, igk_refine_stats* stats);
 
+/* One incremental iteration: igk_apply_modifiers + igk_refine fused (both
+ * kernels launched back to back, one host synchronisation).  If the batch is
+ * invalid, returns IGK_EINVAL exactly as igk_apply_modifiers would (nothing
+ * changed; the refine was skipped) and *bad_index is set.  mods is a HOST
+ * array; igk_step_device takes a DEVICE array. */
+igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_refine_stats* stats,
+                    int64_t* first_new_id, int64_t* bad_index);
+igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,
+                           int64_t* first_new_id, int64_t* bad_index);
+
 /* out[v] for v < n_total: part in [0,k), -1 = deleted, -2 = pending (in the
  * pseudo-partition between apply and refine).  cap_len too small ->
  * IGK_EINVAL with *n_total still set. */
@@ -145,6 +155,15 @@ int64_t igk_kernel_launches(const igk_graph* g);
 /* device-side duration (ms) of the last igk_refine / apply / recount kernel,
  * measured with CUDA events on the handle's stream */
 igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms);
+/* instrumentation: %globaltimer stamps (ns, relative to the kernel start)
+ * taken by CTA 0 after every grid barrier of the last apply (which = 0) or
+ * refine (which = 1) kernel; ids name the phase (see csrc/*.cuh).  Returns
+ * the number of stamps written (<= cap). */
+int32_t igk_debug_phase_times(const igk_graph* g, int32_t which, int32_t* ids, int64_t* t_ns, int32_t cap);
+/* instrumentation (only if the environment had IGK_DEBUG_ARRIVALS set at
+ * igk_create): per-CTA %globaltimer arrival stamps at barrier slot s of the
+ * last kernel, out[s * grid + cta], 128 slots; returns the grid size. */
+int32_t igk_debug_arrivals(const igk_graph* g, int32_t which, int64_t* out, int32_t cap);
 const char* igk_last_error(const igk_graph* g);
 void igk_destroy(igk_graph* g);
 

@@ -23,8 +23,10 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine",
+           "igk_step", "igk_step_device",
            "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
-           "igk_export_csr", "igk_kernel_launches", "igk_last_kernel_ms", "igk_last_error", "igk_destroy"]
+           "igk_export_csr", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
+           "igk_last_error", "igk_destroy"]
 
 
 class Options(C.Structure):
@@ -65,6 +67,10 @@ def lib():
         L.igk_apply_modifiers_device.argtypes = [P, P, i64, i64p, i64p]
         L.igk_refine.restype = C.c_int
         L.igk_refine.argtypes = [P, C.POINTER(Stats)]
+        L.igk_step.restype = C.c_int
+        L.igk_step.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
+        L.igk_step_device.restype = C.c_int
+        L.igk_step_device.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
         L.igk_partition.restype = C.c_int
         L.igk_partition.argtypes = [P, i32p, i64, i64p]
         L.igk_cut_size.restype = C.c_int
@@ -81,6 +87,10 @@ def lib():
         L.igk_kernel_launches.argtypes = [P]
         L.igk_last_kernel_ms.restype = C.c_int
         L.igk_last_kernel_ms.argtypes = [P, C.POINTER(C.c_float), C.POINTER(C.c_float), C.POINTER(C.c_float)]
+        L.igk_debug_phase_times.restype = C.c_int32
+        L.igk_debug_phase_times.argtypes = [P, C.c_int32, i32p, i64p, C.c_int32]
+        L.igk_debug_arrivals.restype = C.c_int32
+        L.igk_debug_arrivals.argtypes = [P, C.c_int32, i64p, C.c_int32]
         L.igk_last_error.restype = C.c_char_p
         L.igk_last_error.argtypes = [P]
         L.igk_destroy.restype = None
@@ -141,6 +151,25 @@ class IGKGraph:
         if s not in (OK, WIMBALANCED):
             raise IGKError(s, self._err())
         return s, {f: int(getattr(st, f)) for f in STATS}
+
+    def step(self, mods):
+        """apply + refine fused (host batch). Returns (status, stats, bad_index)."""
+        m = np.ascontiguousarray(mods, dtype=np.int32).reshape(-1, 4)
+        st = Stats()
+        fid, bad = C.c_int64(0), C.c_int64(-1)
+        s = lib().igk_step(self.h, m.ctypes.data, len(m), C.byref(st), C.byref(fid), C.byref(bad))
+        if s not in (OK, WIMBALANCED, EINVAL):
+            raise IGKError(s, self._err())
+        return s, {f: int(getattr(st, f)) for f in STATS}, bad.value
+
+    def step_device(self, ptr: int, count: int, stats: "Stats | None" = None):
+        """apply + refine fused, batch already in device memory.  Returns (status, Stats)."""
+        st = stats or Stats()
+        fid, bad = C.c_int64(0), C.c_int64(-1)
+        s = lib().igk_step_device(self.h, C.c_void_p(ptr), count, C.byref(st), C.byref(fid), C.byref(bad))
+        if s not in (OK, WIMBALANCED, EINVAL):
+            raise IGKError(s, self._err())
+        return s, st
 
     def num_vertices(self):
         nt, na = C.c_int64(0), C.c_int64(0)
@@ -203,6 +232,19 @@ class IGKGraph:
 
     def kernel_launches(self):
         return int(lib().igk_kernel_launches(self.h))
+
+    def phase_times(self, which):
+        """[(phase id, ns since kernel start)] of the last apply (0) / refine (1) kernel."""
+        ids = np.zeros(128, np.int32)
+        ts = np.zeros(128, np.int64)
+        n = lib().igk_debug_phase_times(self.h, which, _p(ids, C.c_int32), _p(ts, C.c_int64), 128)
+        return list(zip(ids[:n].tolist(), ts[:n].tolist()))
+
+    def arrivals(self, which):
+        """(128, grid) per-CTA barrier arrival stamps (needs IGK_DEBUG_ARRIVALS at create)."""
+        out = np.zeros(128 * 4096, np.int64)
+        gsz = lib().igk_debug_arrivals(self.h, which, _p(out, C.c_int64), len(out))
+        return out[: 128 * gsz].reshape(128, gsz) if gsz else None
 
     def last_ms(self):
         r, a, c = C.c_float(0), C.c_float(0), C.c_float(0)

@@ -1,14 +1,18 @@
 // apply.cuh -- S1: validate and apply one modifier batch on the device.
 //
-// One persistent cooperative kernel; phases are separated by grid barriers:
-//   V0 clear scratch | V1 dup hash, counts | V2 validate, new IDs, allocate
-//   M0 relocate      | M1 edge deletions   | M2 vertex deletions
-//   M3 finalize deletions, compact, vertex insertions | M4 edge insertions
-// Semantics: reading S1 of P:94-98, Alg. 1-2 and Alg. 3 L1-7.
-// Differences from the paper's design: dense-prefix adjacency
-// with slack instead of 32-slot buckets; one directed update per thread or
-// warp after a validation pass, so concurrent updates of one vertex are
-// race-free (the paper's warp-per-modifier bucket insert races, Q10).
+// One persistent cooperative kernel, four phases, three grid barriers:
+//   V1  count VERTEX_INSERTs per CTA chunk, duplicate-edge hash, per-vertex counts
+//   V2  validate against the pre-batch state; new IDs; slot allocation for
+//       growing prefixes; 32-neighbour work chunks of every vertex deletion
+//   M12 edge deletions and vertex deletions (Alg. 2, both directions,
+//       reading Q12) as tombstones; marks (Alg. 3 L6-7); cut / W deltas
+//   M3  finalize deletions; compact dirty prefixes / copy growing ones to their
+//       new slots; vertex insertions (Alg. 2 L7-10, Alg. 3 L2-5)
+//   M4  edge insertions (Alg. 1) appended to the dense prefixes
+// Semantics: reading S1.  Differences from the paper's design
+// (DESIGN.md 5): dense-prefix adjacency with slack instead of 32-slot buckets;
+// all updates of a batch are validated first and then applied as set
+// operations, so concurrent updates of one vertex are race-free (Q10).
 #pragma once
 #include "common.cuh"
 
@@ -17,7 +21,7 @@ namespace igk {
 struct ApplyArgs {
   const int4* mods;
   long long B;
-  long long n0;         // n_total before the batch
+  long long n0;  // n_total before the batch
   uint32_t epD, epT, epG, epA;
   int vw_unit, ew_unit;
 };
@@ -27,36 +31,43 @@ __device__ __forceinline__ unsigned long long edge_key(int u, int v) {
   return ((unsigned long long)a << 32) | b;
 }
 __device__ __forceinline__ long long hslot(unsigned long long key, long long mask) {
-  unsigned long long h = key * 0x9E3779B97F4A7C15ull;
-  return (long long)(h >> 17) & mask;
+  unsigned long long h = key;  // splitmix64 finalizer: every key bit reaches the low bits
+  h = (h ^ (h >> 30)) * 0xBF58476D1CE4E5B9ull;
+  h = (h ^ (h >> 27)) * 0x94D049BB133111EBull;
+  h ^= h >> 31;
+  return (long long)(h & (unsigned long long)mask);
 }
 
-// linear search of x in the dense prefix of u (thread-sequential)
-__device__ __forceinline__ bool has_edge_seq(const Dev& d, int u, int x) {
-  long long o = __ldcg(d.off + u);
-  int dg = __ldcg(d.deg + u);
-  for (int i = 0; i < dg; i++)
-    if (__ldcg(d.adj + o + i) == x) return true;
-  return false;
-}
-
-// warp-cooperative search of x in u's prefix; returns slot index or -1
-__device__ __forceinline__ long long warp_find(const Dev& d, int u, int x) {
-  long long o = __ldcg(d.off + u);
-  int dg = __ldcg(d.deg + u);
-  for (int b = 0; b < dg; b += 32) {
-    int i = b + lane_id();
-    bool hit = i < dg && __ldcg(d.adj + o + i) == x;
-    unsigned m = __ballot_sync(0xffffffffu, hit);
-    if (m) return o + b + __ffs(m) - 1;
+// thread-level search of x in a prefix; 8 independent loads in flight
+__device__ __forceinline__ long long thread_find(const int32_t* adj, long long o, int dg, int x) {
+  for (int i = 0; i < dg; i += 8) {
+    int v[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) v[t] = (i + t < dg) ? __ldcg(adj + o + i + t) : -1;
+#pragma unroll
+    for (int t = 0; t < 8; t++)
+      if (v[t] == x) return o + i + t;
   }
   return -1;
 }
 
-__device__ __forceinline__ void mark_affected(const Dev& d, int x, uint32_t epA) {
-  bool add = stamp_insert(d.markA, x, epA);
-  int slot = agg_append(&d.ctl->nA, add);
-  if (add) d.Alist[slot] = x;
+// warp-cooperative search; 256 entries (8 loads per lane) per round trip
+__device__ __forceinline__ long long warp_find(const int32_t* adj, long long o, int dg, int x) {
+  const int lane = lane_id();
+  for (int b = 0; b < dg; b += 256) {
+    int v[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      int i = b + t * 32 + lane;
+      v[t] = i < dg ? __ldcg(adj + o + i) : -1;
+    }
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      unsigned m = __ballot_sync(0xffffffffu, v[t] == x);
+      if (m) return o + b + t * 32 + __ffs(m) - 1;
+    }
+  }
+  return -1;
 }
 
 // block-wide exclusive scan of one int per thread; returns exclusive prefix, *total
@@ -86,6 +97,16 @@ __device__ __forceinline__ int block_excl_scan(int v, int* total, int* sbuf) {
   return warp_excl + x - v;
 }
 
+__device__ __forceinline__ void mark_dirty_affected(const Dev& d, int x, uint32_t epT, uint32_t epA) {
+  Ctl* ctl = d.ctl;
+  bool nd = stamp_insert(d.markT, x, epT);
+  int s1 = agg_append(&ctl->ndirty, nd);
+  if (nd) d.dlist[s1] = x;
+  bool na = stamp_insert(d.markA, x, epA);
+  int s2 = agg_append(&ctl->nA, na);
+  if (na) d.Alist[s2] = x;
+}
+
 __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
   cg::grid_group grid = cg::this_grid();
   __shared__ int s_scan[64];
@@ -98,21 +119,10 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
   const long long chunk = (B + gridDim.x - 1) / gridDim.x;
   const long long c_lo = min(B, (long long)blockIdx.x * chunk), c_hi = min(B, c_lo + chunk);
 
-  // ---- V0: clear the duplicate hash; reset the error word -------------------
-  for (long long i = tid; i <= d.hmask; i += nthr) {
-    d.hkeys[i] = ~0ull;
-    d.hcnt[i] = 0;
-  }
-  if (tid == 0) {
-    ctl->err_idx = kNoErr;
-    ctl->err_nomem = 0;
-    ctl->slab_top0 = ctl->slab_top;
-    ctl->ngrow = 0;
-    ctl->ndirty = 0;
-  }
-  grid.sync();
-
-  // ---- V1: count VERTEX_INSERTs per block chunk, hash edge keys, count ------
+  if (tid == 0) ctl->nph = 0;
+  stamp_phase(ctl, 100);
+  arrive_stamp(d.dbg, 0);
+  // ---- V1: counts, duplicate hash, per-vertex counters ---------------------
   {
     int cnt = 0;
     for (long long i = c_lo + threadIdx.x; i < c_hi; i += blockDim.x) cnt += (a.mods[i].x == kVertIns);
@@ -120,7 +130,15 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     block_excl_scan(cnt, &tot, s_scan);
     if (threadIdx.x == 0) d.blkcnt[blockIdx.x] = tot;
   }
-  for (long long i = tid; i < B; i += nthr) {
+  if (tid == 0) {
+    ctl->err_idx = kNoErr;
+    ctl->err_nomem = 0;
+    ctl->slab_top0 = ctl->slab_top;
+    ctl->ngrow = 0;
+    ctl->ndirty = 0;
+    ctl->nvdch = 0;
+  }
+  rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
     const long long lim = n0 + B;
     if ((m.x == kEdgeDel || m.x == kEdgeIns) && m.y >= 0 && m.z >= 0 && m.y < lim && m.z < lim) {
@@ -142,18 +160,29 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       atomicAdd(d.vcnt + m.y, 1);
       d.markD[m.y] = a.epD;
     }
-  }
-  grid.sync();
+  });
+  GRID_SYNC_STAMPED(ctl, 101);
 
-  // ---- V2: validate against the pre-batch state; new IDs; allocate slots ----
-  long long n_ins = 0, my_base = 0;
-  for (int b = 0; b < (int)gridDim.x; b++) {
-    int c = __ldcg(d.blkcnt + b);
-    n_ins += c;
-    if (b < (int)blockIdx.x) my_base += c;
+  // ---- V2: validate against the pre-batch state; new IDs; allocate ---------
+  __shared__ long long s_ins[2];
+  if (warp_id() == 0) {  // one warp sums the per-CTA counts
+    long long t = 0, m = 0;
+    for (int b = lane_id(); b < (int)gridDim.x; b += 32) {
+      int c = __ldcg(d.blkcnt + b);
+      t += c;
+      if (b < (int)blockIdx.x) m += c;
+    }
+    t = warp_sum(t);
+    m = warp_sum(m);
+    if (lane_id() == 0) {
+      s_ins[0] = t;
+      s_ins[1] = m;
+    }
   }
+  __syncthreads();
+  const long long n_ins = s_ins[0], my_base = s_ins[1];
   if (tid == 0 && n0 + n_ins > d.n_cap) ctl->err_nomem = 1;
-  {  // IDs of VERTEX_INSERTs: the j-th insertion in batch order gets n0 + j
+  {  // the j-th VERTEX_INSERT in batch order gets ID n0 + j
     long long base = n0 + my_base;
     for (long long t0 = c_lo; t0 < c_hi; t0 += blockDim.x) {
       long long i = t0 + threadIdx.x;
@@ -165,7 +194,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     }
   }
   const long long nlim = n0 + n_ins;
-  for (long long i = tid; i < B; i += nthr) {
+  rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
     bool ok;
     auto old_live = [&](int x) {
@@ -175,16 +204,24 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     auto dup_free = [&](int u, int v) {
       unsigned long long key = edge_key(u, v);
       long long s = hslot(key, d.hmask);
-      while (d.hkeys[s] != key) s = (s + 1) & d.hmask;
+      while (__ldcg(d.hkeys + s) != key) s = (s + 1) & d.hmask;
       return __ldcg(d.hcnt + s) == 1;
     };
-    auto exists = [&](int u, int v) {  // scan the shorter list
-      return __ldcg(d.deg + u) <= __ldcg(d.deg + v) ? has_edge_seq(d, u, v) : has_edge_seq(d, v, u);
+    auto exists = [&](int u, int v) {  // search the shorter prefix
+      int du = __ldcg(d.deg + u), dv = __ldcg(d.deg + v);
+      return du <= dv ? thread_find(d.adj, __ldcg(d.off + u), du, v) >= 0
+                      : thread_find(d.adj, __ldcg(d.off + v), dv, u) >= 0;
     };
     if (m.x == kEdgeDel) {
       ok = m.y != m.z && old_live(m.y) && old_live(m.z) && dup_free(m.y, m.z) && exists(m.y, m.z);
     } else if (m.x == kVertDel) {
       ok = m.y >= 0 && m.y < n0 && __ldcg(d.active + m.y) && __ldcg(d.vcnt + m.y) == 1;
+      if (ok) {  // 32-neighbour work chunks of this deletion
+        int dg = __ldcg(d.deg + m.y);
+        int nch = max(1, (dg + 31) / 32);
+        int s = atomicAdd(&ctl->nvdch, nch);
+        for (int c = 0; c < nch; c++) d.vdch[s + c] = make_int2(m.y, c);
+      }
     } else if (m.x == kVertIns) {
       ok = a.vw_unit ? (m.w == 1) : (m.w >= 1 && m.w <= kVwMax);
     } else if (m.x == kEdgeIns) {
@@ -202,8 +239,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       ok = false;
     }
     if (!ok) atomicMin((long long*)&ctl->err_idx, i);
-    // slot allocation for every endpoint an insertion touches (first touch)
-    if (m.x == kEdgeIns) {
+    if (m.x == kEdgeIns) {  // slots for every endpoint an insertion touches (first touch)
       int ends[2] = {m.y, m.z};
       for (int e = 0; e < 2; e++) {
         int x = ends[e];
@@ -225,53 +261,33 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
         d.reloc[x] = pk;
       }
     }
-  }
-  grid.sync();
+  });
+  GRID_SYNC_STAMPED(ctl, 102);
 
+  // ---- scratch reset (hash, counters) on both the failure and success paths ---
   const bool failed = ldv(&ctl->err_idx) != kNoErr || ldv(&ctl->err_nomem) != 0;
-  // ---- M0: relocate overflowing prefixes (or roll back on failure) ----------
-  {
-    const int ng = ldv(&ctl->ngrow);
-    for (long long t = gwarp; t < ng; t += nwarp) {
-      int x = d.glist[t];
-      long long pk = d.reloc[x];
-      if (lane_id() == 0) d.icnt[x] = 0;
-      if (failed || pk < 0) continue;
-      long long no = pk >> 24;
-      int nc = (int)(pk & 0xffffff);
-      if (x < n0) {
-        long long o = __ldcg(d.off + x);
-        int dg = __ldcg(d.deg + x);
-        for (int i = lane_id(); i < dg; i += 32) {
-          d.adj[no + i] = __ldcg(d.adj + o + i);
-          if (d.adjw) d.adjw[no + i] = __ldcg(d.adjw + o + i);
-        }
-      } else if (lane_id() == 0) {
-        d.deg[x] = 0;
-      }
-      if (lane_id() == 0) {
-        d.off[x] = no;
-        d.capv[x] = nc;
-      }
-    }
-    for (long long i = tid; i < B; i += nthr) {
-      int4 m = a.mods[i];
-      if (m.x == kVertDel && m.y >= 0 && m.y < n0) d.vcnt[m.y] = 0;
-    }
-    if (failed) {  // uniform: every block saw the same error words
-      if (tid == 0) ctl->slab_top = ctl->slab_top0;  // give back the allocations
-      return;
-    }
+  for (long long i = tid; i <= d.hmask; i += nthr) {
+    d.hkeys[i] = ~0ull;
+    d.hcnt[i] = 0;
   }
-  grid.sync();
+  const int ng = ldv(&ctl->ngrow);
+  for (long long t = tid; t < ng; t += nthr) d.icnt[d.glist[t]] = 0;
+  for (long long i = tid; i < B; i += nthr) {
+    int4 m = a.mods[i];
+    if (m.x == kVertDel && m.y >= 0 && m.y < n0) d.vcnt[m.y] = 0;
+  }
+  if (failed) {  // uniform: every CTA read the same error words
+    if (tid == 0) ctl->slab_top = ctl->slab_top0;
+    return;
+  }
 
-  long long cut_acc = 0;
-  // ---- M1: edge deletions ------------------------------------------
-  for (long long i = gwarp; i < B; i += nwarp) {
+  // ---- M12: edge deletions and vertex deletions (tombstones) ---------------
+  long long cut_acc = 0, W_acc = 0;
+  for (long long i = gwarp; i < B; i += nwarp) {  // one warp per edge deletion
     int4 m = a.mods[i];
     if (m.x != kEdgeDel) continue;
-    long long su = warp_find(d, m.y, m.z);
-    long long sv = warp_find(d, m.z, m.y);
+    long long su = warp_find(d.adj, __ldcg(d.off + m.y), __ldcg(d.deg + m.y), m.z);
+    long long sv = warp_find(d.adj, __ldcg(d.off + m.z), __ldcg(d.deg + m.z), m.y);
     if (lane_id() == 0) {
       int w = d.adjw ? __ldcg(d.adjw + su) : 1;
       d.adj[su] = -1;
@@ -279,61 +295,50 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
       if (pu != kPsi && pv != kPsi && pu != pv) cut_acc -= w;
     }
-    int ends[2] = {m.y, m.z};
-    for (int e = 0; e < 2; e++) {
-      if (lane_id() == 0) {
-        int x = ends[e];
-        if (stamp_insert(d.markT, x, a.epT)) d.dlist[atomicAdd(&ctl->ndirty, 1)] = x;
-        if (stamp_insert(d.markA, x, a.epA)) d.Alist[atomicAdd(&ctl->nA, 1)] = x;
-      }
-    }
+    if (lane_id() < 2) mark_dirty_affected(d, lane_id() ? m.z : m.y, a.epT, a.epA);
   }
-  grid.sync();
-
-  // ---- M2: vertex deletions (Alg. 2 L4-6, L11-13; both directions, Q12) ----
-  long long W_acc = 0;
-  for (long long i = gwarp; i < B; i += nwarp) {
-    int4 m = a.mods[i];
-    if (m.x != kVertDel) continue;
-    const int u = m.y;
-    const long long o = __ldcg(d.off + u);
-    const int dg = __ldcg(d.deg + u);
-    const uint8_t pu = ld_part(d.part, u);
-    for (int b = 0; b < dg; b += 32) {
-      int j = b + lane_id();
-      int x = j < dg ? __ldcg(d.adj + o + j) : -1;
+  {
+    const int nch = ldv(&ctl->nvdch);
+    for (long long t = gwarp; t < nch; t += nwarp) {  // one warp per 32 neighbours
+      const int2 ch = d.vdch[t];
+      const int u = ch.x;
+      const long long o = __ldcg(d.off + u);
+      const int dg = __ldcg(d.deg + u);
+      const uint8_t pu = ld_part(d.part, u);
+      const int j = ch.y * 32 + lane_id();
+      int x = j < dg ? __ldcg(d.adj + o + j) : -1;  // -1: tombstone from an edge deletion
       int w = (x >= 0 && d.adjw) ? __ldcg(d.adjw + o + j) : 1;
-      unsigned vm = __ballot_sync(0xffffffffu, x >= 0);
-      while (vm) {
-        int src = __ffs(vm) - 1;
-        vm &= vm - 1;
+      bool xdel = x >= 0 && __ldcg(d.markD + x) == a.epD;
+      int dx = (x >= 0 && !xdel) ? __ldcg(d.deg + x) : 0;
+      bool small = x >= 0 && !xdel && dx <= 32;
+      if (small) {
+        long long s = thread_find(d.adj, __ldcg(d.off + x), dx, u);
+        d.adj[s] = -1;
+      }
+      unsigned hm = __ballot_sync(0xffffffffu, x >= 0 && !xdel && !small);
+      while (hm) {
+        int src = __ffs(hm) - 1;
+        hm &= hm - 1;
         int xx = __shfl_sync(0xffffffffu, x, src);
-        int ww = __shfl_sync(0xffffffffu, w, src);
-        bool xdel = __ldcg(d.markD + xx) == a.epD;
-        if (!xdel) {
-          long long s = warp_find(d, xx, u);
-          if (lane_id() == 0) {
-            d.adj[s] = -1;
-            if (stamp_insert(d.markT, xx, a.epT)) d.dlist[atomicAdd(&ctl->ndirty, 1)] = xx;
-            if (stamp_insert(d.markA, xx, a.epA)) d.Alist[atomicAdd(&ctl->nA, 1)] = xx;
-          }
-        }
-        if (lane_id() == 0) {
-          uint8_t px = ld_part(d.part, xx);
-          if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < xx)) cut_acc -= ww;
-        }
+        long long s = warp_find(d.adj, __ldcg(d.off + xx), __ldcg(d.deg + xx), u);
+        if (lane_id() == 0) d.adj[s] = -1;
+      }
+      if (x >= 0) {
+        uint8_t px = ld_part(d.part, x);
+        if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < x)) cut_acc -= w;
+      }
+      if (x >= 0 && !xdel) mark_dirty_affected(d, x, a.epT, a.epA);
+      if (ch.y == 0 && lane_id() == 0) {
+        int vwu = d.vw ? __ldcg(d.vw + u) : 1;
+        if (pu != kPsi) atomic_add_ll(&ctl->Wp[pu], -(long long)vwu);
+        W_acc -= vwu;
       }
     }
-    if (lane_id() == 0) {
-      int w = d.vw ? __ldcg(d.vw + u) : 1;
-      if (pu != kPsi) atomic_add_ll(&ctl->Wp[pu], -(long long)w);
-      W_acc -= w;
-    }
   }
-  grid.sync();
+  GRID_SYNC_STAMPED(ctl, 103);
 
-  // ---- M3: finalize deletions; compact dirty prefixes; vertex insertions ----
-  for (long long i = tid; i < B; i += nthr) {
+  // ---- M3: finalize deletions; compact / relocate prefixes; insertions ------
+  rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
     if (m.x == kVertDel) {
       d.deg[m.y] = 0;
@@ -350,32 +355,59 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
         d.off[id] = 0;
       }
       W_acc += m.w;
-      int slot = atomicAdd(&ctl->npsi[0], 1);
+      int slot = agg_append(&ctl->npsi[0], true);
       d.psi[0][slot] = id;
+    }
+  });
+  // compact a prefix (dropping tombstones) from `src` into `dst` (may alias)
+  auto compact = [&](int x, long long src, long long dst) {
+    const int dg = __ldcg(d.deg + x);
+    int wr = 0;
+    for (int b = 0; b < dg; b += 128) {  // 4 loads per lane in flight
+      int y[4], w[4];
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        int j = b + t * 32 + lane_id();
+        y[t] = j < dg ? __ldcg(d.adj + src + j) : -1;
+        w[t] = (j < dg && d.adjw) ? __ldcg(d.adjw + src + j) : 0;
+      }
+      __syncwarp();
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        unsigned keep = __ballot_sync(0xffffffffu, y[t] >= 0);
+        if (y[t] >= 0) {
+          int pos = wr + __popc(keep & ((1u << lane_id()) - 1u));
+          d.adj[dst + pos] = y[t];
+          if (d.adjw) d.adjw[dst + pos] = w[t];
+        }
+        wr += __popc(keep);
+      }
+      __syncwarp();
+    }
+    return wr;
+  };
+  for (long long t = gwarp; t < ng; t += nwarp) {  // growing prefixes move to their new slots
+    int x = d.glist[t];
+    long long pk = d.reloc[x];
+    if (pk < 0) continue;
+    long long no = pk >> 24;
+    int nc = (int)(pk & 0xffffff);
+    int wr = 0;
+    if (x < n0) wr = compact(x, __ldcg(d.off + x), no);
+    if (lane_id() == 0) {
+      d.off[x] = no;
+      d.capv[x] = nc;
+      d.deg[x] = wr;
     }
   }
   {
     const int nd = ldv(&ctl->ndirty);
-    for (long long t = gwarp; t < nd; t += nwarp) {
+    for (long long t = gwarp; t < nd; t += nwarp) {  // in-place compaction of the rest
       int x = d.dlist[t];
       if (__ldcg(d.markD + x) == a.epD) continue;
-      const long long o = __ldcg(d.off + x);
-      const int dg = __ldcg(d.deg + x);
-      int wr = 0;
-      for (int b = 0; b < dg; b += 32) {
-        int j = b + lane_id();
-        int y = j < dg ? __ldcg(d.adj + o + j) : -1;
-        int w = (j < dg && d.adjw) ? __ldcg(d.adjw + o + j) : 0;
-        unsigned keep = __ballot_sync(0xffffffffu, y >= 0);
-        __syncwarp();
-        if (y >= 0) {
-          int pos = wr + __popc(keep & ((1u << lane_id()) - 1u));
-          d.adj[o + pos] = y;
-          if (d.adjw) d.adjw[o + pos] = w;
-        }
-        wr += __popc(keep);
-        __syncwarp();
-      }
+      if (__ldcg(d.markG + x) == a.epG && __ldcg(d.reloc + x) >= 0) continue;
+      long long o = __ldcg(d.off + x);
+      int wr = compact(x, o, o);
       if (lane_id() == 0) d.deg[x] = wr;
     }
   }
@@ -383,12 +415,12 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     ctl->n_total = n0 + n_ins;
     ctl->n_ins = (int)n_ins;
   }
-  grid.sync();
+  GRID_SYNC_STAMPED(ctl, 104);
 
-  // ---- M4: edge insertions (Alg. 1): append to the dense prefix -------------
-  for (long long i = tid; i < B; i += nthr) {
+  // ---- M4: edge insertions (Alg. 1): append to the dense prefixes ----------
+  rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
-    if (m.x != kEdgeIns) continue;
+    if (m.x != kEdgeIns) return;
     int pu_pos = atomicAdd(d.deg + m.y, 1);
     int pv_pos = atomicAdd(d.deg + m.z, 1);
     long long su = __ldcg(d.off + m.y) + pu_pos, sv = __ldcg(d.off + m.z) + pv_pos;
@@ -400,11 +432,16 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     }
     uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
     if (pu != kPsi && pv != kPsi && pu != pv) cut_acc += m.w;
-    mark_affected(d, m.y, a.epA);
-    mark_affected(d, m.z, a.epA);
-  }
+    bool na = stamp_insert(d.markA, m.y, a.epA);
+    int s1 = agg_append(&ctl->nA, na);
+    if (na) d.Alist[s1] = m.y;
+    bool nb = stamp_insert(d.markA, m.z, a.epA);
+    int s2 = agg_append(&ctl->nA, nb);
+    if (nb) d.Alist[s2] = m.z;
+  });
   block_atomic_add(&ctl->cut, cut_acc, s_red);
   block_atomic_add(&ctl->W, W_acc, s_red);
+  stamp_phase(ctl, 199);
 }
 
 }  // namespace igk

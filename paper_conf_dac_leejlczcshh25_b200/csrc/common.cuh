@@ -21,7 +21,7 @@ constexpr int kDegMax = 1 << 23;
 constexpr int64_t kNMax = int64_t(1) << 30;
 constexpr int kThreads = 512;       // persistent-kernel block size
 constexpr int kWarps = kThreads / 32;
-constexpr int kThreadDeg = 32;      // degree <= this: one thread per vertex; above: one warp
+constexpr int kThreadDeg = 16;      // degree <= this: one thread per vertex; above: one warp
 constexpr int kDigits = 256;        // radix digit bins (8-bit digits)
 constexpr long long kNoErr = 0x7fffffffffffffffLL;
 
@@ -37,27 +37,35 @@ enum StatIdx {
 };
 
 struct Ctl {
+  // ---- outputs read back after every call (kept first: lean D2H copy) ----
   long long n_total;   // vertex IDs in use
   long long slab_top;  // bump pointer of the adjacency slab
   long long W;         // total active vertex weight
   long long cut;       // maintained cut (placed endpoints only)
-  long long Wp[256];   // part weights
-  long long tot3[3][256];  // per round (mod 3): weight of selected moves per target part
-  long long st_out[ST_N];  // stats of the last refine (copied at its end)
-  long long slab_top0;     // slab_top before the current apply (rollback)
   long long err_idx;   // lowest invalid modifier index (kNoErr = none)
-  long long st[ST_N];  // refine stats
+  long long st_out[ST_N];  // stats of the last refine (copied at its end)
   int err_nomem;
   int n_ins;
+  int refine_skipped;  // fused step: refine skipped because the batch was rejected
+  int nph;             // phase timestamps recorded by the last kernel
+  // ---- device-side state ----
+  long long Wp[256];   // part weights
+  long long tot3[3][256];  // per round (mod 3): weight of selected moves per target part
+  long long slab_top0;     // slab_top before the current apply (rollback)
+  long long st[ST_N];  // refine stats (accumulating)
   int nA;              // affected list length
-  int npsi[2];         // pseudo list lengths (double buffer)
-  int ncand;           // candidate list length
+  int npsi[3];         // pseudo list lengths
+  int ncand;           // candidate list length (C1, R3)
+  int ncand2;          // candidate list length (C2)
   int nN;              // expansion list length
   int ngrow;           // relocation list length
   int ndirty;          // compaction list length
   int nr3;             // restoration candidate list length
+  int nvdch;           // vertex-deletion work chunks
   int applied3[3];     // moves applied per round (mod 3)
   int selected3[3];    // moves selected per round (mod 3)
+  unsigned long long tph[128];  // %globaltimer after each phase (CTA 0)
+  int idph[128];                // phase ids
 };
 
 // ---------------------------------------------------------------------------
@@ -87,17 +95,20 @@ struct Dev {
   int32_t* icnt;     // EDGE_INSERT count per endpoint (zero between calls)
   // lists (n_cap entries each)
   int32_t* Alist;
-  int32_t* psi[2];
+  int32_t* psi[3];    // [0] accumulates Psi (= frontier F); [1],[2] round buffers
   int32_t* cand;
+  int32_t* cand2;
   int32_t* Nlist;
   int32_t* glist;    // grow / relocation list
   int32_t* dlist;    // dirty list
   int2* r3list;      // (vertex, loss) restoration candidates
+  int2* vdch;        // (vertex, chunk) work items of vertex deletions
+  uint32_t* markF;   // frontier membership (entered Psi in this refine cycle)
+  uint8_t* oldp;     // part before entering Psi (kPsi for inserted vertices)
   int64_t* reloc;    // new slab offset for relocated vertices
   // per-vertex move results (rounds)
   uint8_t* tgt;
   int32_t* gain;
-  int32_t* pw;
   uint32_t* meta;    // per psi index: bit31 selected | d0 << 8 | p*
   // selection histograms
   long long* hist0;  // [256][256] digit-0 weights per part
@@ -108,6 +119,7 @@ struct Dev {
   int64_t hmask;
   int32_t* blkcnt;            // per-block counts for chunked scans
   int32_t* newid;             // per modifier: new vertex ID of a VERTEX_INSERT
+  unsigned long long* dbg;    // optional per-CTA barrier arrival stamps [128][grid]
   Ctl* ctl;
 };
 
@@ -120,6 +132,67 @@ __device__ __forceinline__ uint8_t ld_part(const uint8_t* p, int64_t i) { return
 
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+// phase stamp: CTA 0 / thread 0 records (id, time) right after a grid barrier
+__device__ __forceinline__ void stamp_phase(Ctl* ctl, int id) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    int i = ctl->nph;
+    if (i < 128) {
+      ctl->tph[i] = gtimer();
+      ctl->idph[i] = id;
+      ctl->nph = i + 1;
+    }
+  }
+}
+
+// opt-in instrumentation: every CTA stamps its arrival at barrier `slot`
+__device__ __forceinline__ void arrive_stamp(unsigned long long* dbg, int slot) {
+  if (dbg && slot < 128) {
+    __syncthreads();
+    if (threadIdx.x == 0) dbg[(long long)slot * gridDim.x + blockIdx.x] = gtimer();
+  }
+}
+
+// grid barrier with instrumentation (CTA arrival stamp + CTA-0 phase stamp)
+#define GRID_SYNC_STAMPED(ctl_, id_)      \
+  do {                                    \
+    arrive_stamp(d.dbg, (id_) % 100);     \
+    grid.sync();                          \
+    stamp_phase(ctl_, id_);               \
+  } while (0)
+
+// Flat loop over [0, n) in 32-item chunks (one chunk per warp, lanes
+// contiguous so warp-aggregated appends stay one atomic per warp), with the
+// chunks dealt CTA-first: chunk c -> CTA c mod G, warp (c / G) mod W.  A
+// short list thus spreads over all SMs instead of filling the first CTAs.
+template <class F>
+__device__ __forceinline__ void rr_for(long long n, F f) {
+  const long long G = gridDim.x, W = blockDim.x >> 5;
+  const long long my = (long long)(threadIdx.x >> 5) * G + blockIdx.x;  // this warp's rank
+  const long long nw = G * W;
+  const long long nch = (n + 31) >> 5;
+  for (long long c = my; c < nch; c += nw) {
+    long long i = (c << 5) + (threadIdx.x & 31);
+    if (i < n) f(i);
+  }
+}
+
+// per-part accumulation in shared memory with lanes of equal key combined
+// first (one shared atomic per distinct key per warp)
+__device__ __forceinline__ void acc_add(long long* acc, int key, long long v) {
+  unsigned act = __activemask();
+  unsigned grp = __match_any_sync(act, key);
+  int leader = __ffs(grp) - 1;
+  // sum v over the group (lanes of grp) via shuffles from the leader's view
+  long long sum = 0;
+  for (unsigned m = grp; m; m &= m - 1) sum += __shfl_sync(grp, v, __ffs(m) - 1);
+  if ((int)(threadIdx.x & 31) == leader) atomicAdd((unsigned long long*)&acc[key], (unsigned long long)sum);
+}
 
 // warp-aggregated append: returns the slot of this lane (or -1 if !pred)
 __device__ __forceinline__ int agg_append(int* ctr, bool pred) {

@@ -7,6 +7,8 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstddef>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -119,6 +121,7 @@ struct igk_graph {
   long long d_mods_cap = 0;
   long long newid_cap = 0;
   int check = 0;
+  int debug_phases = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
   long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp
@@ -126,6 +129,7 @@ struct igk_graph {
   cudaEvent_t ev[6] = {};
   float ms_refine = 0, ms_apply = 0, ms_recount = 0;
   std::vector<void*> allocs;
+  std::vector<std::pair<int, unsigned long long>> ph[2];  // phase stamps: [0] apply, [1] refine
 };
 
 namespace {
@@ -183,9 +187,16 @@ igk_status launch_recount(igk_graph* g) {
   return IGK_OK;
 }
 
-igk_status sync_ctl(igk_graph* g) {
-  CK(cudaMemcpyAsync(g->h_ctl, g->d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g->stream));
+igk_status sync_ctl(igk_graph* g, int which) {
+  // lean readback: only the output block at the head of Ctl (full copy when debugging)
+  const size_t bytes = (g->debug_phases || g->check) ? sizeof(Ctl) : offsetof(Ctl, Wp);
+  CK(cudaMemcpyAsync(g->h_ctl, g->d.ctl, bytes, cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
+  if (which >= 0 && g->debug_phases) {
+    auto& v = g->ph[which];
+    v.clear();
+    for (int i = 0; i < std::min(g->h_ctl->nph, 128); i++) v.push_back({g->h_ctl->idph[i], g->h_ctl->tph[i]});
+  }
   return IGK_OK;
 }
 
@@ -278,9 +289,10 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.markA, N) && dalloc(g, &d.markT, N) && dalloc(g, &d.markD, N) &&
             dalloc(g, &d.markG, N) && dalloc(g, &d.vcnt, N) && dalloc(g, &d.icnt, N) &&
             dalloc(g, &d.Alist, N) && dalloc(g, &d.psi[0], N) && dalloc(g, &d.psi[1], N) &&
-            dalloc(g, &d.cand, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
+            dalloc(g, &d.psi[2], N) && dalloc(g, &d.cand, N) && dalloc(g, &d.cand2, N) &&
+            dalloc(g, &d.vdch, N + (size_t)(d.slot_cap / 32) + 1024) && dalloc(g, &d.markF, N) && dalloc(g, &d.oldp, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
             dalloc(g, &d.dlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
-            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) &&
+            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.meta, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
             dalloc(g, &g->d_red, 257);
@@ -304,6 +316,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   cudaMemsetAsync(d.markT, 0, N * 4, s);
   cudaMemsetAsync(d.markD, 0, N * 4, s);
   cudaMemsetAsync(d.markG, 0, N * 4, s);
+  cudaMemsetAsync(d.markF, 0, N * 4, s);
   cudaMemsetAsync(d.vcnt, 0, N * 4, s);
   cudaMemsetAsync(d.icnt, 0, N * 4, s);
   cudaMemsetAsync(d.hist0, 0, 256 * kDigits * 8, s);
@@ -369,6 +382,15 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     igk_destroy(g);
     return IGK_ECUDA;
   }
+  g->debug_phases = getenv("IGK_DEBUG_PHASES") != nullptr || getenv("IGK_DEBUG_ARRIVALS") != nullptr;
+  // opt-in per-CTA barrier arrival stamps (tools/phase_profile.py)
+  if (getenv("IGK_DEBUG_ARRIVALS")) {
+    if (!dalloc(g, &d.dbg, 128 * 4096)) {
+      igk_destroy(g);
+      return IGK_ENOMEM;
+    }
+    cudaMemset(d.dbg, 0, 128 * 4096 * 8);
+  }
   // persistent grids
   g->smem_refine = sizeof(RefSmem);
   cudaFuncSetAttribute(k_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
@@ -380,10 +402,8 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   return IGK_OK;
 }
 
-static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t* first_new_id, int64_t* bad_index) {
-  if (bad_index) *bad_index = -1;
-  if (first_new_id) *first_new_id = g->h_ctl->n_total;
-  if (count == 0) return IGK_OK;
+// capacity checks + launch of k_apply (no host synchronisation)
+static igk_status launch_apply(igk_graph* g, const int4* dm, int64_t count) {
   // duplicate-detection hash: >= 2 * count slots, power of two
   long long need = 64;
   while (need < 2 * count + 2) need <<= 1;
@@ -395,6 +415,8 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
     if (cudaMalloc(&g->d.hkeys, need * 8) != cudaSuccess || cudaMalloc(&g->d.hcnt, need * 4) != cudaSuccess)
       return fail(g, IGK_ENOMEM, "hash allocation failed");
     g->hash_cap = need;
+    CK(cudaMemsetAsync(g->d.hkeys, 0xff, need * 8, g->stream));  // empty; kept empty by k_apply
+    CK(cudaMemsetAsync(g->d.hcnt, 0, need * 4, g->stream));
   }
   if (count > g->newid_cap) {
     if (g->d.newid) cudaFree(g->d.newid);
@@ -419,8 +441,11 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
   CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply, kThreads, args, 0, g->stream));
   g->launches++;
   CK(cudaEventRecord(g->ev[3], g->stream));
-  igk_status st = sync_ctl(g);
-  if (st != IGK_OK) return st;
+  return IGK_OK;
+}
+
+// after the control block was read back: apply status
+static igk_status finish_apply(igk_graph* g, int64_t* bad_index) {
   cudaEventElapsedTime(&g->ms_apply, g->ev[2], g->ev[3]);
   if (g->h_ctl->err_idx != kNoErr) {
     if (bad_index) *bad_index = g->h_ctl->err_idx;
@@ -432,6 +457,56 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
   return IGK_OK;
 }
 
+static igk_status launch_refine(igk_graph* g, int after_apply) {
+  RefineArgs a;
+  a.e_ppm = g->e_ppm;
+  a.epC1 = next_epoch(g);
+  a.epN = next_epoch(g);
+  a.epC2 = next_epoch(g);
+  a.epF = next_epoch(g);
+  a.after_apply = after_apply;
+  void* args[] = {(void*)&g->d, (void*)&a};
+  CK(cudaEventRecord(g->ev[0], g->stream));
+  CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
+  g->launches++;
+  CK(cudaEventRecord(g->ev[1], g->stream));
+  return IGK_OK;
+}
+
+static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats);
+
+static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t* first_new_id, int64_t* bad_index) {
+  if (bad_index) *bad_index = -1;
+  if (first_new_id) *first_new_id = g->h_ctl->n_total;
+  if (count == 0) return IGK_OK;
+  igk_status st = launch_apply(g, dm, count);
+  if (st != IGK_OK) return st;
+  st = sync_ctl(g, 0);
+  if (st != IGK_OK) return st;
+  return finish_apply(g, bad_index);
+}
+
+// fused step: apply + refine launched back to back, one host synchronisation
+static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refine_stats* stats,
+                           int64_t* first_new_id, int64_t* bad_index) {
+  if (bad_index) *bad_index = -1;
+  if (first_new_id) *first_new_id = g->h_ctl->n_total;
+  igk_status st;
+  if (count > 0) {
+    st = launch_apply(g, dm, count);
+    if (st != IGK_OK) return st;
+  }
+  st = launch_refine(g, count > 0);
+  if (st != IGK_OK) return st;
+  st = sync_ctl(g, 1);
+  if (st != IGK_OK) return st;
+  if (count > 0) {
+    st = finish_apply(g, bad_index);
+    if (st != IGK_OK) return st;  // the refine kernel exited without touching the state
+  }
+  return finish_refine(g, stats);
+}
+
 igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count, int64_t* first_new_id,
                                int64_t* bad_index) {
   if (!g || g->poisoned) return IGK_ESTATE;
@@ -440,6 +515,7 @@ igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t c
   if (count > g->h_stage_cap) {
     if (g->h_stage) cudaFreeHost(g->h_stage);
     g->h_stage = nullptr;
+    g->h_stage_cap = 0;
     if (cudaMallocHost(&g->h_stage, count * sizeof(igk_modifier)) != cudaSuccess)
       return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
     g->h_stage_cap = count;
@@ -463,21 +539,7 @@ igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, 
   return apply_dev(g, (const int4*)d_mods, count, first_new_id, bad_index);
 }
 
-igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
-  if (!g || g->poisoned) return IGK_ESTATE;
-  RefineArgs a;
-  a.e_ppm = g->e_ppm;
-  a.epC1 = next_epoch(g);
-  a.epN = next_epoch(g);
-  a.epC2 = next_epoch(g);
-  a.epE = next_epoch(g);
-  void* args[] = {(void*)&g->d, (void*)&a};
-  CK(cudaEventRecord(g->ev[0], g->stream));
-  CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
-  g->launches++;
-  CK(cudaEventRecord(g->ev[1], g->stream));
-  igk_status st = sync_ctl(g);
-  if (st != IGK_OK) return st;
+static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
   cudaEventElapsedTime(&g->ms_refine, g->ev[0], g->ev[1]);
   g->epochA = next_epoch(g);
   const long long* so = g->h_ctl->st_out;
@@ -501,7 +563,7 @@ igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
   if (g->check) {  // invariant I1/I2: maintained cut and W_p equal a recount
     int64_t cut = 0;
     int64_t wp[256];
-    st = igk_recount(g, &cut, wp);
+    igk_status st = igk_recount(g, &cut, wp);
     if (st != IGK_OK) return st;
     bool bad = cut != g->h_ctl->cut;
     for (int p = 0; p < g->d.k; p++) bad |= wp[p] != g->h_ctl->Wp[p];
@@ -511,6 +573,48 @@ igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
     }
   }
   return imbal ? IGK_WIMBALANCED : IGK_OK;
+}
+
+igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  igk_status st = launch_refine(g, 0);
+  if (st != IGK_OK) return st;
+  st = sync_ctl(g, 1);
+  if (st != IGK_OK) return st;
+  return finish_refine(g, stats);
+}
+
+igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_refine_stats* stats,
+                    int64_t* first_new_id, int64_t* bad_index) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
+  if (count > g->h_stage_cap) {
+    if (g->h_stage) cudaFreeHost(g->h_stage);
+    g->h_stage = nullptr;
+    g->h_stage_cap = 0;
+    if (cudaMallocHost(&g->h_stage, count * sizeof(igk_modifier)) != cudaSuccess)
+      return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
+    g->h_stage_cap = count;
+  }
+  if (count > g->d_mods_cap) {
+    if (g->d_mods) cudaFree(g->d_mods);
+    g->d_mods = nullptr;
+    g->d_mods_cap = 0;
+    if (cudaMalloc(&g->d_mods, count * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
+    g->d_mods_cap = count;
+  }
+  if (count > 0) {
+    std::memcpy(g->h_stage, mods, count * sizeof(igk_modifier));
+    CK(cudaMemcpyAsync(g->d_mods, g->h_stage, count * 16, cudaMemcpyHostToDevice, g->stream));
+  }
+  return step_dev(g, g->d_mods, count, stats, first_new_id, bad_index);
+}
+
+igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,
+                           int64_t* first_new_id, int64_t* bad_index) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (count < 0 || (count > 0 && !d_mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
+  return step_dev(g, (const int4*)d_mods, count, stats, first_new_id, bad_index);
 }
 
 igk_status igk_partition(const igk_graph* gc, int32_t* out, int64_t cap_len, int64_t* n_total) {
@@ -621,6 +725,26 @@ igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply
   if (apply_ms) *apply_ms = g->ms_apply;
   if (recount_ms) *recount_ms = g->ms_recount;
   return IGK_OK;
+}
+
+int32_t igk_debug_arrivals(const igk_graph* g, int32_t which, int64_t* out, int32_t cap) {
+  if (!g || !g->d.dbg || !out) return 0;
+  int grid = which == 0 ? g->grid_apply : g->grid_refine;
+  std::vector<unsigned long long> h((size_t)128 * grid);
+  if (cudaMemcpy(h.data(), g->d.dbg, h.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return 0;
+  for (size_t i = 0; i < h.size() && (int64_t)i < cap; i++) out[i] = (int64_t)h[i];
+  return grid;
+}
+
+int32_t igk_debug_phase_times(const igk_graph* g, int32_t which, int32_t* ids, int64_t* t_ns, int32_t cap) {
+  if (!g || which < 0 || which > 1) return 0;
+  const auto& v = g->ph[which];
+  int32_t n = (int32_t)std::min<size_t>(v.size(), (size_t)std::max(cap, 0));
+  for (int32_t i = 0; i < n; i++) {
+    if (ids) ids[i] = v[i].first;
+    if (t_ns) t_ns[i] = (int64_t)(v[i].second - v[0].second);
+  }
+  return n;
 }
 
 const char* igk_last_error(const igk_graph* g) { return g ? g->err.c_str() : "null handle"; }

@@ -1,16 +1,18 @@
 // refine.cuh -- incremental refinement (Sec. V.C) as one persistent kernel.
 //
-//   R1 filter over the affected set A          (Alg. 3 L8-24)
-//   deferred commit to the pseudo-partition    (Alg. 3 L25-26)
-//   R2 expansion: neighbours of pseudo vertices, filter, commit
-//   R3 balance restoration (paper silent; reading Q9): evict the minimum-loss
-//      vertices of every overweight part by a weighted device radix select
-//   R4 rounds (Alg. 4) until the pseudo-partition is empty:
-//      select (no smaller-ID pseudo neighbour) + best part (one adjacency
-//      pass, O(deg + k)) | balanced prefix by weighted radix select of the
-//      first violating move in (#nbr desc, ID asc) order | apply.
-// The paper's sort + k*M segmented scan is replaced by a select
-// that finds the same prefix length without sorting.
+//   F0  R1 filter over the affected set A            (Alg. 3 L8-24)
+//   F1  deferred commit of C1 to the pseudo-partition (Alg. 3 L25-26),
+//       fused with the R2 expansion marks (neighbours of pseudo vertices)
+//   F2  R2 filter on sigma2 | F3 commit of C2
+//   R3  balance restoration (paper silent; reading Q9): evict the minimum-loss
+//       vertices of every overweight part via a weighted device radix select
+//   R4  rounds (Alg. 4) until the pseudo-partition is empty:
+//       gain = selection (no smaller-ID pseudo neighbour) + best part in one
+//       adjacency pass, O(deg + k) | balanced prefix = weighted radix select of
+//       the first violating move in (#nbr desc, ID asc) order | apply
+//   FD  cut delta over the frontier F (every vertex that went through Psi)
+// The paper's sort + k x M segmented scan is replaced by a select
+// that yields the same prefix without sorting.
 #pragma once
 #include "common.cuh"
 
@@ -18,49 +20,118 @@ namespace igk {
 
 struct RefineArgs {
   long long e_ppm;
-  uint32_t epC1, epN, epC2, epE;
+  uint32_t epC1, epN, epC2, epF;
+  int after_apply;  // fused step: skip (leave the state untouched) if the batch was rejected
 };
 
 // ---------------------------------------------------------------------------
-// per-vertex scans
+// neighbour iteration with several loads in flight
 // ---------------------------------------------------------------------------
-// internal / external weighted degree on the current partition (
-// pseudo neighbours are external, Q13).  Thread variant.
-__device__ __forceinline__ void int_ext_thread(const Dev& d, int u, uint8_t pu, long long& in,
-                                               long long& ex) {
+// thread: f(x, w, q) for each neighbour; a chunk issues all its ID/weight
+// loads, then all its label loads, before f runs; f returns false to stop
+constexpr int kTC = 16;  // thread chunk (== kThreadDeg: one round trip per vertex)
+template <class F>
+__device__ __forceinline__ void nbrs_thread(const Dev& d, int u, F f) {
   const long long o = __ldg(d.off + u);
   const int dg = __ldg(d.deg + u);
-  long long a = 0, b = 0;
-  for (int i = 0; i < dg; i++) {
-    int x = __ldg(d.adj + o + i);
-    int w = edge_w(d.adjw, o + i);
-    if (ld_part(d.part, x) == pu) a += w; else b += w;
+  for (int i = 0; i < dg; i += kTC) {
+    int x[kTC], w[kTC];
+    uint8_t q[kTC];
+#pragma unroll
+    for (int t = 0; t < kTC; t++) {
+      x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
+      w[t] = (i + t < dg && d.adjw) ? __ldg(d.adjw + o + i + t) : 1;
+    }
+#pragma unroll
+    for (int t = 0; t < kTC; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+#pragma unroll
+    for (int t = 0; t < kTC; t++)
+      if (x[t] >= 0 && !f(x[t], w[t], q[t])) return;
   }
-  in = a;
-  ex = b;
 }
-// warp variant (all lanes get the totals)
-__device__ __forceinline__ void int_ext_warp(const Dev& d, int u, uint8_t pu, long long& in,
-                                             long long& ex) {
+
+// R2 expansion marks for the neighbours of u: the placed ones join N once
+// (stamp epN).  All stamp probes / exchanges of a chunk are in flight
+// together and N is appended with one atomic per lane and chunk.
+template <int C>
+__device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uint8_t* q, uint32_t epN) {
+  bool want[C];
+#pragma unroll
+  for (int t = 0; t < C; t++) want[t] = x[t] >= 0 && q[t] != kPsi && __ldcg(d.markT + x[t]) != epN;
+  unsigned old[C];
+#pragma unroll
+  for (int t = 0; t < C; t++) old[t] = want[t] ? atomicExch(d.markT + x[t], epN) : epN;
+  int c = 0;
+#pragma unroll
+  for (int t = 0; t < C; t++) c += old[t] != epN;
+  int slot = c ? atomicAdd(&d.ctl->nN, c) : 0;  // one reservation per lane and chunk
+#pragma unroll
+  for (int t = 0; t < C; t++)
+    if (old[t] != epN) d.Nlist[slot++] = x[t];
+}
+__device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN) {
   const long long o = __ldg(d.off + u);
   const int dg = __ldg(d.deg + u);
-  long long a = 0, b = 0;
-  for (int i = lane_id(); i < dg; i += 32) {
-    int x = __ldg(d.adj + o + i);
-    int w = edge_w(d.adjw, o + i);
-    if (ld_part(d.part, x) == pu) a += w; else b += w;
+  for (int i = 0; i < dg; i += kTC) {
+    int x[kTC];
+    uint8_t q[kTC];
+#pragma unroll
+    for (int t = 0; t < kTC; t++) x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
+#pragma unroll
+    for (int t = 0; t < kTC; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    mark_chunk<kTC>(d, x, q, epN);
   }
-  in = warp_sum(a);
-  ex = warp_sum(b);
+}
+__device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN) {
+  const long long o = __ldg(d.off + u);
+  const int dg = __ldg(d.deg + u);
+  for (int b = 0; b < dg; b += 256) {
+    int x[8];
+    uint8_t q[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      int i = b + t * 32 + lane_id();
+      x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
+    }
+#pragma unroll
+    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    mark_chunk<8>(d, x, q, epN);
+  }
+}
+// warp: lane-strided, 8 entries per lane per round trip (256 per warp)
+template <class F>
+__device__ __forceinline__ void nbrs_warp(const Dev& d, int u, F f) {
+  const long long o = __ldg(d.off + u);
+  const int dg = __ldg(d.deg + u);
+  for (int b = 0; b < dg; b += 256) {
+    int x[8], w[8];
+    uint8_t q[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      int i = b + t * 32 + lane_id();
+      x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
+      w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+    }
+#pragma unroll
+    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+#pragma unroll
+    for (int t = 0; t < 8; t++)
+      if (x[t] >= 0) f(x[t], w[t], q[t]);
+  }
 }
 
 // Iterate a vertex list: degree <= kThreadDeg -> one thread, else the whole
-// warp cooperates on it.  get(i) -> vertex (or -1); tf(u, i); wf(u, i).
+// warp cooperates on it.  Items are dealt round-robin over ALL warps of the
+// grid (item i -> warp i mod W, lane (i / W) mod 32), so a short list still
+// spreads over every SM and heavy vertices rarely share a warp.
+// get(i) -> vertex (or -1); tf(u, i); wf(u, i).
 template <class Get, class TF, class WF>
 __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get get, TF tf, WF wf) {
-  const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long base = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n; base += stride) {
-    long long i = base + lane_id();
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long per_round = nw * 32;
+  for (long long r0 = 0; r0 < n; r0 += per_round) {
+    long long i = r0 + (long long)lane_id() * nw + gw;
     int u = i < n ? get(i) : -1;
     int dg = u >= 0 ? __ldg(d.deg + u) : 0;
     bool heavy = dg > kThreadDeg;
@@ -70,7 +141,7 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
       int src = __ffs(hm) - 1;
       hm &= hm - 1;
       int uu = __shfl_sync(0xffffffffu, u, src);
-      wf(uu, base + src);
+      wf(uu, r0 + (long long)src * nw + gw);
     }
   }
 }
@@ -78,11 +149,11 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
 // ---------------------------------------------------------------------------
 // weighted radix select (shared by R3 and the round prefix)
 // Per candidate part p: find the first item, in ascending key order among the
-// items of part p, whose inclusive weight prefix reaches T_p.  Key =
-// (d0, R): d0 is an 8-bit digit built in the producing phase; R is the item's
-// vertex ID when bin d0 is exact, else a full 64-bit key.  MSD passes of 8
-// bits over R, one grid barrier per pass; every CTA recomputes the digit
-// choice from the global histograms, so no extra barrier is needed.
+// items of part p, whose inclusive weight prefix reaches T_p.  Key = (d0, R):
+// d0 is an 8-bit digit histogrammed by the producing phase (d.hist0); R is the
+// item's vertex ID when bin d0 is exact, else a full 64-bit key.  MSD passes
+// of 8 bits over R, one grid barrier per pass; every CTA recomputes the digit
+// choice from the global histograms, so the choice needs no extra barrier.
 // ---------------------------------------------------------------------------
 struct SelSmem {
   long long T[256];
@@ -139,7 +210,6 @@ __device__ __forceinline__ bool key_less(int da, unsigned long long ra, int db, 
   return da < db || (da == db && ra < rb);
 }
 
-// digit-0 choice for every candidate part (cands: flags per part in sm.used)
 template <class ExactFn>
 __device__ void sel_digit0(const Dev& d, SelSmem& sm, ExactFn is_exact, int exact_shift) {
   for (int p = threadIdx.x; p < 256; p += blockDim.x) {
@@ -173,7 +243,6 @@ __device__ void sel_digit0(const Dev& d, SelSmem& sm, ExactFn is_exact, int exac
   __syncthreads();
 }
 
-// accumulate pass `pass` histograms; items(j, &p, &d0, &R, &w) -> valid
 template <class Items>
 __device__ void sel_accumulate(const Dev& d, SelSmem& sm, int pass, long long nitems, Items items) {
   long long* hb = d.histR + (long long)(pass % 3) * 256 * kDigits;
@@ -182,17 +251,17 @@ __device__ void sel_accumulate(const Dev& d, SelSmem& sm, int pass, long long ni
   const long long nthr = (long long)gridDim.x * blockDim.x;
   for (long long t = tid; t < (long long)d.k * kDigits; t += nthr)
     if (sm.active[t / kDigits]) hz[t] = 0;
-  for (long long j = tid; j < nitems; j += nthr) {
+  rr_for(nitems, [&](long long j) {
     int p, d0;
     unsigned long long R;
     long long w;
-    if (!items(j, p, d0, R, w)) continue;
-    if (!sm.active[p] || d0 != sm.d0[p]) continue;
+    if (!items(j, p, d0, R, w)) return;
+    if (!sm.active[p] || d0 != sm.d0[p]) return;
     int sh = sm.shift[p];
-    if (sh + 8 < 64 && (R >> (sh + 8)) != (sm.prefix[p] >> (sh + 8))) continue;
+    if (sh + 8 < 64 && (R >> (sh + 8)) != (sm.prefix[p] >> (sh + 8))) return;
     int dig = (int)((R >> sh) & 255);
     atomic_add_ll(hb + (long long)p * kDigits + dig, w);
-  }
+  });
 }
 
 __device__ void sel_choose(const Dev& d, SelSmem& sm, int pass) {
@@ -220,7 +289,6 @@ __device__ void sel_choose(const Dev& d, SelSmem& sm, int pass) {
   __syncthreads();
 }
 
-// full select: digit 0 from d.hist0, then passes; returns after the last pass
 template <class ExactFn, class Items>
 __device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid, ExactFn is_exact,
                                 int exact_shift, long long nitems, Items items) {
@@ -228,15 +296,15 @@ __device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid,
   int pass = 0;
   while (sm.nactive > 0) {
     sel_accumulate(d, sm, pass, nitems, items);
+    arrive_stamp(d.dbg, 300 + pass - 200);
     grid.sync();
+    stamp_phase(d.ctl, 300 + pass);
     sel_choose(d, sm, pass);
     pass++;
   }
-  // every CTA must finish reading the histograms before anyone clears them
-  if (pass > 0) grid.sync();
+  if (pass > 0) grid.sync();  // every CTA finished reading before anyone clears
 }
 
-// zero the histogram rows the select used (call after every CTA finished it)
 __device__ void sel_clear(const Dev& d, const SelSmem& sm) {
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long nthr = (long long)gridDim.x * blockDim.x;
@@ -270,90 +338,72 @@ __device__ __forceinline__ void flush_acc(RefSmem& s, long long* dst, int k) {
   __syncthreads();
 }
 
-// candidate-set commit (Alg. 3 L25-26): cut and W_p deltas on the snapshot
-// before any label changes; edges between two candidates counted once.
-__device__ void commit_delta(const Dev& d, RefSmem& s, int nc, uint32_t ep, long long& cut_acc) {
-  auto get = [&](long long i) { return __ldcg(d.cand + i); };
-  auto delta_thread = [&](int u, long long) {
-    const uint8_t pu = ld_part(d.part, u);
-    const long long o = __ldg(d.off + u);
-    const int dg = __ldg(d.deg + u);
-    long long del = 0;
-    for (int i = 0; i < dg; i++) {
-      int x = __ldg(d.adj + o + i);
-      uint8_t px = ld_part(d.part, x);
-      if (px != kPsi && px != pu && !(x < u && __ldcg(d.markT + x) == ep)) del += edge_w(d.adjw, o + i);
-    }
-    cut_acc -= del;
-    atomicAdd((unsigned long long*)&s.acc[pu], (unsigned long long)(-(long long)vert_w(d.vw, u)));
-  };
-  auto delta_warp = [&](int u, long long) {
-    const uint8_t pu = ld_part(d.part, u);
-    const long long o = __ldg(d.off + u);
-    const int dg = __ldg(d.deg + u);
-    long long del = 0;
-    for (int i = lane_id(); i < dg; i += 32) {
-      int x = __ldg(d.adj + o + i);
-      uint8_t px = ld_part(d.part, x);
-      if (px != kPsi && px != pu && !(x < u && __ldcg(d.markT + x) == ep)) del += edge_w(d.adjw, o + i);
-    }
-    del = warp_sum(del);
-    if (lane_id() == 0) {
-      cut_acc -= del;
-      atomicAdd((unsigned long long*)&s.acc[pu], (unsigned long long)(-(long long)vert_w(d.vw, u)));
-    }
-  };
-  foreach_vertex(d, nc, get, delta_thread, delta_warp);
-}
-
-__device__ void commit_write(const Dev& d, int nc, int* psi_cnt, int32_t* psi_list) {
-  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  const long long nthr = (long long)gridDim.x * blockDim.x;
-  for (long long i = tid; i < nc; i += nthr) {
-    int u = __ldcg(d.cand + i);
-    d.part[u] = kPsi;
-    int slot = agg_append(psi_cnt, true);
-    psi_list[slot] = u;
-  }
-}
-
-// filter (Alg. 3 L8-24): candidates = listed placed vertices with ext > int
+// filter (Alg. 3 L8-24): candidates = listed placed vertices with ext > int;
+// pseudo neighbours count as external (Q13); strict > (Q2)
 template <class Get>
-__device__ void filter_pass(const Dev& d, long long n, Get get, uint32_t ep, long long& scanned,
+__device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, long long& scanned,
                             long long& counted) {
-  Ctl* ctl = d.ctl;
   auto tf = [&](int u, long long) {
     if (!__ldcg(d.active + u)) return;
-    uint8_t pu = ld_part(d.part, u);
+    const uint8_t pu = ld_part(d.part, u);
     if (pu == kPsi) return;
     counted++;
-    long long in, ex;
-    int_ext_thread(d, u, pu, in, ex);
+    long long in = 0, ex = 0;
+    nbrs_thread(d, u, [&](int, int w, uint8_t q) {
+      if (q == pu) in += w; else ex += w;
+      return true;
+    });
     scanned += __ldg(d.deg + u);
     bool c = ex > in;
-    if (c) {
-      d.markT[u] = ep;
-      int slot = atomicAdd(&ctl->ncand, 1);
-      d.cand[slot] = u;
-    }
+    int slot = agg_append(ncand, c);
+    if (c) cand[slot] = u;
   };
   auto wf = [&](int u, long long) {
     if (!__ldcg(d.active + u)) return;
-    uint8_t pu = ld_part(d.part, u);
+    const uint8_t pu = ld_part(d.part, u);
     if (pu == kPsi) return;
-    long long in, ex;
-    int_ext_warp(d, u, pu, in, ex);
+    long long in = 0, ex = 0;
+    nbrs_warp(d, u, [&](int, int w, uint8_t q) {
+      if (q == pu) in += w; else ex += w;
+    });
+    in = warp_sum(in);
+    ex = warp_sum(ex);
     if (lane_id() == 0) {
       counted++;
       scanned += __ldg(d.deg + u);
-      if (ex > in) {
-        d.markT[u] = ep;
-        int slot = atomicAdd(&ctl->ncand, 1);
-        d.cand[slot] = u;
-      }
+      if (ex > in) cand[atomicAdd(ncand, 1)] = u;
     }
   };
   foreach_vertex(d, n, get, tf, wf);
+}
+
+// deferred commit to the pseudo-partition (Alg. 3 L25-26): W_p, label, the
+// frontier list F; with `expand`, also mark the placed neighbours (R2)
+__device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, const int32_t* cand, bool expand,
+                       long long& scanned) {
+  Ctl* ctl = d.ctl;
+  rr_for(nc, [&](long long i) {
+    int u = __ldcg(cand + i);
+    uint8_t pu = ld_part(d.part, u);
+    d.oldp[u] = pu;
+    d.markF[u] = a.epF;
+    acc_add(s.acc, pu, -(long long)vert_w(d.vw, u));
+    d.part[u] = kPsi;
+    int slot = agg_append(&ctl->npsi[0], true);
+    d.psi[0][slot] = u;
+  });
+  if (!expand) return;
+  // labels read here may still show a C1 vertex as placed (written in this
+  // phase): such N entries are pseudo by the R2 filter and skipped there
+  auto mark_t = [&](int u, long long) {
+    scanned += __ldg(d.deg + u);
+    mark_nbrs_thread(d, u, a.epN);
+  };
+  auto mark_w = [&](int u, long long) {
+    if (lane_id() == 0) scanned += __ldg(d.deg + u);
+    mark_nbrs_warp(d, u, a.epN);
+  };
+  foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, mark_t, mark_w);
 }
 
 // better(a, b) on (conn desc, W_p asc, p asc)  (reading Q6)
@@ -372,6 +422,11 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long nthr = (long long)gridDim.x * blockDim.x;
+  if (a.after_apply && (ldv(&ctl->err_idx) != kNoErr || ldv(&ctl->err_nomem) != 0)) {
+    if (tid == 0) ctl->refine_skipped = 1;  // uniform exit: nothing was modified
+    return;
+  }
+  if (tid == 0) ctl->refine_skipped = 0;
   const long long c = cap_of(ldv(&ctl->W), a.e_ppm, k);
   const int exact_shift_id = ((d.idbits + 7) / 8) * 8 - 8;
 
@@ -383,119 +438,117 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
   for (int t = threadIdx.x; t < kWarps * 256; t += blockDim.x) (&s.wconn[0][0])[t] = 0;
   __syncthreads();
 
-  long long cut_acc = 0, scanned = 0, counted = 0, cnt_ins = 0;
-  // ---- F0: stats of the pending set; R1 filter over A on sigma1 -------------
+  if (tid == 0) ctl->nph = 0;
+  stamp_phase(ctl, 200);
+  arrive_stamp(d.dbg, 0);
+  long long scanned = 0, counted = 0, cnt_ins = 0;
+  // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
   const int nA = ldv(&ctl->nA);
   const int np0 = ldv(&ctl->npsi[0]);
-  for (long long i = tid; i < np0; i += nthr) {
+  rr_for(np0, [&](long long i) {
     int u = __ldcg(d.psi[0] + i);
-    if (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) cnt_ins++;
-  }
-  filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, a.epC1, scanned, counted);
+    if (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) {
+      cnt_ins++;
+      d.markF[u] = a.epF;
+      d.oldp[u] = kPsi;
+    }
+  });
+  filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, scanned, counted);
   block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
   block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
-  grid.sync();
+  GRID_SYNC_STAMPED(ctl, 201);
 
-  // ---- F1/F2: commit C1 -------------------------------------------------------
-  int nc = ldv(&ctl->ncand);
-  commit_delta(d, s, nc, a.epC1, cut_acc);
-  flush_acc(s, ctl->Wp, k);
-  grid.sync();
-  commit_write(d, nc, &ctl->npsi[0], d.psi[0]);
-  if (tid == 0) ctl->st[ST_FILTERED_IN] = nc;
-  grid.sync();
-
-  // ---- F3: R2 expansion: placed neighbours of every pseudo vertex ---
+  // ---- F1: commit C1 + R2 expansion marks -----------------------------------
   {
-    const int np = ldv(&ctl->npsi[0]);
-    if (tid == 0) ctl->ncand = 0;
+    const int nc = ldv(&ctl->ncand);
+    if (tid == 0) ctl->st[ST_FILTERED_IN] = nc;
+    commit(d, s, a, nc, d.cand, true, scanned);
+    // neighbours of the pseudo vertices pending since apply
     auto get = [&](long long i) {
       int u = __ldcg(d.psi[0] + i);
-      return (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) ? u : -1;
+      return (__ldcg(d.active + u) && __ldcg(d.markF + u) == a.epF && __ldcg(d.oldp + u) == kPsi) ? u : -1;
     };
-    auto tf = [&](int u, long long) {
-      const long long o = __ldg(d.off + u);
-      const int dg = __ldg(d.deg + u);
-      scanned += dg;
-      for (int i = 0; i < dg; i++) {
-        int x = __ldg(d.adj + o + i);
-        if (ld_part(d.part, x) != kPsi && stamp_insert(d.markT, x, a.epN))
-          d.Nlist[atomicAdd(&ctl->nN, 1)] = x;
-      }
+    auto mt = [&](int u, long long) {
+      scanned += __ldg(d.deg + u);
+      mark_nbrs_thread(d, u, a.epN);
     };
-    auto wf = [&](int u, long long) {
-      const long long o = __ldg(d.off + u);
-      const int dg = __ldg(d.deg + u);
-      if (lane_id() == 0) scanned += dg;
-      for (int i = lane_id(); i < dg; i += 32) {
-        int x = __ldg(d.adj + o + i);
-        bool add = ld_part(d.part, x) != kPsi && stamp_insert(d.markT, x, a.epN);
-        int slot = agg_append(&ctl->nN, add);
-        if (add) d.Nlist[slot] = x;
-      }
+    auto mw = [&](int u, long long) {
+      if (lane_id() == 0) scanned += __ldg(d.deg + u);
+      mark_nbrs_warp(d, u, a.epN);
     };
-    foreach_vertex(d, np, get, tf, wf);
+    foreach_vertex(d, np0, get, mt, mw);
+    flush_acc(s, ctl->Wp, k);
   }
-  grid.sync();
+  GRID_SYNC_STAMPED(ctl, 202);
 
-  // ---- F4: R2 filter on sigma2 ---------------------------------------------
+  // ---- F2: R2 filter on sigma2 ------------------------------------------------
   {
     const int nN = ldv(&ctl->nN);
-    long long dummy = 0;
-    filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, a.epC2, scanned, dummy);
-    if (tid == 0) ctl->st[ST_EXPANDED] = nN;
+    long long cntN = 0;
+    filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, &ctl->ncand2, d.cand2, scanned, cntN);
+    block_atomic_add(&ctl->st[ST_EXPANDED], cntN, s.red);
+    if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
   }
-  grid.sync();
-  nc = ldv(&ctl->ncand);
-  commit_delta(d, s, nc, a.epC2, cut_acc);
-  flush_acc(s, ctl->Wp, k);
-  grid.sync();
-  commit_write(d, nc, &ctl->npsi[0], d.psi[0]);
-  if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc;
-  grid.sync();
+  GRID_SYNC_STAMPED(ctl, 203);
 
-  // ---- R3: balance restoration (reading Q9) -----------------------------------
+  // ---- F3: commit C2 --------------------------------------------------------------
+  {
+    const int nc = ldv(&ctl->ncand2);
+    if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc;
+    commit(d, s, a, nc, d.cand2, false, scanned);
+    flush_acc(s, ctl->Wp, k);
+  }
+  GRID_SYNC_STAMPED(ctl, 204);
+
+  // ---- R3: balance restoration (reading Q9) ----------------------------------------
   {
     bool any = false;
     for (int p = 0; p < k; p++) any |= ldv(&ctl->Wp[p]) > c;
     if (any) {
-      if (tid == 0) ctl->ncand = 0;
       for (int p = threadIdx.x; p < k; p += blockDim.x) {
         long long wp = ldv(&ctl->Wp[p]);
         s.sel.used[p] = wp > c;
         s.sel.T[p] = wp - c;
       }
       __syncthreads();
-      // keys (int - ext, id) for every vertex of an overweight part, sigma3
+      // keys (int - ext, id) of every vertex of an overweight part on sigma3
       const long long ntot = ldv(&ctl->n_total);
       auto get = [&](long long v) {
         if (!__ldcg(d.active + v)) return -1;
         uint8_t p = ld_part(d.part, v);
         return (p != kPsi && s.sel.used[p]) ? (int)v : -1;
       };
-      auto emit = [&](int v, long long loss) {
-        uint8_t p = ld_part(d.part, v);
+      auto emit = [&](int v, uint8_t p, long long loss) {
         int d0 = (int)max(0ll, min(255ll, loss + 128));
         atomic_add_ll(d.hist0 + (long long)p * kDigits + d0, vert_w(d.vw, v));
         int slot = atomicAdd(&ctl->nr3, 1);
         d.r3list[slot] = make_int2(v, (int)loss);
       };
       auto tf = [&](int v, long long) {
-        long long in, ex;
-        int_ext_thread(d, v, ld_part(d.part, v), in, ex);
+        const uint8_t pv = ld_part(d.part, v);
+        long long in = 0, ex = 0;
+        nbrs_thread(d, v, [&](int, int w, uint8_t q) {
+          if (q == pv) in += w; else ex += w;
+          return true;
+        });
         scanned += __ldg(d.deg + v);
-        emit(v, in - ex);
+        emit(v, pv, in - ex);
       };
       auto wf = [&](int v, long long) {
-        long long in, ex;
-        int_ext_warp(d, v, ld_part(d.part, v), in, ex);
+        const uint8_t pv = ld_part(d.part, v);
+        long long in = 0, ex = 0;
+        nbrs_warp(d, v, [&](int, int w, uint8_t q) {
+          if (q == pv) in += w; else ex += w;
+        });
+        in = warp_sum(in);
+        ex = warp_sum(ex);
         if (lane_id() == 0) {
           scanned += __ldg(d.deg + v);
-          emit(v, in - ex);
+          emit(v, pv, in - ex);
         }
       };
       foreach_vertex(d, ntot, get, tf, wf);
-      grid.sync();
+      GRID_SYNC_STAMPED(ctl, 205);
       const int nr3 = ldv(&ctl->nr3);
       auto items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
         int2 e = __ldcg(d.r3list + j);
@@ -509,42 +562,37 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
       };
       weighted_select(d, s.sel, grid, [](int d0) { return d0 != 0 && d0 != 255; }, exact_shift_id, nr3, items);
       // evict every item with key <= the threshold of its part
-      for (long long j = tid; j < nr3; j += nthr) {
+      rr_for(nr3, [&](long long j) {
         int p, d0;
         unsigned long long R;
         long long w;
         items(j, p, d0, R, w);
-        if (!s.sel.found[p]) continue;
-        if (!key_less(s.sel.d0[p], s.sel.prefix[p], d0, R)) {
-          int v = __ldcg(d.r3list + j).x;
-          d.markT[v] = a.epE;
-          d.cand[atomicAdd(&ctl->ncand, 1)] = v;
-        }
-      }
+        bool ev = s.sel.found[p] && !key_less(s.sel.d0[p], s.sel.prefix[p], d0, R);
+        int slot = agg_append(&ctl->ncand, ev);
+        if (ev) d.cand[slot] = __ldcg(d.r3list + j).x;
+      });
       sel_clear(d, s.sel);
-      grid.sync();
-      nc = ldv(&ctl->ncand);
-      commit_delta(d, s, nc, a.epE, cut_acc);
+      GRID_SYNC_STAMPED(ctl, 206);
+      const int nc = ldv(&ctl->ncand);
+      commit(d, s, a, nc, d.cand, false, scanned);
       flush_acc(s, ctl->Wp, k);
-      grid.sync();
-      commit_write(d, nc, &ctl->npsi[0], d.psi[0]);
-      if (tid == 0) {
-        ctl->st[ST_EVICTED] = nc;
-        ctl->nr3 = 0;
-      }
+      if (tid == 0) ctl->st[ST_EVICTED] = nc;
       for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
-      grid.sync();
+      GRID_SYNC_STAMPED(ctl, 207);
     }
   }
 
-  // ---- R4: rounds (Alg. 4) ------------------------------------------------------
+  // ---- R4: rounds (Alg. 4) ------------------------------------------------------------
+  const int nF = ldv(&ctl->npsi[0]);
   int cur = 0;
   long long rounds = 0, rounds_all = 0, applied_tot = 0, deferred_tot = 0;
   while (true) {
     const int np = ldv(&ctl->npsi[cur]);
     if (np == 0) break;
-    int32_t* plist = d.psi[cur];
-    int32_t* pnext = d.psi[cur ^ 1];
+    const int nxt = cur == 1 ? 2 : 1;
+    const int32_t* plist = d.psi[cur];
+    int32_t* pnext = d.psi[nxt];
+    const int r3 = (int)(rounds_all % 3), r3n = (int)((rounds_all + 1) % 3);
     // round-start snapshot of W_p (Q14) and the lightest part (zero-conn choice)
     for (int p = threadIdx.x; p < k; p += blockDim.x) s.Wr[p] = ldv(&ctl->Wp[p]);
     __syncthreads();
@@ -555,20 +603,18 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
       s.best0 = b;
     }
     __syncthreads();
-    const int r3 = (int)(rounds_all % 3), r3n = (int)((rounds_all + 1) % 3);
     if (tid == 0) {
-      ctl->npsi[cur ^ 1] = 0;
+      ctl->npsi[nxt] = 0;
       ctl->applied3[r3n] = 0;
       ctl->selected3[r3n] = 0;
     }
     for (int p = (int)tid; p < k; p += (int)nthr) ctl->tot3[r3n][p] = 0;
     // -- gain: selection + best part, one adjacency pass per vertex
     long long sel_cnt = 0;
-    auto emit_move = [&](long long j, int u, int best, long long g, long long pwv, bool imbal) {
+    auto emit_move = [&](long long j, int u, int best, long long g, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
       d.tgt[u] = (uint8_t)best;
       d.gain[u] = (int)g;
-      d.pw[u] = (int)pwv;
       d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;
       long long w = vert_w(d.vw, u);
       atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
@@ -584,28 +630,22 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
       return u;
     };
     auto tf = [&](int u, long long j) {
-      const long long o = __ldg(d.off + u);
-      const int dg = __ldg(d.deg + u);
       const long long vwu = vert_w(d.vw, u);
-      scanned += dg;
+      scanned += __ldg(d.deg + u);
       int qs[kThreadDeg];
       int ws[kThreadDeg];
       int m = 0;
-      long long pwv = 0;
       bool sel = true;
-      for (int i = 0; i < dg; i++) {
-        int x = __ldg(d.adj + o + i);
-        uint8_t q = ld_part(d.part, x);
+      nbrs_thread(d, u, [&](int x, int w, uint8_t q) {
         if (q == kPsi) {
-          if (x < u) { sel = false; break; }
-          continue;
+          if (x < u) sel = false;  // a smaller-ID pseudo neighbour moves first (Alg. 4 L8)
+          return sel;
         }
-        int w = edge_w(d.adjw, o + i);
         qs[m] = q;
         ws[m] = w;
         m++;
-        pwv += w;
-      }
+        return true;
+      });
       if (!sel) {
         d.meta[j] = 0;
         return;
@@ -620,7 +660,10 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
         long long cc = 0;
         for (int t = i; t < m; t++) cc += qs[t] == p ? ws[t] : 0;
         if (s.Wr[p] + vwu > c) continue;
-        if (better(cc, p, bc, best, s.Wr)) { best = p; bc = cc; }
+        if (better(cc, p, bc, best, s.Wr)) {
+          best = p;
+          bc = cc;
+        }
       }
       bool imbal = false;
       if (best < 0) {  // lightest part: eligible => zero connectivity; else fallback (Q8)
@@ -632,55 +675,42 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
         }
       }
       sel_cnt++;
-      emit_move(j, u, best, bc, pwv, imbal);
+      emit_move(j, u, best, bc, imbal);
     };
     auto wf = [&](int u, long long j) {
-      const long long o = __ldg(d.off + u);
-      const int dg = __ldg(d.deg + u);
       const long long vwu = vert_w(d.vw, u);
       int* wc = s.wconn[warp_id()];
-      if (lane_id() == 0) scanned += dg;
-      long long pwv = 0;
-      bool blocked = false;
-      for (int b = 0; b < dg && !blocked; b += 32) {
-        int i = b + lane_id();
-        bool lb = false;
-        if (i < dg) {
-          int x = __ldg(d.adj + o + i);
-          uint8_t q = ld_part(d.part, x);
-          if (q == kPsi) {
-            lb = x < u;
-          } else {
-            int w = edge_w(d.adjw, o + i);
-            atomicAdd(wc + q, w);
-            pwv += w;
-          }
-        }
-        blocked = __any_sync(0xffffffffu, lb);
-      }
+      if (lane_id() == 0) scanned += __ldg(d.deg + u);
+      bool lb = false;
+      nbrs_warp(d, u, [&](int x, int w, uint8_t q) {
+        if (q == kPsi) lb |= x < u;
+        else atomicAdd(wc + q, w);
+      });
+      const bool blocked = __any_sync(0xffffffffu, lb);
       __syncwarp();
-      if (blocked) {
-        for (int p = lane_id(); p < k; p += 32) wc[p] = 0;
-        __syncwarp();
-        if (lane_id() == 0) d.meta[j] = 0;
-        return;
-      }
-      pwv = warp_sum(pwv);
       long long bc = -1;
       int best = -1;
-      for (int p = lane_id(); p < k; p += 32) {
-        if (s.Wr[p] + vwu > c) continue;
-        long long cc = wc[p];
-        if (better(cc, p, bc, best, s.Wr)) { best = p; bc = cc; }
-      }
+      if (!blocked) {
+        for (int p = lane_id(); p < k; p += 32) {
+          if (s.Wr[p] + vwu > c) continue;
+          long long cc = wc[p];
+          if (better(cc, p, bc, best, s.Wr)) {
+            best = p;
+            bc = cc;
+          }
+        }
 #pragma unroll
-      for (int off = 16; off > 0; off >>= 1) {
-        long long oc = __shfl_xor_sync(0xffffffffu, bc, off);
-        int op = __shfl_xor_sync(0xffffffffu, best, off);
-        if (op >= 0 && better(oc, op, bc, best, s.Wr)) { bc = oc; best = op; }
+        for (int off = 16; off > 0; off >>= 1) {
+          long long oc = __shfl_xor_sync(0xffffffffu, bc, off);
+          int op = __shfl_xor_sync(0xffffffffu, best, off);
+          if (op >= 0 && better(oc, op, bc, best, s.Wr)) {
+            bc = oc;
+            best = op;
+          }
+        }
       }
       bool imbal = false;
-      if (best < 0) {
+      if (!blocked && best < 0) {
         best = s.best0;
         bc = wc[best];
         imbal = true;
@@ -689,8 +719,12 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
       for (int p = lane_id(); p < k; p += 32) wc[p] = 0;
       __syncwarp();
       if (lane_id() == 0) {
-        sel_cnt++;
-        emit_move(j, u, best, bc, pwv, imbal);
+        if (blocked) {
+          d.meta[j] = 0;
+        } else {
+          sel_cnt++;
+          emit_move(j, u, best, bc, imbal);
+        }
       }
     };
     foreach_vertex(d, np, get, tf, wf);
@@ -698,7 +732,7 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
       long long sc = warp_sum(sel_cnt);
       if (lane_id() == 0 && sc) atomicAdd(&ctl->selected3[r3], (int)sc);
     }
-    grid.sync();
+    GRID_SYNC_STAMPED(ctl, 208);
 
     // -- balanced prefix: T_p = c - W_p + 1; K* = min over parts of the first
     //    move whose running weight in (#nbr desc, ID asc) order exceeds c.
@@ -730,9 +764,9 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
     }
     // -- apply the prefix (moves with key < K*); the rest stay pseudo
     long long app = 0;
-    for (long long j = tid; j < np; j += nthr) {
+    rr_for(np, [&](long long j) {
       int u = __ldcg(plist + j);
-      if (u < 0) continue;
+      if (u < 0) return;
       unsigned m = __ldcg(d.meta + j);
       bool keep = true;
       if (m & 0x80000000u) {
@@ -743,42 +777,39 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
         if (key_less(d0, R, kd, kr)) {
           keep = false;
           d.part[u] = (uint8_t)p;
-          atomicAdd((unsigned long long*)&s.acc[p], (unsigned long long)w);
-          cut_acc += (long long)__ldcg(d.pw + u) - __ldcg(d.gain + u);
+          acc_add(s.acc, p, w);
           app++;
         }
       } else if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
         keep = false;  // stale entry (deleted before this refine)
       }
-      int slot = agg_append(&ctl->npsi[cur ^ 1], keep);
+      int slot = agg_append(&ctl->npsi[nxt], keep);
       if (keep) pnext[slot] = u;
-    }
+    });
     flush_acc(s, ctl->Wp, k);
     {
       long long sa = warp_sum(app);
       if (lane_id() == 0 && sa) atomicAdd(&ctl->applied3[r3], (int)sa);
     }
-    // every part that received a selected move has hist0 entries: clear all rows
     for (long long t = tid; t < (long long)k * kDigits; t += nthr) d.hist0[t] = 0;
     sel_clear(d, s.sel);
-    grid.sync();
+    GRID_SYNC_STAMPED(ctl, 209);
     const int napp = ldv(&ctl->applied3[r3]), nsel = ldv(&ctl->selected3[r3]);
     if (napp == 0 && nsel > 0) {
       // L = 0: force the first move (reading Q8); it is the threshold item K*
       const int uf = (int)(kr & 0xffffffffu);
-      const int nn = ldv(&ctl->npsi[cur ^ 1]);
+      const int nn = ldv(&ctl->npsi[nxt]);
       for (long long j = tid; j < nn; j += nthr)
         if (__ldcg(pnext + j) == uf) pnext[j] = -1;
       if (tid == 0) {
         int p = __ldcg(d.tgt + uf);
         d.part[uf] = (uint8_t)p;
         atomic_add_ll(&ctl->Wp[p], vert_w(d.vw, uf));
-        atomic_add_ll(&ctl->cut, (long long)__ldcg(d.pw + uf) - __ldcg(d.gain + uf));
         ctl->st[ST_IMBAL] = 1;
       }
-      grid.sync();
+      GRID_SYNC_STAMPED(ctl, 210);
     }
-    const int napp2 = napp == 0 && nsel > 0 ? 1 : napp;
+    const int napp2 = (napp == 0 && nsel > 0) ? 1 : napp;
     if (nsel > 0) {
       rounds++;
       applied_tot += napp2;
@@ -786,14 +817,85 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
     }
     for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
     __syncthreads();
-    cur ^= 1;
+    cur = nxt;
     rounds_all++;
   }
 
-  // ---- epilogue: stats and counter resets ---------------------------------------
+  // ---- FD: cut delta over the frontier F (edges with an endpoint in F) -------
+  long long cut_acc = 0;
+  {
+    // delta of the edges of u: now (final labels, all placed) minus before
+    // (labels at refine start: oldp for F members); F-F edges once (x > u)
+    auto delta = [&](int u, const int* x, const int* w, const uint8_t* q, const unsigned* mf,
+                     const uint8_t* op, int C) {
+      const uint8_t pu = ld_part(d.part, u), ou = __ldcg(d.oldp + u);
+      long long acc = 0;
+      for (int t = 0; t < C; t++) {
+        if (x[t] < 0) continue;
+        bool xf = mf[t] == a.epF;
+        if (xf && x[t] < u) continue;
+        uint8_t ox = xf ? op[t] : q[t];
+        int was = (ou != kPsi && ox != kPsi && ou != ox) ? w[t] : 0;
+        int now = (pu != q[t]) ? w[t] : 0;
+        acc += now - was;
+      }
+      return acc;
+    };
+    auto get = [&](long long i) {
+      int u = __ldcg(d.psi[0] + i);
+      return __ldcg(d.active + u) ? u : -1;
+    };
+    auto tf = [&](int u, long long) {
+      const long long o = __ldg(d.off + u);
+      const int dg = __ldg(d.deg + u);
+      for (int i = 0; i < dg; i += kTC) {
+        int x[kTC], w[kTC];
+        uint8_t q[kTC], op[kTC];
+        unsigned mf[kTC];
+#pragma unroll
+        for (int t = 0; t < kTC; t++) {
+          x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
+          w[t] = (i + t < dg && d.adjw) ? __ldg(d.adjw + o + i + t) : 1;
+        }
+#pragma unroll
+        for (int t = 0; t < kTC; t++) {
+          q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+          mf[t] = x[t] >= 0 ? __ldcg(d.markF + x[t]) : 0u;
+          op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+        }
+        cut_acc += delta(u, x, w, q, mf, op, kTC);
+      }
+    };
+    auto wf = [&](int u, long long) {
+      const long long o = __ldg(d.off + u);
+      const int dg = __ldg(d.deg + u);
+      long long acc = 0;
+      for (int b = 0; b < dg; b += 256) {
+        int x[8], w[8];
+        uint8_t q[8], op[8];
+        unsigned mf[8];
+#pragma unroll
+        for (int t = 0; t < 8; t++) {
+          int i = b + t * 32 + lane_id();
+          x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
+          w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+        }
+#pragma unroll
+        for (int t = 0; t < 8; t++) {
+          q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+          mf[t] = x[t] >= 0 ? __ldcg(d.markF + x[t]) : 0u;
+          op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+        }
+        acc += delta(u, x, w, q, mf, op, 8);
+      }
+      acc = warp_sum(acc);
+      if (lane_id() == 0) cut_acc += acc;
+    };
+    foreach_vertex(d, nF, get, tf, wf);
+  }
   block_atomic_add(&ctl->cut, cut_acc, s.red);
   block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
-  grid.sync();
+  GRID_SYNC_STAMPED(ctl, 211);
   if (tid == 0) {
     ctl->st[ST_ROUNDS] = rounds;
     ctl->st[ST_MOVES_APPLIED] = applied_tot;
@@ -814,10 +916,12 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
     }
     ctl->nA = 0;
     ctl->ncand = 0;
+    ctl->ncand2 = 0;
     ctl->nN = 0;
     ctl->nr3 = 0;
     ctl->npsi[0] = 0;
     ctl->npsi[1] = 0;
+    ctl->npsi[2] = 0;
   }
 }
 

@@ -240,3 +240,25 @@ def test_edge_cases():
         assert Q.apply(S.next(gi.MODE_MIX, 0.05)) == 0
         Q.refine(f"k254 it{it}")
         Q.compare_state(f"k254 it{it}")
+
+
+def test_fused_step_api():
+    """igk_step (apply + refine in one call) == oracle; an invalid batch is
+    rejected atomically and the refine is skipped."""
+    cfg, g, part, P = _cfg_pair("C1", 1)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(1)) + 1)
+    for it in range(8):
+        b = gi.next_batch(S, cfg)
+        assert P.O.apply(b)[0] == 0
+        so, sto = P.O.refine()
+        sg, stg, bad = P.G.step(b)
+        assert sg == so and bad == -1
+        assert all(sto[f] == stg[f] for f in ("cut", "rounds", "affected", "moves_applied", "evicted"))
+        P.compare_state(f"step it{it}")
+        if it == 3:
+            before = (P.G.partition().tobytes(), P.G.cut())
+            bad_batch = np.array([[0, 0, 0, 0]], np.int32)  # self loop -> invalid
+            sg, stg, bad = P.G.step(bad_batch)
+            assert sg == 1 and bad == 0
+            assert (P.G.partition().tobytes(), P.G.cut()) == before

@@ -1,0 +1,73 @@
+#!/usr/bin/env python
+"""Average per-phase durations inside k_apply / k_refine (globaltimer stamps)
+over C2 iterations.  Usage: python tools/phase_profile.py [iters]"""
+import os
+import sys
+from collections import defaultdict
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+os.environ.setdefault("IGK_DEBUG_PHASES", "1")
+sys.path.insert(0, ROOT)
+import igk_inputs as gi  # noqa: E402
+import paper_conf_dac_leejlczcshh25_b200 as igk  # noqa: E402
+
+NAMES = {100: "start", 101: "V1 hash/counts", 102: "V2 validate/alloc", 103: "M12 deletions",
+         104: "M3 compact/insert-vertices", 199: "M4 insert-edges",
+         200: "start", 201: "F0 R1 filter", 202: "F1 commit C1 + expand", 203: "F2 R2 filter",
+         204: "F3 commit C2"}
+
+
+def main():
+    iters = int(sys.argv[1]) if len(sys.argv) > 1 else 30
+    cfg = gi.CONFIGS["C2"]
+    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(2))
+    part, _ = gi.metis_partition(g, cfg["k"])
+    G = igk.IGKGraph(g.xadj, g.adjncy, cfg["k"], cfg["eps"], part)
+    G.refine()
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(2)))
+    acc = [defaultdict(list), defaultdict(list)]
+    tot = [[], []]
+    for it in range(iters):
+        G.apply(gi.next_batch(S, cfg))
+        pa = G.phase_times(0)
+        _, st = G.refine()
+        pr = G.phase_times(1)
+        if it < 3:
+            continue
+        for w, ph in enumerate((pa, pr)):
+            for (i0, t0), (i1, t1) in zip(ph, ph[1:]):
+                acc[w][(i1, NAMES.get(i1, f"phase {i1}"))].append((t1 - t0) / 1e3)
+            tot[w].append((ph[-1][1] - ph[0][1]) / 1e3)
+    ms = G.last_ms()
+    if os.environ.get("IGK_DEBUG_ARRIVALS"):
+        for w in (0, 1):
+            print(["k_apply", "k_refine"][w], "arrivals (last launch):")
+            arrivals_report(G, w)
+    for w, name in enumerate(("k_apply", "k_refine")):
+        print(f"{name}: stamped span {np.mean(tot[w]):.1f} us (event-timed last launch {ms['apply' if w == 0 else 'refine'] * 1e3:.1f} us)")
+        for key, v in sorted(acc[w].items(), key=lambda kv: kv[0][0]):
+            print(f"   {key[0]:4d} {key[1]:32s} n={len(v):4d} mean {np.mean(v):7.2f} us")
+
+
+
+
+def arrivals_report(G, which):
+    """Per barrier slot: spread of CTA arrivals and the slowest CTA."""
+    A = G.arrivals(which)
+    if A is None:
+        return
+    ph = dict(G.phase_times(which))
+    t0 = min(v for v in A.flatten() if v > 0)
+    for s in range(128):
+        row = A[s]
+        if not row.any():
+            continue
+        r = (row - t0) / 1e3
+        print(f"   slot {s:3d}: arrivals min {r.min():8.2f} med {np.median(r):8.2f} max {r.max():8.2f} us, "
+              f"slowest CTA {int(np.argmax(row))}")
+
+
+if __name__ == "__main__":
+    main()
