@@ -275,11 +275,29 @@ def main():
                "h2d_bytes_per_step": int(np.mean([b.nbytes for b in h_batches])),
                "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches)}
 
+    # ---- S9 cut/weight reduction (full store scan, HBM-bound): own roofline
+    s9 = None
+    if not args.profile:
+        t9 = []
+        for _ in range(5):
+            if flush is not None:
+                flush.zero_()
+            torch.cuda.synchronize()
+            G.recount()
+            t9.append(G.last_ms()["recount"])
+        ss = G.store_stats()
+        b9 = ss["adj_entries"] * 5 + ss["n_total"] * 14  # 4 B ID + 1 B label per entry; 8+4+1+1 B per vertex
+        a9 = b9 / (float(np.median(t9)) / 1e3) / 1e9
+        s9 = {"kernel": "k_recount", "bound": "hbm", "achieved": a9, "unit": "GB/s", "bytes_per_launch": b9,
+              "launch_ms": float(np.median(t9)), "adj_entries": ss["adj_entries"]}
+
     if rank != 0:
         if dist:
             dist.destroy_process_group()
         return
     peak, peak_kind = peaks()
+    if s9:
+        s9.update(peak=peak, peak_kind=peak_kind, frac=s9["achieved"] / peak)
     achieved = rbytes / (refine_ms / 1e3) / 1e9 if refine_ms > 0 else 0.0
     traffic = None
     try:
@@ -308,6 +326,7 @@ def main():
                       "ms_p50": float(np.median([a.elapsed_time(b) for a, b in ev])),
                       "ms_p90": float(np.percentile([a.elapsed_time(b) for a, b in ev], 90))},
         "clocks": clocks,
+        "roofline_s9": s9,
     }
     if e2e:
         line["e2e"] = e2e

@@ -150,6 +150,10 @@ igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp);
  * *n_total and *n_slots. */
 igk_status igk_export_csr(const igk_graph* g, int64_t* xadj, int64_t xadj_len, int32_t* adjncy,
                           int32_t* adjwgt, int64_t adj_len, int64_t* n_total, int64_t* n_slots);
+/* store occupancy: IDs in use, active vertices and adjacency entries as of
+ * the last igk_recount, slab bump pointer and capacity (entries) */
+igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_active, int64_t* adj_entries,
+                           int64_t* slab_top, int64_t* slab_cap);
 /* number of kernels this handle has launched so far (instrumentation) */
 int64_t igk_kernel_launches(const igk_graph* g);
 /* device-side duration (ms) of the last igk_refine / apply / recount kernel,

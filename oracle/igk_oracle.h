@@ -12,6 +12,12 @@
  * DESIGN.md section 4.  A plain, single-threaded, slow implementation on
  * flat arrays; every function cites the passage it follows.
  *
+ * Pins (tests/test_oracle_pins.py): worked examples, exact-rational cap,
+ * brute-force step replay, exhaustive optimum, invariants.  R3 (balance
+ * restoration) follows reading Q9 of a passage the paper leaves silent: its
+ * implementation is pinned by brute force, but the reading itself is
+ * "parity unpinned" against the paper.
+ *
  * Modifiers are passed as int32 quadruples {kind, u, v, w}:
  *   kind 0 = edge deletion  M-(u,v)
  *   kind 1 = vertex deletion M-u      (Alg. 2)

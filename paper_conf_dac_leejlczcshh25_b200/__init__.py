@@ -25,7 +25,7 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine",
            "igk_step", "igk_step_device",
            "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
-           "igk_export_csr", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
+           "igk_export_csr", "igk_store_stats", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
            "igk_last_error", "igk_destroy"]
 
 
@@ -83,6 +83,8 @@ def lib():
         L.igk_recount.argtypes = [P, i64p, i64p]
         L.igk_export_csr.restype = C.c_int
         L.igk_export_csr.argtypes = [P, i64p, i64, i32p, i32p, i64, i64p, i64p]
+        L.igk_store_stats.restype = C.c_int
+        L.igk_store_stats.argtypes = [P, i64p, i64p, i64p, i64p, i64p]
         L.igk_kernel_launches.restype = i64
         L.igk_kernel_launches.argtypes = [P]
         L.igk_last_kernel_ms.restype = C.c_int
@@ -229,6 +231,13 @@ class IGKGraph:
                     adj[a:b] = adj[a:b][o]
                     w[a:b] = w[a:b][o]
         return xadj, adj, w
+
+    def store_stats(self):
+        v = [C.c_int64(0) for _ in range(5)]
+        s = lib().igk_store_stats(self.h, *[C.byref(x) for x in v])
+        if s != OK:
+            raise IGKError(s, self._err())
+        return dict(zip(["n_total", "n_active", "adj_entries", "slab_top", "slab_cap"], [x.value for x in v]))
 
     def kernel_launches(self):
         return int(lib().igk_kernel_launches(self.h))

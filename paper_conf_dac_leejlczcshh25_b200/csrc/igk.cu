@@ -41,7 +41,8 @@ __global__ void k_build(Dev d, const int64_t* xadj, const int32_t* adjncy, const
 // (owner lane found by a shuffle binary search), so slab reads stay
 // coalesced; the 1-byte label gather hits L2.  Edges counted once (u < x).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp) {
+__global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp,
+                                                 long long* out_cnt) {
   __shared__ long long s_wp[256];
   __shared__ long long s_red[32];
   for (int p = threadIdx.x; p < 256; p += blockDim.x) s_wp[p] = 0;
@@ -49,14 +50,26 @@ __global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* 
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   const int lane = lane_id();
-  long long cut = 0;
+  long long cut = 0, ent = 0, nact = 0;
   for (long long base = gw * 32; base < n; base += nw * 32) {
     long long v = base + lane;
-    bool act = v < n && __ldg(d.active + v);
-    uint8_t pv = act ? __ldg(d.part + v) : kPsi;
-    int dg = act ? __ldg(d.deg + v) : 0;
-    long long o = act ? __ldg(d.off + v) : 0;
-    if (act && pv != kPsi) atomicAdd((unsigned long long*)&s_wp[pv], (unsigned long long)vert_w(d.vw, v));
+    bool act = false;
+    uint8_t pv = kPsi;
+    int dg = 0;
+    long long o = 0;
+    if (v < n) {  // independent loads: active, label, degree, offset
+      act = __ldg(d.active + v);
+      pv = __ldg(d.part + v);
+      dg = __ldg(d.deg + v);
+      o = __ldg(d.off + v);
+    }
+    if (!act) {
+      pv = kPsi;
+      dg = 0;
+    }
+    ent += dg;
+    nact += act;
+    if (act && pv != kPsi) acc_add(s_wp, pv, vert_w(d.vw, v));
     if (pv == kPsi) dg = 0;  // pending vertices own no cut edges
     int pre = dg;
 #pragma unroll
@@ -66,28 +79,39 @@ __global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* 
     }
     const int total = __shfl_sync(0xffffffffu, pre, 31);
     pre -= dg;  // exclusive
-    for (int e0 = 0; e0 < total; e0 += 32) {
-      int e = e0 + lane;
-      int lo = 0;
+    for (int e0 = 0; e0 < total; e0 += 128) {  // 4 entries per lane in flight
+      int x[4], w[4], lo[4];
+      long long owner[4];
 #pragma unroll
-      for (int st = 16; st > 0; st >>= 1) {
-        int cand = lo + st;
-        int pc = __shfl_sync(0xffffffffu, pre, cand & 31);
-        if (cand < 32 && pc <= e) lo = cand;
+      for (int t = 0; t < 4; t++) {
+        int e = e0 + t * 32 + lane;
+        int l = 0;
+#pragma unroll
+        for (int st = 16; st > 0; st >>= 1) {
+          int cand = l + st;
+          int pc = __shfl_sync(0xffffffffu, pre, cand & 31);
+          if (cand < 32 && pc <= e) l = cand;
+        }
+        lo[t] = l;
+        long long oo = __shfl_sync(0xffffffffu, o, l);
+        int po = __shfl_sync(0xffffffffu, pre, l);
+        owner[t] = base + l;
+        x[t] = e < total ? __ldg(d.adj + oo + (e - po)) : -1;
+        w[t] = (e < total && d.adjw) ? __ldg(d.adjw + oo + (e - po)) : 1;
       }
-      long long oo = __shfl_sync(0xffffffffu, o, lo);
-      int po = __shfl_sync(0xffffffffu, pre, lo);
-      int pp = __shfl_sync(0xffffffffu, (int)pv, lo);
-      if (e < total) {
-        long long j = oo + (e - po);
-        int x = __ldg(d.adj + j);
-        long long owner = base + lo;
-        uint8_t px = __ldg(d.part + x);
-        if (x > owner && px != kPsi && px != (uint8_t)pp) cut += edge_w(d.adjw, j);
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        int pp = __shfl_sync(0xffffffffu, (int)pv, lo[t]);
+        if (x[t] > owner[t]) {
+          uint8_t px = __ldg(d.part + x[t]);
+          if (px != kPsi && px != (uint8_t)pp) cut += w[t];
+        }
       }
     }
   }
   block_atomic_add(out_cut, cut, s_red);
+  block_atomic_add(out_cnt, ent, s_red);
+  block_atomic_add(out_cnt + 1, nact, s_red);
   for (int p = threadIdx.x; p < d.k; p += blockDim.x)
     if (s_wp[p]) atomicAdd((unsigned long long*)&out_wp[p], (unsigned long long)s_wp[p]);
 }
@@ -124,7 +148,8 @@ struct igk_graph {
   int debug_phases = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
-  long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp
+  long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active
+  long long last_entries = 0, last_active = 0;
   Ctl* h_ctl = nullptr;        // pinned mirror of the control block
   cudaEvent_t ev[6] = {};
   float ms_refine = 0, ms_apply = 0, ms_recount = 0;
@@ -175,12 +200,12 @@ int coop_grid(const void* fn, size_t smem, int want_per_sm) {
 }
 
 igk_status launch_recount(igk_graph* g) {
-  CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 257, g->stream));
+  CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 259, g->stream));
   int sms = 0;
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device));
   long long n = g->h_ctl->n_total;
   CK(cudaEventRecord(g->ev[4], g->stream));
-  k_recount<<<sms * 4, 512, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1);
+  k_recount<<<sms * 4, 512, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
   g->launches++;
   CK(cudaGetLastError());
   CK(cudaEventRecord(g->ev[5], g->stream));
@@ -295,7 +320,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.meta, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
-            dalloc(g, &g->d_red, 257);
+            dalloc(g, &g->d_red, 259);
   if (!ok) {
     igk_destroy(g);
     return IGK_ENOMEM;
@@ -671,10 +696,12 @@ igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp) {
   if (!g || g->poisoned) return IGK_ESTATE;
   igk_status st = launch_recount(g);
   if (st != IGK_OK) return st;
-  long long red[257];
+  long long red[259];
   CK(cudaMemcpyAsync(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
   cudaEventElapsedTime(&g->ms_recount, g->ev[4], g->ev[5]);
+  g->last_entries = red[257];
+  g->last_active = red[258];
   if (out_cut) *out_cut = red[0];
   if (out_wp)
     for (int p = 0; p < g->d.k; p++) out_wp[p] = red[1 + p];
@@ -718,6 +745,17 @@ igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, 
 }
 
 int64_t igk_kernel_launches(const igk_graph* g) { return g ? g->launches : 0; }
+
+igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_active, int64_t* adj_entries,
+                           int64_t* slab_top, int64_t* slab_cap) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (n_total) *n_total = g->h_ctl->n_total;
+  if (n_active) *n_active = g->last_active;
+  if (adj_entries) *adj_entries = g->last_entries;
+  if (slab_top) *slab_top = g->h_ctl->slab_top;
+  if (slab_cap) *slab_cap = g->d.slot_cap;
+  return IGK_OK;
+}
 
 igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms) {
   if (!g) return IGK_ESTATE;

@@ -21,16 +21,22 @@ NAMES = {100: "start", 101: "V1 hash/counts", 102: "V2 validate/alloc", 103: "M1
 
 def main():
     iters = int(sys.argv[1]) if len(sys.argv) > 1 else 30
-    cfg = gi.CONFIGS["C2"]
-    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(2))
-    part, _ = gi.metis_partition(g, cfg["k"])
-    G = igk.IGKGraph(g.xadj, g.adjncy, cfg["k"], cfg["eps"], part)
+    name = sys.argv[2] if len(sys.argv) > 2 else "C2"
+    cfg = dict(gi.CONFIGS[name])
+    k = int(sys.argv[3]) if len(sys.argv) > 3 else (cfg["k"] if isinstance(cfg["k"], int) else cfg["k"][0])
+    if len(sys.argv) > 4:
+        cfg["frac"] = float(sys.argv[4])
+    idx = int(name[1:])
+    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(idx))
+    part, _ = gi.metis_partition(g, k)
+    G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part)
     G.refine()
-    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(2)))
+    region0 = (part == 0).astype(np.int32) if cfg["mode"] == gi.MODE_ADVERSARIAL else None
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(idx)), region0=region0)
     acc = [defaultdict(list), defaultdict(list)]
     tot = [[], []]
     for it in range(iters):
-        G.apply(gi.next_batch(S, cfg))
+        G.apply(gi.next_batch(S, cfg, cfg.get("frac") if cfg["mode"] == gi.MODE_MIX else None))
         pa = G.phase_times(0)
         _, st = G.refine()
         pr = G.phase_times(1)
