@@ -36,28 +36,32 @@ __global__ void k_build(Dev d, const int64_t* xadj, const int32_t* adjncy, const
 }
 
 // ---------------------------------------------------------------------------
-// S9: cut / part-weight reduction.  Each warp owns 32 consecutive
-// vertices and walks their concatenated adjacency 32 entries at a time
-// (owner lane found by a shuffle binary search), so slab reads stay
-// coalesced; the 1-byte label gather hits L2.  Edges counted once (u < x).
+// S9: cut / part-weight reduction, a full store scan.  One thread per
+// vertex (consecutive lanes = consecutive IDs, so the per-vertex arrays are
+// read coalesced); every prefix starts 16-byte aligned (capacities are
+// multiples of 4), so a list is read with int4 loads; vertices of degree > 64
+// are walked by the whole warp (8 loads per lane in flight).  Labels are a
+// 1-byte gather that stays in L2.  Edges are counted once (x > v).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp,
+constexpr int kRcHeavy = 64;
+__global__ void __launch_bounds__(512, 2) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp,
                                                  long long* out_cnt) {
   __shared__ long long s_wp[256];
   __shared__ long long s_red[32];
   for (int p = threadIdx.x; p < 256; p += blockDim.x) s_wp[p] = 0;
   __syncthreads();
-  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   const int lane = lane_id();
+  const bool ballot_wp = d.vw == nullptr && d.k <= 32;  // unit weights: W_p by popc(ballot)
   long long cut = 0, ent = 0, nact = 0;
-  for (long long base = gw * 32; base < n; base += nw * 32) {
-    long long v = base + lane;
+  long long wp_lane = 0;  // ballot mode: lane p accumulates W_p
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long base = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n; base += stride) {
+    const long long v = base + lane;
     bool act = false;
     uint8_t pv = kPsi;
     int dg = 0;
     long long o = 0;
-    if (v < n) {  // independent loads: active, label, degree, offset
+    if (v < n) {
       act = __ldg(d.active + v);
       pv = __ldg(d.part + v);
       dg = __ldg(d.deg + v);
@@ -69,46 +73,62 @@ __global__ void __launch_bounds__(512) k_recount(Dev d, long long n, long long* 
     }
     ent += dg;
     nact += act;
-    if (act && pv != kPsi) acc_add(s_wp, pv, vert_w(d.vw, v));
-    if (pv == kPsi) dg = 0;  // pending vertices own no cut edges
-    int pre = dg;
-#pragma unroll
-    for (int s = 1; s < 32; s <<= 1) {
-      int y = __shfl_up_sync(0xffffffffu, pre, s);
-      if (lane >= s) pre += y;
-    }
-    const int total = __shfl_sync(0xffffffffu, pre, 31);
-    pre -= dg;  // exclusive
-    for (int e0 = 0; e0 < total; e0 += 128) {  // 4 entries per lane in flight
-      int x[4], w[4], lo[4];
-      long long owner[4];
-#pragma unroll
-      for (int t = 0; t < 4; t++) {
-        int e = e0 + t * 32 + lane;
-        int l = 0;
-#pragma unroll
-        for (int st = 16; st > 0; st >>= 1) {
-          int cand = l + st;
-          int pc = __shfl_sync(0xffffffffu, pre, cand & 31);
-          if (cand < 32 && pc <= e) l = cand;
-        }
-        lo[t] = l;
-        long long oo = __shfl_sync(0xffffffffu, o, l);
-        int po = __shfl_sync(0xffffffffu, pre, l);
-        owner[t] = base + l;
-        x[t] = e < total ? __ldg(d.adj + oo + (e - po)) : -1;
-        w[t] = (e < total && d.adjw) ? __ldg(d.adjw + oo + (e - po)) : 1;
+    const bool placed = act && pv != kPsi;
+    if (ballot_wp) {
+      for (int p = 0; p < d.k; p++) {
+        unsigned m = __ballot_sync(0xffffffffu, placed && pv == p);
+        if (lane == p) wp_lane += __popc(m);
       }
+    } else if (placed) {
+      acc_add(s_wp, pv, vert_w(d.vw, v));
+    }
+    if (!placed) dg = 0;  // pending vertices own no cut edges
+    const bool heavy = dg > kRcHeavy;
+    if (!heavy && dg > 0) {
+      const int4* a4 = reinterpret_cast<const int4*>(d.adj + o);
+      const int4* w4 = d.adjw ? reinterpret_cast<const int4*>(d.adjw + o) : nullptr;
+      for (int i = 0; i < dg; i += 8) {  // two int4 per round trip, then 8 label gathers
+        int4 a0 = __ldg(a4 + (i >> 2));
+        int4 a1 = (i + 4 < dg) ? __ldg(a4 + (i >> 2) + 1) : make_int4(-1, -1, -1, -1);
+        int4 w0 = w4 ? __ldg(w4 + (i >> 2)) : make_int4(1, 1, 1, 1);
+        int4 w1 = (w4 && i + 4 < dg) ? __ldg(w4 + (i >> 2) + 1) : make_int4(1, 1, 1, 1);
+        const int xs[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const int ws[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
+        uint8_t qs[8];
 #pragma unroll
-      for (int t = 0; t < 4; t++) {
-        int pp = __shfl_sync(0xffffffffu, (int)pv, lo[t]);
-        if (x[t] > owner[t]) {
-          uint8_t px = __ldg(d.part + x[t]);
-          if (px != kPsi && px != (uint8_t)pp) cut += w[t];
+        for (int t = 0; t < 8; t++) qs[t] = (i + t < dg && xs[t] > v) ? __ldg(d.part + xs[t]) : pv;
+#pragma unroll
+        for (int t = 0; t < 8; t++)
+          if (qs[t] != kPsi && qs[t] != pv) cut += ws[t];
+      }
+    }
+    unsigned hm = __ballot_sync(0xffffffffu, heavy);
+    while (hm) {
+      const int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      const long long hv = base + src;
+      const long long ho = __shfl_sync(0xffffffffu, o, src);
+      const int hd = __shfl_sync(0xffffffffu, dg, src);
+      const uint8_t hp = (uint8_t)__shfl_sync(0xffffffffu, (int)pv, src);
+      for (int b = 0; b < hd; b += 128) {
+        int x[4], w[4];
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+          int i = b + 32 * t + lane;
+          x[t] = i < hd ? __ldg(d.adj + ho + i) : -1;
+          w[t] = (i < hd && d.adjw) ? __ldg(d.adjw + ho + i) : 1;
+        }
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+          if (x[t] > hv) {
+            uint8_t q = __ldg(d.part + x[t]);
+            if (q != kPsi && q != hp) cut += w[t];
+          }
         }
       }
     }
   }
+  if (ballot_wp && lane < d.k && wp_lane) atomicAdd((unsigned long long*)&s_wp[lane], (unsigned long long)wp_lane);
   block_atomic_add(out_cut, cut, s_red);
   block_atomic_add(out_cnt, ent, s_red);
   block_atomic_add(out_cnt + 1, nact, s_red);

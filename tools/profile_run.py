@@ -21,4 +21,12 @@ S = gi.Stream(g, gi.stream_seed(gi.graph_seed(idx)))
 for it in range(iters):
     G.apply(gi.next_batch(S, cfg))
     G.refine()
+if "--recount" in sys.argv:
+    import torch
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    for _ in range(3):
+        flush.zero_()
+        torch.cuda.synchronize()
+        G.recount()
+    print("recount ms", G.last_ms()["recount"], G.store_stats())
 print("done", G.cut())
