@@ -231,8 +231,8 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       ok = ok && dup_free(m.y, m.z);
       if (ok && uo && vo) ok = !exists(m.y, m.z);
       if (ok) {
-        long long du = (m.y < n0 ? __ldcg(d.deg + m.y) : 0) + __ldcg(d.icnt + m.y);
-        long long dv = (m.z < n0 ? __ldcg(d.deg + m.z) : 0) + __ldcg(d.icnt + m.z);
+        long long du = (m.y < n0 ? __ldcg(d.ldeg + m.y) : 0) + __ldcg(d.icnt + m.y);
+        long long dv = (m.z < n0 ? __ldcg(d.ldeg + m.z) : 0) + __ldcg(d.icnt + m.z);
         ok = du <= kDegMax && dv <= kDegMax;
       }
     } else {
@@ -283,20 +283,49 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
 
   // ---- M12: edge deletions and vertex deletions (tombstones) ---------------
   long long cut_acc = 0, W_acc = 0;
-  for (long long i = gwarp; i < B; i += nwarp) {  // one warp per edge deletion
-    int4 m = a.mods[i];
-    if (m.x != kEdgeDel) continue;
-    long long su = warp_find(d.adj, __ldcg(d.off + m.y), __ldcg(d.deg + m.y), m.z);
-    long long sv = warp_find(d.adj, __ldcg(d.off + m.z), __ldcg(d.deg + m.z), m.y);
-    if (lane_id() == 0) {
+  // edge deletions: one thread per modifier; a search in a prefix longer than
+  // 32 entries is done by the whole warp (ballot loop)
+  rr_for_warp(B, [&](long long i, bool valid) {
+    int4 m = valid ? a.mods[i] : make_int4(-1, 0, 0, 0);
+    const bool ed = m.x == kEdgeDel;
+    long long ou = 0, ox = 0;
+    int du = 0, dx = 0;
+    if (ed) {
+      ou = __ldcg(d.off + m.y);
+      du = __ldcg(d.deg + m.y);
+      ox = __ldcg(d.off + m.z);
+      dx = __ldcg(d.deg + m.z);
+    }
+    long long su = (ed && du <= 32) ? thread_find(d.adj, ou, du, m.z) : -1;
+    long long sx = (ed && dx <= 32) ? thread_find(d.adj, ox, dx, m.y) : -1;
+    unsigned hm = __ballot_sync(0xffffffffu, ed && du > 32);
+    while (hm) {
+      int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      long long s = warp_find(d.adj, __shfl_sync(0xffffffffu, ou, src), __shfl_sync(0xffffffffu, du, src),
+                              __shfl_sync(0xffffffffu, m.z, src));
+      if (lane_id() == src) su = s;
+    }
+    hm = __ballot_sync(0xffffffffu, ed && dx > 32);
+    while (hm) {
+      int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      long long s = warp_find(d.adj, __shfl_sync(0xffffffffu, ox, src), __shfl_sync(0xffffffffu, dx, src),
+                              __shfl_sync(0xffffffffu, m.y, src));
+      if (lane_id() == src) sx = s;
+    }
+    if (ed) {
       int w = d.adjw ? __ldcg(d.adjw + su) : 1;
       d.adj[su] = -1;
-      d.adj[sv] = -1;
+      d.adj[sx] = -1;
+      atomicSub(d.ldeg + m.y, 1);
+      atomicSub(d.ldeg + m.z, 1);
       uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
       if (pu != kPsi && pv != kPsi && pu != pv) cut_acc -= w;
+      mark_dirty_affected(d, m.y, a.epT, a.epA);
+      mark_dirty_affected(d, m.z, a.epT, a.epA);
     }
-    if (lane_id() < 2) mark_dirty_affected(d, lane_id() ? m.z : m.y, a.epT, a.epA);
-  }
+  });
   {
     const int nch = ldv(&ctl->nvdch);
     for (long long t = gwarp; t < nch; t += nwarp) {  // one warp per 32 neighbours
@@ -315,6 +344,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
         long long s = thread_find(d.adj, __ldcg(d.off + x), dx, u);
         d.adj[s] = -1;
       }
+      if (x >= 0 && !xdel) atomicSub(d.ldeg + x, 1);
       unsigned hm = __ballot_sync(0xffffffffu, x >= 0 && !xdel && !small);
       while (hm) {
         int src = __ffs(hm) - 1;
@@ -342,6 +372,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     int4 m = a.mods[i];
     if (m.x == kVertDel) {
       d.deg[m.y] = 0;
+      d.ldeg[m.y] = 0;
       d.active[m.y] = 0;
       d.part[m.y] = kDel;
     } else if (m.x == kVertIns) {
@@ -354,6 +385,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
         d.capv[id] = 0;
         d.off[id] = 0;
       }
+      d.ldeg[id] = 0;
       W_acc += m.w;
       int slot = agg_append(&ctl->npsi[0], true);
       d.psi[0][slot] = id;
@@ -406,6 +438,9 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       int x = d.dlist[t];
       if (__ldcg(d.markD + x) == a.epD) continue;
       if (__ldcg(d.markG + x) == a.epG && __ldcg(d.reloc + x) >= 0) continue;
+      // lazy compaction: tombstones stay until they are more than half the prefix
+      const int dg = __ldcg(d.deg + x), live = __ldcg(d.ldeg + x);
+      if (2 * (dg - live) <= dg) continue;
       long long o = __ldcg(d.off + x);
       int wr = compact(x, o, o);
       if (lane_id() == 0) d.deg[x] = wr;
@@ -423,6 +458,8 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     if (m.x != kEdgeIns) return;
     int pu_pos = atomicAdd(d.deg + m.y, 1);
     int pv_pos = atomicAdd(d.deg + m.z, 1);
+    atomicAdd(d.ldeg + m.y, 1);
+    atomicAdd(d.ldeg + m.z, 1);
     long long su = __ldcg(d.off + m.y) + pu_pos, sv = __ldcg(d.off + m.z) + pv_pos;
     d.adj[su] = m.z;
     d.adj[sv] = m.y;

@@ -79,7 +79,8 @@ struct Dev {
   int32_t idbits;    // bits to hold any vertex ID < n_cap
   // graph store (S0)
   int64_t* off;      // slab offset of each vertex's dense prefix
-  int32_t* deg;      // prefix length
+  int32_t* deg;      // prefix length (live entries + tombstones, -1)
+  int32_t* ldeg;     // live degree (tombstones excluded)
   int32_t* capv;     // capacity
   int32_t* adj;      // neighbour IDs
   int32_t* adjw;     // edge weights (nullptr = unit)
@@ -179,6 +180,21 @@ __device__ __forceinline__ void rr_for(long long n, F f) {
   for (long long c = my; c < nch; c += nw) {
     long long i = (c << 5) + (threadIdx.x & 31);
     if (i < n) f(i);
+  }
+}
+
+// Warp-uniform variant of rr_for: f(i, valid) runs on every lane of the warp
+// in every iteration (valid == false past the end), so f may use warp
+// collectives (ballot loops for heavy items).
+template <class F>
+__device__ __forceinline__ void rr_for_warp(long long n, F f) {
+  const long long G = gridDim.x, W = blockDim.x >> 5;
+  const long long my = (long long)(threadIdx.x >> 5) * G + blockIdx.x;
+  const long long nw = G * W;
+  const long long nch = (n + 31) >> 5;
+  for (long long c = my; c < nch; c += nw) {
+    long long i = (c << 5) + (threadIdx.x & 31);
+    f(i, i < n);
   }
 }
 

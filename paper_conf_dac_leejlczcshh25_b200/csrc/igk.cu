@@ -328,7 +328,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     return IGK_EINVAL;
   }
   const size_t N = (size_t)d.n_cap;
-  bool ok = dalloc(g, &d.off, N) && dalloc(g, &d.deg, N) && dalloc(g, &d.capv, N) &&
+  bool ok = dalloc(g, &d.off, N) && dalloc(g, &d.deg, N) && dalloc(g, &d.ldeg, N) && dalloc(g, &d.capv, N) &&
             dalloc(g, &d.adj, (size_t)d.slot_cap) && (g->ew_unit || dalloc(g, &d.adjw, (size_t)d.slot_cap)) &&
             dalloc(g, &d.active, N) && (g->vw_unit || dalloc(g, &d.vw, N)) && dalloc(g, &d.part, N) &&
             dalloc(g, &d.markA, N) && dalloc(g, &d.markT, N) && dalloc(g, &d.markD, N) &&
@@ -355,6 +355,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   cudaMemsetAsync(d.active, 0, N, s);
   cudaMemsetAsync(d.part, kDel, N, s);
   cudaMemsetAsync(d.deg, 0, N * 4, s);
+  cudaMemsetAsync(d.ldeg, 0, N * 4, s);
   cudaMemsetAsync(d.capv, 0, N * 4, s);
   cudaMemsetAsync(d.off, 0, N * 8, s);
   cudaMemsetAsync(d.markA, 0, N * 4, s);
@@ -386,6 +387,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     if (e == cudaSuccess && m2 && d_adjwgt) e = cudaMemcpy(d_adjwgt, adjwgt, m2 * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.off, off.data(), n * 8, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.deg, deg.data(), n * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d.ldeg, deg.data(), n * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.capv, capv.data(), n * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.part, part8.data(), n, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.active, act.data(), n, cudaMemcpyHostToDevice);
@@ -734,33 +736,38 @@ igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, 
   if (!g || g->poisoned) return IGK_ESTATE;
   long long n = g->h_ctl->n_total;
   std::vector<int64_t> off((size_t)std::max<long long>(n, 1));
-  std::vector<int32_t> deg((size_t)std::max<long long>(n, 1));
+  std::vector<int32_t> deg((size_t)std::max<long long>(n, 1)), ldeg((size_t)std::max<long long>(n, 1));
   if (n) {
     CK(cudaMemcpy(off.data(), g->d.off, n * 8, cudaMemcpyDeviceToHost));
     CK(cudaMemcpy(deg.data(), g->d.deg, n * 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(ldeg.data(), g->d.ldeg, n * 4, cudaMemcpyDeviceToHost));
   }
   long long tot = 0;
-  for (long long v = 0; v < n; v++) tot += deg[v];
+  for (long long v = 0; v < n; v++) tot += ldeg[v];
   if (n_total) *n_total = n;
   if (n_slots) *n_slots = tot;
   if (!xadj) return IGK_OK;
   if (xadj_len < n + 1 || adj_len < tot || !adjncy) return fail(g, IGK_EINVAL, "export buffers too small");
   xadj[0] = 0;
   long long pos = 0;
+  std::vector<int32_t> row, roww;
   for (long long v = 0; v < n; v++) {
-    if (deg[v]) {
-      CK(cudaMemcpy(adjncy + pos, g->d.adj + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
-      if (adjwgt) {
-        if (g->d.adjw) {
-          CK(cudaMemcpy(adjwgt + pos, g->d.adjw + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
-        } else {
-          for (int i = 0; i < deg[v]; i++) adjwgt[pos + i] = 1;
-        }
+    if (deg[v]) {  // copy the prefix, drop tombstones (-1)
+      row.resize(deg[v]);
+      roww.assign(deg[v], 1);
+      CK(cudaMemcpy(row.data(), g->d.adj + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
+      if (g->d.adjw) CK(cudaMemcpy(roww.data(), g->d.adjw + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
+      for (int i = 0; i < deg[v]; i++) {
+        if (row[i] < 0) continue;
+        if (pos >= adj_len) return fail(g, IGK_ESTATE, "export: live degree mismatch");
+        adjncy[pos] = row[i];
+        if (adjwgt) adjwgt[pos] = roww[i];
+        pos++;
       }
     }
-    pos += deg[v];
     xadj[v + 1] = pos;
   }
+  if (pos != tot) return fail(g, IGK_ESTATE, "export: live degree mismatch");
   return IGK_OK;
 }
 

@@ -262,3 +262,37 @@ def test_fused_step_api():
             sg, stg, bad = P.G.step(bad_batch)
             assert sg == 1 and bad == 0
             assert (P.G.partition().tobytes(), P.G.cut()) == before
+
+
+def test_c4_full_size_10m():
+    """BASELINE C4 at full size (10M vertices, heavy fanout <= 1e4, k=16, 5%
+    modified per iteration): full partition vectors, cuts and part weights
+    bit-exact for 3 iterations (the oracle needs ~0.7 s per iteration)."""
+    cfg, g, part, P = _cfg_pair("C4", 4, check=False)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(4)))
+    for it in range(3):
+        b = gi.next_batch(S, cfg)
+        assert P.apply(b, f"C4 it{it}") == 0
+        P.refine(f"C4 it{it}")
+        P.compare_state(f"C4 it{it}")
+
+
+def test_c5_full_size_adversarial():
+    """BASELINE C5 at full size (4M vertices, k=8): deletions concentrated in
+    one region; after warm-up the restoration (R3) fires every iteration."""
+    cfg = gi.CONFIGS["C5"]
+    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(5))
+    part, _ = gi.metis_partition(g, cfg["k"])
+    P = Pair(g.xadj, g.adjncy, cfg["k"], cfg["eps"], part, check=False)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(5)), region0=(part == 0).astype(np.int32))
+    evicted = []
+    for it in range(10):
+        b = gi.next_batch(S, cfg)
+        assert P.apply(b, f"C5 it{it}") == 0
+        sto, stg = P.refine(f"C5 it{it}")
+        evicted.append(stg["evicted"])
+        if it % 3 == 2 or it == 9:
+            P.compare_state(f"C5 it{it}")
+    assert sum(e > 0 for e in evicted) >= 3, evicted
