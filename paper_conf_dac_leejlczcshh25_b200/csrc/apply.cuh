@@ -6,9 +6,13 @@
 //       growing prefixes; 32-neighbour work chunks of every vertex deletion
 //   M12 edge deletions and vertex deletions (Alg. 2, both directions,
 //       reading Q12) as tombstones; marks (Alg. 3 L6-7); cut / W deltas
-//   M3  finalize deletions; compact dirty prefixes / copy growing ones to their
-//       new slots; vertex insertions (Alg. 2 L7-10, Alg. 3 L2-5)
-//   M4  edge insertions (Alg. 1) appended to the dense prefixes
+//   M3  finalize deletions; growing prefixes move (compacted) to new slots,
+//       leaving forward marks; vertex insertions (Alg. 2 L7-10, Alg. 3 L2-5)
+//   M4  edge insertions (Alg. 1) appended to the prefixes; twin fix-ups
+// Every slot keeps the slot of its reverse entry ("twin"), so an edge deletion
+// searches only the shorter of the two prefixes and a vertex deletion needs
+// no search at all; hub prefixes (degree up to 10^4) are never scanned.
+// Tombstones (-1) stay in a prefix until it relocates (lazy compaction).
 // Semantics: reading S1.  Differences from the paper's design
 // (DESIGN.md 5): dense-prefix adjacency with slack instead of 32-slot buckets;
 // all updates of a batch are validated first and then applied as set
@@ -97,13 +101,9 @@ __device__ __forceinline__ int block_excl_scan(int v, int* total, int* sbuf) {
   return warp_excl + x - v;
 }
 
-__device__ __forceinline__ void mark_dirty_affected(const Dev& d, int x, uint32_t epT, uint32_t epA) {
-  Ctl* ctl = d.ctl;
-  bool nd = stamp_insert(d.markT, x, epT);
-  int s1 = agg_append(&ctl->ndirty, nd);
-  if (nd) d.dlist[s1] = x;
+__device__ __forceinline__ void mark_affected(const Dev& d, int x, uint32_t epA) {
   bool na = stamp_insert(d.markA, x, epA);
-  int s2 = agg_append(&ctl->nA, na);
+  int s2 = agg_append(&d.ctl->nA, na);
   if (na) d.Alist[s2] = x;
 }
 
@@ -288,42 +288,39 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
   rr_for_warp(B, [&](long long i, bool valid) {
     int4 m = valid ? a.mods[i] : make_int4(-1, 0, 0, 0);
     const bool ed = m.x == kEdgeDel;
-    long long ou = 0, ox = 0;
-    int du = 0, dx = 0;
+    // search the shorter prefix; the twin gives the reverse slot
+    int a0 = m.y, b0 = m.z;
+    long long oa = 0;
+    int da = 0;
     if (ed) {
-      ou = __ldcg(d.off + m.y);
-      du = __ldcg(d.deg + m.y);
-      ox = __ldcg(d.off + m.z);
-      dx = __ldcg(d.deg + m.z);
+      int du = __ldcg(d.deg + m.y), dv = __ldcg(d.deg + m.z);
+      if (dv < du) {
+        a0 = m.z;
+        b0 = m.y;
+      }
+      oa = __ldcg(d.off + a0);
+      da = min(du, dv);
     }
-    long long su = (ed && du <= 32) ? thread_find(d.adj, ou, du, m.z) : -1;
-    long long sx = (ed && dx <= 32) ? thread_find(d.adj, ox, dx, m.y) : -1;
-    unsigned hm = __ballot_sync(0xffffffffu, ed && du > 32);
+    long long sa = (ed && da <= 32) ? thread_find(d.adj, oa, da, b0) : -1;
+    unsigned hm = __ballot_sync(0xffffffffu, ed && da > 32);
     while (hm) {
       int src = __ffs(hm) - 1;
       hm &= hm - 1;
-      long long s = warp_find(d.adj, __shfl_sync(0xffffffffu, ou, src), __shfl_sync(0xffffffffu, du, src),
-                              __shfl_sync(0xffffffffu, m.z, src));
-      if (lane_id() == src) su = s;
-    }
-    hm = __ballot_sync(0xffffffffu, ed && dx > 32);
-    while (hm) {
-      int src = __ffs(hm) - 1;
-      hm &= hm - 1;
-      long long s = warp_find(d.adj, __shfl_sync(0xffffffffu, ox, src), __shfl_sync(0xffffffffu, dx, src),
-                              __shfl_sync(0xffffffffu, m.y, src));
-      if (lane_id() == src) sx = s;
+      long long s = warp_find(d.adj, __shfl_sync(0xffffffffu, oa, src), __shfl_sync(0xffffffffu, da, src),
+                              __shfl_sync(0xffffffffu, b0, src));
+      if (lane_id() == src) sa = s;
     }
     if (ed) {
-      int w = d.adjw ? __ldcg(d.adjw + su) : 1;
-      d.adj[su] = -1;
-      d.adj[sx] = -1;
+      long long sb = __ldcg(d.twin + sa);
+      int w = d.adjw ? __ldcg(d.adjw + sa) : 1;
+      d.adj[sa] = -1;
+      d.adj[sb] = -1;
       atomicSub(d.ldeg + m.y, 1);
       atomicSub(d.ldeg + m.z, 1);
       uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
       if (pu != kPsi && pv != kPsi && pu != pv) cut_acc -= w;
-      mark_dirty_affected(d, m.y, a.epT, a.epA);
-      mark_dirty_affected(d, m.z, a.epT, a.epA);
+      mark_affected(d, m.y, a.epA);
+      mark_affected(d, m.z, a.epA);
     }
   });
   {
@@ -338,26 +335,15 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       int x = j < dg ? __ldcg(d.adj + o + j) : -1;  // -1: tombstone from an edge deletion
       int w = (x >= 0 && d.adjw) ? __ldcg(d.adjw + o + j) : 1;
       bool xdel = x >= 0 && __ldcg(d.markD + x) == a.epD;
-      int dx = (x >= 0 && !xdel) ? __ldcg(d.deg + x) : 0;
-      bool small = x >= 0 && !xdel && dx <= 32;
-      if (small) {
-        long long s = thread_find(d.adj, __ldcg(d.off + x), dx, u);
-        d.adj[s] = -1;
-      }
-      if (x >= 0 && !xdel) atomicSub(d.ldeg + x, 1);
-      unsigned hm = __ballot_sync(0xffffffffu, x >= 0 && !xdel && !small);
-      while (hm) {
-        int src = __ffs(hm) - 1;
-        hm &= hm - 1;
-        int xx = __shfl_sync(0xffffffffu, x, src);
-        long long s = warp_find(d.adj, __ldcg(d.off + xx), __ldcg(d.deg + xx), u);
-        if (lane_id() == 0) d.adj[s] = -1;
+      if (x >= 0 && !xdel) {  // the twin is u's entry in x's prefix
+        d.adj[__ldcg(d.twin + o + j)] = -1;
+        atomicSub(d.ldeg + x, 1);
       }
       if (x >= 0) {
         uint8_t px = ld_part(d.part, x);
         if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < x)) cut_acc -= w;
       }
-      if (x >= 0 && !xdel) mark_dirty_affected(d, x, a.epT, a.epA);
+      if (x >= 0 && !xdel) mark_affected(d, x, a.epA);
       if (ch.y == 0 && lane_id() == 0) {
         int vwu = d.vw ? __ldcg(d.vw + u) : 1;
         if (pu != kPsi) atomic_add_ll(&ctl->Wp[pu], -(long long)vwu);
@@ -391,19 +377,21 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
       d.psi[0][slot] = id;
     }
   });
-  // compact a prefix (dropping tombstones) from `src` into `dst` (may alias)
-  auto compact = [&](int x, long long src, long long dst) {
+  // move a prefix (dropping tombstones) from `src` to the fresh region `dst`;
+  // every moved slot's twin is copied and the old slot's twin becomes a
+  // forward mark -(new slot + 2), resolved in M4
+  auto relocate = [&](int x, long long src, long long dst) {
     const int dg = __ldcg(d.deg + x);
     int wr = 0;
     for (int b = 0; b < dg; b += 128) {  // 4 loads per lane in flight
-      int y[4], w[4];
+      int y[4], w[4], tw[4];
 #pragma unroll
       for (int t = 0; t < 4; t++) {
         int j = b + t * 32 + lane_id();
         y[t] = j < dg ? __ldcg(d.adj + src + j) : -1;
         w[t] = (j < dg && d.adjw) ? __ldcg(d.adjw + src + j) : 0;
+        tw[t] = y[t] >= 0 ? __ldcg(d.twin + src + j) : 0;
       }
-      __syncwarp();
 #pragma unroll
       for (int t = 0; t < 4; t++) {
         unsigned keep = __ballot_sync(0xffffffffu, y[t] >= 0);
@@ -411,10 +399,11 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
           int pos = wr + __popc(keep & ((1u << lane_id()) - 1u));
           d.adj[dst + pos] = y[t];
           if (d.adjw) d.adjw[dst + pos] = w[t];
+          d.twin[dst + pos] = tw[t];
+          d.twin[src + b + t * 32 + lane_id()] = -(int)(dst + pos) - 2;
         }
         wr += __popc(keep);
       }
-      __syncwarp();
     }
     return wr;
   };
@@ -425,25 +414,12 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     long long no = pk >> 24;
     int nc = (int)(pk & 0xffffff);
     int wr = 0;
-    if (x < n0) wr = compact(x, __ldcg(d.off + x), no);
+    if (x < n0) wr = relocate(x, __ldcg(d.off + x), no);
     if (lane_id() == 0) {
       d.off[x] = no;
       d.capv[x] = nc;
       d.deg[x] = wr;
-    }
-  }
-  {
-    const int nd = ldv(&ctl->ndirty);
-    for (long long t = gwarp; t < nd; t += nwarp) {  // in-place compaction of the rest
-      int x = d.dlist[t];
-      if (__ldcg(d.markD + x) == a.epD) continue;
-      if (__ldcg(d.markG + x) == a.epG && __ldcg(d.reloc + x) >= 0) continue;
-      // lazy compaction: tombstones stay until they are more than half the prefix
-      const int dg = __ldcg(d.deg + x), live = __ldcg(d.ldeg + x);
-      if (2 * (dg - live) <= dg) continue;
-      long long o = __ldcg(d.off + x);
-      int wr = compact(x, o, o);
-      if (lane_id() == 0) d.deg[x] = wr;
+      d.icnt[x] = wr;  // moved entries to fix up in M4 (icnt is free again after V2)
     }
   }
   if (tid == 0) {
@@ -463,6 +439,8 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     long long su = __ldcg(d.off + m.y) + pu_pos, sv = __ldcg(d.off + m.z) + pv_pos;
     d.adj[su] = m.z;
     d.adj[sv] = m.y;
+    d.twin[su] = (int)sv;
+    d.twin[sv] = (int)su;
     if (d.adjw) {
       d.adjw[su] = m.w;
       d.adjw[sv] = m.w;
@@ -476,6 +454,24 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
     int s2 = agg_append(&ctl->nA, nb);
     if (nb) d.Alist[s2] = m.z;
   });
+  // twin fix-ups of moved entries: resolve forward marks of moved partners,
+  // then point the partner back at the new slot (idempotent when both moved)
+  for (long long t = gwarp; t < ng; t += nwarp) {
+    int x = d.glist[t];
+    if (d.reloc[x] < 0) continue;
+    const long long o = __ldcg(d.off + x);
+    const int cnt = __ldcg(d.icnt + x);
+    for (int j = lane_id(); j < cnt; j += 32) {
+      long long s = o + j;
+      int tp = __ldcg(d.twin + s);
+      int f = __ldcg(d.twin + tp);
+      if (f < -1) tp = -f - 2;  // the partner moved too
+      d.twin[s] = tp;
+      d.twin[tp] = (int)s;
+    }
+    __syncwarp();
+    if (lane_id() == 0) d.icnt[x] = 0;
+  }
   block_atomic_add(&ctl->cut, cut_acc, s_red);
   block_atomic_add(&ctl->W, W_acc, s_red);
   stamp_phase(ctl, 199);

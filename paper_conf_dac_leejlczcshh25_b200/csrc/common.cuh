@@ -82,7 +82,8 @@ struct Dev {
   int32_t* deg;      // prefix length (live entries + tombstones, -1)
   int32_t* ldeg;     // live degree (tombstones excluded)
   int32_t* capv;     // capacity
-  int32_t* adj;      // neighbour IDs
+  int32_t* adj;      // neighbour IDs (-1 = tombstone)
+  int32_t* twin;     // slot of the reverse entry (x -> u) of every live slot (u -> x)
   int32_t* adjw;     // edge weights (nullptr = unit)
   uint8_t* active;
   int32_t* vw;       // vertex weights (nullptr = unit)

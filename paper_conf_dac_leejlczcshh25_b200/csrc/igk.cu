@@ -266,27 +266,31 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     if (init_part[u] < 0 || init_part[u] >= k) return IGK_EINVAL;
     if (vwgt && (vwgt[u] < 1 || vwgt[u] > kVwMax)) return IGK_EINVAL;
   }
-  {
-    std::vector<std::pair<int32_t, int32_t>> rows((size_t)m2);
-    for (int64_t u = 0; u < n; u++) {
-      for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
-        int32_t x = adjncy[j], w = adjwgt ? adjwgt[j] : 1;
-        if (x < 0 || x >= n || x == u || w < 1 || w > kEwMax) return IGK_EINVAL;
-        rows[j] = {x, w};
-      }
-      std::sort(rows.begin() + xadj[u], rows.begin() + xadj[u + 1]);
-      for (int64_t j = xadj[u] + 1; j < xadj[u + 1]; j++)
-        if (rows[j].first == rows[j - 1].first) return IGK_EINVAL;
+  // rows sorted by neighbour (neighbour, position in row): duplicate check,
+  // symmetry check with equal weights, and the twin of every entry
+  std::vector<std::pair<int32_t, int32_t>> rows((size_t)m2);
+  for (int64_t u = 0; u < n; u++) {
+    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+      int32_t x = adjncy[j], w = adjwgt ? adjwgt[j] : 1;
+      if (x < 0 || x >= n || x == u || w < 1 || w > kEwMax) return IGK_EINVAL;
+      rows[j] = {x, (int32_t)(j - xadj[u])};
     }
-    for (int64_t u = 0; u < n; u++) {
-      for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
-        int32_t x = rows[j].first;
-        auto b = rows.begin() + xadj[x], e = rows.begin() + xadj[x + 1];
-        auto it = std::lower_bound(b, e, std::make_pair((int32_t)u, INT32_MIN));
-        if (it == e || it->first != u || it->second != rows[j].second) return IGK_EINVAL;
-      }
+    std::sort(rows.begin() + xadj[u], rows.begin() + xadj[u + 1]);
+    for (int64_t j = xadj[u] + 1; j < xadj[u + 1]; j++)
+      if (rows[j].first == rows[j - 1].first) return IGK_EINVAL;
+  }
+  std::vector<int32_t> twin_pos((size_t)std::max<long long>(m2, 1));  // position of u in row x
+  for (int64_t u = 0; u < n; u++) {
+    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+      int32_t x = adjncy[j];
+      auto b = rows.begin() + xadj[x], e = rows.begin() + xadj[x + 1];
+      auto it = std::lower_bound(b, e, std::make_pair((int32_t)u, INT32_MIN));
+      if (it == e || it->first != u) return IGK_EINVAL;
+      if (adjwgt && adjwgt[xadj[x] + it->second] != adjwgt[j]) return IGK_EINVAL;
+      twin_pos[j] = it->second;
     }
   }
+  std::vector<std::pair<int32_t, int32_t>>().swap(rows);
   igk_graph* g = new igk_graph();
   g->device = o.device;
   g->stream = (cudaStream_t)o.stream;
@@ -323,13 +327,15 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     used += c;
   }
   d.slot_cap = o.max_slots > 0 ? o.max_slots : 4 * used + (1ll << 22);
+  d.slot_cap = std::min<long long>(d.slot_cap, (1ll << 31) - 2);  // slots are int32 (twin pointers)
   if (d.slot_cap < used) {
     delete g;
     return IGK_EINVAL;
   }
   const size_t N = (size_t)d.n_cap;
   bool ok = dalloc(g, &d.off, N) && dalloc(g, &d.deg, N) && dalloc(g, &d.ldeg, N) && dalloc(g, &d.capv, N) &&
-            dalloc(g, &d.adj, (size_t)d.slot_cap) && (g->ew_unit || dalloc(g, &d.adjw, (size_t)d.slot_cap)) &&
+            dalloc(g, &d.adj, (size_t)d.slot_cap) && dalloc(g, &d.twin, (size_t)d.slot_cap) &&
+            (g->ew_unit || dalloc(g, &d.adjw, (size_t)d.slot_cap)) &&
             dalloc(g, &d.active, N) && (g->vw_unit || dalloc(g, &d.vw, N)) && dalloc(g, &d.part, N) &&
             dalloc(g, &d.markA, N) && dalloc(g, &d.markT, N) && dalloc(g, &d.markD, N) &&
             dalloc(g, &d.markG, N) && dalloc(g, &d.vcnt, N) && dalloc(g, &d.icnt, N) &&
@@ -378,6 +384,13 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     igk_destroy(g);
     return IGK_ENOMEM;
   }
+  std::vector<int32_t> twin_h((size_t)std::max<long long>(used, 1));
+  for (int64_t u = 0; u < n; u++)
+    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+      int32_t x = adjncy[j];
+      twin_h[off[u] + (j - xadj[u])] = (int32_t)(off[x] + twin_pos[j]);
+    }
+  std::vector<int32_t>().swap(twin_pos);
   std::vector<uint8_t> part8((size_t)std::max<int64_t>(n, 1)), act((size_t)std::max<int64_t>(n, 1), 1);
   for (int64_t u = 0; u < n; u++) part8[u] = (uint8_t)init_part[u];
   cudaError_t e = cudaSuccess;
@@ -386,6 +399,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     if (e == cudaSuccess && m2) e = cudaMemcpy(d_adjncy, adjncy, m2 * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess && m2 && d_adjwgt) e = cudaMemcpy(d_adjwgt, adjwgt, m2 * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.off, off.data(), n * 8, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && used) e = cudaMemcpy(d.twin, twin_h.data(), used * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.deg, deg.data(), n * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.ldeg, deg.data(), n * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.capv, capv.data(), n * 4, cudaMemcpyHostToDevice);
