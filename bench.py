@@ -228,10 +228,10 @@ def main():
         ev[i][1].record(stream)
         st = {f: int(getattr(st_buf, f)) for f in igk.STATS}
         ms = G.last_ms()
-        refine_ms += ms["refine"]
+        refine_ms += ms["refine"]  # igk_step: ONE fused kernel (k_step = apply + refine)
         apply_ms += ms["apply"]
         aff += st["affected"]
-        rbytes += refine_bytes(st)
+        rbytes += refine_bytes(st) + 16 * len(b)  # + the batch itself
         stats.append(st)
         gpu_cuts.append(st["cut"])
     torch.cuda.synchronize()
@@ -313,11 +313,11 @@ def main():
                    "l2": "flushed between iterations (256 MiB write)" if flush is not None else "not flushed",
                    "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]]))},
         "gpu_launches": launches,
-        "roofline": {"kernel": "k_refine", "bound": "hbm", "achieved": achieved, "peak": peak,
+        "roofline": {"kernel": "k_step (apply+refine fused)", "bound": "hbm", "achieved": achieved, "peak": peak,
                      "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
                      "bytes_per_launch": rbytes / K, "launch_ms": refine_ms / K,
                      "share_of_step": refine_ms / t_ms if t_ms else None},
-        "kernel_ms": {"k_apply": apply_ms / K, "k_refine": refine_ms / K},
+        "kernel_ms": {"k_step": refine_ms / K},
         "iteration": {"affected": aff / K, "rounds": float(np.mean([s["rounds"] for s in stats])),
                       "moves": float(np.mean([s["moves_applied"] for s in stats])),
                       "evicted": float(np.mean([s["evicted"] for s in stats])),

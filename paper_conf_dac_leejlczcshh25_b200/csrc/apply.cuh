@@ -107,10 +107,16 @@ __device__ __forceinline__ void mark_affected(const Dev& d, int x, uint32_t epA)
   if (na) d.Alist[s2] = x;
 }
 
-__global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
-  cg::grid_group grid = cg::this_grid();
-  __shared__ int s_scan[64];
-  __shared__ long long s_red[32];
+struct ApplySmem {
+  int scan[64];
+  long long red[32];
+  long long ins[2];
+};
+
+// the whole apply; returns false (uniformly) if the batch was rejected
+__device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg::grid_group& grid, ApplySmem& sm) {
+  int* s_scan = sm.scan;
+  long long* s_red = sm.red;
   Ctl* ctl = d.ctl;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long nthr = (long long)gridDim.x * blockDim.x;
@@ -164,7 +170,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
   GRID_SYNC_STAMPED(ctl, 101);
 
   // ---- V2: validate against the pre-batch state; new IDs; allocate ---------
-  __shared__ long long s_ins[2];
+  long long* s_ins = sm.ins;
   if (warp_id() == 0) {  // one warp sums the per-CTA counts
     long long t = 0, m = 0;
     for (int b = lane_id(); b < (int)gridDim.x; b += 32) {
@@ -278,7 +284,7 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
   }
   if (failed) {  // uniform: every CTA read the same error words
     if (tid == 0) ctl->slab_top = ctl->slab_top0;
-    return;
+    return false;
   }
 
   // ---- M12: edge deletions and vertex deletions (tombstones) ---------------
@@ -475,6 +481,13 @@ __global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
   block_atomic_add(&ctl->cut, cut_acc, s_red);
   block_atomic_add(&ctl->W, W_acc, s_red);
   stamp_phase(ctl, 199);
+  return true;
+}
+
+__global__ void __launch_bounds__(kThreads) k_apply(Dev d, ApplyArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ ApplySmem sm;
+  apply_body(d, a, grid, sm);
 }
 
 }  // namespace igk

@@ -17,6 +17,7 @@
 #include "apply.cuh"
 #include "common.cuh"
 #include "refine.cuh"
+#include "step.cuh"
 
 using namespace igk;
 
@@ -157,7 +158,7 @@ struct igk_graph {
   uint32_t epoch = 1;   // last stamp value handed out
   uint32_t epochA = 0;  // stamp of the current affected set
   int grid_apply = 0, grid_refine = 0;
-  size_t smem_refine = 0;
+  size_t smem_refine = 0, smem_step = 0;
   long long launches = 0;
   igk_modifier* h_stage = nullptr;  // pinned staging for host batches
   long long h_stage_cap = 0;
@@ -454,17 +455,23 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   }
   // persistent grids
   g->smem_refine = sizeof(RefSmem);
+  g->smem_step = sizeof(StepSmem);
   cudaFuncSetAttribute(k_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
+  cudaFuncSetAttribute(k_step, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_step);
   g->grid_apply = coop_grid((const void*)k_apply, 0, o.blocks_per_sm);
   g->grid_refine = coop_grid((const void*)k_refine, g->smem_refine, o.blocks_per_sm);
+  g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_step, g->smem_step, o.blocks_per_sm));
   if (g->grid_apply > 4096) g->grid_apply = 4096;
   g->epochA = next_epoch(g);
   *out = g;
   return IGK_OK;
 }
 
-// capacity checks + launch of k_apply (no host synchronisation)
-static igk_status launch_apply(igk_graph* g, const int4* dm, int64_t count) {
+static ApplyArgs make_apply_args(igk_graph* g, const int4* dm, int64_t count);
+static RefineArgs make_refine_args(igk_graph* g, int after_apply);
+
+// capacity of the per-batch scratch (hash, new IDs)
+static igk_status prepare_apply(igk_graph* g, int64_t count) {
   // duplicate-detection hash: >= 2 * count slots, power of two
   long long need = 64;
   while (need < 2 * count + 2) need <<= 1;
@@ -487,16 +494,14 @@ static igk_status launch_apply(igk_graph* g, const int4* dm, int64_t count) {
     g->newid_cap = count;
   }
   g->d.hmask = g->hash_cap - 1;
-  ApplyArgs a;
-  a.mods = dm;
-  a.B = count;
-  a.n0 = g->h_ctl->n_total;
-  a.epD = next_epoch(g);
-  a.epT = next_epoch(g);
-  a.epG = next_epoch(g);
-  a.epA = g->epochA;
-  a.vw_unit = g->vw_unit;
-  a.ew_unit = g->ew_unit;
+  return IGK_OK;
+}
+
+// launch of k_apply alone (no host synchronisation)
+static igk_status launch_apply(igk_graph* g, const int4* dm, int64_t count) {
+  igk_status st = prepare_apply(g, count);
+  if (st != IGK_OK) return st;
+  ApplyArgs a = make_apply_args(g, dm, count);
   void* args[] = {(void*)&g->d, (void*)&a};
   CK(cudaEventRecord(g->ev[2], g->stream));
   CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply, kThreads, args, 0, g->stream));
@@ -518,7 +523,21 @@ static igk_status finish_apply(igk_graph* g, int64_t* bad_index) {
   return IGK_OK;
 }
 
-static igk_status launch_refine(igk_graph* g, int after_apply) {
+static ApplyArgs make_apply_args(igk_graph* g, const int4* dm, int64_t count) {
+  ApplyArgs a;
+  a.mods = dm;
+  a.B = count;
+  a.n0 = g->h_ctl->n_total;
+  a.epD = next_epoch(g);
+  a.epT = next_epoch(g);
+  a.epG = next_epoch(g);
+  a.epA = g->epochA;
+  a.vw_unit = g->vw_unit;
+  a.ew_unit = g->ew_unit;
+  return a;
+}
+
+static RefineArgs make_refine_args(igk_graph* g, int after_apply) {
   RefineArgs a;
   a.e_ppm = g->e_ppm;
   a.epC1 = next_epoch(g);
@@ -526,6 +545,11 @@ static igk_status launch_refine(igk_graph* g, int after_apply) {
   a.epC2 = next_epoch(g);
   a.epF = next_epoch(g);
   a.after_apply = after_apply;
+  return a;
+}
+
+static igk_status launch_refine(igk_graph* g, int after_apply) {
+  RefineArgs a = make_refine_args(g, after_apply);
   void* args[] = {(void*)&g->d, (void*)&a};
   CK(cudaEventRecord(g->ev[0], g->stream));
   CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
@@ -548,22 +572,39 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
 }
 
 // fused step: apply + refine launched back to back, one host synchronisation
+static igk_status prepare_apply(igk_graph* g, int64_t count);
+
 static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refine_stats* stats,
                            int64_t* first_new_id, int64_t* bad_index) {
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   igk_status st;
-  if (count > 0) {
-    st = launch_apply(g, dm, count);
+  if (count == 0) {
+    st = launch_refine(g, 0);
     if (st != IGK_OK) return st;
+  } else {  // apply + refine in ONE persistent launch (k_step)
+    st = prepare_apply(g, count);
+    if (st != IGK_OK) return st;
+    ApplyArgs aa = make_apply_args(g, dm, count);
+    RefineArgs ra = make_refine_args(g, 1);
+    void* args[] = {(void*)&g->d, (void*)&aa, (void*)&ra};
+    CK(cudaEventRecord(g->ev[0], g->stream));
+    CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
+    g->launches++;
+    CK(cudaEventRecord(g->ev[1], g->stream));
+    g->h_ctl->refine_skipped = 0;
   }
-  st = launch_refine(g, count > 0);
-  if (st != IGK_OK) return st;
   st = sync_ctl(g, 1);
   if (st != IGK_OK) return st;
   if (count > 0) {
-    st = finish_apply(g, bad_index);
-    if (st != IGK_OK) return st;  // the refine kernel exited without touching the state
+    g->ms_apply = 0;  // fused: the whole step is in ms_refine
+    if (g->h_ctl->err_idx != kNoErr) {
+      if (bad_index) *bad_index = g->h_ctl->err_idx;
+      char buf[128];
+      snprintf(buf, sizeof buf, "invalid modifier at index %lld", g->h_ctl->err_idx);
+      return fail(g, IGK_EINVAL, buf);  // the kernel ended before the refine: state unchanged
+    }
+    if (g->h_ctl->err_nomem) return fail(g, IGK_ENOMEM, "vertex or slot capacity exhausted");
   }
   return finish_refine(g, stats);
 }

@@ -414,10 +414,7 @@ __device__ __forceinline__ bool better(long long ca, int pa, long long cb, int p
   return pa < pb;
 }
 
-__global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
-  cg::grid_group grid = cg::this_grid();
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  RefSmem& s = *reinterpret_cast<RefSmem*>(smem_raw);
+__device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s) {
   Ctl* ctl = d.ctl;
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -923,6 +920,12 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
     ctl->npsi[1] = 0;
     ctl->npsi[2] = 0;
   }
+}
+
+__global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  refine_body(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw));
 }
 
 }  // namespace igk
