@@ -33,6 +33,7 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+import benchdist  # noqa: E402
 import igk_inputs as gi  # noqa: E402
 
 METRIC = "ms per incremental iteration & affected vertices/s; cut vs full repartition"
@@ -62,7 +63,7 @@ def workload(args, rank):
     n = args.n or cfg["n"]
     k = args.k or (cfg["k"] if isinstance(cfg["k"], int) else cfg["k"][0])
     frac = args.frac or (cfg.get("frac") if not isinstance(cfg.get("frac"), tuple) else cfg["frac"][2])
-    gseed = gi.graph_seed(idx) + 1000 * rank  # rank 0 = the canonical instance
+    gseed = benchdist.rank_graph_seed(idx, rank)  # rank 0 = the canonical instance
     g = gi.make_graph(n, cfg["fmax"], gseed)
     part, metis_cut = gi.metis_partition(g, k)
     region0 = (part == 0).astype(np.int32) if cfg["mode"] == gi.MODE_ADVERSARIAL else None
@@ -184,9 +185,7 @@ def run_reference(args, rank, world):
 
 def main():
     args = parse()
-    rank = int(os.environ.get("RANK", 0))
-    world = int(os.environ.get("WORLD_SIZE", 1))
-    local = int(os.environ.get("LOCAL_RANK", 0))
+    rank, world, local = benchdist.env_ranks()
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
@@ -240,14 +239,7 @@ def main():
     clocks = clk.stop()
     launches = G.kernel_launches() - l0
     t_ms = sum(a.elapsed_time(b) for a, b in ev)
-    if dist:
-        tt = torch.tensor([t_ms], device="cuda", dtype=torch.float64)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ta = torch.tensor([float(aff)], device="cuda", dtype=torch.float64)
-        dist.all_reduce(ta, op=dist.ReduceOp.SUM)
-        t_ms, aff_all = tt.item(), ta.item()
-    else:
-        aff_all = aff
+    t_ms, aff_all = benchdist.reduce_time_and_work(t_ms, aff, dist, "cuda")
     value = aff_all / (t_ms / 1e3)
 
     # ---- e2e: public C ABI with HOST batches; H2D + D2H inside the timed region
@@ -265,12 +257,7 @@ def main():
         e1.record(stream)
         torch.cuda.synchronize()
         te = e0.elapsed_time(e1)
-        if dist:
-            tt = torch.tensor([te], device="cuda", dtype=torch.float64)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            ta = torch.tensor([float(aff_e)], device="cuda", dtype=torch.float64)
-            dist.all_reduce(ta, op=dist.ReduceOp.SUM)
-            te, aff_e = tt.item(), ta.item()
+        te, aff_e = benchdist.reduce_time_and_work(te, aff_e, dist, "cuda")
         e2e = {"value": aff_e / (te / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": int(np.mean([b.nbytes for b in h_batches])),
                "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches)}
