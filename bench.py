@@ -289,7 +289,7 @@ def main():
     traffic = None
     try:
         tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        traffic = tj.get(args.config, {}).get("k_refine")
+        traffic = tj.get(args.config, {}).get("k_step")
     except Exception:
         pass
     line = {
