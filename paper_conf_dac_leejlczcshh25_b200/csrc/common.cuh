@@ -111,6 +111,7 @@ struct Dev {
   // per-vertex move results (rounds)
   uint8_t* tgt;
   int32_t* gain;
+  int32_t* pw;       // placed-neighbour weight at round start (cut delta of a placement)
   uint32_t* meta;    // per psi index: bit31 selected | d0 << 8 | p*
   // selection histograms
   long long* hist0;  // [256][256] digit-0 weights per part

@@ -344,7 +344,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.psi[2], N) && dalloc(g, &d.cand, N) && dalloc(g, &d.cand2, N) &&
             dalloc(g, &d.vdch, N + (size_t)(d.slot_cap / 32) + 1024) && dalloc(g, &d.markF, N) && dalloc(g, &d.oldp, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
             dalloc(g, &d.dlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
-            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.meta, N) &&
+            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
             dalloc(g, &g->d_red, 259);
@@ -544,6 +544,7 @@ static RefineArgs make_refine_args(igk_graph* g, int after_apply) {
   a.epN = next_epoch(g);
   a.epC2 = next_epoch(g);
   a.epF = next_epoch(g);
+  a.epE = next_epoch(g);
   a.after_apply = after_apply;
   return a;
 }

@@ -10,7 +10,10 @@
 //       gain = selection (no smaller-ID pseudo neighbour) + best part in one
 //       adjacency pass, O(deg + k) | balanced prefix = weighted radix select of
 //       the first violating move in (#nbr desc, ID asc) order | apply
-//   FD  cut delta over the frontier F (every vertex that went through Psi)
+// The cut is kept exact inside the same phases: a commit subtracts the cut
+// edges of its candidates (read on the snapshot via candidate stamps + saved
+// labels, edges between two candidates once), a placement adds its placed-
+// neighbour weight minus its gain (the selected set is independent).
 // The paper's sort + k x M segmented scan is replaced by a select
 // that yields the same prefix without sorting.
 #pragma once
@@ -20,7 +23,7 @@ namespace igk {
 
 struct RefineArgs {
   long long e_ppm;
-  uint32_t epC1, epN, epC2, epF;
+  uint32_t epC1, epN, epC2, epF, epE;
   int after_apply;  // fused step: skip (leave the state untouched) if the batch was rejected
 };
 
@@ -54,10 +57,14 @@ __device__ __forceinline__ void nbrs_thread(const Dev& d, int u, F f) {
 // (stamp epN).  All stamp probes / exchanges of a chunk are in flight
 // together and N is appended with one atomic per lane and chunk.
 template <int C>
-__device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uint8_t* q, uint32_t epN) {
+__device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uint8_t* q, uint32_t epN,
+                                           uint32_t epC) {
   bool want[C];
 #pragma unroll
-  for (int t = 0; t < C; t++) want[t] = x[t] >= 0 && q[t] != kPsi && __ldcg(d.markT + x[t]) != epN;
+  for (int t = 0; t < C; t++) {
+    unsigned mk = x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN;
+    want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC;  // C1 members are pseudo on sigma2
+  }
   unsigned old[C];
 #pragma unroll
   for (int t = 0; t < C; t++) old[t] = want[t] ? atomicExch(d.markT + x[t], epN) : epN;
@@ -69,7 +76,7 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
   for (int t = 0; t < C; t++)
     if (old[t] != epN) d.Nlist[slot++] = x[t];
 }
-__device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN) {
+__device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN, uint32_t epC) {
   const long long o = __ldg(d.off + u);
   const int dg = __ldg(d.deg + u);
   for (int i = 0; i < dg; i += kTC) {
@@ -79,10 +86,10 @@ __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t e
     for (int t = 0; t < kTC; t++) x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
 #pragma unroll
     for (int t = 0; t < kTC; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
-    mark_chunk<kTC>(d, x, q, epN);
+    mark_chunk<kTC>(d, x, q, epN, epC);
   }
 }
-__device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN) {
+__device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN, uint32_t epC) {
   const long long o = __ldg(d.off + u);
   const int dg = __ldg(d.deg + u);
   for (int b = 0; b < dg; b += 256) {
@@ -95,7 +102,7 @@ __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN
     }
 #pragma unroll
     for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
-    mark_chunk<8>(d, x, q, epN);
+    mark_chunk<8>(d, x, q, epN, epC);
   }
 }
 // warp: lane-strided, 8 entries per lane per round trip (256 per warp)
@@ -144,6 +151,44 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
       wf(uu, r0 + (long long)src * nw + gw);
     }
   }
+}
+
+// Scoped variants: kBlock = true restricts the work to the calling CTA (used
+// by CTA 0 alone for the last, small rounds; barriers become __syncthreads).
+template <bool kBlock, class Get, class TF, class WF>
+__device__ __forceinline__ void foreach_vertex_s(const Dev& d, long long n, Get get, TF tf, WF wf) {
+  if (!kBlock) {
+    foreach_vertex(d, n, get, tf, wf);
+    return;
+  }
+  const long long nw = blockDim.x >> 5, gw = threadIdx.x >> 5;
+  for (long long r0 = 0; r0 < n; r0 += nw * 32) {
+    long long i = r0 + (long long)lane_id() * nw + gw;
+    int u = i < n ? get(i) : -1;
+    int dg = u >= 0 ? __ldg(d.deg + u) : 0;
+    bool heavy = dg > kThreadDeg;
+    if (u >= 0 && !heavy) tf(u, i);
+    unsigned hm = __ballot_sync(0xffffffffu, heavy);
+    while (hm) {
+      int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      int uu = __shfl_sync(0xffffffffu, u, src);
+      wf(uu, r0 + (long long)src * nw + gw);
+    }
+  }
+}
+template <bool kBlock, class F>
+__device__ __forceinline__ void rr_for_s(long long n, F f) {
+  if (!kBlock) {
+    rr_for(n, f);
+    return;
+  }
+  for (long long i = threadIdx.x; i < n; i += blockDim.x) f(i);
+}
+template <bool kBlock>
+__device__ __forceinline__ void scope_sync(cg::grid_group& grid) {
+  if (kBlock) __syncthreads();
+  else grid.sync();
 }
 
 // ---------------------------------------------------------------------------
@@ -243,15 +288,14 @@ __device__ void sel_digit0(const Dev& d, SelSmem& sm, ExactFn is_exact, int exac
   __syncthreads();
 }
 
-template <class Items>
+template <bool kBlock, class Items>
 __device__ void sel_accumulate(const Dev& d, SelSmem& sm, int pass, long long nitems, Items items) {
   long long* hb = d.histR + (long long)(pass % 3) * 256 * kDigits;
   long long* hz = d.histR + (long long)((pass + 1) % 3) * 256 * kDigits;
-  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  const long long nthr = (long long)gridDim.x * blockDim.x;
-  for (long long t = tid; t < (long long)d.k * kDigits; t += nthr)
+  rr_for_s<kBlock>((long long)d.k * kDigits, [&](long long t) {
     if (sm.active[t / kDigits]) hz[t] = 0;
-  rr_for(nitems, [&](long long j) {
+  });
+  rr_for_s<kBlock>(nitems, [&](long long j) {
     int p, d0;
     unsigned long long R;
     long long w;
@@ -289,32 +333,31 @@ __device__ void sel_choose(const Dev& d, SelSmem& sm, int pass) {
   __syncthreads();
 }
 
-template <class ExactFn, class Items>
+template <bool kBlock = false, class ExactFn, class Items>
 __device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid, ExactFn is_exact,
                                 int exact_shift, long long nitems, Items items) {
   sel_digit0(d, sm, is_exact, exact_shift);
   int pass = 0;
   while (sm.nactive > 0) {
-    sel_accumulate(d, sm, pass, nitems, items);
-    arrive_stamp(d.dbg, 300 + pass - 200);
-    grid.sync();
+    sel_accumulate<kBlock>(d, sm, pass, nitems, items);
+    if (!kBlock) arrive_stamp(d.dbg, 300 + pass - 200);
+    scope_sync<kBlock>(grid);
     stamp_phase(d.ctl, 300 + pass);
     sel_choose(d, sm, pass);
     pass++;
   }
-  if (pass > 0) grid.sync();  // every CTA finished reading before anyone clears
+  if (pass > 0) scope_sync<kBlock>(grid);  // every CTA finished reading before anyone clears
 }
 
+template <bool kBlock = false>
 __device__ void sel_clear(const Dev& d, const SelSmem& sm) {
-  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  const long long nthr = (long long)gridDim.x * blockDim.x;
-  for (long long t = tid; t < (long long)d.k * kDigits; t += nthr) {
-    if (!sm.used[t / kDigits]) continue;
+  rr_for_s<kBlock>((long long)d.k * kDigits, [&](long long t) {
+    if (!sm.used[t / kDigits]) return;
     d.hist0[t] = 0;
     d.histR[t] = 0;
     d.histR[256 * kDigits + t] = 0;
     d.histR[2 * 256 * kDigits + t] = 0;
-  }
+  });
 }
 
 // ---------------------------------------------------------------------------
@@ -341,8 +384,8 @@ __device__ __forceinline__ void flush_acc(RefSmem& s, long long* dst, int k) {
 // filter (Alg. 3 L8-24): candidates = listed placed vertices with ext > int;
 // pseudo neighbours count as external (Q13); strict > (Q2)
 template <class Get>
-__device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, long long& scanned,
-                            long long& counted) {
+__device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, uint32_t ep,
+                            long long& scanned, long long& counted) {
   auto tf = [&](int u, long long) {
     if (!__ldcg(d.active + u)) return;
     const uint8_t pu = ld_part(d.part, u);
@@ -355,6 +398,10 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     });
     scanned += __ldg(d.deg + u);
     bool c = ex > in;
+    if (c) {  // stamp + snapshot label: the commit reads it while labels change
+      d.markT[u] = ep;
+      d.oldp[u] = pu;
+    }
     int slot = agg_append(ncand, c);
     if (c) cand[slot] = u;
   };
@@ -371,39 +418,103 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     if (lane_id() == 0) {
       counted++;
       scanned += __ldg(d.deg + u);
-      if (ex > in) cand[atomicAdd(ncand, 1)] = u;
+      if (ex > in) {
+        d.markT[u] = ep;
+        d.oldp[u] = pu;
+        cand[atomicAdd(ncand, 1)] = u;
+      }
     }
   };
   foreach_vertex(d, n, get, tf, wf);
 }
 
-// deferred commit to the pseudo-partition (Alg. 3 L25-26): W_p, label, the
-// frontier list F; with `expand`, also mark the placed neighbours (R2)
-__device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, const int32_t* cand, bool expand,
-                       long long& scanned) {
+// deferred commit to the pseudo-partition (Alg. 3 L25-26) of the candidates
+// stamped `ep`: W_p, label, frontier list, and the exact cut delta.  A
+// neighbour's snapshot label is its saved label if it is a candidate (its
+// current label may already be psi), else its current label.  With `expand`,
+// the placed-on-sigma2 neighbours are marked for R2.
+__device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, const int32_t* cand, uint32_t ep,
+                       bool expand, long long& scanned, long long& cut_acc) {
   Ctl* ctl = d.ctl;
-  rr_for(nc, [&](long long i) {
-    int u = __ldcg(cand + i);
-    uint8_t pu = ld_part(d.part, u);
-    d.oldp[u] = pu;
-    d.markF[u] = a.epF;
+  auto finish = [&](int u, uint8_t pu) {
     acc_add(s.acc, pu, -(long long)vert_w(d.vw, u));
     d.part[u] = kPsi;
     int slot = agg_append(&ctl->npsi[0], true);
     d.psi[0][slot] = u;
-  });
-  if (!expand) return;
-  // labels read here may still show a C1 vertex as placed (written in this
-  // phase): such N entries are pseudo by the R2 filter and skipped there
-  auto mark_t = [&](int u, long long) {
-    scanned += __ldg(d.deg + u);
-    mark_nbrs_thread(d, u, a.epN);
   };
-  auto mark_w = [&](int u, long long) {
-    if (lane_id() == 0) scanned += __ldg(d.deg + u);
-    mark_nbrs_warp(d, u, a.epN);
+  auto tf = [&](int u, long long) {
+    const uint8_t pu = __ldcg(d.oldp + u);
+    const long long o = __ldg(d.off + u);
+    const int dg = __ldg(d.deg + u);
+    scanned += dg;
+    long long del = 0;
+    for (int i = 0; i < dg; i += kTC) {
+      int x[kTC], w[kTC];
+      uint8_t q[kTC];
+      unsigned mk[kTC];
+#pragma unroll
+      for (int t = 0; t < kTC; t++) {
+        x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
+        w[t] = (i + t < dg && d.adjw) ? __ldg(d.adjw + o + i + t) : 1;
+      }
+      uint8_t op[kTC];
+#pragma unroll
+      for (int t = 0; t < kTC; t++) {  // label, stamp and saved label in one round trip
+        q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+        mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
+        op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+      }
+#pragma unroll
+      for (int t = 0; t < kTC; t++) {
+        if (x[t] < 0) continue;
+        const bool xc = mk[t] == ep;
+        const uint8_t qx = xc ? op[t] : q[t];
+        if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
+      }
+      if (expand) mark_chunk<kTC>(d, x, q, a.epN, ep);
+    }
+    cut_acc -= del;
+    finish(u, pu);
   };
-  foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, mark_t, mark_w);
+  auto wf = [&](int u, long long) {
+    const uint8_t pu = __ldcg(d.oldp + u);
+    const long long o = __ldg(d.off + u);
+    const int dg = __ldg(d.deg + u);
+    if (lane_id() == 0) scanned += dg;
+    long long del = 0;
+    for (int b = 0; b < dg; b += 256) {
+      int x[8], w[8];
+      uint8_t q[8];
+      unsigned mk[8];
+#pragma unroll
+      for (int t = 0; t < 8; t++) {
+        int i = b + t * 32 + lane_id();
+        x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
+        w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+      }
+      uint8_t op[8];
+#pragma unroll
+      for (int t = 0; t < 8; t++) {
+        q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+        mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
+        op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+      }
+#pragma unroll
+      for (int t = 0; t < 8; t++) {
+        if (x[t] < 0) continue;
+        const bool xc = mk[t] == ep;
+        const uint8_t qx = xc ? op[t] : q[t];
+        if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
+      }
+      if (expand) mark_chunk<8>(d, x, q, a.epN, ep);
+    }
+    del = warp_sum(del);
+    if (lane_id() == 0) {
+      cut_acc -= del;
+      finish(u, pu);
+    }
+  };
+  foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, tf, wf);
 }
 
 // better(a, b) on (conn desc, W_p asc, p asc)  (reading Q6)
@@ -412,6 +523,281 @@ __device__ __forceinline__ bool better(long long ca, int pa, long long cb, int p
   if (ca != cb) return ca > cb;
   if (Wr[pa] != Wr[pb]) return Wr[pa] < Wr[pb];
   return pa < pb;
+}
+
+// ---------------------------------------------------------------------------
+// R4 rounds (Alg. 4) until the pseudo-partition is empty.
+// kBlock = false: all CTAs with grid barriers (the only mode in use);
+// kBlock = true: the calling CTA alone with __syncthreads barriers.
+// ---------------------------------------------------------------------------
+constexpr int kSmallPsi = 0;  // > 0: hand tails of <= kSmallPsi pending vertices to kBlock mode
+struct RoundState {
+  int cur = 0;
+  long long rounds = 0, rounds_all = 0, applied_tot = 0, deferred_tot = 0;
+};
+template <bool kBlock>
+__device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long long c, int exact_shift_id,
+                           RoundState& rs, long long& scanned, long long& cut_acc) {
+  Ctl* ctl = d.ctl;
+  const int k = d.k;
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  int& cur = rs.cur;
+  long long& rounds = rs.rounds;
+  long long& rounds_all = rs.rounds_all;
+  long long& applied_tot = rs.applied_tot;
+  long long& deferred_tot = rs.deferred_tot;
+  auto round_sync = [&](int id) {
+    if (!kBlock) arrive_stamp(d.dbg, id % 100);
+    scope_sync<kBlock>(grid);
+    stamp_phase(ctl, kBlock ? id + 20 : id);
+  };
+  while (true) {
+    const int np = ldv(&ctl->npsi[cur]);
+    if (np == 0 || (!kBlock && np <= kSmallPsi)) break;
+    const int nxt = cur == 1 ? 2 : 1;
+    const int32_t* plist = d.psi[cur];
+    int32_t* pnext = d.psi[nxt];
+    const int r3 = (int)(rounds_all % 3), r3n = (int)((rounds_all + 1) % 3);
+    // round-start snapshot of W_p (Q14) and the lightest part (zero-conn choice)
+    for (int p = threadIdx.x; p < k; p += blockDim.x) s.Wr[p] = ldv(&ctl->Wp[p]);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int b = 0;
+      for (int p = 1; p < k; p++)
+        if (s.Wr[p] < s.Wr[b]) b = p;
+      s.best0 = b;
+    }
+    __syncthreads();
+    if (tid == 0) {
+      ctl->npsi[nxt] = 0;
+      ctl->applied3[r3n] = 0;
+      ctl->selected3[r3n] = 0;
+    }
+    rr_for_s<kBlock>(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
+    // -- gain: selection + best part, one adjacency pass per vertex
+    long long sel_cnt = 0;
+    auto emit_move = [&](long long j, int u, int best, long long g, long long pwv, bool imbal) {
+      int d0 = 255 - (int)min(g, 255ll);
+      d.tgt[u] = (uint8_t)best;
+      d.gain[u] = (int)g;
+      d.pw[u] = (int)pwv;
+      d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;
+      long long w = vert_w(d.vw, u);
+      atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
+      atomic_add_ll(&ctl->tot3[r3][best], w);
+      if (imbal) ctl->st[ST_IMBAL] = 1;
+    };
+    auto get = [&](long long i) {
+      int u = __ldcg(plist + i);
+      if (u < 0 || !__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
+        d.meta[i] = 0;
+        return -1;
+      }
+      return u;
+    };
+    auto tf = [&](int u, long long j) {
+      const long long vwu = vert_w(d.vw, u);
+      scanned += __ldg(d.deg + u);
+      int qs[kThreadDeg];
+      int ws[kThreadDeg];
+      int m = 0;
+      bool sel = true;
+      long long pwv = 0;
+      nbrs_thread(d, u, [&](int x, int w, uint8_t q) {
+        if (q == kPsi) {
+          if (x < u) sel = false;  // a smaller-ID pseudo neighbour moves first (Alg. 4 L8)
+          return sel;
+        }
+        qs[m] = q;
+        ws[m] = w;
+        m++;
+        pwv += w;
+        return true;
+      });
+      if (!sel) {
+        d.meta[j] = 0;
+        return;
+      }
+      int best = -1;
+      long long bc = -1;
+      for (int i = 0; i < m; i++) {
+        int p = qs[i];
+        bool seen = false;
+        for (int t = 0; t < i; t++) seen |= qs[t] == p;
+        if (seen) continue;
+        long long cc = 0;
+        for (int t = i; t < m; t++) cc += qs[t] == p ? ws[t] : 0;
+        if (s.Wr[p] + vwu > c) continue;
+        if (better(cc, p, bc, best, s.Wr)) {
+          best = p;
+          bc = cc;
+        }
+      }
+      bool imbal = false;
+      if (best < 0) {  // lightest part: eligible => zero connectivity; else fallback (Q8)
+        best = s.best0;
+        bc = 0;
+        if (s.Wr[best] + vwu > c) {
+          imbal = true;
+          for (int t = 0; t < m; t++) bc += qs[t] == best ? ws[t] : 0;
+        }
+      }
+      sel_cnt++;
+      emit_move(j, u, best, bc, pwv, imbal);
+    };
+    auto wf = [&](int u, long long j) {
+      const long long vwu = vert_w(d.vw, u);
+      int* wc = s.wconn[warp_id()];
+      if (lane_id() == 0) scanned += __ldg(d.deg + u);
+      bool lb = false;
+      long long pwv = 0;
+      nbrs_warp(d, u, [&](int x, int w, uint8_t q) {
+        if (q == kPsi) {
+          lb |= x < u;
+        } else {
+          atomicAdd(wc + q, w);
+          pwv += w;
+        }
+      });
+      const bool blocked = __any_sync(0xffffffffu, lb);
+      pwv = warp_sum(pwv);
+      __syncwarp();
+      long long bc = -1;
+      int best = -1;
+      if (!blocked) {
+        for (int p = lane_id(); p < k; p += 32) {
+          if (s.Wr[p] + vwu > c) continue;
+          long long cc = wc[p];
+          if (better(cc, p, bc, best, s.Wr)) {
+            best = p;
+            bc = cc;
+          }
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) {
+          long long oc = __shfl_xor_sync(0xffffffffu, bc, off);
+          int op = __shfl_xor_sync(0xffffffffu, best, off);
+          if (op >= 0 && better(oc, op, bc, best, s.Wr)) {
+            bc = oc;
+            best = op;
+          }
+        }
+      }
+      bool imbal = false;
+      if (!blocked && best < 0) {
+        best = s.best0;
+        bc = wc[best];
+        imbal = true;
+      }
+      __syncwarp();
+      for (int p = lane_id(); p < k; p += 32) wc[p] = 0;
+      __syncwarp();
+      if (lane_id() == 0) {
+        if (blocked) {
+          d.meta[j] = 0;
+        } else {
+          sel_cnt++;
+          emit_move(j, u, best, bc, pwv, imbal);
+        }
+      }
+    };
+    foreach_vertex_s<kBlock>(d, np, get, tf, wf);
+    {
+      long long sc = warp_sum(sel_cnt);
+      if (lane_id() == 0 && sc) atomicAdd(&ctl->selected3[r3], (int)sc);
+    }
+    round_sync(208);
+
+    // -- balanced prefix: T_p = c - W_p + 1; K* = min over parts of the first
+    //    move whose running weight in (#nbr desc, ID asc) order exceeds c.
+    for (int p = threadIdx.x; p < k; p += blockDim.x) {
+      long long T = c - s.Wr[p] + 1;
+      s.sel.T[p] = T;
+      s.sel.used[p] = ldv(&ctl->tot3[r3][p]) >= T;
+    }
+    __syncthreads();
+    auto items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
+      unsigned m = __ldcg(d.meta + j);
+      if (!(m & 0x80000000u)) return false;
+      int u = __ldcg(plist + j);
+      p = (int)(m & 255u);
+      d0 = (int)((m >> 8) & 255u);
+      R = d0 ? (unsigned long long)u
+             : (((unsigned long long)(0x7fffffffu - (unsigned)__ldcg(d.gain + u))) << 32) | (unsigned)u;
+      w = vert_w(d.vw, u);
+      return true;
+    };
+    weighted_select<kBlock>(d, s.sel, grid, [](int d0) { return d0 != 0; }, exact_shift_id, np, items);
+    int kd = 1 << 30;
+    unsigned long long kr = ~0ull;
+    for (int p = 0; p < k; p++) {
+      if (s.sel.used[p] && s.sel.found[p] && key_less(s.sel.d0[p], s.sel.prefix[p], kd, kr)) {
+        kd = s.sel.d0[p];
+        kr = s.sel.prefix[p];
+      }
+    }
+    // -- apply the prefix (moves with key < K*); the rest stay pseudo
+    long long app = 0;
+    rr_for_s<kBlock>(np, [&](long long j) {
+      int u = __ldcg(plist + j);
+      if (u < 0) return;
+      unsigned m = __ldcg(d.meta + j);
+      bool keep = true;
+      if (m & 0x80000000u) {
+        int p, d0;
+        unsigned long long R;
+        long long w;
+        items(j, p, d0, R, w);
+        if (key_less(d0, R, kd, kr)) {
+          keep = false;
+          d.part[u] = (uint8_t)p;
+          acc_add(s.acc, p, w);
+          cut_acc += (long long)__ldcg(d.pw + u) - __ldcg(d.gain + u);  // independent set: exact
+          app++;
+        }
+      } else if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
+        keep = false;  // stale entry (deleted before this refine)
+      }
+      int slot = agg_append(&ctl->npsi[nxt], keep);
+      if (keep) pnext[slot] = u;
+    });
+    flush_acc(s, ctl->Wp, k);
+    {
+      long long sa = warp_sum(app);
+      if (lane_id() == 0 && sa) atomicAdd(&ctl->applied3[r3], (int)sa);
+    }
+    rr_for_s<kBlock>((long long)k * kDigits, [&](long long t) { d.hist0[t] = 0; });
+    sel_clear<kBlock>(d, s.sel);
+    round_sync(209);
+    const int napp = ldv(&ctl->applied3[r3]), nsel = ldv(&ctl->selected3[r3]);
+    if (napp == 0 && nsel > 0) {
+      // L = 0: force the first move (reading Q8); it is the threshold item K*
+      const int uf = (int)(kr & 0xffffffffu);
+      const int nn = ldv(&ctl->npsi[nxt]);
+      rr_for_s<kBlock>(nn, [&](long long j) {
+        if (__ldcg(pnext + j) == uf) pnext[j] = -1;
+      });
+      if (tid == 0) {
+        int p = __ldcg(d.tgt + uf);
+        d.part[uf] = (uint8_t)p;
+        atomic_add_ll(&ctl->Wp[p], vert_w(d.vw, uf));
+        atomic_add_ll(&ctl->cut, (long long)__ldcg(d.pw + uf) - __ldcg(d.gain + uf));
+        ctl->st[ST_IMBAL] = 1;
+      }
+      round_sync(210);
+    }
+    const int napp2 = (napp == 0 && nsel > 0) ? 1 : napp;
+    if (nsel > 0) {
+      rounds++;
+      applied_tot += napp2;
+      deferred_tot += nsel - napp2;
+    }
+    for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
+    __syncthreads();
+    cur = nxt;
+    rounds_all++;
+  }
+
 }
 
 __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s) {
@@ -438,19 +824,16 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   if (tid == 0) ctl->nph = 0;
   stamp_phase(ctl, 200);
   arrive_stamp(d.dbg, 0);
-  long long scanned = 0, counted = 0, cnt_ins = 0;
+  long long scanned = 0, counted = 0, cnt_ins = 0, cut_acc = 0;
   // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
   const int nA = ldv(&ctl->nA);
   const int np0 = ldv(&ctl->npsi[0]);
   rr_for(np0, [&](long long i) {
     int u = __ldcg(d.psi[0] + i);
-    if (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) {
-      cnt_ins++;
-      d.markF[u] = a.epF;
-      d.oldp[u] = kPsi;
-    }
+    if (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) cnt_ins++;
   });
-  filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, scanned, counted);
+  filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
+              counted);
   block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
   block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
   GRID_SYNC_STAMPED(ctl, 201);
@@ -459,19 +842,19 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   {
     const int nc = ldv(&ctl->ncand);
     if (tid == 0) ctl->st[ST_FILTERED_IN] = nc;
-    commit(d, s, a, nc, d.cand, true, scanned);
+    commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
     // neighbours of the pseudo vertices pending since apply
     auto get = [&](long long i) {
       int u = __ldcg(d.psi[0] + i);
-      return (__ldcg(d.active + u) && __ldcg(d.markF + u) == a.epF && __ldcg(d.oldp + u) == kPsi) ? u : -1;
+      return (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) ? u : -1;  // C1 joins beyond np0
     };
     auto mt = [&](int u, long long) {
       scanned += __ldg(d.deg + u);
-      mark_nbrs_thread(d, u, a.epN);
+      mark_nbrs_thread(d, u, a.epN, a.epC1);
     };
     auto mw = [&](int u, long long) {
       if (lane_id() == 0) scanned += __ldg(d.deg + u);
-      mark_nbrs_warp(d, u, a.epN);
+      mark_nbrs_warp(d, u, a.epN, a.epC1);
     };
     foreach_vertex(d, np0, get, mt, mw);
     flush_acc(s, ctl->Wp, k);
@@ -482,7 +865,8 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   {
     const int nN = ldv(&ctl->nN);
     long long cntN = 0;
-    filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, &ctl->ncand2, d.cand2, scanned, cntN);
+    filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, &ctl->ncand2, d.cand2, a.epC2, scanned,
+                cntN);
     block_atomic_add(&ctl->st[ST_EXPANDED], cntN, s.red);
     if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
   }
@@ -492,7 +876,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   {
     const int nc = ldv(&ctl->ncand2);
     if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc;
-    commit(d, s, a, nc, d.cand2, false, scanned);
+    commit(d, s, a, nc, d.cand2, a.epC2, false, scanned, cut_acc);
     flush_acc(s, ctl->Wp, k);
   }
   GRID_SYNC_STAMPED(ctl, 204);
@@ -566,12 +950,17 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         items(j, p, d0, R, w);
         bool ev = s.sel.found[p] && !key_less(s.sel.d0[p], s.sel.prefix[p], d0, R);
         int slot = agg_append(&ctl->ncand, ev);
-        if (ev) d.cand[slot] = __ldcg(d.r3list + j).x;
+        if (ev) {
+          int v = __ldcg(d.r3list + j).x;
+          d.cand[slot] = v;
+          d.markT[v] = a.epE;
+          d.oldp[v] = (uint8_t)p;
+        }
       });
       sel_clear(d, s.sel);
       GRID_SYNC_STAMPED(ctl, 206);
       const int nc = ldv(&ctl->ncand);
-      commit(d, s, a, nc, d.cand, false, scanned);
+      commit(d, s, a, nc, d.cand, a.epE, false, scanned, cut_acc);
       flush_acc(s, ctl->Wp, k);
       if (tid == 0) ctl->st[ST_EVICTED] = nc;
       for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
@@ -579,317 +968,12 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     }
   }
 
-  // ---- R4: rounds (Alg. 4) ------------------------------------------------------------
-  const int nF = ldv(&ctl->npsi[0]);
-  int cur = 0;
-  long long rounds = 0, rounds_all = 0, applied_tot = 0, deferred_tot = 0;
-  while (true) {
-    const int np = ldv(&ctl->npsi[cur]);
-    if (np == 0) break;
-    const int nxt = cur == 1 ? 2 : 1;
-    const int32_t* plist = d.psi[cur];
-    int32_t* pnext = d.psi[nxt];
-    const int r3 = (int)(rounds_all % 3), r3n = (int)((rounds_all + 1) % 3);
-    // round-start snapshot of W_p (Q14) and the lightest part (zero-conn choice)
-    for (int p = threadIdx.x; p < k; p += blockDim.x) s.Wr[p] = ldv(&ctl->Wp[p]);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      int b = 0;
-      for (int p = 1; p < k; p++)
-        if (s.Wr[p] < s.Wr[b]) b = p;
-      s.best0 = b;
-    }
-    __syncthreads();
-    if (tid == 0) {
-      ctl->npsi[nxt] = 0;
-      ctl->applied3[r3n] = 0;
-      ctl->selected3[r3n] = 0;
-    }
-    for (int p = (int)tid; p < k; p += (int)nthr) ctl->tot3[r3n][p] = 0;
-    // -- gain: selection + best part, one adjacency pass per vertex
-    long long sel_cnt = 0;
-    auto emit_move = [&](long long j, int u, int best, long long g, bool imbal) {
-      int d0 = 255 - (int)min(g, 255ll);
-      d.tgt[u] = (uint8_t)best;
-      d.gain[u] = (int)g;
-      d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;
-      long long w = vert_w(d.vw, u);
-      atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
-      atomic_add_ll(&ctl->tot3[r3][best], w);
-      if (imbal) ctl->st[ST_IMBAL] = 1;
-    };
-    auto get = [&](long long i) {
-      int u = __ldcg(plist + i);
-      if (u < 0 || !__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
-        d.meta[i] = 0;
-        return -1;
-      }
-      return u;
-    };
-    auto tf = [&](int u, long long j) {
-      const long long vwu = vert_w(d.vw, u);
-      scanned += __ldg(d.deg + u);
-      int qs[kThreadDeg];
-      int ws[kThreadDeg];
-      int m = 0;
-      bool sel = true;
-      nbrs_thread(d, u, [&](int x, int w, uint8_t q) {
-        if (q == kPsi) {
-          if (x < u) sel = false;  // a smaller-ID pseudo neighbour moves first (Alg. 4 L8)
-          return sel;
-        }
-        qs[m] = q;
-        ws[m] = w;
-        m++;
-        return true;
-      });
-      if (!sel) {
-        d.meta[j] = 0;
-        return;
-      }
-      int best = -1;
-      long long bc = -1;
-      for (int i = 0; i < m; i++) {
-        int p = qs[i];
-        bool seen = false;
-        for (int t = 0; t < i; t++) seen |= qs[t] == p;
-        if (seen) continue;
-        long long cc = 0;
-        for (int t = i; t < m; t++) cc += qs[t] == p ? ws[t] : 0;
-        if (s.Wr[p] + vwu > c) continue;
-        if (better(cc, p, bc, best, s.Wr)) {
-          best = p;
-          bc = cc;
-        }
-      }
-      bool imbal = false;
-      if (best < 0) {  // lightest part: eligible => zero connectivity; else fallback (Q8)
-        best = s.best0;
-        bc = 0;
-        if (s.Wr[best] + vwu > c) {
-          imbal = true;
-          for (int t = 0; t < m; t++) bc += qs[t] == best ? ws[t] : 0;
-        }
-      }
-      sel_cnt++;
-      emit_move(j, u, best, bc, imbal);
-    };
-    auto wf = [&](int u, long long j) {
-      const long long vwu = vert_w(d.vw, u);
-      int* wc = s.wconn[warp_id()];
-      if (lane_id() == 0) scanned += __ldg(d.deg + u);
-      bool lb = false;
-      nbrs_warp(d, u, [&](int x, int w, uint8_t q) {
-        if (q == kPsi) lb |= x < u;
-        else atomicAdd(wc + q, w);
-      });
-      const bool blocked = __any_sync(0xffffffffu, lb);
-      __syncwarp();
-      long long bc = -1;
-      int best = -1;
-      if (!blocked) {
-        for (int p = lane_id(); p < k; p += 32) {
-          if (s.Wr[p] + vwu > c) continue;
-          long long cc = wc[p];
-          if (better(cc, p, bc, best, s.Wr)) {
-            best = p;
-            bc = cc;
-          }
-        }
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) {
-          long long oc = __shfl_xor_sync(0xffffffffu, bc, off);
-          int op = __shfl_xor_sync(0xffffffffu, best, off);
-          if (op >= 0 && better(oc, op, bc, best, s.Wr)) {
-            bc = oc;
-            best = op;
-          }
-        }
-      }
-      bool imbal = false;
-      if (!blocked && best < 0) {
-        best = s.best0;
-        bc = wc[best];
-        imbal = true;
-      }
-      __syncwarp();
-      for (int p = lane_id(); p < k; p += 32) wc[p] = 0;
-      __syncwarp();
-      if (lane_id() == 0) {
-        if (blocked) {
-          d.meta[j] = 0;
-        } else {
-          sel_cnt++;
-          emit_move(j, u, best, bc, imbal);
-        }
-      }
-    };
-    foreach_vertex(d, np, get, tf, wf);
-    {
-      long long sc = warp_sum(sel_cnt);
-      if (lane_id() == 0 && sc) atomicAdd(&ctl->selected3[r3], (int)sc);
-    }
-    GRID_SYNC_STAMPED(ctl, 208);
+  // ---- R4: rounds (Alg. 4), grid-wide (a CTA-local variant for small tails
+  //      measured slower: the rounds are load-latency bound, not barrier bound)
+  RoundState rs;
+  run_rounds<false>(d, s, grid, c, exact_shift_id, rs, scanned, cut_acc);
+  const long long rounds = rs.rounds, applied_tot = rs.applied_tot, deferred_tot = rs.deferred_tot;
 
-    // -- balanced prefix: T_p = c - W_p + 1; K* = min over parts of the first
-    //    move whose running weight in (#nbr desc, ID asc) order exceeds c.
-    for (int p = threadIdx.x; p < k; p += blockDim.x) {
-      long long T = c - s.Wr[p] + 1;
-      s.sel.T[p] = T;
-      s.sel.used[p] = ldv(&ctl->tot3[r3][p]) >= T;
-    }
-    __syncthreads();
-    auto items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
-      unsigned m = __ldcg(d.meta + j);
-      if (!(m & 0x80000000u)) return false;
-      int u = __ldcg(plist + j);
-      p = (int)(m & 255u);
-      d0 = (int)((m >> 8) & 255u);
-      R = d0 ? (unsigned long long)u
-             : (((unsigned long long)(0x7fffffffu - (unsigned)__ldcg(d.gain + u))) << 32) | (unsigned)u;
-      w = vert_w(d.vw, u);
-      return true;
-    };
-    weighted_select(d, s.sel, grid, [](int d0) { return d0 != 0; }, exact_shift_id, np, items);
-    int kd = 1 << 30;
-    unsigned long long kr = ~0ull;
-    for (int p = 0; p < k; p++) {
-      if (s.sel.used[p] && s.sel.found[p] && key_less(s.sel.d0[p], s.sel.prefix[p], kd, kr)) {
-        kd = s.sel.d0[p];
-        kr = s.sel.prefix[p];
-      }
-    }
-    // -- apply the prefix (moves with key < K*); the rest stay pseudo
-    long long app = 0;
-    rr_for(np, [&](long long j) {
-      int u = __ldcg(plist + j);
-      if (u < 0) return;
-      unsigned m = __ldcg(d.meta + j);
-      bool keep = true;
-      if (m & 0x80000000u) {
-        int p, d0;
-        unsigned long long R;
-        long long w;
-        items(j, p, d0, R, w);
-        if (key_less(d0, R, kd, kr)) {
-          keep = false;
-          d.part[u] = (uint8_t)p;
-          acc_add(s.acc, p, w);
-          app++;
-        }
-      } else if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
-        keep = false;  // stale entry (deleted before this refine)
-      }
-      int slot = agg_append(&ctl->npsi[nxt], keep);
-      if (keep) pnext[slot] = u;
-    });
-    flush_acc(s, ctl->Wp, k);
-    {
-      long long sa = warp_sum(app);
-      if (lane_id() == 0 && sa) atomicAdd(&ctl->applied3[r3], (int)sa);
-    }
-    for (long long t = tid; t < (long long)k * kDigits; t += nthr) d.hist0[t] = 0;
-    sel_clear(d, s.sel);
-    GRID_SYNC_STAMPED(ctl, 209);
-    const int napp = ldv(&ctl->applied3[r3]), nsel = ldv(&ctl->selected3[r3]);
-    if (napp == 0 && nsel > 0) {
-      // L = 0: force the first move (reading Q8); it is the threshold item K*
-      const int uf = (int)(kr & 0xffffffffu);
-      const int nn = ldv(&ctl->npsi[nxt]);
-      for (long long j = tid; j < nn; j += nthr)
-        if (__ldcg(pnext + j) == uf) pnext[j] = -1;
-      if (tid == 0) {
-        int p = __ldcg(d.tgt + uf);
-        d.part[uf] = (uint8_t)p;
-        atomic_add_ll(&ctl->Wp[p], vert_w(d.vw, uf));
-        ctl->st[ST_IMBAL] = 1;
-      }
-      GRID_SYNC_STAMPED(ctl, 210);
-    }
-    const int napp2 = (napp == 0 && nsel > 0) ? 1 : napp;
-    if (nsel > 0) {
-      rounds++;
-      applied_tot += napp2;
-      deferred_tot += nsel - napp2;
-    }
-    for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
-    __syncthreads();
-    cur = nxt;
-    rounds_all++;
-  }
-
-  // ---- FD: cut delta over the frontier F (edges with an endpoint in F) -------
-  long long cut_acc = 0;
-  {
-    // delta of the edges of u: now (final labels, all placed) minus before
-    // (labels at refine start: oldp for F members); F-F edges once (x > u)
-    auto delta = [&](int u, const int* x, const int* w, const uint8_t* q, const unsigned* mf,
-                     const uint8_t* op, int C) {
-      const uint8_t pu = ld_part(d.part, u), ou = __ldcg(d.oldp + u);
-      long long acc = 0;
-      for (int t = 0; t < C; t++) {
-        if (x[t] < 0) continue;
-        bool xf = mf[t] == a.epF;
-        if (xf && x[t] < u) continue;
-        uint8_t ox = xf ? op[t] : q[t];
-        int was = (ou != kPsi && ox != kPsi && ou != ox) ? w[t] : 0;
-        int now = (pu != q[t]) ? w[t] : 0;
-        acc += now - was;
-      }
-      return acc;
-    };
-    auto get = [&](long long i) {
-      int u = __ldcg(d.psi[0] + i);
-      return __ldcg(d.active + u) ? u : -1;
-    };
-    auto tf = [&](int u, long long) {
-      const long long o = __ldg(d.off + u);
-      const int dg = __ldg(d.deg + u);
-      for (int i = 0; i < dg; i += kTC) {
-        int x[kTC], w[kTC];
-        uint8_t q[kTC], op[kTC];
-        unsigned mf[kTC];
-#pragma unroll
-        for (int t = 0; t < kTC; t++) {
-          x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
-          w[t] = (i + t < dg && d.adjw) ? __ldg(d.adjw + o + i + t) : 1;
-        }
-#pragma unroll
-        for (int t = 0; t < kTC; t++) {
-          q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
-          mf[t] = x[t] >= 0 ? __ldcg(d.markF + x[t]) : 0u;
-          op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
-        }
-        cut_acc += delta(u, x, w, q, mf, op, kTC);
-      }
-    };
-    auto wf = [&](int u, long long) {
-      const long long o = __ldg(d.off + u);
-      const int dg = __ldg(d.deg + u);
-      long long acc = 0;
-      for (int b = 0; b < dg; b += 256) {
-        int x[8], w[8];
-        uint8_t q[8], op[8];
-        unsigned mf[8];
-#pragma unroll
-        for (int t = 0; t < 8; t++) {
-          int i = b + t * 32 + lane_id();
-          x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
-          w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
-        }
-#pragma unroll
-        for (int t = 0; t < 8; t++) {
-          q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
-          mf[t] = x[t] >= 0 ? __ldcg(d.markF + x[t]) : 0u;
-          op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
-        }
-        acc += delta(u, x, w, q, mf, op, 8);
-      }
-      acc = warp_sum(acc);
-      if (lane_id() == 0) cut_acc += acc;
-    };
-    foreach_vertex(d, nF, get, tf, wf);
-  }
   block_atomic_add(&ctl->cut, cut_acc, s.red);
   block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
   GRID_SYNC_STAMPED(ctl, 211);
