@@ -62,6 +62,9 @@ struct Ctl {
   int ndirty;          // compaction list length
   int nr3;             // restoration candidate list length
   int nvdch;           // vertex-deletion work chunks
+  int ntie;            // tie-group buffer length (round prefix select)
+  int tiecnt[256];     // tie-group size per part
+  unsigned long long kres[256];  // per-part threshold keys from the CTA-local select
   int applied3[3];     // moves applied per round (mod 3)
   int selected3[3];    // moves selected per round (mod 3)
   unsigned long long tph[128];  // %globaltimer after each phase (CTA 0)

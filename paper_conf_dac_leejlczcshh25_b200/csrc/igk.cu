@@ -210,6 +210,14 @@ bool dalloc(igk_graph* g, T** p, size_t count) {
 
 uint32_t next_epoch(igk_graph* g) { return ++g->epoch; }
 
+// capacities grow geometrically so that slowly growing batches do not
+// re-allocate (pinned host allocations are expensive)
+long long grow_cap(long long need) {
+  long long c = 1024;
+  while (c < need) c <<= 1;
+  return c;
+}
+
 int coop_grid(const void* fn, size_t smem, int want_per_sm) {
   int dev = 0, sms = 0, occ = 0;
   cudaGetDevice(&dev);
@@ -490,8 +498,9 @@ static igk_status prepare_apply(igk_graph* g, int64_t count) {
     if (g->d.newid) cudaFree(g->d.newid);
     g->d.newid = nullptr;
     g->newid_cap = 0;
-    if (cudaMalloc(&g->d.newid, count * 4) != cudaSuccess) return fail(g, IGK_ENOMEM, "newid allocation failed");
-    g->newid_cap = count;
+    long long cap = grow_cap(count);
+    if (cudaMalloc(&g->d.newid, cap * 4) != cudaSuccess) return fail(g, IGK_ENOMEM, "newid allocation failed");
+    g->newid_cap = cap;
   }
   g->d.hmask = g->hash_cap - 1;
   return IGK_OK;
@@ -619,16 +628,18 @@ igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t c
     if (g->h_stage) cudaFreeHost(g->h_stage);
     g->h_stage = nullptr;
     g->h_stage_cap = 0;
-    if (cudaMallocHost(&g->h_stage, count * sizeof(igk_modifier)) != cudaSuccess)
+    long long cap = grow_cap(count);
+    if (cudaMallocHost(&g->h_stage, cap * sizeof(igk_modifier)) != cudaSuccess)
       return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
-    g->h_stage_cap = count;
+    g->h_stage_cap = cap;
   }
   if (count > g->d_mods_cap) {
     if (g->d_mods) cudaFree(g->d_mods);
     g->d_mods = nullptr;
     g->d_mods_cap = 0;
-    if (cudaMalloc(&g->d_mods, count * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
-    g->d_mods_cap = count;
+    long long cap = grow_cap(count);
+    if (cudaMalloc(&g->d_mods, cap * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
+    g->d_mods_cap = cap;
   }
   std::memcpy(g->h_stage, mods, count * sizeof(igk_modifier));
   CK(cudaMemcpyAsync(g->d_mods, g->h_stage, count * 16, cudaMemcpyHostToDevice, g->stream));
@@ -695,16 +706,18 @@ igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_r
     if (g->h_stage) cudaFreeHost(g->h_stage);
     g->h_stage = nullptr;
     g->h_stage_cap = 0;
-    if (cudaMallocHost(&g->h_stage, count * sizeof(igk_modifier)) != cudaSuccess)
+    long long cap = grow_cap(count);
+    if (cudaMallocHost(&g->h_stage, cap * sizeof(igk_modifier)) != cudaSuccess)
       return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
-    g->h_stage_cap = count;
+    g->h_stage_cap = cap;
   }
   if (count > g->d_mods_cap) {
     if (g->d_mods) cudaFree(g->d_mods);
     g->d_mods = nullptr;
     g->d_mods_cap = 0;
-    if (cudaMalloc(&g->d_mods, count * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
-    g->d_mods_cap = count;
+    long long cap = grow_cap(count);
+    if (cudaMalloc(&g->d_mods, cap * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
+    g->d_mods_cap = cap;
   }
   if (count > 0) {
     std::memcpy(g->h_stage, mods, count * sizeof(igk_modifier));

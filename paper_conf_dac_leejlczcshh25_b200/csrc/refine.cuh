@@ -333,10 +333,8 @@ __device__ void sel_choose(const Dev& d, SelSmem& sm, int pass) {
   __syncthreads();
 }
 
-template <bool kBlock = false, class ExactFn, class Items>
-__device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid, ExactFn is_exact,
-                                int exact_shift, long long nitems, Items items) {
-  sel_digit0(d, sm, is_exact, exact_shift);
+template <bool kBlock = false, class Items>
+__device__ void sel_passes(const Dev& d, SelSmem& sm, cg::grid_group& grid, long long nitems, Items items) {
   int pass = 0;
   while (sm.nactive > 0) {
     sel_accumulate<kBlock>(d, sm, pass, nitems, items);
@@ -347,6 +345,13 @@ __device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid,
     pass++;
   }
   if (pass > 0) scope_sync<kBlock>(grid);  // every CTA finished reading before anyone clears
+}
+
+template <bool kBlock = false, class ExactFn, class Items>
+__device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid, ExactFn is_exact,
+                                int exact_shift, long long nitems, Items items) {
+  sel_digit0(d, sm, is_exact, exact_shift);
+  sel_passes<kBlock>(d, sm, grid, nitems, items);
 }
 
 template <bool kBlock = false>
@@ -363,8 +368,15 @@ __device__ void sel_clear(const Dev& d, const SelSmem& sm) {
 // ---------------------------------------------------------------------------
 // the refine kernel
 // ---------------------------------------------------------------------------
+constexpr int kTieMax = 4096;  // tie groups up to this size finish in one CTA's shared memory
 struct RefSmem {
   SelSmem sel;
+  int tie_u[kTieMax];     // CTA-local select: vertex IDs of one part's tie group
+  int tie_w[kTieMax];     //                   and their weights
+  long long tie_h[256];
+  unsigned long long tie_prefix;
+  long long tie_base;
+  int tie_n;
   long long Wr[256];      // round-start part weights (Q14)
   long long acc[256];     // per-part weight deltas of this CTA
   long long red[32];
@@ -379,6 +391,67 @@ __device__ __forceinline__ void flush_acc(RefSmem& s, long long* dst, int k) {
     s.acc[p] = 0;
   }
   __syncthreads();
+}
+
+// CTA-local weighted select over one part's tie group (vertex IDs < 2^31):
+// the first ID, ascending, whose inclusive weight prefix (after `base`)
+// reaches T.  Four 8-bit MSD passes over a shared-memory histogram.
+__device__ unsigned block_select_ids(RefSmem& s, int cnt, long long base, long long T) {
+  if (threadIdx.x == 0) {
+    s.tie_prefix = 0;
+    s.tie_base = base;
+  }
+  for (int shift = 24; shift >= 0; shift -= 8) {
+    for (int b = threadIdx.x; b < 256; b += blockDim.x) s.tie_h[b] = 0;
+    __syncthreads();
+    const unsigned pre = (unsigned)s.tie_prefix;
+    for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
+      unsigned u = (unsigned)s.tie_u[i];
+      if (shift == 24 || (u >> (shift + 8)) == (pre >> (shift + 8)))
+        atomicAdd((unsigned long long*)&s.tie_h[(u >> shift) & 255], (unsigned long long)s.tie_w[i]);
+    }
+    __syncthreads();
+    if (warp_id() == 0) {
+      const int l = lane_id();
+      long long v[8], sum = 0;
+#pragma unroll
+      for (int t = 0; t < 8; t++) {
+        v[t] = s.tie_h[8 * l + t];
+        sum += v[t];
+      }
+      long long incl = sum;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        long long y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (l >= o) incl += y;
+      }
+      long long run = s.tie_base + incl - sum;
+      int cd = -1;
+      long long cb = 0;
+#pragma unroll
+      for (int t = 0; t < 8; t++) {
+        if (cd < 0 && v[t] > 0) {
+          if (run + v[t] >= T) {
+            cd = 8 * l + t;
+            cb = run;
+          }
+          run += v[t];
+        }
+      }
+      unsigned m = __ballot_sync(0xffffffffu, cd >= 0);
+      if (m) {
+        int src = __ffs(m) - 1;
+        int dd = __shfl_sync(0xffffffffu, cd, src);
+        long long bb = __shfl_sync(0xffffffffu, cb, src);
+        if (l == 0) {
+          s.tie_prefix |= (unsigned long long)dd << shift;
+          s.tie_base = bb;
+        }
+      }
+    }
+    __syncthreads();
+  }
+  return (unsigned)s.tie_prefix;
 }
 
 // filter (Alg. 3 L8-24): candidates = listed placed vertices with ext > int;
@@ -546,8 +619,9 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
   long long& rounds_all = rs.rounds_all;
   long long& applied_tot = rs.applied_tot;
   long long& deferred_tot = rs.deferred_tot;
-  auto round_sync = [&](int id) {
-    if (!kBlock) arrive_stamp(d.dbg, id % 100);
+  auto round_sync = [&](int id) {  // per-round arrival slots 20 + 2r (gain), 21 + 2r (apply)
+    const bool per_round = (id == 208 || id == 209) && rounds_all < 40;
+    if (!kBlock) arrive_stamp(d.dbg, per_round ? 20 + 2 * (int)rounds_all + (id - 208) : id % 100);
     scope_sync<kBlock>(grid);
     stamp_phase(ctl, kBlock ? id + 20 : id);
   };
@@ -727,7 +801,65 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
       w = vert_w(d.vw, u);
       return true;
     };
-    weighted_select<kBlock>(d, s.sel, grid, [](int d0) { return d0 != 0; }, exact_shift_id, np, items);
+    sel_digit0(d, s.sel, [](int d0) { return d0 != 0; }, exact_shift_id);
+    if (s.sel.nactive > 0) {
+      // tie groups (moves of an overflowing part with its threshold digit 0)
+      rr_for_s<kBlock>(np, [&](long long j) {
+        int p, d0;
+        unsigned long long R;
+        long long w;
+        bool in = items(j, p, d0, R, w) && s.sel.active[p] && d0 == s.sel.d0[p];
+        int slot = agg_append(&ctl->ntie, in);
+        if (in) {
+          d.r3list[slot] = make_int2(__ldcg(plist + j), p | ((int)w << 8));
+          atomicAdd(&ctl->tiecnt[p], 1);
+        }
+      });
+      round_sync(212);
+      const int ntie = ldv(&ctl->ntie);
+      bool local_ok = true;
+      for (int p = 0; p < k; p++)
+        if (s.sel.active[p]) local_ok &= s.sel.exact[p] && ldv(&ctl->tiecnt[p]) <= kTieMax;
+      if (local_ok) {
+        // one CTA per overflowing part finishes its select in shared memory
+        for (int p = kBlock ? 0 : (int)blockIdx.x; p < k; p += kBlock ? 1 : (int)gridDim.x) {
+          if (!s.sel.active[p]) continue;
+          if (threadIdx.x == 0) s.tie_n = 0;
+          __syncthreads();
+          for (int i = threadIdx.x; i < ntie; i += blockDim.x) {
+            int2 e = __ldcg(d.r3list + i);
+            if ((e.y & 255) == p) {
+              int q = atomicAdd(&s.tie_n, 1);
+              s.tie_u[q] = e.x;
+              s.tie_w[q] = e.y >> 8;
+            }
+          }
+          __syncthreads();
+          unsigned key = block_select_ids(s, s.tie_n, s.sel.base[p], s.sel.T[p]);
+          if (threadIdx.x == 0) ctl->kres[p] = key;
+          __syncthreads();
+        }
+        round_sync(213);
+        for (int p = threadIdx.x; p < k; p += blockDim.x)
+          if (s.sel.active[p]) {
+            s.sel.prefix[p] = ldv((const long long*)&ctl->kres[p]);
+            s.sel.active[p] = 0;
+          }
+        __syncthreads();
+      } else {  // fallback: grid-wide radix passes over the tie buffer only
+        auto tie_items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
+          int2 e = __ldcg(d.r3list + j);
+          p = e.y & 255;
+          w = e.y >> 8;
+          d0 = s.sel.d0[p];
+          R = s.sel.exact[p] ? (unsigned long long)e.x
+                             : (((unsigned long long)(0x7fffffffu - (unsigned)__ldcg(d.gain + e.x))) << 32) |
+                                   (unsigned)e.x;
+          return true;
+        };
+        sel_passes<kBlock>(d, s.sel, grid, ntie, tie_items);
+      }
+    }
     int kd = 1 << 30;
     unsigned long long kr = ~0ull;
     for (int p = 0; p < k; p++) {
@@ -767,6 +899,8 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
       if (lane_id() == 0 && sa) atomicAdd(&ctl->applied3[r3], (int)sa);
     }
     rr_for_s<kBlock>((long long)k * kDigits, [&](long long t) { d.hist0[t] = 0; });
+    rr_for_s<kBlock>(k, [&](long long p) { ctl->tiecnt[p] = 0; });
+    if (tid == 0) ctl->ntie = 0;
     sel_clear<kBlock>(d, s.sel);
     round_sync(209);
     const int napp = ldv(&ctl->applied3[r3]), nsel = ldv(&ctl->selected3[r3]);
