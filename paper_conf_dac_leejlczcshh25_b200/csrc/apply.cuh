@@ -101,10 +101,16 @@ __device__ __forceinline__ int block_excl_scan(int v, int* total, int* sbuf) {
   return warp_excl + x - v;
 }
 
-__device__ __forceinline__ void mark_affected(const Dev& d, int x, uint32_t epA) {
+// x joins the affected set A (Alg. 3 L6-7); a vertex of degree >
+// kBlockDeg is also listed (and stamped) for CTA-cooperative filtering
+__device__ __forceinline__ void mark_affected(const Dev& d, int x, uint32_t epA, int dgx) {
   bool na = stamp_insert(d.markA, x, epA);
   int s2 = agg_append(&d.ctl->nA, na);
   if (na) d.Alist[s2] = x;
+  if (na && dgx > kBlockDeg) {
+    d.markH[x] = epA;
+    d.hubA[atomicAdd(&d.ctl->nhubA, 1)] = x;
+  }
 }
 
 struct ApplySmem {
@@ -297,9 +303,10 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     // search the shorter prefix; the twin gives the reverse slot
     int a0 = m.y, b0 = m.z;
     long long oa = 0;
-    int da = 0;
+    int da = 0, du = 0, dv = 0;
     if (ed) {
-      int du = __ldcg(d.deg + m.y), dv = __ldcg(d.deg + m.z);
+      du = __ldcg(d.deg + m.y);
+      dv = __ldcg(d.deg + m.z);
       if (dv < du) {
         a0 = m.z;
         b0 = m.y;
@@ -325,8 +332,8 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       atomicSub(d.ldeg + m.z, 1);
       uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
       if (pu != kPsi && pv != kPsi && pu != pv) cut_acc -= w;
-      mark_affected(d, m.y, a.epA);
-      mark_affected(d, m.z, a.epA);
+      mark_affected(d, m.y, a.epA, du);
+      mark_affected(d, m.z, a.epA, dv);
     }
   });
   {
@@ -341,6 +348,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       int x = j < dg ? __ldcg(d.adj + o + j) : -1;  // -1: tombstone from an edge deletion
       int w = (x >= 0 && d.adjw) ? __ldcg(d.adjw + o + j) : 1;
       bool xdel = x >= 0 && __ldcg(d.markD + x) == a.epD;
+      const int dx = x >= 0 ? __ldcg(d.deg + x) : 0;
       if (x >= 0 && !xdel) {  // the twin is u's entry in x's prefix
         d.adj[__ldcg(d.twin + o + j)] = -1;
         atomicSub(d.ldeg + x, 1);
@@ -349,7 +357,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
         uint8_t px = ld_part(d.part, x);
         if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < x)) cut_acc -= w;
       }
-      if (x >= 0 && !xdel) mark_affected(d, x, a.epA);
+      if (x >= 0 && !xdel) mark_affected(d, x, a.epA, dx);
       if (ch.y == 0 && lane_id() == 0) {
         int vwu = d.vw ? __ldcg(d.vw + u) : 1;
         if (pu != kPsi) atomic_add_ll(&ctl->Wp[pu], -(long long)vwu);
@@ -453,12 +461,8 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     }
     uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
     if (pu != kPsi && pv != kPsi && pu != pv) cut_acc += m.w;
-    bool na = stamp_insert(d.markA, m.y, a.epA);
-    int s1 = agg_append(&ctl->nA, na);
-    if (na) d.Alist[s1] = m.y;
-    bool nb = stamp_insert(d.markA, m.z, a.epA);
-    int s2 = agg_append(&ctl->nA, nb);
-    if (nb) d.Alist[s2] = m.z;
+    mark_affected(d, m.y, a.epA, pu_pos + 1);
+    mark_affected(d, m.z, a.epA, pv_pos + 1);
   });
   // twin fix-ups of moved entries: resolve forward marks of moved partners,
   // then point the partner back at the new slot (idempotent when both moved)

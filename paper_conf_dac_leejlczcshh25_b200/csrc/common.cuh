@@ -22,6 +22,7 @@ constexpr int64_t kNMax = int64_t(1) << 30;
 constexpr int kThreads = 512;       // persistent-kernel block size
 constexpr int kWarps = kThreads / 32;
 constexpr int kThreadDeg = 16;      // degree <= this: one thread per vertex; above: one warp
+constexpr int kBlockDeg = 1024;     // degree > this (hubs): one whole CTA per vertex
 constexpr int kDigits = 256;        // radix digit bins (8-bit digits)
 constexpr long long kNoErr = 0x7fffffffffffffffLL;
 
@@ -54,6 +55,7 @@ struct Ctl {
   long long slab_top0;     // slab_top before the current apply (rollback)
   long long st[ST_N];  // refine stats (accumulating)
   int nA;              // affected list length
+  int nhubA, nhubC, nhubN, nhubC2, nhubP;  // hub (degree > kBlockDeg) work lists
   int npsi[3];         // pseudo list lengths
   int ncand;           // candidate list length (C1, R3)
   int ncand2;          // candidate list length (C2)
@@ -109,6 +111,12 @@ struct Dev {
   int2* r3list;      // (vertex, loss) restoration candidates
   int2* vdch;        // (vertex, chunk) work items of vertex deletions
   uint32_t* markF;   // frontier membership (entered Psi in this refine cycle)
+  uint32_t* markH;   // hub routed to a CTA-cooperative list (epoch = the list's cycle)
+  int32_t* hubA;     // hubs in A
+  int32_t* hubC;     // hub candidates of R1 / R2 / R3 (commit lists)
+  int32_t* hubN;     // hubs in N (R2)
+  int32_t* hubC2;
+  int32_t* hubP;     // hubs in the pseudo-partition (rounds)
   uint8_t* oldp;     // part before entering Psi (kPsi for inserted vertices)
   int64_t* reloc;    // new slab offset for relocated vertices
   // per-vertex move results (rounds)
@@ -116,6 +124,7 @@ struct Dev {
   int32_t* gain;
   int32_t* pw;       // placed-neighbour weight at round start (cut delta of a placement)
   uint32_t* meta;    // per psi index: bit31 selected | d0 << 8 | p*
+  uint32_t* metav;   // per vertex: the same record for CTA-processed hubs
   // selection histograms
   long long* hist0;  // [256][256] digit-0 weights per part
   long long* histR;  // [3][256][256] pass histograms

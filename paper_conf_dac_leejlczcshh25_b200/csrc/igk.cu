@@ -350,9 +350,11 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.markG, N) && dalloc(g, &d.vcnt, N) && dalloc(g, &d.icnt, N) &&
             dalloc(g, &d.Alist, N) && dalloc(g, &d.psi[0], N) && dalloc(g, &d.psi[1], N) &&
             dalloc(g, &d.psi[2], N) && dalloc(g, &d.cand, N) && dalloc(g, &d.cand2, N) &&
-            dalloc(g, &d.vdch, N + (size_t)(d.slot_cap / 32) + 1024) && dalloc(g, &d.markF, N) && dalloc(g, &d.oldp, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
+            dalloc(g, &d.vdch, N + (size_t)(d.slot_cap / 32) + 1024) && dalloc(g, &d.markF, N) && dalloc(g, &d.oldp, N) && dalloc(g, &d.markH, N) &&
+            dalloc(g, &d.hubA, N) && dalloc(g, &d.hubC, N) && dalloc(g, &d.hubN, N) && dalloc(g, &d.hubC2, N) &&
+            dalloc(g, &d.hubP, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
             dalloc(g, &d.dlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
-            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) &&
+            dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) && dalloc(g, &d.metav, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
             dalloc(g, &g->d_red, 259);
@@ -378,6 +380,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   cudaMemsetAsync(d.markD, 0, N * 4, s);
   cudaMemsetAsync(d.markG, 0, N * 4, s);
   cudaMemsetAsync(d.markF, 0, N * 4, s);
+  cudaMemsetAsync(d.markH, 0, N * 4, s);
   cudaMemsetAsync(d.vcnt, 0, N * 4, s);
   cudaMemsetAsync(d.icnt, 0, N * 4, s);
   cudaMemsetAsync(d.hist0, 0, 256 * kDigits * 8, s);
@@ -554,6 +557,7 @@ static RefineArgs make_refine_args(igk_graph* g, int after_apply) {
   a.epC2 = next_epoch(g);
   a.epF = next_epoch(g);
   a.epE = next_epoch(g);
+  a.epA = g->epochA;
   a.after_apply = after_apply;
   return a;
 }

@@ -24,6 +24,7 @@ namespace igk {
 struct RefineArgs {
   long long e_ppm;
   uint32_t epC1, epN, epC2, epF, epE;
+  uint32_t epA;     // stamp of the affected set (hubs in A carry markH == epA)
   int after_apply;  // fused step: skip (leave the state untouched) if the batch was rejected
 };
 
@@ -60,21 +61,30 @@ template <int C>
 __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uint8_t* q, uint32_t epN,
                                            uint32_t epC) {
   bool want[C];
+  int dgx[C];
 #pragma unroll
   for (int t = 0; t < C; t++) {
     unsigned mk = x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN;
+    dgx[t] = x[t] >= 0 ? __ldg(d.deg + x[t]) : 0;
     want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC;  // C1 members are pseudo on sigma2
   }
   unsigned old[C];
 #pragma unroll
   for (int t = 0; t < C; t++) old[t] = want[t] ? atomicExch(d.markT + x[t], epN) : epN;
-  int c = 0;
+  int c = 0, ch = 0;
 #pragma unroll
-  for (int t = 0; t < C; t++) c += old[t] != epN;
+  for (int t = 0; t < C; t++) {
+    c += old[t] != epN && dgx[t] <= kBlockDeg;
+    ch += old[t] != epN && dgx[t] > kBlockDeg;
+  }
   int slot = c ? atomicAdd(&d.ctl->nN, c) : 0;  // one reservation per lane and chunk
+  int hslot = ch ? atomicAdd(&d.ctl->nhubN, ch) : 0;
 #pragma unroll
-  for (int t = 0; t < C; t++)
-    if (old[t] != epN) d.Nlist[slot++] = x[t];
+  for (int t = 0; t < C; t++) {
+    if (old[t] == epN) continue;
+    if (dgx[t] > kBlockDeg) d.hubN[hslot++] = x[t];  // hubs are filtered by a whole CTA
+    else d.Nlist[slot++] = x[t];
+  }
 }
 __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN, uint32_t epC) {
   const long long o = __ldg(d.off + u);
@@ -368,7 +378,8 @@ __device__ void sel_clear(const Dev& d, const SelSmem& sm) {
 // ---------------------------------------------------------------------------
 // the refine kernel
 // ---------------------------------------------------------------------------
-constexpr int kTieMax = 4096;  // tie groups up to this size finish in one CTA's shared memory
+constexpr int kTieMax = 4096;
+constexpr unsigned kMetaHub = 0x40000000u;  // move record kept per vertex (metav): CTA-processed hub  // tie groups up to this size finish in one CTA's shared memory
 struct RefSmem {
   SelSmem sel;
   int tie_u[kTieMax];     // CTA-local select: vertex IDs of one part's tie group
@@ -454,15 +465,87 @@ __device__ unsigned block_select_ids(RefSmem& s, int cnt, long long base, long l
   return (unsigned)s.tie_prefix;
 }
 
+// ---------------------------------------------------------------------------
+// CTA-cooperative processing of hubs (degree > kBlockDeg): the "block" bucket
+// of the degree-bucketed work assignment (thread <= 16 < warp <= 1024 < CTA)
+// ---------------------------------------------------------------------------
+// sum of (a, b) over the CTA, result in every thread
+__device__ __forceinline__ void block_sum2(RefSmem& s, long long& a, long long& b) {
+  a = warp_sum(a);
+  b = warp_sum(b);
+  __syncthreads();
+  if (lane_id() == 0) {
+    s.red[warp_id()] = a;
+    s.red[16 + warp_id()] = b;
+  }
+  __syncthreads();
+  a = 0;
+  b = 0;
+  for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+    a += s.red[w];
+    b += s.red[16 + w];
+  }
+  __syncthreads();
+}
+// CTA-strided walk over u's prefix, 4 entries per thread per round trip
+template <class F>
+__device__ __forceinline__ void nbrs_block(const Dev& d, int u, F f) {
+  const long long o = __ldg(d.off + u);
+  const int dg = __ldg(d.deg + u);
+  for (int b = 0; b < dg; b += 4 * (int)blockDim.x) {
+    int x[4], w[4];
+    uint8_t q[4];
+#pragma unroll
+    for (int t = 0; t < 4; t++) {
+      int i = b + t * (int)blockDim.x + (int)threadIdx.x;
+      x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
+      w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+    }
+#pragma unroll
+    for (int t = 0; t < 4; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    f(x, w, q);
+  }
+}
+// hub filter (Alg. 3 L8-24) by a whole CTA; candidates go to `hout`
+__device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh, uint32_t ep, int* nout,
+                           int32_t* hout, long long& scanned, long long& counted) {
+  for (int h = blockIdx.x; h < nh; h += gridDim.x) {
+    const int u = __ldcg(hubs + h);
+    if (!__ldcg(d.active + u)) continue;  // uniform over the CTA
+    const uint8_t pu = ld_part(d.part, u);
+    if (pu == kPsi) continue;
+    long long in = 0, ex = 0;
+    nbrs_block(d, u, [&](const int* x, const int* w, const uint8_t* q) {
+#pragma unroll
+      for (int t = 0; t < 4; t++)
+        if (x[t] >= 0) {
+          if (q[t] == pu) in += w[t]; else ex += w[t];
+        }
+    });
+    block_sum2(s, in, ex);
+    if (threadIdx.x == 0) {
+      counted++;
+      scanned += __ldg(d.deg + u);
+      if (ex > in) {
+        d.markT[u] = ep;
+        d.oldp[u] = pu;
+        hout[atomicAdd(nout, 1)] = u;
+      }
+    }
+  }
+}
+
 // filter (Alg. 3 L8-24): candidates = listed placed vertices with ext > int;
 // pseudo neighbours count as external (Q13); strict > (Q2)
+// (vertices stamped markH == hub_ep are left to the CTA-cooperative hub pass)
 template <class Get>
 __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, uint32_t ep,
-                            long long& scanned, long long& counted) {
+                            long long& scanned, long long& counted, uint32_t hub_ep = 0) {
   auto tf = [&](int u, long long) {
-    if (!__ldcg(d.active + u)) return;
+    const bool act = __ldcg(d.active + u);
     const uint8_t pu = ld_part(d.part, u);
-    if (pu == kPsi) return;
+    const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
+    if (!act || hub || pu == kPsi) return;
     counted++;
     long long in = 0, ex = 0;
     nbrs_thread(d, u, [&](int, int w, uint8_t q) {
@@ -479,9 +562,10 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     if (c) cand[slot] = u;
   };
   auto wf = [&](int u, long long) {
-    if (!__ldcg(d.active + u)) return;
+    const bool act = __ldcg(d.active + u);
     const uint8_t pu = ld_part(d.part, u);
-    if (pu == kPsi) return;
+    const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
+    if (!act || hub || pu == kPsi) return;
     long long in = 0, ex = 0;
     nbrs_warp(d, u, [&](int, int w, uint8_t q) {
       if (q == pu) in += w; else ex += w;
@@ -590,6 +674,46 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
   foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, tf, wf);
 }
 
+// commit of hub candidates by a whole CTA each (same arithmetic as commit());
+// committed hubs are stamped and listed for CTA-cooperative rounds
+__device__ void hub_commit(const Dev& d, RefSmem& s, const RefineArgs& a, const int32_t* hubs, int nh, uint32_t ep,
+                           bool expand, long long& scanned, long long& cut_acc) {
+  Ctl* ctl = d.ctl;
+  for (int h = blockIdx.x; h < nh; h += gridDim.x) {
+    const int u = __ldcg(hubs + h);
+    const uint8_t pu = __ldcg(d.oldp + u);
+    long long del = 0, dummy = 0;
+    nbrs_block(d, u, [&](const int* x, const int* w, const uint8_t* q) {
+      unsigned mk[4];
+      uint8_t op[4];
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
+        op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+      }
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        if (x[t] < 0) continue;
+        const bool xc = mk[t] == ep;
+        const uint8_t qx = xc ? op[t] : q[t];
+        if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
+      }
+      if (expand) mark_chunk<4>(d, x, q, a.epN, ep);
+    });
+    block_sum2(s, del, dummy);
+    if (threadIdx.x == 0) {
+      scanned += __ldg(d.deg + u);
+      cut_acc -= del;
+      atomic_add_ll(&ctl->Wp[pu], -(long long)vert_w(d.vw, u));
+      d.part[u] = kPsi;
+      d.psi[0][atomicAdd(&ctl->npsi[0], 1)] = u;
+      d.markH[u] = a.epF;  // rounds: handled by a whole CTA
+      d.hubP[atomicAdd(&ctl->nhubP, 1)] = u;
+    }
+    __syncthreads();
+  }
+}
+
 // better(a, b) on (conn desc, W_p asc, p asc)  (reading Q6)
 __device__ __forceinline__ bool better(long long ca, int pa, long long cb, int pb, const long long* Wr) {
   if (pb < 0) return true;
@@ -609,8 +733,8 @@ struct RoundState {
   long long rounds = 0, rounds_all = 0, applied_tot = 0, deferred_tot = 0;
 };
 template <bool kBlock>
-__device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long long c, int exact_shift_id,
-                           RoundState& rs, long long& scanned, long long& cut_acc) {
+__device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::grid_group& grid, long long c,
+                           int exact_shift_id, RoundState& rs, long long& scanned, long long& cut_acc) {
   Ctl* ctl = d.ctl;
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -619,6 +743,7 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
   long long& rounds_all = rs.rounds_all;
   long long& applied_tot = rs.applied_tot;
   long long& deferred_tot = rs.deferred_tot;
+  const int nhp = ldv(&ctl->nhubP);  // final after F3: hubs pending in the rounds
   auto round_sync = [&](int id) {  // per-round arrival slots 20 + 2r (gain), 21 + 2r (apply)
     const bool per_round = (id == 208 || id == 209) && rounds_all < 40;
     if (!kBlock) arrive_stamp(d.dbg, per_round ? 20 + 2 * (int)rounds_all + (id - 208) : id % 100);
@@ -655,7 +780,18 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
       d.tgt[u] = (uint8_t)best;
       d.gain[u] = (int)g;
       d.pw[u] = (int)pwv;
-      d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;
+      d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;  // j: list position (hubs: vertex id)
+      long long w = vert_w(d.vw, u);
+      atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
+      atomic_add_ll(&ctl->tot3[r3][best], w);
+      if (imbal) ctl->st[ST_IMBAL] = 1;
+    };
+    auto emit_move_v = [&](int u, int best, long long g, long long pwv, bool imbal) {
+      int d0 = 255 - (int)min(g, 255ll);
+      d.tgt[u] = (uint8_t)best;
+      d.gain[u] = (int)g;
+      d.pw[u] = (int)pwv;
+      d.metav[u] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;
       long long w = vert_w(d.vw, u);
       atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
       atomic_add_ll(&ctl->tot3[r3][best], w);
@@ -663,8 +799,19 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
     };
     auto get = [&](long long i) {
       int u = __ldcg(plist + i);
-      if (u < 0 || !__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
+      if (u < 0) {
         d.meta[i] = 0;
+        return -1;
+      }
+      const bool act = __ldcg(d.active + u);
+      const uint8_t pu = ld_part(d.part, u);
+      const bool hub = __ldcg(d.markH + u) == a.epF;
+      if (!act || pu != kPsi) {
+        d.meta[i] = 0;
+        return -1;
+      }
+      if (hub) {  // CTA-cooperative below; its record is kept per vertex in metav
+        d.meta[i] = kMetaHub;
         return -1;
       }
       return u;
@@ -776,6 +923,86 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
       }
     };
     foreach_vertex_s<kBlock>(d, np, get, tf, wf);
+    if (!kBlock) {  // hubs in the pseudo-partition: one CTA each
+      int* conn = s.wconn[0];
+      for (int h = blockIdx.x; h < nhp; h += gridDim.x) {
+        const int u = __ldcg(d.hubP + h);
+        if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) continue;  // uniform: placed earlier
+        const long long vwu = vert_w(d.vw, u);
+        __syncthreads();
+        for (int p = threadIdx.x; p < 256; p += blockDim.x) conn[p] = 0;
+        __syncthreads();
+        bool lb = false;
+        long long pwv = 0, dummy = 0;
+        nbrs_block(d, u, [&](const int* x, const int* w, const uint8_t* q) {
+#pragma unroll
+          for (int t = 0; t < 4; t++) {
+            if (x[t] < 0) continue;
+            if (q[t] == kPsi) {
+              lb |= x[t] < u;
+            } else {
+              atomicAdd(conn + q[t], w[t]);
+              pwv += w[t];
+            }
+          }
+        });
+        const bool blocked = __syncthreads_or(lb);
+        block_sum2(s, pwv, dummy);
+        long long bc = -1;
+        int best = -1;
+        if (!blocked) {
+          for (int p = threadIdx.x; p < k; p += blockDim.x) {
+            if (s.Wr[p] + vwu > c) continue;
+            if (better(conn[p], p, bc, best, s.Wr)) {
+              best = p;
+              bc = conn[p];
+            }
+          }
+#pragma unroll
+          for (int off = 16; off > 0; off >>= 1) {
+            long long oc = __shfl_xor_sync(0xffffffffu, bc, off);
+            int op = __shfl_xor_sync(0xffffffffu, best, off);
+            if (op >= 0 && better(oc, op, bc, best, s.Wr)) {
+              bc = oc;
+              best = op;
+            }
+          }
+          if (lane_id() == 0) {
+            s.red[warp_id()] = bc;
+            s.red[16 + warp_id()] = best;
+          }
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+          if (blocked) {
+            d.metav[u] = 0;
+          } else {
+            bc = -1;
+            best = -1;
+            for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+              int op = (int)s.red[16 + w];
+              if (op >= 0 && better(s.red[w], op, bc, best, s.Wr)) {
+                bc = s.red[w];
+                best = op;
+              }
+            }
+            bool imbal = false;
+            if (best < 0) {  // E(u) empty (Q8)
+              best = s.best0;
+              bc = conn[best];
+              imbal = true;
+            }
+            sel_cnt++;
+            scanned += __ldg(d.deg + u);
+            emit_move_v(u, best, bc, pwv, imbal);
+          }
+        }
+        __syncthreads();
+        // conn is warp 0's histogram: the warp path expects it zeroed
+        for (int p = threadIdx.x; p < 256; p += blockDim.x) conn[p] = 0;
+        __syncthreads();
+      }
+    }
     {
       long long sc = warp_sum(sel_cnt);
       if (lane_id() == 0 && sc) atomicAdd(&ctl->selected3[r3], (int)sc);
@@ -792,8 +1019,9 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
     __syncthreads();
     auto items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
       unsigned m = __ldcg(d.meta + j);
+      const int u = __ldcg(plist + j);
+      if (m == kMetaHub) m = __ldcg(d.metav + u);
       if (!(m & 0x80000000u)) return false;
-      int u = __ldcg(plist + j);
       p = (int)(m & 255u);
       d0 = (int)((m >> 8) & 255u);
       R = d0 ? (unsigned long long)u
@@ -874,6 +1102,7 @@ __device__ void run_rounds(const Dev& d, RefSmem& s, cg::grid_group& grid, long 
       int u = __ldcg(plist + j);
       if (u < 0) return;
       unsigned m = __ldcg(d.meta + j);
+      if (m == kMetaHub) m = __ldcg(d.metav + u);
       bool keep = true;
       if (m & 0x80000000u) {
         int p, d0;
@@ -962,21 +1191,24 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
   const int nA = ldv(&ctl->nA);
   const int np0 = ldv(&ctl->npsi[0]);
+  const int nhA = ldv(&ctl->nhubA);
   rr_for(np0, [&](long long i) {
     int u = __ldcg(d.psi[0] + i);
     if (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) cnt_ins++;
   });
   filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
-              counted);
+              counted, a.epA);  // hubs of A: CTA-cooperative below
+  hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
   block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
   block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
   GRID_SYNC_STAMPED(ctl, 201);
 
   // ---- F1: commit C1 + R2 expansion marks -----------------------------------
   {
-    const int nc = ldv(&ctl->ncand);
-    if (tid == 0) ctl->st[ST_FILTERED_IN] = nc;
+    const int nc = ldv(&ctl->ncand), nhC = ldv(&ctl->nhubC);
+    if (tid == 0) ctl->st[ST_FILTERED_IN] = nc + nhC;
     commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
+    hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
     // neighbours of the pseudo vertices pending since apply
     auto get = [&](long long i) {
       int u = __ldcg(d.psi[0] + i);
@@ -997,10 +1229,11 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
 
   // ---- F2: R2 filter on sigma2 ------------------------------------------------
   {
-    const int nN = ldv(&ctl->nN);
+    const int nN = ldv(&ctl->nN), nhN = ldv(&ctl->nhubN);
     long long cntN = 0;
     filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, &ctl->ncand2, d.cand2, a.epC2, scanned,
                 cntN);
+    hub_filter(d, s, d.hubN, nhN, a.epC2, &ctl->nhubC2, d.hubC2, scanned, cntN);
     block_atomic_add(&ctl->st[ST_EXPANDED], cntN, s.red);
     if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
   }
@@ -1008,9 +1241,10 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
 
   // ---- F3: commit C2 --------------------------------------------------------------
   {
-    const int nc = ldv(&ctl->ncand2);
-    if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc;
+    const int nc = ldv(&ctl->ncand2), nhC2 = ldv(&ctl->nhubC2);
+    if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc + nhC2;
     commit(d, s, a, nc, d.cand2, a.epC2, false, scanned, cut_acc);
+    hub_commit(d, s, a, d.hubC2, nhC2, a.epC2, false, scanned, cut_acc);
     flush_acc(s, ctl->Wp, k);
   }
   GRID_SYNC_STAMPED(ctl, 204);
@@ -1105,7 +1339,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   // ---- R4: rounds (Alg. 4), grid-wide (a CTA-local variant for small tails
   //      measured slower: the rounds are load-latency bound, not barrier bound)
   RoundState rs;
-  run_rounds<false>(d, s, grid, c, exact_shift_id, rs, scanned, cut_acc);
+  run_rounds<false>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc);
   const long long rounds = rs.rounds, applied_tot = rs.applied_tot, deferred_tot = rs.deferred_tot;
 
   block_atomic_add(&ctl->cut, cut_acc, s.red);
@@ -1130,6 +1364,11 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       for (int p = 0; p < k; p++) ctl->tot3[r][p] = 0;
     }
     ctl->nA = 0;
+    ctl->nhubA = 0;
+    ctl->nhubC = 0;
+    ctl->nhubN = 0;
+    ctl->nhubC2 = 0;
+    ctl->nhubP = 0;
     ctl->ncand = 0;
     ctl->ncand2 = 0;
     ctl->nN = 0;

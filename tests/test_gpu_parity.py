@@ -296,3 +296,69 @@ def test_c5_full_size_adversarial():
         if it % 3 == 2 or it == 9:
             P.compare_state(f"C5 it{it}")
     assert sum(e > 0 for e in evicted) >= 3, evicted
+
+
+def _hub_graph(seed, n=12_000, hubs=6, leaves=(1100, 3000)):
+    """Sparse random graph plus star hubs of degree > 1024 whose leaves sit
+    mostly in other parts, so hubs enter A, C1, N and the rounds."""
+    rng = np.random.default_rng(seed)
+    edges = set()
+    for u in range(n):
+        for v in rng.integers(max(0, u - 40), min(n, u + 40), size=2):
+            if u != v:
+                edges.add((min(u, int(v)), max(u, int(v))))
+    hub_ids = rng.choice(n, size=hubs, replace=False)
+    for h in hub_ids:
+        for v in rng.choice(n, size=int(rng.integers(*leaves)), replace=False):
+            if v != h:
+                edges.add((min(int(h), int(v)), max(int(h), int(v))))
+    xadj, adj = _csr(n, sorted(edges))
+    return xadj, adj, hub_ids
+
+
+def test_hub_cta_paths():
+    k = 4
+    xadj, adj, hubs = _hub_graph(7)
+    n = len(xadj) - 1
+    part = gi.block_partition(n, k)
+    for i, h in enumerate(hubs):  # hubs start in a part where few of their leaves are
+        part[h] = (part[h] + 1 + i) % k
+    P = Pair(xadj, adj, k, 0.05, part)
+    P.refine("settle")
+    P.compare_state("settle")
+    g = gi.Graph(*P.O.export_csr()[:2], None, None)
+    rng = np.random.default_rng(3)
+    for it in range(6):
+        xa, aj, _ = P.O.export_csr()
+        cur = P.O.partition()
+        live = np.nonzero(cur >= 0)[0]
+        batch, used = [], set()
+        for h in hubs:  # touch every hub: new edges to random live vertices
+            if cur[h] < 0:
+                continue
+            nb = set(aj[xa[h]:xa[h + 1]].tolist())
+            for v in rng.choice(live, size=4, replace=False):
+                key = (min(int(h), int(v)), max(int(h), int(v)))
+                if v != h and int(v) not in nb and key not in used:
+                    used.add(key)
+                    batch.append([3, int(h), int(v), 1])
+            # and delete one existing hub edge
+            if xa[h + 1] > xa[h]:
+                v = int(aj[xa[h] + it])
+                key = (min(int(h), v), max(int(h), v))
+                if key not in used:
+                    used.add(key)
+                    batch.append([0, int(h), v, 0])
+        # a couple of vertex insertions attached to hubs (pseudo neighbours of hubs)
+        base = len(cur)
+        for j in range(3):
+            batch.append([2, 0, 0, 1])
+            batch.append([3, base + j, int(hubs[j % len(hubs)]), 1])
+        b = np.array(batch, np.int32)
+        assert P.apply(b, f"hub it{it}") == 0
+        sto, stg = P.refine(f"hub it{it}")
+        P.compare_state(f"hub it{it}", full_csr=(it % 2 == 0))
+    # a hub deletion
+    assert P.apply(np.array([[1, int(hubs[0]), 0, 0]], np.int32), "hub delete") == 0
+    P.refine("hub delete")
+    P.compare_state("hub delete", full_csr=True)
