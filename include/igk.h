@@ -132,6 +132,25 @@ igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_r
 igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,
                            int64_t* first_new_id, int64_t* bad_index);
 
+/* Vertex-range sharded refinement across nranks processes (one per GPU).
+ * Every rank holds the replicated store and state (it applies the same
+ * batches); the per-round gain (the adjacency scans of the pending vertices,
+ * Alg. 4 L1-23) is split by owner = vertex ID mod nranks, and each round the
+ * selected moves are exchanged as 16-byte records {u, meta, #nbr, placed
+ * weight} through `allgather`; every rank then computes the same balanced
+ * prefix and applies all moves.  Results are identical to
+ * igk_refine on one GPU (and to the oracle).
+ * allgather(ctx, send, nsend, recv, recv_cap): collective over the ranks;
+ * send/recv are HOST buffers of 16-byte records (recv may alias send); must
+ * write the concatenation of all ranks' records in rank order to recv and
+ * return their total count (<= recv_cap), or -1 on failure (-> IGK_ENCCL). */
+typedef struct {
+  int32_t nranks, rank;
+  void* ctx;
+  int64_t (*allgather)(void* ctx, const void* send, int64_t nsend, void* recv, int64_t recv_cap);
+} igk_comm;
+igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_stats* stats);
+
 /* out[v] for v < n_total: part in [0,k), -1 = deleted, -2 = pending (in the
  * pseudo-partition between apply and refine).  cap_len too small ->
  * IGK_EINVAL with *n_total still set. */

@@ -23,7 +23,7 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine",
-           "igk_step", "igk_step_device",
+           "igk_step", "igk_step_device", "igk_refine_sharded",
            "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
            "igk_last_error", "igk_destroy"]
@@ -37,6 +37,63 @@ class Options(C.Structure):
 
 class Stats(C.Structure):
     _fields_ = [(s, C.c_int64) for s in STATS]
+
+
+ALLGATHER_FN = C.CFUNCTYPE(C.c_int64, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64)
+
+
+class Comm(C.Structure):
+    _fields_ = [("nranks", C.c_int32), ("rank", C.c_int32), ("ctx", C.c_void_p), ("allgather", ALLGATHER_FN)]
+
+
+class TorchComm:
+    """igk_comm over torch.distributed: the per-round all-gather of 16-byte
+    move records (igk_refine_sharded).  gloo moves host tensors; NCCL moves
+    device tensors.  Plumbing only: the records are produced and consumed by
+    the CUDA kernels."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist, self.group = dist, group
+        self.nranks = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.backend = dist.get_backend(group)
+        self.calls = 0
+        self._cb = ALLGATHER_FN(self._allgather)
+        self.struct = Comm(self.nranks, self.rank, None, self._cb)
+
+    def gather_records(self, recs: np.ndarray) -> np.ndarray:
+        """all ranks' (n_i, 4) int32 record arrays, concatenated in rank order"""
+        import torch
+        dev = torch.device("cuda", torch.cuda.current_device()) if self.backend == "nccl" else torch.device("cpu")
+        cnt = torch.tensor([len(recs)], dtype=torch.int64, device=dev)
+        cnts = [torch.zeros_like(cnt) for _ in range(self.nranks)]
+        self.dist.all_gather(cnts, cnt, group=self.group)
+        counts = [int(c.item()) for c in cnts]
+        mx = max(max(counts), 1)
+        buf = np.zeros((mx, 4), np.int32)
+        buf[: len(recs)] = recs
+        t = torch.from_numpy(buf).to(dev)
+        outs = [torch.empty_like(t) for _ in range(self.nranks)]
+        self.dist.all_gather(outs, t, group=self.group)
+        self.calls += 1
+        return np.concatenate([o.cpu().numpy()[:c] for o, c in zip(outs, counts)]).reshape(-1, 4)
+
+    def _allgather(self, ctx, send, nsend, recv, cap):
+        try:
+            recs = np.empty((nsend, 4), np.int32)
+            if nsend:
+                C.memmove(recs.ctypes.data, send, nsend * 16)
+            out = self.gather_records(recs)
+            if len(out) > cap:
+                return -1
+            if len(out):
+                C.memmove(recv, np.ascontiguousarray(out).ctypes.data, len(out) * 16)
+            return len(out)
+        except Exception:  # never let an exception cross the C ABI
+            import traceback
+            traceback.print_exc()
+            return -1
 
 
 class IGKError(RuntimeError):
@@ -71,6 +128,8 @@ def lib():
         L.igk_step.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
         L.igk_step_device.restype = C.c_int
         L.igk_step_device.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
+        L.igk_refine_sharded.restype = C.c_int
+        L.igk_refine_sharded.argtypes = [P, C.POINTER(Comm), C.POINTER(Stats)]
         L.igk_partition.restype = C.c_int
         L.igk_partition.argtypes = [P, i32p, i64, i64p]
         L.igk_cut_size.restype = C.c_int
@@ -150,6 +209,14 @@ class IGKGraph:
     def refine(self):
         st = Stats()
         s = lib().igk_refine(self.h, C.byref(st))
+        if s not in (OK, WIMBALANCED):
+            raise IGKError(s, self._err())
+        return s, {f: int(getattr(st, f)) for f in STATS}
+
+    def refine_sharded(self, comm: "TorchComm"):
+        """igk_refine_sharded: round gain split by owner, move records all-gathered."""
+        st = Stats()
+        s = lib().igk_refine_sharded(self.h, C.byref(comm.struct), C.byref(st))
         if s not in (OK, WIMBALANCED):
             raise IGKError(s, self._err())
         return s, {f: int(getattr(st, f)) for f in STATS}

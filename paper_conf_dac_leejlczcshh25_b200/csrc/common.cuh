@@ -49,6 +49,10 @@ struct Ctl {
   int n_ins;
   int refine_skipped;  // fused step: refine skipped because the batch was rejected
   int nph;             // phase timestamps recorded by the last kernel
+  int nrec;            // sharded round: move records emitted by this rank
+  int rs_cur;          // sharded refine: round state between host-driven launches
+  long long rs_rounds, rs_rounds_all, rs_applied, rs_deferred;
+  int rs_pending;      // pending vertices left for the next sharded round
   // ---- device-side state ----
   long long Wp[256];   // part weights
   long long tot3[3][256];  // per round (mod 3): weight of selected moves per target part

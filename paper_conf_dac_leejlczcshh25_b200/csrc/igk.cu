@@ -167,6 +167,10 @@ struct igk_graph {
   long long newid_cap = 0;
   int check = 0;
   int debug_phases = 0;
+  int4* d_rec_out = nullptr;  // sharded rounds: this rank's move records
+  int4* d_rec_in = nullptr;   //                 all ranks' records
+  int4* h_rec = nullptr;      //                 pinned host staging (out, then in)
+  long long rec_cap = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
   long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active
@@ -468,10 +472,12 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   g->smem_refine = sizeof(RefSmem);
   g->smem_step = sizeof(StepSmem);
   cudaFuncSetAttribute(k_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
+  cudaFuncSetAttribute(k_refine_sh, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
   cudaFuncSetAttribute(k_step, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_step);
   g->grid_apply = coop_grid((const void*)k_apply, 0, o.blocks_per_sm);
   g->grid_refine = coop_grid((const void*)k_refine, g->smem_refine, o.blocks_per_sm);
   g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_step, g->smem_step, o.blocks_per_sm));
+  g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_refine_sh, g->smem_refine, o.blocks_per_sm));
   if (g->grid_apply > 4096) g->grid_apply = 4096;
   g->epochA = next_epoch(g);
   *out = g;
@@ -560,6 +566,13 @@ static RefineArgs make_refine_args(igk_graph* g, int after_apply) {
   a.epA = g->epochA;
   a.after_apply = after_apply;
   return a;
+}
+
+static igk_status launch_refine_sh(igk_graph* g, const RefineArgs& a, const ShardArgs& sh) {
+  void* args[] = {(void*)&g->d, (void*)&a, (void*)&sh};
+  CK(cudaLaunchCooperativeKernel((const void*)k_refine_sh, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
+  g->launches++;
+  return IGK_OK;
 }
 
 static igk_status launch_refine(igk_graph* g, int after_apply) {
@@ -697,6 +710,63 @@ igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
   igk_status st = launch_refine(g, 0);
   if (st != IGK_OK) return st;
+  st = sync_ctl(g, 1);
+  if (st != IGK_OK) return st;
+  return finish_refine(g, stats);
+}
+
+igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_stats* stats) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (!comm || !comm->allgather || comm->nranks < 1 || comm->rank < 0 || comm->rank >= comm->nranks)
+    return fail(g, IGK_EINVAL, "bad communicator");
+  RefineArgs ra = make_refine_args(g, 0);
+  ShardArgs sh{};
+  sh.nranks = comm->nranks;
+  sh.rank = comm->rank;
+  sh.mode = kModePre;  // F0..R3 replicated on every rank
+  CK(cudaEventRecord(g->ev[0], g->stream));
+  igk_status st = launch_refine_sh(g, ra, sh);
+  if (st == IGK_OK) st = sync_ctl(g, -1);
+  while (st == IGK_OK && g->h_ctl->rs_pending > 0) {
+    const long long np = g->h_ctl->rs_pending;
+    if (np > g->rec_cap) {  // records of one round <= pending vertices
+      cudaFree(g->d_rec_out);
+      cudaFree(g->d_rec_in);
+      if (g->h_rec) cudaFreeHost(g->h_rec);
+      g->d_rec_out = g->d_rec_in = g->h_rec = nullptr;
+      g->rec_cap = 0;
+      long long cap = grow_cap(np);
+      if (cudaMalloc(&g->d_rec_out, cap * 16) != cudaSuccess || cudaMalloc(&g->d_rec_in, cap * 16) != cudaSuccess ||
+          cudaMallocHost(&g->h_rec, cap * 16) != cudaSuccess)
+        return fail(g, IGK_ENOMEM, "record buffers");
+      g->rec_cap = cap;
+    }
+    CK(cudaMemsetAsync(&g->d.ctl->nrec, 0, sizeof(int), g->stream));
+    sh.mode = kModeGain;  // this rank's share of the round gain
+    sh.out = g->d_rec_out;
+    st = launch_refine_sh(g, ra, sh);
+    if (st == IGK_OK) st = sync_ctl(g, -1);
+    if (st != IGK_OK) break;
+    const long long nout = g->h_ctl->nrec;
+    if (nout) CK(cudaMemcpy(g->h_rec, g->d_rec_out, nout * 16, cudaMemcpyDeviceToHost));
+    // the exchange: all-gather of the move records (host buffers, in place)
+    const long long tot = comm->allgather(comm->ctx, g->h_rec, nout, g->h_rec, g->rec_cap);
+    if (tot < 0 || tot > g->rec_cap) {
+      g->poisoned = true;
+      return fail(g, IGK_ENCCL, "all-gather of move records failed");
+    }
+    if (tot) CK(cudaMemcpyAsync(g->d_rec_in, g->h_rec, tot * 16, cudaMemcpyHostToDevice, g->stream));
+    sh.mode = kModeFinish;  // install remote moves, balanced prefix, apply (replicated)
+    sh.recs = g->d_rec_in;
+    sh.nrecs = tot;
+    st = launch_refine_sh(g, ra, sh);
+    if (st == IGK_OK) st = sync_ctl(g, -1);
+  }
+  if (st != IGK_OK) return st;
+  sh.mode = kModePost;
+  st = launch_refine_sh(g, ra, sh);
+  if (st != IGK_OK) return st;
+  CK(cudaEventRecord(g->ev[1], g->stream));
   st = sync_ctl(g, 1);
   if (st != IGK_OK) return st;
   return finish_refine(g, stats);
@@ -896,6 +966,9 @@ void igk_destroy(igk_graph* g) {
   if (g->d.newid) cudaFree(g->d.newid);
   if (g->d_mods) cudaFree(g->d_mods);
   if (g->h_stage) cudaFreeHost(g->h_stage);
+  if (g->d_rec_out) cudaFree(g->d_rec_out);
+  if (g->d_rec_in) cudaFree(g->d_rec_in);
+  if (g->h_rec) cudaFreeHost(g->h_rec);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
   for (auto& e : g->ev)
     if (e) cudaEventDestroy(e);

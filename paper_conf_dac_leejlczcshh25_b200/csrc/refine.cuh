@@ -28,6 +28,20 @@ struct RefineArgs {
   int after_apply;  // fused step: skip (leave the state untouched) if the batch was rejected
 };
 
+// Sharded refine: every rank holds the replicated store and
+// state; the round gain is split by owner (u mod nranks) and the selected
+// moves are all-gathered as 16-byte records {u, meta | imbal << 30, gain, pw}.
+enum RefineMode { kModeFull = 0, kModePre = 1, kModeGain = 2, kModeFinish = 3, kModePost = 4 };
+struct ShardArgs {
+  int mode;            // RefineMode
+  int nranks, rank;    // owner(u) = u mod nranks
+  const int4* recs;    // kModeFinish: all ranks' move records of this round
+  long long nrecs;
+  int4* out;           // kModeGain: this rank's move records (count in ctl->nrec)
+};
+__device__ __forceinline__ bool owned(const ShardArgs& sh, int u) { return sh.nranks <= 1 || u % sh.nranks == sh.rank; }
+#define IGK_OWNED(sh, u) (!kSh || owned(sh, u))
+
 // ---------------------------------------------------------------------------
 // neighbour iteration with several loads in flight
 // ---------------------------------------------------------------------------
@@ -732,9 +746,17 @@ struct RoundState {
   int cur = 0;
   long long rounds = 0, rounds_all = 0, applied_tot = 0, deferred_tot = 0;
 };
-template <bool kBlock>
+template <bool kBlock, bool kSh>
 __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::grid_group& grid, long long c,
-                           int exact_shift_id, RoundState& rs, long long& scanned, long long& cut_acc) {
+                           int exact_shift_id, RoundState& rs, long long& scanned, long long& cut_acc,
+                           const ShardArgs& sh_in) {
+  // kSh = false: the single-GPU kernels, all sharding code compiled out
+  ShardArgs sh = sh_in;
+  if (!kSh) {
+    sh.mode = kModeFull;
+    sh.nranks = 1;
+  }
+  const bool sharded = kSh && (sh.mode == kModeGain || sh.mode == kModeFinish);
   Ctl* ctl = d.ctl;
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -767,24 +789,29 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       s.best0 = b;
     }
     __syncthreads();
-    if (tid == 0) {
+    if (tid == 0 && (!kSh || sh.mode != kModeFinish)) {
       ctl->npsi[nxt] = 0;
       ctl->applied3[r3n] = 0;
       ctl->selected3[r3n] = 0;
     }
-    rr_for_s<kBlock>(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
     // -- gain: selection + best part, one adjacency pass per vertex
     long long sel_cnt = 0;
+    if (!kSh || sh.mode != kModeFinish) {  // (the finish kernel of a sharded round skips to the install)
+    rr_for_s<kBlock>(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
     auto emit_move = [&](long long j, int u, int best, long long g, long long pwv, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
       d.tgt[u] = (uint8_t)best;
       d.gain[u] = (int)g;
       d.pw[u] = (int)pwv;
-      d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;  // j: list position (hubs: vertex id)
+      d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;  // j: list position
       long long w = vert_w(d.vw, u);
       atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
       atomic_add_ll(&ctl->tot3[r3][best], w);
       if (imbal) ctl->st[ST_IMBAL] = 1;
+      if (sharded)
+        sh.out[atomicAdd(&ctl->nrec, 1)] =
+            make_int4(u, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)), (int)g,
+                      (int)pwv);
     };
     auto emit_move_v = [&](int u, int best, long long g, long long pwv, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
@@ -796,6 +823,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
       atomic_add_ll(&ctl->tot3[r3][best], w);
       if (imbal) ctl->st[ST_IMBAL] = 1;
+      if (sharded)
+        sh.out[atomicAdd(&ctl->nrec, 1)] =
+            make_int4(u, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)), (int)g,
+                      (int)pwv);
     };
     auto get = [&](long long i) {
       int u = __ldcg(plist + i);
@@ -808,6 +839,11 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       const bool hub = __ldcg(d.markH + u) == a.epF;
       if (!act || pu != kPsi) {
         d.meta[i] = 0;
+        return -1;
+      }
+      if (!IGK_OWNED(sh, u)) {  // another rank's vertex: its record arrives per vertex (metav)
+        d.meta[i] = kMetaHub;
+        if (!hub) d.metav[u] = 0;
         return -1;
       }
       if (hub) {  // CTA-cooperative below; its record is kept per vertex in metav
@@ -928,6 +964,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       for (int h = blockIdx.x; h < nhp; h += gridDim.x) {
         const int u = __ldcg(d.hubP + h);
         if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) continue;  // uniform: placed earlier
+        if (!IGK_OWNED(sh, u)) {  // another rank's hub: its record arrives in the finish
+          if (threadIdx.x == 0) d.metav[u] = 0;
+          continue;
+        }
         const long long vwu = vert_w(d.vw, u);
         __syncthreads();
         for (int p = threadIdx.x; p < 256; p += blockDim.x) conn[p] = 0;
@@ -1006,6 +1046,27 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     {
       long long sc = warp_sum(sel_cnt);
       if (lane_id() == 0 && sc) atomicAdd(&ctl->selected3[r3], (int)sc);
+    }
+    }  // gain
+    if (kSh && sh.mode == kModeGain) return;  // the host all-gathers the move records
+    if (kSh && sh.mode == kModeFinish) {
+      // install the other ranks' moves of this round (per vertex, metav)
+      rr_for_s<kBlock>(sh.nrecs, [&](long long r) {
+        const int4 e = sh.recs[r];
+        const int u = e.x;
+        if (IGK_OWNED(sh, u)) return;
+        const unsigned m = (unsigned)e.y & ~(1u << 30);
+        const int best = (int)(m & 255u), d0 = (int)((m >> 8) & 255u);
+        d.tgt[u] = (uint8_t)best;
+        d.gain[u] = e.z;
+        d.pw[u] = e.w;
+        d.metav[u] = m;
+        const long long w = vert_w(d.vw, u);
+        atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
+        atomic_add_ll(&ctl->tot3[r3][best], w);
+        atomicAdd(&ctl->selected3[r3], 1);
+        if ((unsigned)e.y & (1u << 30)) ctl->st[ST_IMBAL] = 1;
+      });
     }
     round_sync(208);
 
@@ -1159,11 +1220,14 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     __syncthreads();
     cur = nxt;
     rounds_all++;
+    if (kSh && sh.mode == kModeFinish) return;  // one round per sharded finish launch
   }
 
 }
 
-__device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s) {
+template <bool kSh>
+__device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s,
+                                            const ShardArgs& sh) {
   Ctl* ctl = d.ctl;
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -1188,6 +1252,31 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   stamp_phase(ctl, 200);
   arrive_stamp(d.dbg, 0);
   long long scanned = 0, counted = 0, cnt_ins = 0, cut_acc = 0;
+  auto flush_partial = [&]() {  // split (sharded) modes: per-kernel accumulators to the control block
+    block_atomic_add(&ctl->cut, cut_acc, s.red);
+    block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
+  };
+  if (kSh && (sh.mode == kModeGain || sh.mode == kModeFinish)) {  // one sharded round
+    RoundState rs;
+    rs.cur = ldv(&ctl->rs_cur);
+    rs.rounds = ldv(&ctl->rs_rounds);
+    rs.rounds_all = ldv(&ctl->rs_rounds_all);
+    rs.applied_tot = ldv(&ctl->rs_applied);
+    rs.deferred_tot = ldv(&ctl->rs_deferred);
+    run_rounds<false, kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
+    flush_partial();
+    grid.sync();  // every CTA read the round state before it is written back
+    if (tid == 0 && sh.mode == kModeFinish) {
+      ctl->rs_pending = ctl->npsi[rs.cur];
+      ctl->rs_cur = rs.cur;
+      ctl->rs_rounds = rs.rounds;
+      ctl->rs_rounds_all = rs.rounds_all;
+      ctl->rs_applied = rs.applied_tot;
+      ctl->rs_deferred = rs.deferred_tot;
+    }
+    return;
+  }
+  if (!kSh || sh.mode != kModePost) {
   // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
   const int nA = ldv(&ctl->nA);
   const int np0 = ldv(&ctl->npsi[0]);
@@ -1336,10 +1425,26 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     }
   }
 
+  if (kSh && sh.mode == kModePre) {  // sharded: the host drives the rounds
+    flush_partial();
+    if (tid == 0) {
+      ctl->rs_cur = 0;
+      ctl->rs_rounds = ctl->rs_rounds_all = ctl->rs_applied = ctl->rs_deferred = 0;
+      ctl->rs_pending = ctl->npsi[0];
+    }
+    return;
+  }
+  }  // pre-round phases
   // ---- R4: rounds (Alg. 4), grid-wide (a CTA-local variant for small tails
   //      measured slower: the rounds are load-latency bound, not barrier bound)
   RoundState rs;
-  run_rounds<false>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc);
+  if (kSh && sh.mode == kModePost) {
+    rs.rounds = ldv(&ctl->rs_rounds);
+    rs.applied_tot = ldv(&ctl->rs_applied);
+    rs.deferred_tot = ldv(&ctl->rs_deferred);
+  } else {
+    run_rounds<false, kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
+  }
   const long long rounds = rs.rounds, applied_tot = rs.applied_tot, deferred_tot = rs.deferred_tot;
 
   block_atomic_add(&ctl->cut, cut_acc, s.red);
@@ -1382,7 +1487,17 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
 __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
   cg::grid_group grid = cg::this_grid();
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  refine_body(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw));
+  ShardArgs sh{};
+  sh.mode = kModeFull;
+  sh.nranks = 1;
+  refine_body<false>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh);
+}
+
+// sharded refine: one launch per mode (pre | round gain | round finish | post)
+__global__ void __launch_bounds__(kThreads) k_refine_sh(Dev d, RefineArgs a, ShardArgs sh) {
+  cg::grid_group grid = cg::this_grid();
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  refine_body<true>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh);
 }
 
 }  // namespace igk

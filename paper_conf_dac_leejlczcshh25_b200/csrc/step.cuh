@@ -21,7 +21,10 @@ __global__ void __launch_bounds__(kThreads) k_step(Dev d, ApplyArgs aa, RefineAr
     return;
   }
   grid.sync();  // the refine starts from the complete applied state
-  refine_body(d, ra, grid, sm.rf);
+  ShardArgs sh{};
+  sh.mode = kModeFull;
+  sh.nranks = 1;
+  refine_body<false>(d, ra, grid, sm.rf, sh);
 }
 
 }  // namespace igk
