@@ -54,10 +54,15 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
+    ap.add_argument("--shard", action="store_true",
+                    help="N>1: ONE graph, round gain split over the ranks (igk_refine_sharded, strong scaling) "
+                         "instead of independent replicas")
     return ap.parse_args()
 
 
 def workload(args, rank):
+    if args.shard:
+        rank = 0  # every rank holds the same (canonical) graph
     idx = int(args.config[1:])
     cfg = dict(gi.CONFIGS[args.config])
     n = args.n or cfg["n"]
@@ -191,14 +196,20 @@ def main():
         return
     import torch
     import paper_conf_dac_leejlczcshh25_b200 as igk
+    one_gpu_test = os.environ.get("IGK_BENCH_ONE_GPU") == "1"  # plumbing test: all ranks on cuda:0 over gloo
+    if one_gpu_test:
+        local = 0
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_gpu_test:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     g, part, metis_cut, S, cfg, k, desc = workload(args, rank)
     W, K = args.warmup, args.steps
-    e2e_steps = 0 if args.profile else K
+    e2e_steps = 0 if (args.profile or args.shard) else K
     batches = [gi.next_batch(S, cfg) for _ in range(W + K + e2e_steps)]
     stream = torch.cuda.current_stream()
     G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part, device=local, stream=stream.cuda_stream)
@@ -207,9 +218,17 @@ def main():
     flush = None if args.no_flush else torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     gpu_cuts = []
     st_buf = igk.Stats()
+    comm = igk.TorchComm() if (args.shard and dist) else None
+
+    def one_step(i, b):
+        if comm is None:
+            G.step_device(dev_batches[i].data_ptr(), len(b), st_buf)  # igk_step_device: apply + refine
+            return {f: int(getattr(st_buf, f)) for f in igk.STATS}
+        G.apply_device(dev_batches[i].data_ptr(), len(b))  # replicated apply
+        return G.refine_sharded(comm)[1]  # owner-split round gain + per-round record all-gather
+
     for i in range(W):
-        G.step_device(dev_batches[i].data_ptr(), len(batches[i]), st_buf)
-        gpu_cuts.append(st_buf.cut)
+        gpu_cuts.append(one_step(i, batches[i])["cut"])
     torch.cuda.synchronize()
     if dist:
         dist.barrier()
@@ -223,9 +242,8 @@ def main():
         if flush is not None:
             flush.zero_()  # L2 flush (256 MiB > 126 MB L2), outside the timed events
         ev[i][0].record(stream)
-        s, _ = G.step_device(dev_batches[W + i].data_ptr(), len(b), st_buf)  # igk_step_device: apply + refine
+        st = one_step(W + i, b)
         ev[i][1].record(stream)
-        st = {f: int(getattr(st_buf, f)) for f in igk.STATS}
         ms = G.last_ms()
         refine_ms += ms["refine"]  # igk_step: ONE fused kernel (k_step = apply + refine)
         apply_ms += ms["apply"]
@@ -240,6 +258,8 @@ def main():
     launches = G.kernel_launches() - l0
     t_ms = sum(a.elapsed_time(b) for a, b in ev)
     t_ms, aff_all = benchdist.reduce_time_and_work(t_ms, aff, dist, "cuda")
+    if comm is not None:
+        aff_all = aff  # one shared graph: the work is not multiplied by the ranks
     value = aff_all / (t_ms / 1e3)
 
     # ---- e2e: public C ABI with HOST batches; H2D + D2H inside the timed region
@@ -294,9 +314,11 @@ def main():
         pass
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": W,
-        "ms_per_step": t_ms / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": t_ms / K, "higher_is_better": True, "scaling": "strong" if args.shard else "weak",
+        "vs_baseline": None,
         "dtype": "int32", "data": "synthetic",
-        "config": {"workload": desc, "n": g.n, "k": k, "parallelism": "replicas" if world > 1 else "single",
+        "config": {"workload": desc, "n": g.n, "k": k,
+                   "parallelism": ("sharded" if args.shard else "replicas") if world > 1 else "single",
                    "l2": "flushed between iterations (256 MiB write)" if flush is not None else "not flushed",
                    "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]]))},
         "gpu_launches": launches,

@@ -28,6 +28,8 @@ def reduce_time_and_work(t_ms: float, work: float, dist=None, device="cpu"):
     if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
         return float(t_ms), float(work)
     import torch
+    if dist.get_backend() == "gloo":
+        device = "cpu"
     t = torch.tensor([float(t_ms)], dtype=torch.float64, device=device)
     w = torch.tensor([float(work)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
