@@ -173,6 +173,12 @@ igk_status igk_export_csr(const igk_graph* g, int64_t* xadj, int64_t xadj_len, i
  * the last igk_recount, slab bump pointer and capacity (entries) */
 igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_active, int64_t* adj_entries,
                            int64_t* slab_top, int64_t* slab_cap);
+/* Store maintenance (NEXT-4): rewrite the adjacency slab densely (drops
+ * tombstones and the holes relocations leave), growing it if needed.  Also
+ * done automatically: when a batch fails validation only for capacity (vertex
+ * IDs or slab slots; nothing is modified then), the library grows the vertex
+ * arrays and/or compacts the slab and re-runs the batch once. */
+igk_status igk_compact(igk_graph* g);
 /* number of kernels this handle has launched so far (instrumentation) */
 int64_t igk_kernel_launches(const igk_graph* g);
 /* device-side duration (ms) of the last igk_refine / apply / recount kernel,

@@ -25,7 +25,7 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine",
            "igk_step", "igk_step_device", "igk_refine_sharded",
            "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
-           "igk_export_csr", "igk_store_stats", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
+           "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
            "igk_last_error", "igk_destroy"]
 
 
@@ -144,6 +144,8 @@ def lib():
         L.igk_export_csr.argtypes = [P, i64p, i64, i32p, i32p, i64, i64p, i64p]
         L.igk_store_stats.restype = C.c_int
         L.igk_store_stats.argtypes = [P, i64p, i64p, i64p, i64p, i64p]
+        L.igk_compact.restype = C.c_int
+        L.igk_compact.argtypes = [P]
         L.igk_kernel_launches.restype = i64
         L.igk_kernel_launches.argtypes = [P]
         L.igk_last_kernel_ms.restype = C.c_int
@@ -305,6 +307,11 @@ class IGKGraph:
         if s != OK:
             raise IGKError(s, self._err())
         return dict(zip(["n_total", "n_active", "adj_entries", "slab_top", "slab_cap"], [x.value for x in v]))
+
+    def compact(self):
+        s = lib().igk_compact(self.h)
+        if s != OK:
+            raise IGKError(s, self._err())
 
     def kernel_launches(self):
         return int(lib().igk_kernel_launches(self.h))

@@ -193,7 +193,10 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   }
   __syncthreads();
   const long long n_ins = s_ins[0], my_base = s_ins[1];
-  if (tid == 0 && n0 + n_ins > d.n_cap) ctl->err_nomem = 1;
+  if (tid == 0) {
+    ctl->n_ins = (int)n_ins;  // read by the host when capacity must grow
+    if (n0 + n_ins > d.n_cap) atomicOr(&ctl->err_nomem, 1);  // 1: vertex IDs exhausted
+  }
   {  // the j-th VERTEX_INSERT in batch order gets ID n0 + j
     long long base = n0 + my_base;
     for (long long t0 = c_lo; t0 < c_hi; t0 += blockDim.x) {
@@ -267,7 +270,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
           long long nc = need + max((long long)d.slack_min, need / 4);
           nc = (nc + 3) & ~3ll;
           long long no = atomicAdd((unsigned long long*)&ctl->slab_top, (unsigned long long)nc);
-          if (no + nc > d.slot_cap) ctl->err_nomem = 1;
+          if (no + nc > d.slot_cap) atomicOr(&ctl->err_nomem, 2);  // 2: adjacency slab exhausted
           pk = (no << 24) | nc;
         }
         d.reloc[x] = pk;

@@ -137,6 +137,41 @@ __global__ void __launch_bounds__(512, 2) k_recount(Dev d, long long n, long lon
     if (s_wp[p]) atomicAdd((unsigned long long*)&out_wp[p], (unsigned long long)s_wp[p]);
 }
 
+// ---------------------------------------------------------------------------
+// store maintenance: compaction of the slab into fresh arrays.
+// Relocations leave holes and tombstones stay until a prefix moves; this
+// copies every live entry to a new dense layout (warp per vertex), recording
+// old slot -> new slot, then rewrites every twin through that map.
+// ---------------------------------------------------------------------------
+__global__ void k_compact_copy(Dev d, long long n, const int64_t* noff, int32_t* nadj, int32_t* nadjw,
+                               int32_t* ntwin, int32_t* fwd) {
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long v = gw; v < n; v += nw) {
+    const long long o = d.off[v], no = noff[v];
+    const int dg = d.active[v] ? d.deg[v] : 0;
+    int wr = 0;
+    for (int b = 0; b < dg; b += 32) {
+      int j = b + lane_id();
+      int y = j < dg ? d.adj[o + j] : -1;
+      unsigned keep = __ballot_sync(0xffffffffu, y >= 0);
+      if (y >= 0) {
+        long long pos = no + wr + __popc(keep & ((1u << lane_id()) - 1u));
+        nadj[pos] = y;
+        if (nadjw) nadjw[pos] = d.adjw[o + j];
+        ntwin[pos] = d.twin[o + j];  // still an old slot: rewritten below
+        fwd[o + j] = (int32_t)pos;
+      }
+      wr += __popc(keep);
+    }
+  }
+}
+__global__ void k_compact_twins(long long used, const int32_t* nadj, int32_t* ntwin, const int32_t* fwd) {
+  for (long long s = (long long)blockIdx.x * blockDim.x + threadIdx.x; s < used;
+       s += (long long)gridDim.x * blockDim.x)
+    if (nadj[s] >= 0) ntwin[s] = fwd[ntwin[s]];
+}
+
 __global__ void k_export_part(Dev d, long long n, int32_t* out) {
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
     uint8_t p = d.part[v];
@@ -171,6 +206,7 @@ struct igk_graph {
   int4* d_rec_in = nullptr;   //                 all ranks' records
   int4* h_rec = nullptr;      //                 pinned host staging (out, then in)
   long long rec_cap = 0;
+  long long compactions = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
   long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active
@@ -255,6 +291,131 @@ igk_status sync_ctl(igk_graph* g, int which) {
     v.clear();
     for (int i = 0; i < std::min(g->h_ctl->nph, 128); i++) v.push_back({g->h_ctl->idph[i], g->h_ctl->tph[i]});
   }
+  return IGK_OK;
+}
+
+// replace *p (count_old elements of `elem` bytes) by a fresh allocation of
+// count_new elements: old content copied, the tail filled with byte `fill`
+bool regrow(igk_graph* g, void** p, size_t elem, size_t count_old, size_t count_new, int fill) {
+  void* q = nullptr;
+  if (cudaMalloc(&q, std::max<size_t>(count_new, 1) * elem) != cudaSuccess) return false;
+  if (*p && count_old) cudaMemcpyAsync(q, *p, count_old * elem, cudaMemcpyDeviceToDevice, g->stream);
+  if (count_new > count_old) cudaMemsetAsync((char*)q + count_old * elem, fill, (count_new - count_old) * elem, g->stream);
+  for (auto& a : g->allocs)
+    if (a == *p) a = q;
+  if (*p) {
+    cudaStreamSynchronize(g->stream);
+    cudaFree(*p);
+  }
+  *p = q;
+  return true;
+}
+
+// grow every per-vertex array to new_cap vertex IDs (contents kept)
+igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
+  Dev& d = g->d;
+  const size_t o = (size_t)d.n_cap, n = (size_t)new_cap;
+  struct A {
+    void** p;
+    size_t elem;
+    int fill;
+  } arrs[] = {
+      {(void**)&d.off, 8, 0},      {(void**)&d.deg, 4, 0},     {(void**)&d.ldeg, 4, 0},   {(void**)&d.capv, 4, 0},
+      {(void**)&d.active, 1, 0},   {(void**)&d.part, 1, kDel}, {(void**)&d.markA, 4, 0},  {(void**)&d.markT, 4, 0},
+      {(void**)&d.markD, 4, 0},    {(void**)&d.markG, 4, 0},   {(void**)&d.markF, 4, 0},  {(void**)&d.markH, 4, 0},
+      {(void**)&d.vcnt, 4, 0},     {(void**)&d.icnt, 4, 0},    {(void**)&d.Alist, 4, 0},  {(void**)&d.psi[0], 4, 0},
+      {(void**)&d.psi[1], 4, 0},   {(void**)&d.psi[2], 4, 0},  {(void**)&d.cand, 4, 0},   {(void**)&d.cand2, 4, 0},
+      {(void**)&d.Nlist, 4, 0},    {(void**)&d.glist, 4, 0},   {(void**)&d.dlist, 4, 0},  {(void**)&d.r3list, 8, 0},
+      {(void**)&d.reloc, 8, 0},    {(void**)&d.tgt, 1, 0},     {(void**)&d.gain, 4, 0},   {(void**)&d.pw, 4, 0},
+      {(void**)&d.meta, 4, 0},     {(void**)&d.metav, 4, 0},   {(void**)&d.oldp, 1, 0},   {(void**)&d.hubA, 4, 0},
+      {(void**)&d.hubC, 4, 0},     {(void**)&d.hubN, 4, 0},    {(void**)&d.hubC2, 4, 0},  {(void**)&d.hubP, 4, 0},
+      {(void**)&g->d_out, 4, 0},
+  };
+  for (auto& a : arrs)
+    if (!regrow(g, a.p, a.elem, o, n, a.fill)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
+  if (d.vw && !regrow(g, (void**)&d.vw, 4, o, n, 0)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
+  const size_t vdo = o + (size_t)(d.slot_cap / 32) + 1024, vdn = n + (size_t)(d.slot_cap / 32) + 1024;
+  if (!regrow(g, (void**)&d.vdch, 8, 0, vdn, 0)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
+  (void)vdo;
+  d.n_cap = new_cap;
+  int ib = 1;
+  while ((1ll << ib) < d.n_cap) ib++;
+  d.idbits = ib;
+  CK(cudaStreamSynchronize(g->stream));
+  return IGK_OK;
+}
+
+// compact the slab into fresh arrays (capacity >= min_cap); live entries only
+igk_status compact_slab(igk_graph* g, long long min_cap) {
+  Dev& d = g->d;
+  const long long n = g->h_ctl->n_total;
+  std::vector<int32_t> ldeg((size_t)std::max<long long>(n, 1));
+  std::vector<uint8_t> act((size_t)std::max<long long>(n, 1));
+  if (n) {
+    CK(cudaMemcpy(ldeg.data(), d.ldeg, n * 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(act.data(), d.active, n, cudaMemcpyDeviceToHost));
+  }
+  std::vector<int64_t> noff((size_t)std::max<long long>(n, 1));
+  std::vector<int32_t> ncap((size_t)std::max<long long>(n, 1));
+  long long used = 0;
+  for (long long v = 0; v < n; v++) {
+    long long dg = act[v] ? ldeg[v] : 0;
+    ldeg[v] = (int32_t)dg;  // deleted vertices keep no prefix
+    long long c = act[v] ? ((dg + std::max<long long>(d.slack_min, dg / 4) + 3) & ~3ll) : 0;
+    noff[v] = used;
+    ncap[v] = (int32_t)c;
+    used += c;
+  }
+  long long cap = std::max<long long>(d.slot_cap, min_cap);
+  while (cap < 2 * used + (1ll << 20)) cap *= 2;  // keep at least half free after compaction
+  cap = std::min<long long>(cap, (1ll << 31) - 2);
+  if (used > cap) return fail(g, IGK_ENOMEM, "adjacency slab cannot hold the graph");
+  int32_t *nadj = nullptr, *nadjw = nullptr, *ntwin = nullptr, *fwd = nullptr;
+  int64_t* d_noff = nullptr;
+  const long long old_top = g->h_ctl->slab_top;
+  bool ok = cudaMalloc(&nadj, cap * 4) == cudaSuccess && cudaMalloc(&ntwin, cap * 4) == cudaSuccess &&
+            (!d.adjw || cudaMalloc(&nadjw, cap * 4) == cudaSuccess) &&
+            cudaMalloc(&fwd, std::max<long long>(old_top, 1) * 4) == cudaSuccess &&
+            cudaMalloc(&d_noff, std::max<long long>(n, 1) * 8) == cudaSuccess;
+  if (!ok) {
+    cudaFree(nadj); cudaFree(ntwin); cudaFree(nadjw); cudaFree(fwd); cudaFree(d_noff);
+    return fail(g, IGK_ENOMEM, "slab compaction: allocation failed");
+  }
+  CK(cudaMemsetAsync(nadj, 0xff, cap * 4, g->stream));
+  if (n) CK(cudaMemcpyAsync(d_noff, noff.data(), n * 8, cudaMemcpyHostToDevice, g->stream));
+  int sms = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
+  k_compact_copy<<<sms * 8, 256, 0, g->stream>>>(d, n, d_noff, nadj, nadjw, ntwin, fwd);
+  k_compact_twins<<<sms * 8, 256, 0, g->stream>>>(used, nadj, ntwin, fwd);
+  g->launches += 2;
+  CK(cudaGetLastError());
+  if (n) {
+    CK(cudaMemcpyAsync(d.off, d_noff, n * 8, cudaMemcpyDeviceToDevice, g->stream));
+    CK(cudaMemcpyAsync(d.capv, ncap.data(), n * 4, cudaMemcpyHostToDevice, g->stream));
+    CK(cudaMemcpyAsync(d.deg, ldeg.data(), n * 4, cudaMemcpyHostToDevice, g->stream));  // no tombstones left
+    CK(cudaMemcpyAsync(d.ldeg, ldeg.data(), n * 4, cudaMemcpyHostToDevice, g->stream));
+  }
+  CK(cudaStreamSynchronize(g->stream));
+  int32_t* olds[3] = {d.adj, d.twin, d.adjw};
+  int32_t* news[3] = {nadj, ntwin, nadjw};
+  for (int i = 0; i < 3; i++) {
+    if (!olds[i]) continue;
+    for (auto& a : g->allocs)
+      if (a == olds[i]) a = news[i];
+    cudaFree(olds[i]);
+  }
+  d.adj = nadj;
+  d.twin = ntwin;
+  d.adjw = nadjw;
+  cudaFree(fwd);
+  cudaFree(d_noff);
+  // the vertex-deletion chunk list is sized by the slab: regrow it
+  if (!regrow(g, (void**)&d.vdch, 8, 0, (size_t)d.n_cap + (size_t)(cap / 32) + 1024, 0))
+    return fail(g, IGK_ENOMEM, "slab compaction: allocation failed");
+  d.slot_cap = cap;
+  g->h_ctl->slab_top = used;
+  CK(cudaMemcpy(&d.ctl->slab_top, &used, 8, cudaMemcpyHostToDevice));
+  g->compactions++;
   return IGK_OK;
 }
 
@@ -587,18 +748,39 @@ static igk_status launch_refine(igk_graph* g, int after_apply) {
 
 static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats);
 
+// after a capacity failure (detected in validation: nothing was mutated),
+// grow the vertex arrays and/or compact the slab so the batch can be re-run
+static igk_status make_room(igk_graph* g) {
+  const int why = g->h_ctl->err_nomem;
+  igk_status st = IGK_OK;
+  if (why & 1) {
+    long long need = g->h_ctl->n_total + g->h_ctl->n_ins;
+    if (need > kNMax) return fail(g, IGK_ENOMEM, "vertex ID space (2^30) exhausted");
+    st = grow_vertex_capacity(g, std::min<long long>(kNMax, std::max<long long>(2 * g->d.n_cap, need + 65536)));
+  }
+  if (st == IGK_OK && (why & 2)) st = compact_slab(g, 0);
+  return st;
+}
+
 static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t* first_new_id, int64_t* bad_index) {
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   if (count == 0) return IGK_OK;
-  igk_status st = launch_apply(g, dm, count);
-  if (st != IGK_OK) return st;
-  st = sync_ctl(g, 0);
-  if (st != IGK_OK) return st;
-  return finish_apply(g, bad_index);
+  for (int attempt = 0;; attempt++) {
+    igk_status st = launch_apply(g, dm, count);
+    if (st != IGK_OK) return st;
+    st = sync_ctl(g, 0);
+    if (st != IGK_OK) return st;
+    // a vertex-ID shortfall hides the slab demand of the new vertices: up to two rounds of growth
+    if (g->h_ctl->err_idx == kNoErr && g->h_ctl->err_nomem && attempt < 2) {
+      st = make_room(g);
+      if (st != IGK_OK) return st;
+      continue;
+    }
+    return finish_apply(g, bad_index);
+  }
 }
 
-// fused step: apply + refine launched back to back, one host synchronisation
 static igk_status prepare_apply(igk_graph* g, int64_t count);
 
 static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refine_stats* stats,
@@ -606,23 +788,30 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   igk_status st;
-  if (count == 0) {
-    st = launch_refine(g, 0);
+  for (int attempt = 0;; attempt++) {
+    if (count == 0) {
+      st = launch_refine(g, 0);
+      if (st != IGK_OK) return st;
+    } else {  // apply + refine in ONE persistent launch (k_step)
+      st = prepare_apply(g, count);
+      if (st != IGK_OK) return st;
+      ApplyArgs aa = make_apply_args(g, dm, count);
+      RefineArgs ra = make_refine_args(g, 1);
+      void* args[] = {(void*)&g->d, (void*)&aa, (void*)&ra};
+      CK(cudaEventRecord(g->ev[0], g->stream));
+      CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
+      g->launches++;
+      CK(cudaEventRecord(g->ev[1], g->stream));
+    }
+    st = sync_ctl(g, 1);
     if (st != IGK_OK) return st;
-  } else {  // apply + refine in ONE persistent launch (k_step)
-    st = prepare_apply(g, count);
-    if (st != IGK_OK) return st;
-    ApplyArgs aa = make_apply_args(g, dm, count);
-    RefineArgs ra = make_refine_args(g, 1);
-    void* args[] = {(void*)&g->d, (void*)&aa, (void*)&ra};
-    CK(cudaEventRecord(g->ev[0], g->stream));
-    CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
-    g->launches++;
-    CK(cudaEventRecord(g->ev[1], g->stream));
-    g->h_ctl->refine_skipped = 0;
+    if (count > 0 && g->h_ctl->err_idx == kNoErr && g->h_ctl->err_nomem && attempt < 2) {
+      st = make_room(g);  // the kernel stopped before any mutation: grow / compact, then re-run
+      if (st != IGK_OK) return st;
+      continue;
+    }
+    break;
   }
-  st = sync_ctl(g, 1);
-  if (st != IGK_OK) return st;
   if (count > 0) {
     g->ms_apply = 0;  // fused: the whole step is in ms_refine
     if (g->h_ctl->err_idx != kNoErr) {
@@ -915,6 +1104,13 @@ igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, 
 }
 
 int64_t igk_kernel_launches(const igk_graph* g) { return g ? g->launches : 0; }
+
+igk_status igk_compact(igk_graph* g) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  igk_status st = sync_ctl(g, -1);
+  if (st != IGK_OK) return st;
+  return compact_slab(g, 0);
+}
 
 igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_active, int64_t* adj_entries,
                            int64_t* slab_top, int64_t* slab_cap) {

@@ -362,3 +362,41 @@ def test_hub_cta_paths():
     assert P.apply(np.array([[1, int(hubs[0]), 0, 0]], np.int32), "hub delete") == 0
     P.refine("hub delete")
     P.compare_state("hub delete", full_csr=True)
+
+
+def test_store_maintenance_growth_and_compaction():
+    """Store maintenance (NEXT-4): a store created with almost no
+    spare vertex IDs or slab slots must grow / compact itself transparently
+    (capacity failures are detected before any mutation, then the batch is
+    re-run) and stay bit-exact with the oracle, through both the two-call and
+    the fused-step entry points and an explicit igk_compact."""
+    cfg = dict(gi.CONFIGS["C1"])
+    k = cfg["k"] if isinstance(cfg["k"], int) else cfg["k"][0]
+    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(1))
+    part, _ = gi.metis_partition(g, k)
+    deg = np.diff(g.xadj)
+    used = int((((deg + np.maximum(2, deg // 4)) + 3) & ~3).sum())
+    P = Pair(g.xadj, g.adjncy, k, cfg["eps"], part, g.vwgt, g.adjwgt, check=True,
+             max_vertices=cfg["n"] + 8, max_slots=used + 64)
+    cap0 = P.G.store_stats()["slab_cap"]
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(1)))
+    for it in range(cfg["iters"]):
+        b = gi.next_batch(S, cfg)
+        if it % 2 == 0:
+            assert P.apply(b, f"it{it}") == 0
+            P.refine(f"it{it}")
+        else:
+            assert P.O.apply(b)[0] == 0
+            so, sto = P.O.refine()
+            sg, stg, bad = P.G.step(b)
+            assert sg == so == 0 and bad == -1
+            assert sto["cut"] == stg["cut"] and sto["rounds"] == stg["rounds"]
+        P.compare_state(f"it{it}", full_csr=(it % 5 == 4))
+        if it == 10:
+            P.G.compact()
+            P.compare_state("after explicit compact", full_csr=True)
+    ss = P.G.store_stats()
+    assert ss["n_total"] > cfg["n"] + 8     # vertex arrays grew
+    assert ss["slab_cap"] > cap0            # the slab was compacted into a larger one
+    assert ss["slab_top"] <= ss["slab_cap"]
