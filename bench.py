@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--cpu-iters", type=int, default=150, help="oracle sample size (iterations)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--no-repartition", action="store_true", help="skip the METIS full-repartition comparison")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
     ap.add_argument("--shard", action="store_true",
                     help="N>1: ONE graph, round gain split over the ranks (igk_refine_sharded, strong scaling) "
@@ -157,6 +158,32 @@ def cpu_baseline(g, part, k, eps, batches, gpu_cuts, iters):
                       f"{tt:.1f}s; setup {t_setup:.1f}s excluded)",
             "ms_per_iteration": 1e3 * tt / n_it,
             "parity_cut_checked_iters": min(n_it, len(gpu_cuts)), "parity_cut_match": cut_ok}
+
+
+def full_repartition(G, k, igk_cut, ms_per_step):
+    """The metric's "cut vs full repartition": METIS k-way
+    (default options, ufactor 30 = the same 3% imbalance) from scratch on the
+    CURRENT graph (exported from the device store, deleted IDs dropped and the
+    active vertices relabelled densely), single-threaded on the host.  Reports
+    both cuts and the repartition wall time against one incremental step."""
+    xadj, adj, w = G.export_csr(sort_rows=False)
+    part = G.partition()
+    act = part >= 0
+    new_id = np.cumsum(act) - 1
+    deg = np.diff(xadj)[act]
+    cx = np.zeros(int(act.sum()) + 1, dtype=np.int64)
+    np.cumsum(deg, out=cx[1:])
+    # inactive rows are empty (I6), so the exported entries are exactly the active rows' entries
+    assert int(xadj[-1]) == int(deg.sum()), "exported CSR has entries in deleted rows"
+    ca = new_id[adj].astype(np.int32)
+    g = gi.Graph(cx, ca, None, None if (w == 1).all() else w.astype(np.int32))
+    t = time.perf_counter()
+    mpart, mcut = gi.metis_partition(g, k)
+    t_metis = time.perf_counter() - t
+    return {"igk_cut": int(igk_cut), "metis_cut": int(mcut), "cut_ratio": igk_cut / max(mcut, 1),
+            "metis_s": t_metis, "metis_vs_step": 1e3 * t_metis / ms_per_step,
+            "n_active": int(act.sum()), "how": "METIS_PartGraphKway default options (ufactor 30), 1 host core, "
+                                               "on the graph as it stands after the timed iterations"}
 
 
 def run_reference(args, rank, world):
@@ -339,6 +366,8 @@ def main():
     }
     if e2e:
         line["e2e"] = e2e
+    if not args.no_repartition and not args.profile:
+        line["full_repartition"] = full_repartition(G, k, G.cut(), t_ms / K)
     if not args.no_cpu_baseline and not args.profile:
         line["cpu_baseline"] = cpu_baseline(g, part, k, cfg["eps"], batches, gpu_cuts, args.cpu_iters)
     print(json.dumps(line), flush=True)

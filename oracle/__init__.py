@@ -47,6 +47,7 @@ def lib():
         L.ora_last_error.argtypes = [P]
         L.ora_apply.argtypes = [P, i32p, C.c_int64, i64p, i64p]
         L.ora_refine.argtypes = [P, i64p]
+        L.ora_refine_global.argtypes = [P, i64p]
         L.ora_n_total.restype = C.c_int64
         L.ora_n_total.argtypes = [P]
         L.ora_n_active.restype = C.c_int64
@@ -117,6 +118,12 @@ class Oracle:
     def refine(self):
         st = np.zeros(len(STATS), dtype=np.int64)
         s = lib().ora_refine(self.h, _p(st, C.c_int64))
+        return int(s), dict(zip(STATS, (int(x) for x in st)))
+
+    def refine_global(self):
+        """NEXT-1: every boundary vertex (adj_ext != 0) joins A, then refine."""
+        st = np.zeros(len(STATS), dtype=np.int64)
+        s = lib().ora_refine_global(self.h, _p(st, C.c_int64))
         return int(s), dict(zip(STATS, (int(x) for x in st)))
 
     @property

@@ -681,6 +681,22 @@ int ora_refine(ora_graph* g, int64_t* stats) {
   return g->last_imbalanced ? ORA_WIMBALANCED : ORA_OK;
 }
 
+/* NEXT-1 global boundary refinement: G-kway's
+ * refinement "refines all vertices on the partition boundary (i.e.,
+ * vertices with adj_ext != 0)".  Reading B1: the boundary is
+ * taken on the partition as it stands when the call is made (a pending
+ * pseudo neighbour is external, reading Q13); every boundary vertex joins
+ * the affected set A, then the ordinary refine runs (R1-R4 unchanged). */
+int ora_refine_global(ora_graph* g, int64_t* stats) {
+  for (int64_t u = 0; u < g->n; u++) {
+    if (!g->active[u] || g->part[u] == PSI) continue;
+    int64_t in, ex;
+    int_ext(g, g->part, (int32_t)u, &in, &ex);
+    if (ex != 0) g->inA[u] = 1;
+  }
+  return ora_refine(g, stats);
+}
+
 /* ------------------------------------------------------------------ */
 /* queries                                                              */
 /* ------------------------------------------------------------------ */

@@ -67,6 +67,8 @@ const char* ora_last_error(const ora_graph* g);
 int ora_apply(ora_graph* g, const int32_t* mods, int64_t count,
               int64_t* first_new_id, int64_t* bad_index);
 int ora_refine(ora_graph* g, int64_t* stats /* ORA_NSTATS, nullable */);
+/* NEXT-1: A |= every boundary vertex (adj_ext != 0), then refine */
+int ora_refine_global(ora_graph* g, int64_t* stats /* ORA_NSTATS, nullable */);
 
 int64_t ora_n_total(const ora_graph* g);
 int64_t ora_n_active(const ora_graph* g);
