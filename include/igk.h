@@ -122,6 +122,18 @@ igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, 
  * IGK_WIMBALANCED in the weighted corner case (result still valid). */
 igk_status igk_refine(igk_graph* g, igk_refine_stats* stats);
 
+/* Global boundary refinement (G-kway "refines all
+ * vertices on the partition boundary (i.e., vertices with adj_ext != 0)").
+ * Every active placed vertex with a neighbour in another part -- or a pending
+ * (pseudo) neighbour, which counts as external (reading Q13) -- joins the
+ * affected set A on the partition as it stands when the call is made (reading
+ * B1); then the ordinary refine (R1-R4) runs in the SAME kernel
+ * launch.  A from earlier applies is kept (A |= boundary).  Intended to be
+ * called periodically to undo the cut drift of many incremental iterations
+ * (P:322).  Same arguments, stats and return codes as igk_refine;
+ * stats->affected counts the boundary as affected. */
+igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats);
+
 /* One incremental iteration: igk_apply_modifiers + igk_refine fused (both
  * kernels launched back to back, one host synchronisation).  If the batch is
  * invalid, returns IGK_EINVAL exactly as igk_apply_modifiers would (nothing

@@ -22,7 +22,7 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
          "adj_entries_scanned"]
 
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
-SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine",
+SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine", "igk_refine_global",
            "igk_step", "igk_step_device", "igk_refine_sharded",
            "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
@@ -124,6 +124,8 @@ def lib():
         L.igk_apply_modifiers_device.argtypes = [P, P, i64, i64p, i64p]
         L.igk_refine.restype = C.c_int
         L.igk_refine.argtypes = [P, C.POINTER(Stats)]
+        L.igk_refine_global.restype = C.c_int
+        L.igk_refine_global.argtypes = [P, C.POINTER(Stats)]
         L.igk_step.restype = C.c_int
         L.igk_step.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
         L.igk_step_device.restype = C.c_int
@@ -211,6 +213,14 @@ class IGKGraph:
     def refine(self):
         st = Stats()
         s = lib().igk_refine(self.h, C.byref(st))
+        if s not in (OK, WIMBALANCED):
+            raise IGKError(s, self._err())
+        return s, {f: int(getattr(st, f)) for f in STATS}
+
+    def refine_global(self):
+        """igk_refine_global: the partition boundary (adj_ext != 0) joins A, then refine."""
+        st = Stats()
+        s = lib().igk_refine_global(self.h, C.byref(st))
         if s not in (OK, WIMBALANCED):
             raise IGKError(s, self._err())
         return s, {f: int(getattr(st, f)) for f in STATS}

@@ -646,7 +646,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
 }
 
 static ApplyArgs make_apply_args(igk_graph* g, const int4* dm, int64_t count);
-static RefineArgs make_refine_args(igk_graph* g, int after_apply);
+static RefineArgs make_refine_args(igk_graph* g, int after_apply, int global = 0);
 
 // capacity of the per-batch scratch (hash, new IDs)
 static igk_status prepare_apply(igk_graph* g, int64_t count) {
@@ -716,7 +716,7 @@ static ApplyArgs make_apply_args(igk_graph* g, const int4* dm, int64_t count) {
   return a;
 }
 
-static RefineArgs make_refine_args(igk_graph* g, int after_apply) {
+static RefineArgs make_refine_args(igk_graph* g, int after_apply, int global) {
   RefineArgs a;
   a.e_ppm = g->e_ppm;
   a.epC1 = next_epoch(g);
@@ -726,6 +726,7 @@ static RefineArgs make_refine_args(igk_graph* g, int after_apply) {
   a.epE = next_epoch(g);
   a.epA = g->epochA;
   a.after_apply = after_apply;
+  a.global = global;
   return a;
 }
 
@@ -736,8 +737,8 @@ static igk_status launch_refine_sh(igk_graph* g, const RefineArgs& a, const Shar
   return IGK_OK;
 }
 
-static igk_status launch_refine(igk_graph* g, int after_apply) {
-  RefineArgs a = make_refine_args(g, after_apply);
+static igk_status launch_refine(igk_graph* g, int after_apply, int global = 0) {
+  RefineArgs a = make_refine_args(g, after_apply, global);
   void* args[] = {(void*)&g->d, (void*)&a};
   CK(cudaEventRecord(g->ev[0], g->stream));
   CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
@@ -898,6 +899,15 @@ static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
 igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
   igk_status st = launch_refine(g, 0);
+  if (st != IGK_OK) return st;
+  st = sync_ctl(g, 1);
+  if (st != IGK_OK) return st;
+  return finish_refine(g, stats);
+}
+
+igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  igk_status st = launch_refine(g, 0, 1);  // boundary scan + refine: one launch
   if (st != IGK_OK) return st;
   st = sync_ctl(g, 1);
   if (st != IGK_OK) return st;

@@ -18,6 +18,7 @@
 // that yields the same prefix without sorting.
 #pragma once
 #include "common.cuh"
+#include "apply.cuh"  // mark_affected (A membership), shared with the apply
 
 namespace igk {
 
@@ -26,6 +27,7 @@ struct RefineArgs {
   uint32_t epC1, epN, epC2, epF, epE;
   uint32_t epA;     // stamp of the affected set (hubs in A carry markH == epA)
   int after_apply;  // fused step: skip (leave the state untouched) if the batch was rejected
+  int global;       // NEXT-1: the partition boundary joins A before F0 (igk_refine_global)
 };
 
 // Sharded refine: every rank holds the replicated store and
@@ -1225,6 +1227,73 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
 
 }
 
+// NEXT-1 global boundary refinement: every active placed vertex with
+// adj_ext != 0 (a pseudo neighbour is external, reading Q13) joins A on the
+// labels as they stand (reading B1).  A full-store scan: 32 consecutive
+// vertices per warp (per-vertex arrays read coalesced), each thread walks its
+// own prefix with int4 loads and stops at the first external neighbour;
+// prefixes longer than kBndHeavy are walked by the whole warp.
+constexpr int kBndHeavy = 32;
+__device__ __forceinline__ void boundary_mark(const Dev& d, uint32_t epA) {
+  const long long n = ldv(&d.ctl->n_total);
+  const int lane = lane_id();
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long base = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n; base += stride) {
+    const long long v = base + lane;
+    bool placed = false;
+    uint8_t pv = kPsi;
+    int dg = 0;
+    long long o = 0;
+    if (v < n) {
+      placed = __ldcg(d.active + v);
+      pv = ld_part(d.part, v);
+      placed = placed && pv != kPsi;
+      if (placed) {
+        dg = __ldg(d.deg + v);
+        o = __ldg(d.off + v);
+      }
+    }
+    bool bnd = false;
+    const bool heavy = placed && dg > kBndHeavy;
+    if (placed && !heavy) {
+      const int4* a4 = reinterpret_cast<const int4*>(d.adj + o);
+      for (int i = 0; i < dg && !bnd; i += 8) {  // two int4 per round trip, then 8 label gathers
+        int4 a0 = __ldg(a4 + (i >> 2));
+        int4 a1 = (i + 4 < dg) ? __ldg(a4 + (i >> 2) + 1) : make_int4(-1, -1, -1, -1);
+        const int xs[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        uint8_t qs[8];
+#pragma unroll
+        for (int t = 0; t < 8; t++) qs[t] = (i + t < dg && xs[t] >= 0) ? ld_part(d.part, xs[t]) : pv;
+#pragma unroll
+        for (int t = 0; t < 8; t++) bnd |= qs[t] != pv;
+      }
+    }
+    unsigned hm = __ballot_sync(0xffffffffu, heavy);
+    while (hm) {
+      const int src = __ffs(hm) - 1;
+      hm &= hm - 1;
+      const long long ho = __shfl_sync(0xffffffffu, o, src);
+      const int hd = __shfl_sync(0xffffffffu, dg, src);
+      const uint8_t hp = (uint8_t)__shfl_sync(0xffffffffu, (int)pv, src);
+      bool hb = false;
+      for (int b = 0; b < hd && !hb; b += 256) {
+        int x[8];
+#pragma unroll
+        for (int t = 0; t < 8; t++) {
+          int i = b + 32 * t + lane;
+          x[t] = i < hd ? __ldg(d.adj + ho + i) : -1;
+        }
+        bool e = false;
+#pragma unroll
+        for (int t = 0; t < 8; t++) e |= x[t] >= 0 && ld_part(d.part, x[t]) != hp;
+        hb = __any_sync(0xffffffffu, e);
+      }
+      if (lane == src) bnd = hb;
+    }
+    if (bnd) mark_affected(d, (int)v, epA, dg);
+  }
+}
+
 template <bool kSh>
 __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s,
                                             const ShardArgs& sh) {
@@ -1277,6 +1346,10 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     return;
   }
   if (!kSh || sh.mode != kModePost) {
+  if (!kSh && a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
+    boundary_mark(d, a.epA);
+    GRID_SYNC_STAMPED(ctl, 220);
+  }
   // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
   const int nA = ldv(&ctl->nA);
   const int np0 = ldv(&ctl->npsi[0]);

@@ -50,6 +50,14 @@ class Pair:
         assert not diff, f"{where}: stats differ (oracle, gpu): {diff}"
         return sto, stg
 
+    def refine_global(self, where=""):
+        so, sto = self.O.refine_global()
+        sg, stg = self.G.refine_global()
+        assert so == sg, where
+        diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
+        assert not diff, f"{where}: global refine stats differ (oracle, gpu): {diff}"
+        return sto, stg
+
 
 def run_stream(pair: Pair, batches, full_csr_every=0, tag=""):
     stats = []
