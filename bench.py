@@ -180,8 +180,20 @@ def full_repartition(G, k, igk_cut, ms_per_step):
     t = time.perf_counter()
     mpart, mcut = gi.metis_partition(g, k)
     t_metis = time.perf_counter() - t
+    # NEXT-1: one global boundary refinement (igk_refine_global) on the
+    # same graph -- how much of the incremental drift it recovers, and at what cost
+    import torch
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record()
+    _, gst = G.refine_global()
+    e1.record()
+    torch.cuda.synchronize()
+    gcut = G.cut()
     return {"igk_cut": int(igk_cut), "metis_cut": int(mcut), "cut_ratio": igk_cut / max(mcut, 1),
             "metis_s": t_metis, "metis_vs_step": 1e3 * t_metis / ms_per_step,
+            "global_refine": {"cut": int(gcut), "cut_ratio": gcut / max(mcut, 1), "ms": e0.elapsed_time(e1),
+                              "boundary_affected": gst["affected"], "rounds": gst["rounds"]},
             "n_active": int(act.sum()), "how": "METIS_PartGraphKway default options (ufactor 30), 1 host core, "
                                                "on the graph as it stands after the timed iterations"}
 
@@ -292,22 +304,32 @@ def main():
     # ---- e2e: public C ABI with HOST batches; H2D + D2H inside the timed region
     e2e = None
     if e2e_steps:
-        h_batches = batches[W + K:]
+        # the caller's batches live in page-locked host memory (DMA'd straight
+        # to the device by igk_step); filling them is the caller's own work
+        h_batches = []
+        for b in batches[W + K:]:
+            hb = torch.empty(b.shape, dtype=torch.int32, pin_memory=True).numpy()
+            hb[...] = b
+            h_batches.append(hb)
         torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(len(h_batches) + 1)]
         aff_e = 0
-        e0.record(stream)
-        for b in h_batches:
-            _, st, _ = G.step(b)  # igk_step: pinned staging + H2D copy, apply + refine
+        slab0 = G.store_stats()["slab_cap"]
+        evs[0].record(stream)
+        for j, b in enumerate(h_batches):
+            _, st, _ = G.step(b)  # igk_step: H2D DMA from pinned host memory, apply + refine
             G.cut()               # D2H read of the step's result
             aff_e += st["affected"]
-        e1.record(stream)
+            evs[j + 1].record(stream)
         torch.cuda.synchronize()
-        te = e0.elapsed_time(e1)
+        te = evs[0].elapsed_time(evs[-1])
+        per = [evs[j].elapsed_time(evs[j + 1]) for j in range(len(h_batches))]
         te, aff_e = benchdist.reduce_time_and_work(te, aff_e, dist, "cuda")
         e2e = {"value": aff_e / (te / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": int(np.mean([b.nbytes for b in h_batches])),
-               "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches)}
+               "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches),
+               "ms_p50": float(np.median(per)), "ms_max": float(np.max(per)),
+               "store_compacted": G.store_stats()["slab_cap"] != slab0}
 
     # ---- S9 cut/weight reduction (full store scan, HBM-bound): own roofline
     s9 = None
@@ -333,10 +355,13 @@ def main():
     if s9:
         s9.update(peak=peak, peak_kind=peak_kind, frac=s9["achieved"] / peak)
     achieved = rbytes / (refine_ms / 1e3) / 1e9 if refine_ms > 0 else 0.0
+    # batches of >= kSplitB modifiers run as k_apply + k_refine (2 launches per step)
+    split = launches >= 2 * K and comm is None
+    kname = "k_apply+k_refine (split launch, one step)" if split else "k_step (apply+refine fused)"
     traffic = None
     try:
         tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        traffic = tj.get(args.config, {}).get("k_step")
+        traffic = tj.get(args.config, {}).get("k_apply+k_refine" if split else "k_step")
     except Exception:
         pass
     line = {
@@ -349,11 +374,11 @@ def main():
                    "l2": "flushed between iterations (256 MiB write)" if flush is not None else "not flushed",
                    "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]]))},
         "gpu_launches": launches,
-        "roofline": {"kernel": "k_step (apply+refine fused)", "bound": "hbm", "achieved": achieved, "peak": peak,
+        "roofline": {"kernel": kname, "bound": "hbm", "achieved": achieved, "peak": peak,
                      "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
                      "bytes_per_launch": rbytes / K, "launch_ms": refine_ms / K,
                      "share_of_step": refine_ms / t_ms if t_ms else None},
-        "kernel_ms": {"k_step": refine_ms / K},
+        "kernel_ms": {kname.split(" ")[0]: refine_ms / K},
         "iteration": {"affected": aff / K, "rounds": float(np.mean([s["rounds"] for s in stats])),
                       "moves": float(np.mean([s["moves_applied"] for s in stats])),
                       "evicted": float(np.mean([s["evicted"] for s in stats])),

@@ -110,7 +110,10 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj,
  * n_total + j); weights in range.  Phase order: edge deletions, vertex
  * deletions, vertex insertions, edge insertions; inside a phase the batch
  * order is irrelevant.  *first_new_id (nullable) = ID of the 1st insertion.
- * mods is a HOST array. */
+ * mods is a HOST array, copied before the call returns: a page-locked
+ * buffer (cudaHostAlloc / cudaHostRegister / torch pin_memory) is DMA'd
+ * straight to the device, pageable memory through an internal pinned
+ * staging buffer. */
 igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count,
                                int64_t* first_new_id, int64_t* bad_index);
 /* Same, with mods in DEVICE memory (count entries on the handle's device). */
@@ -138,7 +141,7 @@ igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats);
  * kernels launched back to back, one host synchronisation).  If the batch is
  * invalid, returns IGK_EINVAL exactly as igk_apply_modifiers would (nothing
  * changed; the refine was skipped) and *bad_index is set.  mods is a HOST
- * array; igk_step_device takes a DEVICE array. */
+ * array (staged as in igk_apply_modifiers); igk_step_device takes a DEVICE array. */
 igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_refine_stats* stats,
                     int64_t* first_new_id, int64_t* bad_index);
 igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,

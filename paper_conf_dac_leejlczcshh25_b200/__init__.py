@@ -12,7 +12,9 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "libigk.so")
+# IGK_LIB: load another in-tree build of the same library instead (A/B timing
+# of kernel variants by tools/; the product default is libigk.so here)
+_SO = os.environ.get("IGK_LIB") or os.path.join(_HERE, "libigk.so")
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE, WIMBALANCED = 0, 1, 2, 3, 4, 5, 6
 EDGE_DELETE, VERTEX_DELETE, VERTEX_INSERT, EDGE_INSERT = 0, 1, 2, 3

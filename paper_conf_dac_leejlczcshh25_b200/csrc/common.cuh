@@ -23,6 +23,7 @@ constexpr int kThreads = 512;       // persistent-kernel block size
 constexpr int kWarps = kThreads / 32;
 constexpr int kThreadDeg = 16;      // degree <= this: one thread per vertex; above: one warp
 constexpr int kBlockDeg = 1024;     // degree > this (hubs): one whole CTA per vertex
+constexpr int kVdC = 8;            // vertex deletion: prefix entries per work item (one thread each)
 constexpr int kDigits = 256;        // radix digit bins (8-bit digits)
 constexpr long long kNoErr = 0x7fffffffffffffffLL;
 
@@ -65,7 +66,7 @@ struct Ctl {
   int ncand2;          // candidate list length (C2)
   int nN;              // expansion list length
   int ngrow;           // relocation list length
-  int ndirty;          // compaction list length
+  int nreloc;          // relocation list length
   int nr3;             // restoration candidate list length
   int nvdch;           // vertex-deletion work chunks
   int ntie;            // tie-group buffer length (round prefix select)
@@ -111,9 +112,9 @@ struct Dev {
   int32_t* cand2;
   int32_t* Nlist;
   int32_t* glist;    // grow / relocation list
-  int32_t* dlist;    // dirty list
+  int32_t* rlist;    // relocation list: first-touched vertices whose prefix moves (V2)
   int2* r3list;      // (vertex, loss) restoration candidates
-  int2* vdch;        // (vertex, chunk) work items of vertex deletions
+  int2* vdch;        // (vertex, chunk) work items of vertex deletions, kVdC entries each
   uint32_t* markF;   // frontier membership (entered Psi in this refine cycle)
   uint32_t* markH;   // hub routed to a CTA-cooperative list (epoch = the list's cycle)
   int32_t* hubA;     // hubs in A

@@ -21,6 +21,12 @@
 
 using namespace igk;
 
+// igk_step runs batches of at least this many modifiers as two launches
+// (k_apply at full occupancy + k_refine) instead of the fused k_step; the
+// fused launch wins or ties up to C3-10% batches (~56K modifiers, measured)
+constexpr long long kSplitB = 131072;
+
+
 // ---------------------------------------------------------------------------
 // create-time store build: copy every CSR row into its slab prefix
 // ---------------------------------------------------------------------------
@@ -37,15 +43,23 @@ __global__ void k_build(Dev d, const int64_t* xadj, const int32_t* adjncy, const
 }
 
 // ---------------------------------------------------------------------------
-// S9: cut / part-weight reduction, a full store scan.  One thread per
-// vertex (consecutive lanes = consecutive IDs, so the per-vertex arrays are
-// read coalesced); every prefix starts 16-byte aligned (capacities are
-// multiples of 4), so a list is read with int4 loads; vertices of degree > 64
-// are walked by the whole warp (8 loads per lane in flight).  Labels are a
-// 1-byte gather that stays in L2.  Edges are counted once (x > v).
+// S9: cut / part-weight reduction, a full store scan, HBM-bound.
+// Work unit = a warp tile of 32 consecutive vertex IDs: the per-vertex arrays
+// (active, part, deg, off) are read coalesced, one vertex per lane.  Every
+// adjacency prefix starts 16-byte aligned (capacities are multiples of 4), so
+// a prefix is a run of int4 chunks; the tile's chunks are flattened (warp
+// prefix sum of ceil(deg/4)) and dealt lane-strided, kRcU chunks per lane per
+// round trip, so a tile costs ceil(chunks / (32 kRcU)) dependent load trips
+// whatever its degree mix -- hubs of 10^4 neighbours and degree-1 leaves share
+// one schedule (no divergent per-thread loops).  A chunk's owner lane is found
+// by a 5-step shuffle search over the inclusive chunk prefix.  (Measured: a
+// variant that first reads every lane's own first chunk without the search
+// was slower, C4 282 -> 333 us.)  Labels are a
+// 1-byte gather that stays in L2.  Edges are counted once (x > v); pending
+// (psi) vertices own no cut edges and count for no part.
 // ---------------------------------------------------------------------------
-constexpr int kRcHeavy = 64;
-__global__ void __launch_bounds__(512, 2) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp,
+constexpr int kRcU = 2;  // int4 chunks per lane in flight
+__global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* out_cut, long long* out_wp,
                                                  long long* out_cnt) {
   __shared__ long long s_wp[256];
   __shared__ long long s_red[32];
@@ -55,8 +69,9 @@ __global__ void __launch_bounds__(512, 2) k_recount(Dev d, long long n, long lon
   const bool ballot_wp = d.vw == nullptr && d.k <= 32;  // unit weights: W_p by popc(ballot)
   long long cut = 0, ent = 0, nact = 0;
   long long wp_lane = 0;  // ballot mode: lane p accumulates W_p
-  const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long base = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n; base += stride) {
+  const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; base < n;
+       base += nwarps * 32) {
     const long long v = base + lane;
     bool act = false;
     uint8_t pv = kPsi;
@@ -84,48 +99,54 @@ __global__ void __launch_bounds__(512, 2) k_recount(Dev d, long long n, long lon
       acc_add(s_wp, pv, vert_w(d.vw, v));
     }
     if (!placed) dg = 0;  // pending vertices own no cut edges
-    const bool heavy = dg > kRcHeavy;
-    if (!heavy && dg > 0) {
-      const int4* a4 = reinterpret_cast<const int4*>(d.adj + o);
-      const int4* w4 = d.adjw ? reinterpret_cast<const int4*>(d.adjw + o) : nullptr;
-      for (int i = 0; i < dg; i += 8) {  // two int4 per round trip, then 8 label gathers
-        int4 a0 = __ldg(a4 + (i >> 2));
-        int4 a1 = (i + 4 < dg) ? __ldg(a4 + (i >> 2) + 1) : make_int4(-1, -1, -1, -1);
-        int4 w0 = w4 ? __ldg(w4 + (i >> 2)) : make_int4(1, 1, 1, 1);
-        int4 w1 = (w4 && i + 4 < dg) ? __ldg(w4 + (i >> 2) + 1) : make_int4(1, 1, 1, 1);
-        const int xs[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-        const int ws[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
-        uint8_t qs[8];
+    // inclusive prefix of the tile's chunk counts
+    int incl = (dg + 3) >> 2;
 #pragma unroll
-        for (int t = 0; t < 8; t++) qs[t] = (i + t < dg && xs[t] > v) ? __ldg(d.part + xs[t]) : pv;
-#pragma unroll
-        for (int t = 0; t < 8; t++)
-          if (qs[t] != kPsi && qs[t] != pv) cut += ws[t];
-      }
+    for (int sh = 1; sh < 32; sh <<= 1) {
+      int t = __shfl_up_sync(0xffffffffu, incl, sh);
+      if (lane >= sh) incl += t;
     }
-    unsigned hm = __ballot_sync(0xffffffffu, heavy);
-    while (hm) {
-      const int src = __ffs(hm) - 1;
-      hm &= hm - 1;
-      const long long hv = base + src;
-      const long long ho = __shfl_sync(0xffffffffu, o, src);
-      const int hd = __shfl_sync(0xffffffffu, dg, src);
-      const uint8_t hp = (uint8_t)__shfl_sync(0xffffffffu, (int)pv, src);
-      for (int b = 0; b < hd; b += 128) {
-        int x[4], w[4];
+    const int total = __shfl_sync(0xffffffffu, incl, 31);
+    const int excl = incl - ((dg + 3) >> 2);
+    const long long c0 = o >> 2;  // chunk index of the prefix start (off is a multiple of 4)
+    const int4* a4 = reinterpret_cast<const int4*>(d.adj);
+    const int4* w4 = reinterpret_cast<const int4*>(d.adjw);
+    for (int e0 = 0; e0 < total; e0 += 32 * kRcU) {
+      int4 xa[kRcU], wa[kRcU];
+      int vl[kRcU], pl[kRcU], rem[kRcU];
 #pragma unroll
-        for (int t = 0; t < 4; t++) {
-          int i = b + 32 * t + lane;
-          x[t] = i < hd ? __ldg(d.adj + ho + i) : -1;
-          w[t] = (i < hd && d.adjw) ? __ldg(d.adjw + ho + i) : 1;
-        }
+      for (int t = 0; t < kRcU; t++) {
+        const int e = e0 + t * 32 + lane;
+        // owner lane j = #lanes with incl <= e (uniform 5-step search)
+        int j = 0;
 #pragma unroll
-        for (int t = 0; t < 4; t++) {
-          if (x[t] > hv) {
-            uint8_t q = __ldg(d.part + x[t]);
-            if (q != kPsi && q != hp) cut += w[t];
-          }
+        for (int b = 16; b; b >>= 1) {
+          int c = __shfl_sync(0xffffffffu, incl, j + b - 1);
+          if (c <= e) j += b;
         }
+        const long long oj = __shfl_sync(0xffffffffu, c0, j);
+        const int ej = __shfl_sync(0xffffffffu, excl, j);
+        const int dj = __shfl_sync(0xffffffffu, dg, j);
+        pl[t] = __shfl_sync(0xffffffffu, (int)pv, j);
+        vl[t] = (int)(base + j);
+        const int ci = e - ej;  // chunk within the owner's prefix
+        rem[t] = e < total ? dj - 4 * ci : 0;  // live entries in this chunk (>= 4: all)
+        xa[t] = e < total ? __ldg(a4 + oj + ci) : make_int4(-1, -1, -1, -1);
+        wa[t] = (e < total && w4) ? __ldg(w4 + oj + ci) : make_int4(1, 1, 1, 1);
+      }
+      uint8_t q[kRcU][4];
+#pragma unroll
+      for (int t = 0; t < kRcU; t++) {
+        const int xs[4] = {xa[t].x, xa[t].y, xa[t].z, xa[t].w};
+#pragma unroll
+        for (int c = 0; c < 4; c++) q[t][c] = (c < rem[t] && xs[c] > vl[t]) ? __ldg(d.part + xs[c]) : (uint8_t)pl[t];
+      }
+#pragma unroll
+      for (int t = 0; t < kRcU; t++) {
+        const int ws[4] = {wa[t].x, wa[t].y, wa[t].z, wa[t].w};
+#pragma unroll
+        for (int c = 0; c < 4; c++)
+          if (q[t][c] != kPsi && q[t][c] != (uint8_t)pl[t]) cut += ws[c];
       }
     }
   }
@@ -193,6 +214,8 @@ struct igk_graph {
   uint32_t epoch = 1;   // last stamp value handed out
   uint32_t epochA = 0;  // stamp of the current affected set
   int grid_apply = 0, grid_refine = 0;
+  int grid_apply_wide = 0;   // k_apply at full occupancy (split step of large batches)
+  long long split_b = 0;     // igk_step: batches of >= split_b modifiers run k_apply + k_refine
   size_t smem_refine = 0, smem_step = 0;
   long long launches = 0;
   igk_modifier* h_stage = nullptr;  // pinned staging for host batches
@@ -274,7 +297,7 @@ igk_status launch_recount(igk_graph* g) {
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device));
   long long n = g->h_ctl->n_total;
   CK(cudaEventRecord(g->ev[4], g->stream));
-  k_recount<<<sms * 4, 512, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
+  k_recount<<<sms * 4, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
   g->launches++;
   CK(cudaGetLastError());
   CK(cudaEventRecord(g->ev[5], g->stream));
@@ -325,7 +348,7 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
       {(void**)&d.markD, 4, 0},    {(void**)&d.markG, 4, 0},   {(void**)&d.markF, 4, 0},  {(void**)&d.markH, 4, 0},
       {(void**)&d.vcnt, 4, 0},     {(void**)&d.icnt, 4, 0},    {(void**)&d.Alist, 4, 0},  {(void**)&d.psi[0], 4, 0},
       {(void**)&d.psi[1], 4, 0},   {(void**)&d.psi[2], 4, 0},  {(void**)&d.cand, 4, 0},   {(void**)&d.cand2, 4, 0},
-      {(void**)&d.Nlist, 4, 0},    {(void**)&d.glist, 4, 0},   {(void**)&d.dlist, 4, 0},  {(void**)&d.r3list, 8, 0},
+      {(void**)&d.Nlist, 4, 0},    {(void**)&d.glist, 4, 0},   {(void**)&d.rlist, 4, 0},  {(void**)&d.r3list, 8, 0},
       {(void**)&d.reloc, 8, 0},    {(void**)&d.tgt, 1, 0},     {(void**)&d.gain, 4, 0},   {(void**)&d.pw, 4, 0},
       {(void**)&d.meta, 4, 0},     {(void**)&d.metav, 4, 0},   {(void**)&d.oldp, 1, 0},   {(void**)&d.hubA, 4, 0},
       {(void**)&d.hubC, 4, 0},     {(void**)&d.hubN, 4, 0},    {(void**)&d.hubC2, 4, 0},  {(void**)&d.hubP, 4, 0},
@@ -334,7 +357,7 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
   for (auto& a : arrs)
     if (!regrow(g, a.p, a.elem, o, n, a.fill)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
   if (d.vw && !regrow(g, (void**)&d.vw, 4, o, n, 0)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
-  const size_t vdo = o + (size_t)(d.slot_cap / 32) + 1024, vdn = n + (size_t)(d.slot_cap / 32) + 1024;
+  const size_t vdo = o + (size_t)(d.slot_cap / kVdC) + 1024, vdn = n + (size_t)(d.slot_cap / kVdC) + 1024;
   if (!regrow(g, (void**)&d.vdch, 8, 0, vdn, 0)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
   (void)vdo;
   d.n_cap = new_cap;
@@ -410,7 +433,7 @@ igk_status compact_slab(igk_graph* g, long long min_cap) {
   cudaFree(fwd);
   cudaFree(d_noff);
   // the vertex-deletion chunk list is sized by the slab: regrow it
-  if (!regrow(g, (void**)&d.vdch, 8, 0, (size_t)d.n_cap + (size_t)(cap / 32) + 1024, 0))
+  if (!regrow(g, (void**)&d.vdch, 8, 0, (size_t)d.n_cap + (size_t)(cap / kVdC) + 1024, 0))
     return fail(g, IGK_ENOMEM, "slab compaction: allocation failed");
   d.slot_cap = cap;
   g->h_ctl->slab_top = used;
@@ -515,10 +538,10 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.markG, N) && dalloc(g, &d.vcnt, N) && dalloc(g, &d.icnt, N) &&
             dalloc(g, &d.Alist, N) && dalloc(g, &d.psi[0], N) && dalloc(g, &d.psi[1], N) &&
             dalloc(g, &d.psi[2], N) && dalloc(g, &d.cand, N) && dalloc(g, &d.cand2, N) &&
-            dalloc(g, &d.vdch, N + (size_t)(d.slot_cap / 32) + 1024) && dalloc(g, &d.markF, N) && dalloc(g, &d.oldp, N) && dalloc(g, &d.markH, N) &&
+            dalloc(g, &d.vdch, N + (size_t)(d.slot_cap / kVdC) + 1024) && dalloc(g, &d.markF, N) && dalloc(g, &d.oldp, N) && dalloc(g, &d.markH, N) &&
             dalloc(g, &d.hubA, N) && dalloc(g, &d.hubC, N) && dalloc(g, &d.hubN, N) && dalloc(g, &d.hubC2, N) &&
             dalloc(g, &d.hubP, N) && dalloc(g, &d.Nlist, N) && dalloc(g, &d.glist, N) &&
-            dalloc(g, &d.dlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
+            dalloc(g, &d.rlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
             dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) && dalloc(g, &d.metav, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
@@ -640,6 +663,9 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_step, g->smem_step, o.blocks_per_sm));
   g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_refine_sh, g->smem_refine, o.blocks_per_sm));
   if (g->grid_apply > 4096) g->grid_apply = 4096;
+  g->grid_apply_wide = std::min(4096, coop_grid((const void*)k_apply, 0, 64));
+  g->split_b = kSplitB;
+  if (const char* e = getenv("IGK_SPLIT_B")) g->split_b = atoll(e);
   g->epochA = next_epoch(g);
   *out = g;
   return IGK_OK;
@@ -793,6 +819,22 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
     if (count == 0) {
       st = launch_refine(g, 0);
       if (st != IGK_OK) return st;
+    } else if (count >= g->split_b) {
+      // large batch: k_apply at full occupancy (64 registers: 2x the warps
+      // of the fused kernel for its latency-bound gathers and atomics), then
+      // k_refine on the same stream -- no host round trip between them; a
+      // rejected batch makes the refine exit untouched (after_apply)
+      st = prepare_apply(g, count);
+      if (st != IGK_OK) return st;
+      ApplyArgs aa = make_apply_args(g, dm, count);
+      RefineArgs ra = make_refine_args(g, 1);
+      void* a1[] = {(void*)&g->d, (void*)&aa};
+      void* a2[] = {(void*)&g->d, (void*)&ra};
+      CK(cudaEventRecord(g->ev[0], g->stream));
+      CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply_wide, kThreads, a1, 0, g->stream));
+      CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, a2, g->smem_refine, g->stream));
+      g->launches += 2;
+      CK(cudaEventRecord(g->ev[1], g->stream));
     } else {  // apply + refine in ONE persistent launch (k_step)
       st = prepare_apply(g, count);
       if (st != IGK_OK) return st;
@@ -826,11 +868,26 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
   return finish_refine(g, stats);
 }
 
-igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count, int64_t* first_new_id,
-                               int64_t* bad_index) {
-  if (!g || g->poisoned) return IGK_ESTATE;
-  if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
-  if (count == 0) return apply_dev(g, nullptr, 0, first_new_id, bad_index);
+// host batch -> g->d_mods on the handle stream.  A page-locked caller buffer
+// (cudaHostAlloc / cudaHostRegister / torch pin_memory) is DMA'd directly;
+// pageable memory goes through the handle's pinned staging buffer.  The copy
+// is complete before the call returns (the step synchronises the stream).
+static igk_status stage_batch(igk_graph* g, const igk_modifier* mods, int64_t count) {
+  if (count > g->d_mods_cap) {
+    if (g->d_mods) cudaFree(g->d_mods);
+    g->d_mods = nullptr;
+    g->d_mods_cap = 0;
+    long long cap = grow_cap(count);
+    if (cudaMalloc(&g->d_mods, cap * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
+    g->d_mods_cap = cap;
+  }
+  cudaPointerAttributes at{};
+  const bool pinned = cudaPointerGetAttributes(&at, mods) == cudaSuccess && at.type == cudaMemoryTypeHost;
+  cudaGetLastError();  // a pageable pointer is not an error
+  if (pinned) {
+    CK(cudaMemcpyAsync(g->d_mods, mods, count * 16, cudaMemcpyHostToDevice, g->stream));
+    return IGK_OK;
+  }
   if (count > g->h_stage_cap) {
     if (g->h_stage) cudaFreeHost(g->h_stage);
     g->h_stage = nullptr;
@@ -840,16 +897,18 @@ igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t c
       return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
     g->h_stage_cap = cap;
   }
-  if (count > g->d_mods_cap) {
-    if (g->d_mods) cudaFree(g->d_mods);
-    g->d_mods = nullptr;
-    g->d_mods_cap = 0;
-    long long cap = grow_cap(count);
-    if (cudaMalloc(&g->d_mods, cap * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
-    g->d_mods_cap = cap;
-  }
   std::memcpy(g->h_stage, mods, count * sizeof(igk_modifier));
   CK(cudaMemcpyAsync(g->d_mods, g->h_stage, count * 16, cudaMemcpyHostToDevice, g->stream));
+  return IGK_OK;
+}
+
+igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count, int64_t* first_new_id,
+                               int64_t* bad_index) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
+  if (count == 0) return apply_dev(g, nullptr, 0, first_new_id, bad_index);
+  igk_status st = stage_batch(g, mods, count);
+  if (st != IGK_OK) return st;
   return apply_dev(g, g->d_mods, count, first_new_id, bad_index);
 }
 
@@ -975,26 +1034,9 @@ igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_r
                     int64_t* first_new_id, int64_t* bad_index) {
   if (!g || g->poisoned) return IGK_ESTATE;
   if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
-  if (count > g->h_stage_cap) {
-    if (g->h_stage) cudaFreeHost(g->h_stage);
-    g->h_stage = nullptr;
-    g->h_stage_cap = 0;
-    long long cap = grow_cap(count);
-    if (cudaMallocHost(&g->h_stage, cap * sizeof(igk_modifier)) != cudaSuccess)
-      return fail(g, IGK_ENOMEM, "pinned staging allocation failed");
-    g->h_stage_cap = cap;
-  }
-  if (count > g->d_mods_cap) {
-    if (g->d_mods) cudaFree(g->d_mods);
-    g->d_mods = nullptr;
-    g->d_mods_cap = 0;
-    long long cap = grow_cap(count);
-    if (cudaMalloc(&g->d_mods, cap * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
-    g->d_mods_cap = cap;
-  }
   if (count > 0) {
-    std::memcpy(g->h_stage, mods, count * sizeof(igk_modifier));
-    CK(cudaMemcpyAsync(g->d_mods, g->h_stage, count * 16, cudaMemcpyHostToDevice, g->stream));
+    igk_status st = stage_batch(g, mods, count);
+    if (st != IGK_OK) return st;
   }
   return step_dev(g, g->d_mods, count, stats, first_new_id, bad_index);
 }

@@ -14,7 +14,7 @@ import numpy as np
 import pytest
 
 import igk_inputs as gi
-from tests.parity import Pair, run_stream
+from tests.parity import COMMON, Pair, run_stream
 from tests.tinycases import random_batch, random_graph
 
 pytestmark = pytest.mark.gpu
@@ -242,9 +242,14 @@ def test_edge_cases():
         Q.compare_state(f"k254 it{it}")
 
 
-def test_fused_step_api():
+@pytest.mark.parametrize("split", ["fused", "split"])
+def test_fused_step_api(split, monkeypatch):
     """igk_step (apply + refine in one call) == oracle; an invalid batch is
-    rejected atomically and the refine is skipped."""
+    rejected atomically and the refine is skipped.  "split" forces the
+    large-batch launch pair (k_apply at full occupancy + k_refine) that
+    igk_step uses from kSplitB modifiers on."""
+    if split == "split":
+        monkeypatch.setenv("IGK_SPLIT_B", "1")  # read when the handle is created
     cfg, g, part, P = _cfg_pair("C1", 1)
     P.refine("settle")
     S = gi.Stream(g, gi.stream_seed(gi.graph_seed(1)) + 1)
@@ -276,6 +281,25 @@ def test_c4_full_size_10m():
         assert P.apply(b, f"C4 it{it}") == 0
         P.refine(f"C4 it{it}")
         P.compare_state(f"C4 it{it}")
+
+
+def test_c4_full_size_step_split_launch():
+    """C4 through igk_step: its ~280K-modifier batches take the split launch
+    (k_apply at full occupancy, then k_refine without a host round trip);
+    bit-exact with the oracle for 2 iterations."""
+    cfg, g, part, P = _cfg_pair("C4", 4, check=False)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(4)))
+    for it in range(2):
+        b = gi.next_batch(S, cfg)
+        assert len(b) >= 32768
+        assert P.O.apply(b)[0] == 0
+        so, sto = P.O.refine()
+        sg, stg, bad = P.G.step(b)
+        assert sg == so and bad == -1
+        diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
+        assert not diff, diff
+        P.compare_state(f"C4 step it{it}")
 
 
 def test_c5_full_size_adversarial():

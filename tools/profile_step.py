@@ -31,3 +31,6 @@ for it in range(iters):
     _, st, _ = G.step(gi.next_batch(S, cfg))
     print(it, "affected", st["affected"], "rounds", st["rounds"], "ms", G.last_ms())
 print("done", G.cut())
+rc = G.recount()  # S9 full-store scan (k_recount), captured by `ncu -k regex:k_recount`
+assert rc[0] == G.cut(), (rc, G.cut())
+print("recount ok", rc[0])
