@@ -253,16 +253,16 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     if (yo) {
       acty = __ldcg(d.active + m.y);
       mdy = __ldcg(d.markD + m.y);
-      dgy = __ldcg(d.deg + m.y);
-      ofy = __ldcg(d.off + m.y);
-      ldy = __ldcg(d.ldeg + m.y);
+      dgy = __ldcg(&d.vr[m.y].deg);
+      ofy = __ldcg(&d.vr[m.y].off);
+      ldy = __ldcg(&d.vr[m.y].ldeg);
     }
     if (zo) {
       actz = __ldcg(d.active + m.z);
       mdz = __ldcg(d.markD + m.z);
-      dgz = __ldcg(d.deg + m.z);
-      ofz = __ldcg(d.off + m.z);
-      ldz = __ldcg(d.ldeg + m.z);
+      dgz = __ldcg(&d.vr[m.z].deg);
+      ofz = __ldcg(&d.vr[m.z].off);
+      ldz = __ldcg(&d.vr[m.z].ldeg);
     }
     const bool yr = m.y >= 0 && m.y < d.n_cap, zr = m.z >= 0 && m.z < d.n_cap;
     if (m.x == kEdgeIns) {
@@ -325,7 +325,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
         int slot = agg_append(&ctl->ngrow, first);
         if (!first) continue;
         d.glist[slot] = x;
-        long long need = (x < n0 ? __ldcg(d.deg + x) : 0) + __ldcg(d.icnt + x);
+        long long need = (x < n0 ? __ldcg(&d.vr[x].deg) : 0) + __ldcg(d.icnt + x);
         long long have = x < n0 ? __ldcg(d.capv + x) : 0;
         long long pk = -1;
         if (need > have) {
@@ -371,13 +371,13 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     long long oa = 0;
     int da = 0, du = 0, dv = 0;
     if (ed) {
-      du = __ldcg(d.deg + m.y);
-      dv = __ldcg(d.deg + m.z);
+      du = __ldcg(&d.vr[m.y].deg);
+      dv = __ldcg(&d.vr[m.z].deg);
       if (dv < du) {
         a0 = m.z;
         b0 = m.y;
       }
-      oa = __ldcg(d.off + a0);
+      oa = __ldcg(&d.vr[a0].off);
       da = min(du, dv);
     }
     long long sa = (ed && da <= 32) ? thread_find(d.adj, oa, da, b0) : -1;
@@ -394,8 +394,8 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       int w = d.adjw ? __ldcg(d.adjw + sa) : 1;
       d.adj[sa] = -1;
       d.adj[sb] = -1;
-      atomicSub(d.ldeg + m.y, 1);
-      atomicSub(d.ldeg + m.z, 1);
+      atomicSub(&d.vr[m.y].ldeg, 1);
+      atomicSub(&d.vr[m.z].ldeg, 1);
       uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
       if (pu != kPsi && pv != kPsi && pu != pv) cut_acc -= w;
       mark_affected(d, m.y, a.epA, du);
@@ -413,17 +413,17 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     for (long long t = gwarp; t < nvd; t += nwarp) {
       const int2 ch = __ldcg(d.vdch + t);
       const int u = ch.x;
-      const long long o = __ldcg(d.off + u);
-      const int dg = __ldcg(d.deg + u);
+      const long long o = __ldcg(&d.vr[u].off);
+      const int dg = __ldcg(&d.vr[u].deg);
       const uint8_t pu = ld_part(d.part, u);
       const int j = ch.y * kVdC + lane_id();
       const int x = (lane_id() < kVdC && j < dg) ? __ldcg(d.adj + o + j) : -1;  // -1: tombstone
       const int w = (x >= 0 && d.adjw) ? __ldcg(d.adjw + o + j) : 1;
       const bool xdel = x >= 0 && __ldcg(d.markD + x) == a.epD;
-      const int dx = x >= 0 ? __ldcg(d.deg + x) : 0;
+      const int dx = x >= 0 ? __ldcg(&d.vr[x].deg) : 0;
       if (x >= 0 && !xdel) {  // the twin is u's entry in x's prefix
         d.adj[__ldcg(d.twin + o + j)] = -1;
-        atomicSub(d.ldeg + x, 1);
+        atomicSub(&d.vr[x].ldeg, 1);
       }
       if (x >= 0) {
         const uint8_t px = ld_part(d.part, x);
@@ -439,8 +439,8 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   } else rr_for(nvd, [&](long long t) {
     const int2 ch = __ldcg(d.vdch + t);
     const int u = ch.x;
-    const long long o = __ldcg(d.off + u);
-    const int dg = __ldcg(d.deg + u);
+    const long long o = __ldcg(&d.vr[u].off);
+    const int dg = __ldcg(&d.vr[u].deg);
     const uint8_t pu = ld_part(d.part, u);
     const int j0 = ch.y * kVdC;
     int x[kVdC], w[kVdC], dx[kVdC], tw[kVdC];
@@ -453,7 +453,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
 #pragma unroll
     for (int e = 0; e < kVdC; e++) {
       xdel[e] = x[e] >= 0 && __ldcg(d.markD + x[e]) == a.epD;
-      dx[e] = x[e] >= 0 ? __ldcg(d.deg + x[e]) : 0;
+      dx[e] = x[e] >= 0 ? __ldcg(&d.vr[x[e]].deg) : 0;
       tw[e] = x[e] >= 0 ? __ldcg(d.twin + o + j0 + e) : 0;
     }
 #pragma unroll
@@ -463,7 +463,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       if (pu != kPsi && px != kPsi && pu != px && (!xdel[e] || u < x[e])) cut_acc -= w[e];
       if (!xdel[e]) {  // the twin is u's entry in x's prefix
         d.adj[tw[e]] = -1;
-        atomicSub(d.ldeg + x[e], 1);
+        atomicSub(&d.vr[x[e]].ldeg, 1);
       }
     }
     bool want[kVdC];
@@ -482,8 +482,8 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
     if (m.x == kVertDel) {
-      d.deg[m.y] = 0;
-      d.ldeg[m.y] = 0;
+      d.vr[m.y].deg = 0;
+      d.vr[m.y].ldeg = 0;
       d.active[m.y] = 0;
       d.part[m.y] = kDel;
     } else if (m.x == kVertIns) {
@@ -492,11 +492,11 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       if (d.vw) d.vw[id] = m.w;
       d.part[id] = kPsi;  // Alg. 3 L2-5: straight to the pseudo-partition
       if (__ldcg(d.markG + id) != a.epG) {
-        d.deg[id] = 0;
+        d.vr[id].deg = 0;
         d.capv[id] = 0;
-        d.off[id] = 0;
+        d.vr[id].off = 0;
       }
-      d.ldeg[id] = 0;
+      d.vr[id].ldeg = 0;
       W_acc += m.w;
       int slot = agg_append(&ctl->npsi[0], true);
       d.psi[0][slot] = id;
@@ -506,7 +506,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   // every moved slot's twin is copied and the old slot's twin becomes a
   // forward mark -(new slot + 2), resolved in M4
   auto relocate = [&](int x, long long src, long long dst) {
-    const int dg = __ldcg(d.deg + x);
+    const int dg = __ldcg(&d.vr[x].deg);
     int wr = 0;
     for (int b = 0; b < dg; b += 128) {  // 4 loads per lane in flight
       int y[4], w[4], tw[4];
@@ -539,11 +539,11 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     long long no = pk >> 24;
     int nc = (int)(pk & 0xffffff);
     int wr = 0;
-    if (x < n0) wr = relocate(x, __ldcg(d.off + x), no);
+    if (x < n0) wr = relocate(x, __ldcg(&d.vr[x].off), no);
     if (lane_id() == 0) {
-      d.off[x] = no;
+      d.vr[x].off = no;
       d.capv[x] = nc;
-      d.deg[x] = wr;
+      d.vr[x].deg = wr;
       d.icnt[x] = wr;  // moved entries to fix up in M4 (icnt is free again after V2)
     }
   }
@@ -557,11 +557,11 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
     if (m.x != kEdgeIns) return;
-    int pu_pos = atomicAdd(d.deg + m.y, 1);
-    int pv_pos = atomicAdd(d.deg + m.z, 1);
-    atomicAdd(d.ldeg + m.y, 1);
-    atomicAdd(d.ldeg + m.z, 1);
-    long long su = __ldcg(d.off + m.y) + pu_pos, sv = __ldcg(d.off + m.z) + pv_pos;
+    int pu_pos = atomicAdd(&d.vr[m.y].deg, 1);
+    int pv_pos = atomicAdd(&d.vr[m.z].deg, 1);
+    atomicAdd(&d.vr[m.y].ldeg, 1);
+    atomicAdd(&d.vr[m.z].ldeg, 1);
+    long long su = __ldcg(&d.vr[m.y].off) + pu_pos, sv = __ldcg(&d.vr[m.z].off) + pv_pos;
     d.adj[su] = m.z;
     d.adj[sv] = m.y;
     d.twin[su] = (int)sv;
@@ -579,7 +579,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   // then point the partner back at the new slot (idempotent when both moved)
   for (long long t = gwarp; t < nrl; t += nwarp) {
     int x = __ldcg(d.rlist + t);
-    const long long o = __ldcg(d.off + x);
+    const long long o = __ldcg(&d.vr[x].off);
     const int cnt = __ldcg(d.icnt + x);
     for (int j = lane_id(); j < cnt; j += 32) {
       long long s = o + j;

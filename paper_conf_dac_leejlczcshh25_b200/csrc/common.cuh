@@ -81,6 +81,15 @@ struct Ctl {
 // ---------------------------------------------------------------------------
 // all device pointers of one handle, passed by value to every kernel
 // ---------------------------------------------------------------------------
+// Per-vertex store record, 16 bytes = one aligned half-sector: the fields a
+// vertex visit reads together (offset and length of its dense prefix) come
+// in ONE memory transaction instead of one cold miss per array.
+struct __align__(16) VRec {
+  int64_t off;   // slab offset of the vertex's dense prefix (multiple of 4)
+  int32_t deg;   // prefix length (live entries + tombstones, -1)
+  int32_t ldeg;  // live degree (tombstones excluded)
+};
+
 struct Dev {
   int32_t k;
   int64_t n_cap;     // vertex capacity
@@ -88,9 +97,7 @@ struct Dev {
   int32_t slack_min;
   int32_t idbits;    // bits to hold any vertex ID < n_cap
   // graph store (S0)
-  int64_t* off;      // slab offset of each vertex's dense prefix
-  int32_t* deg;      // prefix length (live entries + tombstones, -1)
-  int32_t* ldeg;     // live degree (tombstones excluded)
+  VRec* vr;          // per-vertex record: prefix offset, length, live degree (one sector)
   int32_t* capv;     // capacity
   int32_t* adj;      // neighbour IDs (-1 = tombstone)
   int32_t* twin;     // slot of the reverse entry (x -> u) of every live slot (u -> x)

@@ -34,7 +34,7 @@ __global__ void k_build(Dev d, const int64_t* xadj, const int32_t* adjncy, const
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   for (long long u = gw; u < n; u += nw) {
-    const long long s = xadj[u], e = xadj[u + 1], o = d.off[u];
+    const long long s = xadj[u], e = xadj[u + 1], o = d.vr[u].off;
     for (long long j = s + lane_id(); j < e; j += 32) {
       d.adj[o + j - s] = adjncy[j];
       if (d.adjw) d.adjw[o + j - s] = adjwgt[j];
@@ -80,8 +80,8 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
     if (v < n) {
       act = __ldg(d.active + v);
       pv = __ldg(d.part + v);
-      dg = __ldg(d.deg + v);
-      o = __ldg(d.off + v);
+      dg = __ldg(&d.vr[v].deg);
+      o = __ldg(&d.vr[v].off);
     }
     if (!act) {
       pv = kPsi;
@@ -169,8 +169,8 @@ __global__ void k_compact_copy(Dev d, long long n, const int64_t* noff, int32_t*
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   for (long long v = gw; v < n; v += nw) {
-    const long long o = d.off[v], no = noff[v];
-    const int dg = d.active[v] ? d.deg[v] : 0;
+    const long long o = d.vr[v].off, no = noff[v];
+    const int dg = d.active[v] ? d.vr[v].deg : 0;
     int wr = 0;
     for (int b = 0; b < dg; b += 32) {
       int j = b + lane_id();
@@ -281,6 +281,19 @@ long long grow_cap(long long need) {
   return c;
 }
 
+// strided copies between the packed per-vertex records and a plain array of
+// one field (host or device side)
+static cudaError_t vr_put(VRec* vr, size_t field, const void* src, size_t elem, long long n, cudaMemcpyKind kind,
+                          cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  return cudaMemcpy2DAsync((char*)vr + field, sizeof(VRec), src, elem, elem, (size_t)n, kind, s);
+}
+static cudaError_t vr_get(void* dst, const VRec* vr, size_t field, size_t elem, long long n, cudaMemcpyKind kind,
+                          cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  return cudaMemcpy2DAsync(dst, elem, (const char*)vr + field, sizeof(VRec), elem, (size_t)n, kind, s);
+}
+
 int coop_grid(const void* fn, size_t smem, int want_per_sm) {
   int dev = 0, sms = 0, occ = 0;
   cudaGetDevice(&dev);
@@ -343,7 +356,7 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
     size_t elem;
     int fill;
   } arrs[] = {
-      {(void**)&d.off, 8, 0},      {(void**)&d.deg, 4, 0},     {(void**)&d.ldeg, 4, 0},   {(void**)&d.capv, 4, 0},
+      {(void**)&d.vr, sizeof(VRec), 0},                                                        {(void**)&d.capv, 4, 0},
       {(void**)&d.active, 1, 0},   {(void**)&d.part, 1, kDel}, {(void**)&d.markA, 4, 0},  {(void**)&d.markT, 4, 0},
       {(void**)&d.markD, 4, 0},    {(void**)&d.markG, 4, 0},   {(void**)&d.markF, 4, 0},  {(void**)&d.markH, 4, 0},
       {(void**)&d.vcnt, 4, 0},     {(void**)&d.icnt, 4, 0},    {(void**)&d.Alist, 4, 0},  {(void**)&d.psi[0], 4, 0},
@@ -375,7 +388,8 @@ igk_status compact_slab(igk_graph* g, long long min_cap) {
   std::vector<int32_t> ldeg((size_t)std::max<long long>(n, 1));
   std::vector<uint8_t> act((size_t)std::max<long long>(n, 1));
   if (n) {
-    CK(cudaMemcpy(ldeg.data(), d.ldeg, n * 4, cudaMemcpyDeviceToHost));
+    CK(vr_get(ldeg.data(), d.vr, offsetof(VRec, ldeg), 4, n, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
     CK(cudaMemcpy(act.data(), d.active, n, cudaMemcpyDeviceToHost));
   }
   std::vector<int64_t> noff((size_t)std::max<long long>(n, 1));
@@ -413,10 +427,10 @@ igk_status compact_slab(igk_graph* g, long long min_cap) {
   g->launches += 2;
   CK(cudaGetLastError());
   if (n) {
-    CK(cudaMemcpyAsync(d.off, d_noff, n * 8, cudaMemcpyDeviceToDevice, g->stream));
+    CK(vr_put(d.vr, offsetof(VRec, off), d_noff, 8, n, cudaMemcpyDeviceToDevice, g->stream));
     CK(cudaMemcpyAsync(d.capv, ncap.data(), n * 4, cudaMemcpyHostToDevice, g->stream));
-    CK(cudaMemcpyAsync(d.deg, ldeg.data(), n * 4, cudaMemcpyHostToDevice, g->stream));  // no tombstones left
-    CK(cudaMemcpyAsync(d.ldeg, ldeg.data(), n * 4, cudaMemcpyHostToDevice, g->stream));
+    CK(vr_put(d.vr, offsetof(VRec, deg), ldeg.data(), 4, n, cudaMemcpyHostToDevice, g->stream));  // no tombstones left
+    CK(vr_put(d.vr, offsetof(VRec, ldeg), ldeg.data(), 4, n, cudaMemcpyHostToDevice, g->stream));
   }
   CK(cudaStreamSynchronize(g->stream));
   int32_t* olds[3] = {d.adj, d.twin, d.adjw};
@@ -530,7 +544,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     return IGK_EINVAL;
   }
   const size_t N = (size_t)d.n_cap;
-  bool ok = dalloc(g, &d.off, N) && dalloc(g, &d.deg, N) && dalloc(g, &d.ldeg, N) && dalloc(g, &d.capv, N) &&
+  bool ok = dalloc(g, &d.vr, N) && dalloc(g, &d.capv, N) &&
             dalloc(g, &d.adj, (size_t)d.slot_cap) && dalloc(g, &d.twin, (size_t)d.slot_cap) &&
             (g->ew_unit || dalloc(g, &d.adjw, (size_t)d.slot_cap)) &&
             dalloc(g, &d.active, N) && (g->vw_unit || dalloc(g, &d.vw, N)) && dalloc(g, &d.part, N) &&
@@ -559,10 +573,8 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   cudaStream_t s = g->stream;
   cudaMemsetAsync(d.active, 0, N, s);
   cudaMemsetAsync(d.part, kDel, N, s);
-  cudaMemsetAsync(d.deg, 0, N * 4, s);
-  cudaMemsetAsync(d.ldeg, 0, N * 4, s);
+  cudaMemsetAsync(d.vr, 0, N * sizeof(VRec), s);
   cudaMemsetAsync(d.capv, 0, N * 4, s);
-  cudaMemsetAsync(d.off, 0, N * 8, s);
   cudaMemsetAsync(d.markA, 0, N * 4, s);
   cudaMemsetAsync(d.markT, 0, N * 4, s);
   cudaMemsetAsync(d.markD, 0, N * 4, s);
@@ -598,10 +610,11 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     e = cudaMemcpy(d_xadj, xadj, (n + 1) * 8, cudaMemcpyHostToDevice);
     if (e == cudaSuccess && m2) e = cudaMemcpy(d_adjncy, adjncy, m2 * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess && m2 && d_adjwgt) e = cudaMemcpy(d_adjwgt, adjwgt, m2 * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(d.off, off.data(), n * 8, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, off), off.data(), 8, n, cudaMemcpyHostToDevice, s);
     if (e == cudaSuccess && used) e = cudaMemcpy(d.twin, twin_h.data(), used * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(d.deg, deg.data(), n * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(d.ldeg, deg.data(), n * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, deg), deg.data(), 4, n, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, ldeg), deg.data(), 4, n, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess) e = cudaMemcpy(d.capv, capv.data(), n * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.part, part8.data(), n, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(d.active, act.data(), n, cudaMemcpyHostToDevice);
@@ -1122,9 +1135,10 @@ igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, 
   std::vector<int64_t> off((size_t)std::max<long long>(n, 1));
   std::vector<int32_t> deg((size_t)std::max<long long>(n, 1)), ldeg((size_t)std::max<long long>(n, 1));
   if (n) {
-    CK(cudaMemcpy(off.data(), g->d.off, n * 8, cudaMemcpyDeviceToHost));
-    CK(cudaMemcpy(deg.data(), g->d.deg, n * 4, cudaMemcpyDeviceToHost));
-    CK(cudaMemcpy(ldeg.data(), g->d.ldeg, n * 4, cudaMemcpyDeviceToHost));
+    CK(vr_get(off.data(), g->d.vr, offsetof(VRec, off), 8, n, cudaMemcpyDeviceToHost, g->stream));
+    CK(vr_get(deg.data(), g->d.vr, offsetof(VRec, deg), 4, n, cudaMemcpyDeviceToHost, g->stream));
+    CK(vr_get(ldeg.data(), g->d.vr, offsetof(VRec, ldeg), 4, n, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
   }
   long long tot = 0;
   for (long long v = 0; v < n; v++) tot += ldeg[v];

@@ -52,8 +52,8 @@ __device__ __forceinline__ bool owned(const ShardArgs& sh, int u) { return sh.nr
 constexpr int kTC = 16;  // thread chunk (== kThreadDeg: one round trip per vertex)
 template <class F>
 __device__ __forceinline__ void nbrs_thread(const Dev& d, int u, F f) {
-  const long long o = __ldg(d.off + u);
-  const int dg = __ldg(d.deg + u);
+  const long long o = __ldg(&d.vr[u].off);
+  const int dg = __ldg(&d.vr[u].deg);
   for (int i = 0; i < dg; i += kTC) {
     int x[kTC], w[kTC];
     uint8_t q[kTC];
@@ -81,7 +81,7 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
 #pragma unroll
   for (int t = 0; t < C; t++) {
     unsigned mk = x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN;
-    dgx[t] = x[t] >= 0 ? __ldg(d.deg + x[t]) : 0;
+    dgx[t] = x[t] >= 0 ? __ldg(&d.vr[x[t]].deg) : 0;
     want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC;  // C1 members are pseudo on sigma2
   }
   unsigned old[C];
@@ -103,8 +103,8 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
   }
 }
 __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN, uint32_t epC) {
-  const long long o = __ldg(d.off + u);
-  const int dg = __ldg(d.deg + u);
+  const long long o = __ldg(&d.vr[u].off);
+  const int dg = __ldg(&d.vr[u].deg);
   for (int i = 0; i < dg; i += kTC) {
     int x[kTC];
     uint8_t q[kTC];
@@ -116,8 +116,8 @@ __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t e
   }
 }
 __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN, uint32_t epC) {
-  const long long o = __ldg(d.off + u);
-  const int dg = __ldg(d.deg + u);
+  const long long o = __ldg(&d.vr[u].off);
+  const int dg = __ldg(&d.vr[u].deg);
   for (int b = 0; b < dg; b += 256) {
     int x[8];
     uint8_t q[8];
@@ -134,8 +134,8 @@ __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN
 // warp: lane-strided, 8 entries per lane per round trip (256 per warp)
 template <class F>
 __device__ __forceinline__ void nbrs_warp(const Dev& d, int u, F f) {
-  const long long o = __ldg(d.off + u);
-  const int dg = __ldg(d.deg + u);
+  const long long o = __ldg(&d.vr[u].off);
+  const int dg = __ldg(&d.vr[u].deg);
   for (int b = 0; b < dg; b += 256) {
     int x[8], w[8];
     uint8_t q[8];
@@ -166,7 +166,7 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
   for (long long r0 = 0; r0 < n; r0 += per_round) {
     long long i = r0 + (long long)lane_id() * nw + gw;
     int u = i < n ? get(i) : -1;
-    int dg = u >= 0 ? __ldg(d.deg + u) : 0;
+    int dg = u >= 0 ? __ldg(&d.vr[u].deg) : 0;
     bool heavy = dg > kThreadDeg;
     if (u >= 0 && !heavy) tf(u, i);
     unsigned hm = __ballot_sync(0xffffffffu, heavy);
@@ -191,7 +191,7 @@ __device__ __forceinline__ void foreach_vertex_s(const Dev& d, long long n, Get 
   for (long long r0 = 0; r0 < n; r0 += nw * 32) {
     long long i = r0 + (long long)lane_id() * nw + gw;
     int u = i < n ? get(i) : -1;
-    int dg = u >= 0 ? __ldg(d.deg + u) : 0;
+    int dg = u >= 0 ? __ldg(&d.vr[u].deg) : 0;
     bool heavy = dg > kThreadDeg;
     if (u >= 0 && !heavy) tf(u, i);
     unsigned hm = __ballot_sync(0xffffffffu, heavy);
@@ -506,8 +506,8 @@ __device__ __forceinline__ void block_sum2(RefSmem& s, long long& a, long long& 
 // CTA-strided walk over u's prefix, 4 entries per thread per round trip
 template <class F>
 __device__ __forceinline__ void nbrs_block(const Dev& d, int u, F f) {
-  const long long o = __ldg(d.off + u);
-  const int dg = __ldg(d.deg + u);
+  const long long o = __ldg(&d.vr[u].off);
+  const int dg = __ldg(&d.vr[u].deg);
   for (int b = 0; b < dg; b += 4 * (int)blockDim.x) {
     int x[4], w[4];
     uint8_t q[4];
@@ -541,7 +541,7 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
     block_sum2(s, in, ex);
     if (threadIdx.x == 0) {
       counted++;
-      scanned += __ldg(d.deg + u);
+      scanned += __ldg(&d.vr[u].deg);
       if (ex > in) {
         d.markT[u] = ep;
         d.oldp[u] = pu;
@@ -568,7 +568,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
       if (q == pu) in += w; else ex += w;
       return true;
     });
-    scanned += __ldg(d.deg + u);
+    scanned += __ldg(&d.vr[u].deg);
     bool c = ex > in;
     if (c) {  // stamp + snapshot label: the commit reads it while labels change
       d.markT[u] = ep;
@@ -590,7 +590,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     ex = warp_sum(ex);
     if (lane_id() == 0) {
       counted++;
-      scanned += __ldg(d.deg + u);
+      scanned += __ldg(&d.vr[u].deg);
       if (ex > in) {
         d.markT[u] = ep;
         d.oldp[u] = pu;
@@ -617,8 +617,8 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
   };
   auto tf = [&](int u, long long) {
     const uint8_t pu = __ldcg(d.oldp + u);
-    const long long o = __ldg(d.off + u);
-    const int dg = __ldg(d.deg + u);
+    const long long o = __ldg(&d.vr[u].off);
+    const int dg = __ldg(&d.vr[u].deg);
     scanned += dg;
     long long del = 0;
     for (int i = 0; i < dg; i += kTC) {
@@ -651,8 +651,8 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
   };
   auto wf = [&](int u, long long) {
     const uint8_t pu = __ldcg(d.oldp + u);
-    const long long o = __ldg(d.off + u);
-    const int dg = __ldg(d.deg + u);
+    const long long o = __ldg(&d.vr[u].off);
+    const int dg = __ldg(&d.vr[u].deg);
     if (lane_id() == 0) scanned += dg;
     long long del = 0;
     for (int b = 0; b < dg; b += 256) {
@@ -718,7 +718,7 @@ __device__ void hub_commit(const Dev& d, RefSmem& s, const RefineArgs& a, const 
     });
     block_sum2(s, del, dummy);
     if (threadIdx.x == 0) {
-      scanned += __ldg(d.deg + u);
+      scanned += __ldg(&d.vr[u].deg);
       cut_acc -= del;
       atomic_add_ll(&ctl->Wp[pu], -(long long)vert_w(d.vw, u));
       d.part[u] = kPsi;
@@ -856,7 +856,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     };
     auto tf = [&](int u, long long j) {
       const long long vwu = vert_w(d.vw, u);
-      scanned += __ldg(d.deg + u);
+      scanned += __ldg(&d.vr[u].deg);
       int qs[kThreadDeg];
       int ws[kThreadDeg];
       int m = 0;
@@ -907,7 +907,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     auto wf = [&](int u, long long j) {
       const long long vwu = vert_w(d.vw, u);
       int* wc = s.wconn[warp_id()];
-      if (lane_id() == 0) scanned += __ldg(d.deg + u);
+      if (lane_id() == 0) scanned += __ldg(&d.vr[u].deg);
       bool lb = false;
       long long pwv = 0;
       nbrs_warp(d, u, [&](int x, int w, uint8_t q) {
@@ -1035,7 +1035,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
               imbal = true;
             }
             sel_cnt++;
-            scanned += __ldg(d.deg + u);
+            scanned += __ldg(&d.vr[u].deg);
             emit_move_v(u, best, bc, pwv, imbal);
           }
         }
@@ -1249,8 +1249,8 @@ __device__ __forceinline__ void boundary_mark(const Dev& d, uint32_t epA) {
       pv = ld_part(d.part, v);
       placed = placed && pv != kPsi;
       if (placed) {
-        dg = __ldg(d.deg + v);
-        o = __ldg(d.off + v);
+        dg = __ldg(&d.vr[v].deg);
+        o = __ldg(&d.vr[v].off);
       }
     }
     bool bnd = false;
@@ -1377,11 +1377,11 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       return (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) ? u : -1;  // C1 joins beyond np0
     };
     auto mt = [&](int u, long long) {
-      scanned += __ldg(d.deg + u);
+      scanned += __ldg(&d.vr[u].deg);
       mark_nbrs_thread(d, u, a.epN, a.epC1);
     };
     auto mw = [&](int u, long long) {
-      if (lane_id() == 0) scanned += __ldg(d.deg + u);
+      if (lane_id() == 0) scanned += __ldg(&d.vr[u].deg);
       mark_nbrs_warp(d, u, a.epN, a.epC1);
     };
     foreach_vertex(d, np0, get, mt, mw);
@@ -1442,7 +1442,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
           if (q == pv) in += w; else ex += w;
           return true;
         });
-        scanned += __ldg(d.deg + v);
+        scanned += __ldg(&d.vr[v].deg);
         emit(v, pv, in - ex);
       };
       auto wf = [&](int v, long long) {
@@ -1454,7 +1454,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         in = warp_sum(in);
         ex = warp_sum(ex);
         if (lane_id() == 0) {
-          scanned += __ldg(d.deg + v);
+          scanned += __ldg(&d.vr[v].deg);
           emit(v, pv, in - ex);
         }
       };
