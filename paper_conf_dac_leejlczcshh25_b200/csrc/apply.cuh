@@ -253,16 +253,18 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     if (yo) {
       acty = __ldcg(d.active + m.y);
       mdy = __ldcg(d.markD + m.y);
-      dgy = __ldcg(&d.vr[m.y].deg);
-      ofy = __ldcg(&d.vr[m.y].off);
-      ldy = __ldcg(&d.vr[m.y].ldeg);
+      const longlong2 r = __ldcg(reinterpret_cast<const longlong2*>(d.vr + m.y));  // one 16-byte record
+      ofy = r.x;
+      dgy = (int)(unsigned)(unsigned long long)r.y;
+      ldy = (int)(r.y >> 32);
     }
     if (zo) {
       actz = __ldcg(d.active + m.z);
       mdz = __ldcg(d.markD + m.z);
-      dgz = __ldcg(&d.vr[m.z].deg);
-      ofz = __ldcg(&d.vr[m.z].off);
-      ldz = __ldcg(&d.vr[m.z].ldeg);
+      const longlong2 r = __ldcg(reinterpret_cast<const longlong2*>(d.vr + m.z));  // one 16-byte record
+      ofz = r.x;
+      dgz = (int)(unsigned)(unsigned long long)r.y;
+      ldz = (int)(r.y >> 32);
     }
     const bool yr = m.y >= 0 && m.y < d.n_cap, zr = m.z >= 0 && m.z < d.n_cap;
     if (m.x == kEdgeIns) {
@@ -413,8 +415,9 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     for (long long t = gwarp; t < nvd; t += nwarp) {
       const int2 ch = __ldcg(d.vdch + t);
       const int u = ch.x;
-      const long long o = __ldcg(&d.vr[u].off);
-      const int dg = __ldcg(&d.vr[u].deg);
+      long long o;
+      int dg;
+      vr_ldcg(d, u, o, dg);
       const uint8_t pu = ld_part(d.part, u);
       const int j = ch.y * kVdC + lane_id();
       const int x = (lane_id() < kVdC && j < dg) ? __ldcg(d.adj + o + j) : -1;  // -1: tombstone
@@ -439,8 +442,9 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   } else rr_for(nvd, [&](long long t) {
     const int2 ch = __ldcg(d.vdch + t);
     const int u = ch.x;
-    const long long o = __ldcg(&d.vr[u].off);
-    const int dg = __ldcg(&d.vr[u].deg);
+    long long o;
+    int dg;
+    vr_ldcg(d, u, o, dg);
     const uint8_t pu = ld_part(d.part, u);
     const int j0 = ch.y * kVdC;
     int x[kVdC], w[kVdC], dx[kVdC], tw[kVdC];

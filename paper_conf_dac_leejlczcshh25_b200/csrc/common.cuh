@@ -157,6 +157,19 @@ __device__ __forceinline__ long long ldv(const long long* p) { return *(volatile
 __device__ __forceinline__ int ldv(const int* p) { return *(volatile const int*)p; }
 __device__ __forceinline__ uint8_t ld_part(const uint8_t* p, int64_t i) { return __ldcg(p + i); }
 
+// one 16-byte load of a vertex record's (offset, prefix length): read-only
+// path (__ldg) and L2-coherent path (__ldcg, for fields written in-kernel)
+__device__ __forceinline__ void vr_ld(const Dev& d, int64_t u, long long& o, int& dg) {
+  const longlong2 r = __ldg(reinterpret_cast<const longlong2*>(d.vr + u));
+  o = r.x;
+  dg = (int)(unsigned)(unsigned long long)r.y;
+}
+__device__ __forceinline__ void vr_ldcg(const Dev& d, int64_t u, long long& o, int& dg) {
+  const longlong2 r = __ldcg(reinterpret_cast<const longlong2*>(d.vr + u));
+  o = r.x;
+  dg = (int)(unsigned)(unsigned long long)r.y;
+}
+
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
 

@@ -78,10 +78,9 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
     int dg = 0;
     long long o = 0;
     if (v < n) {
-      act = __ldg(d.active + v);
       pv = __ldg(d.part + v);
-      dg = __ldg(&d.vr[v].deg);
-      o = __ldg(&d.vr[v].off);
+      act = pv != kDel;  // the label doubles as the active flag
+      vr_ld(d, v, o, dg);
     }
     if (!act) {
       pv = kPsi;

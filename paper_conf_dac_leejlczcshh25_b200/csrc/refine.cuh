@@ -52,8 +52,9 @@ __device__ __forceinline__ bool owned(const ShardArgs& sh, int u) { return sh.nr
 constexpr int kTC = 16;  // thread chunk (== kThreadDeg: one round trip per vertex)
 template <class F>
 __device__ __forceinline__ void nbrs_thread(const Dev& d, int u, F f) {
-  const long long o = __ldg(&d.vr[u].off);
-  const int dg = __ldg(&d.vr[u].deg);
+  long long o;
+  int dg;
+  vr_ld(d, u, o, dg);
   for (int i = 0; i < dg; i += kTC) {
     int x[kTC], w[kTC];
     uint8_t q[kTC];
@@ -103,8 +104,9 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
   }
 }
 __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN, uint32_t epC) {
-  const long long o = __ldg(&d.vr[u].off);
-  const int dg = __ldg(&d.vr[u].deg);
+  long long o;
+  int dg;
+  vr_ld(d, u, o, dg);
   for (int i = 0; i < dg; i += kTC) {
     int x[kTC];
     uint8_t q[kTC];
@@ -116,8 +118,9 @@ __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t e
   }
 }
 __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN, uint32_t epC) {
-  const long long o = __ldg(&d.vr[u].off);
-  const int dg = __ldg(&d.vr[u].deg);
+  long long o;
+  int dg;
+  vr_ld(d, u, o, dg);
   for (int b = 0; b < dg; b += 256) {
     int x[8];
     uint8_t q[8];
@@ -134,8 +137,9 @@ __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN
 // warp: lane-strided, 8 entries per lane per round trip (256 per warp)
 template <class F>
 __device__ __forceinline__ void nbrs_warp(const Dev& d, int u, F f) {
-  const long long o = __ldg(&d.vr[u].off);
-  const int dg = __ldg(&d.vr[u].deg);
+  long long o;
+  int dg;
+  vr_ld(d, u, o, dg);
   for (int b = 0; b < dg; b += 256) {
     int x[8], w[8];
     uint8_t q[8];
@@ -506,8 +510,9 @@ __device__ __forceinline__ void block_sum2(RefSmem& s, long long& a, long long& 
 // CTA-strided walk over u's prefix, 4 entries per thread per round trip
 template <class F>
 __device__ __forceinline__ void nbrs_block(const Dev& d, int u, F f) {
-  const long long o = __ldg(&d.vr[u].off);
-  const int dg = __ldg(&d.vr[u].deg);
+  long long o;
+  int dg;
+  vr_ld(d, u, o, dg);
   for (int b = 0; b < dg; b += 4 * (int)blockDim.x) {
     int x[4], w[4];
     uint8_t q[4];
@@ -527,9 +532,8 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
                            int32_t* hout, long long& scanned, long long& counted) {
   for (int h = blockIdx.x; h < nh; h += gridDim.x) {
     const int u = __ldcg(hubs + h);
-    if (!__ldcg(d.active + u)) continue;  // uniform over the CTA
-    const uint8_t pu = ld_part(d.part, u);
-    if (pu == kPsi) continue;
+    const uint8_t pu = ld_part(d.part, u);  // deleted vertices carry kDel (== !active)
+    if (pu == kDel || pu == kPsi) continue;  // uniform over the CTA
     long long in = 0, ex = 0;
     nbrs_block(d, u, [&](const int* x, const int* w, const uint8_t* q) {
 #pragma unroll
@@ -558,8 +562,8 @@ template <class Get>
 __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, uint32_t ep,
                             long long& scanned, long long& counted, uint32_t hub_ep = 0) {
   auto tf = [&](int u, long long) {
-    const bool act = __ldcg(d.active + u);
     const uint8_t pu = ld_part(d.part, u);
+    const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
     if (!act || hub || pu == kPsi) return;
     counted++;
@@ -578,8 +582,8 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     if (c) cand[slot] = u;
   };
   auto wf = [&](int u, long long) {
-    const bool act = __ldcg(d.active + u);
     const uint8_t pu = ld_part(d.part, u);
+    const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
     if (!act || hub || pu == kPsi) return;
     long long in = 0, ex = 0;
@@ -617,8 +621,9 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
   };
   auto tf = [&](int u, long long) {
     const uint8_t pu = __ldcg(d.oldp + u);
-    const long long o = __ldg(&d.vr[u].off);
-    const int dg = __ldg(&d.vr[u].deg);
+    long long o;
+    int dg;
+    vr_ld(d, u, o, dg);
     scanned += dg;
     long long del = 0;
     for (int i = 0; i < dg; i += kTC) {
@@ -651,8 +656,9 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
   };
   auto wf = [&](int u, long long) {
     const uint8_t pu = __ldcg(d.oldp + u);
-    const long long o = __ldg(&d.vr[u].off);
-    const int dg = __ldg(&d.vr[u].deg);
+    long long o;
+    int dg;
+    vr_ld(d, u, o, dg);
     if (lane_id() == 0) scanned += dg;
     long long del = 0;
     for (int b = 0; b < dg; b += 256) {
@@ -836,8 +842,8 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         d.meta[i] = 0;
         return -1;
       }
-      const bool act = __ldcg(d.active + u);
       const uint8_t pu = ld_part(d.part, u);
+      const bool act = pu != kDel;  // the label doubles as the active flag
       const bool hub = __ldcg(d.markH + u) == a.epF;
       if (!act || pu != kPsi) {
         d.meta[i] = 0;
@@ -965,7 +971,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       int* conn = s.wconn[0];
       for (int h = blockIdx.x; h < nhp; h += gridDim.x) {
         const int u = __ldcg(d.hubP + h);
-        if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) continue;  // uniform: placed earlier
+        if (ld_part(d.part, u) != kPsi) continue;  // uniform: placed earlier (or deleted)
         if (!IGK_OWNED(sh, u)) {  // another rank's hub: its record arrives in the finish
           if (threadIdx.x == 0) d.metav[u] = 0;
           continue;
@@ -1179,7 +1185,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
           cut_acc += (long long)__ldcg(d.pw + u) - __ldcg(d.gain + u);  // independent set: exact
           app++;
         }
-      } else if (!__ldcg(d.active + u) || ld_part(d.part, u) != kPsi) {
+      } else if (ld_part(d.part, u) != kPsi) {
         keep = false;  // stale entry (deleted before this refine)
       }
       int slot = agg_append(&ctl->npsi[nxt], keep);
@@ -1245,12 +1251,10 @@ __device__ __forceinline__ void boundary_mark(const Dev& d, uint32_t epA) {
     int dg = 0;
     long long o = 0;
     if (v < n) {
-      placed = __ldcg(d.active + v);
       pv = ld_part(d.part, v);
-      placed = placed && pv != kPsi;
+      placed = pv != kDel && pv != kPsi;
       if (placed) {
-        dg = __ldg(&d.vr[v].deg);
-        o = __ldg(&d.vr[v].off);
+        vr_ld(d, v, o, dg);
       }
     }
     bool bnd = false;
@@ -1356,7 +1360,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   const int nhA = ldv(&ctl->nhubA);
   rr_for(np0, [&](long long i) {
     int u = __ldcg(d.psi[0] + i);
-    if (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) cnt_ins++;
+    if (ld_part(d.part, u) == kPsi) cnt_ins++;
   });
   filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
               counted, a.epA);  // hubs of A: CTA-cooperative below
@@ -1374,7 +1378,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     // neighbours of the pseudo vertices pending since apply
     auto get = [&](long long i) {
       int u = __ldcg(d.psi[0] + i);
-      return (__ldcg(d.active + u) && ld_part(d.part, u) == kPsi) ? u : -1;  // C1 joins beyond np0
+      return ld_part(d.part, u) == kPsi ? u : -1;  // C1 joins beyond np0
     };
     auto mt = [&](int u, long long) {
       scanned += __ldg(&d.vr[u].deg);
@@ -1425,9 +1429,8 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       // keys (int - ext, id) of every vertex of an overweight part on sigma3
       const long long ntot = ldv(&ctl->n_total);
       auto get = [&](long long v) {
-        if (!__ldcg(d.active + v)) return -1;
         uint8_t p = ld_part(d.part, v);
-        return (p != kPsi && s.sel.used[p]) ? (int)v : -1;
+        return (p != kDel && p != kPsi && s.sel.used[p]) ? (int)v : -1;
       };
       auto emit = [&](int v, uint8_t p, long long loss) {
         int d0 = (int)max(0ll, min(255ll, loss + 128));
