@@ -4,6 +4,7 @@
 #pragma once
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
+#include <stddef.h>
 #include <stdint.h>
 
 namespace igk {
@@ -76,6 +77,7 @@ struct Ctl {
   int selected3[3];    // moves selected per round (mod 3)
   unsigned long long tph[128];  // %globaltimer after each phase (CTA 0)
   int idph[128];                // phase ids
+  int ndone;                    // CTAs finished (publish: the last one posts the notice)
 };
 
 // ---------------------------------------------------------------------------
@@ -148,6 +150,9 @@ struct Dev {
   int32_t* newid;             // per modifier: new vertex ID of a VERTEX_INSERT
   unsigned long long* dbg;    // optional per-CTA barrier arrival stamps [128][grid]
   Ctl* ctl;
+  Ctl* hmap;                  // host-mapped copy of the output head (igk_step fast path)
+  volatile unsigned* hflag;   // host-mapped completion notice
+  unsigned seq;               // notice value of this launch (0 = no notice)
 };
 
 // ---------------------------------------------------------------------------
@@ -178,6 +183,35 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
   return t;
 }
+// Completion notice for the host (igk_step fast path): the last CTA to
+// finish copies the output head of Ctl into host-mapped memory, fences at
+// system scope and raises the flag to this launch's sequence number.  The
+// host polls the flag instead of a D2H copy + stream synchronisation.  Every
+// CTA of the grid must call it exactly once, at its exit.
+__device__ __forceinline__ void publish(const Dev& d) {
+  if (d.seq == 0) return;
+  __shared__ int s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(&d.ctl->ndone, 1) == (int)gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  const int nw = (int)(offsetof(Ctl, Wp) / 8);
+  const long long* src = reinterpret_cast<const long long*>(d.ctl);
+  long long* dst = reinterpret_cast<long long*>(d.hmap);
+  for (int i = threadIdx.x; i < nw; i += blockDim.x) dst[i] = __ldcg(src + i);
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    d.ctl->ndone = 0;
+    *d.hflag = d.seq;
+    __threadfence_system();
+  }
+}
+
 // phase stamp: CTA 0 / thread 0 records (id, time) right after a grid barrier
 __device__ __forceinline__ void stamp_phase(Ctl* ctl, int id) {
   if (blockIdx.x == 0 && threadIdx.x == 0) {

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <cstddef>
 #include <cstdlib>
@@ -234,6 +235,10 @@ struct igk_graph {
   long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active
   long long last_entries = 0, last_active = 0;
   Ctl* h_ctl = nullptr;        // pinned mirror of the control block
+  Ctl* h_map = nullptr;        // host-mapped output head written by the kernel (igk_step fast path)
+  unsigned* h_flag = nullptr;  // host-mapped completion notice
+  unsigned seq = 0;            // last notice value
+  int ms_pending = 0;          // ev[0] -> ev[1] not yet converted (fast path returns before ev[1])
   cudaEvent_t ev[6] = {};
   float ms_refine = 0, ms_apply = 0, ms_recount = 0;
   std::vector<void*> allocs;
@@ -317,6 +322,7 @@ igk_status launch_recount(igk_graph* g) {
 }
 
 igk_status sync_ctl(igk_graph* g, int which) {
+  g->ms_pending = 0;  // the stream is synchronised below: every event is complete
   // lean readback: only the output block at the head of Ctl (full copy when debugging)
   const size_t bytes = (g->debug_phases || g->check) ? sizeof(Ctl) : offsetof(Ctl, Wp);
   CK(cudaMemcpyAsync(g->h_ctl, g->d.ctl, bytes, cudaMemcpyDeviceToHost, g->stream));
@@ -563,10 +569,16 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     igk_destroy(g);
     return IGK_ENOMEM;
   }
-  if (cudaMallocHost(&g->h_ctl, sizeof(Ctl)) != cudaSuccess) {
+  if (cudaMallocHost(&g->h_ctl, sizeof(Ctl)) != cudaSuccess ||
+      cudaHostAlloc(&g->h_map, sizeof(Ctl), cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostAlloc(&g->h_flag, 64, cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostGetDevicePointer((void**)&d.hmap, g->h_map, 0) != cudaSuccess ||
+      cudaHostGetDevicePointer((void**)&d.hflag, g->h_flag, 0) != cudaSuccess) {
     igk_destroy(g);
     return IGK_ENOMEM;
   }
+  *g->h_flag = 0;
+  d.seq = 0;
   for (auto& e : g->ev) cudaEventCreate(&e);
   // zero-init
   cudaStream_t s = g->stream;
@@ -822,12 +834,42 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
 
 static igk_status prepare_apply(igk_graph* g, int64_t count);
 
+// igk_step fast path: the kernel posts its output head into host-mapped
+// memory and raises a flag (publish, common.cuh); the host polls the flag
+// instead of a D2H copy + stream synchronisation.  Debug / check modes keep
+// the full copy.
+static bool notice_begin(igk_graph* g) {
+  if (g->debug_phases || g->check) {
+    g->d.seq = 0;
+    return false;
+  }
+  if (++g->seq == 0) ++g->seq;  // 0 means "no notice"
+  g->d.seq = g->seq;
+  return true;
+}
+static igk_status notice_wait(igk_graph* g) {
+  volatile unsigned* f = g->h_flag;
+  for (long long i = 1; *f != g->seq; i++) {
+    if ((i & 255) == 0) {  // the kernel failed or ended without a notice: fall back
+      cudaError_t e = cudaStreamQuery(g->stream);
+      if (e == cudaErrorNotReady) continue;
+      if (e != cudaSuccess) CK(e);
+      if (*f != g->seq) return sync_ctl(g, 1);
+    }
+  }
+  std::atomic_thread_fence(std::memory_order_acquire);
+  std::memcpy(g->h_ctl, (const void*)g->h_map, offsetof(Ctl, Wp));
+  g->ms_pending = 1;  // ev[1] completes after the kernel exits: convert lazily
+  return IGK_OK;
+}
+
 static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refine_stats* stats,
                            int64_t* first_new_id, int64_t* bad_index) {
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   igk_status st;
   for (int attempt = 0;; attempt++) {
+    bool posted = false;  // this launch posts a host-mapped completion notice
     if (count == 0) {
       st = launch_refine(g, 0);
       if (st != IGK_OK) return st;
@@ -842,23 +884,32 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
       RefineArgs ra = make_refine_args(g, 1);
       void* a1[] = {(void*)&g->d, (void*)&aa};
       void* a2[] = {(void*)&g->d, (void*)&ra};
+      Dev dn = g->d;  // the refine posts the completion notice, not the apply
+      const bool fast = notice_begin(g);
+      void* a1n[] = {(void*)&dn, (void*)&aa};
       CK(cudaEventRecord(g->ev[0], g->stream));
-      CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply_wide, kThreads, a1, 0, g->stream));
+      CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply_wide, kThreads, fast ? a1n : a1, 0,
+                                     g->stream));
       CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, a2, g->smem_refine, g->stream));
+      g->d.seq = 0;
       g->launches += 2;
       CK(cudaEventRecord(g->ev[1], g->stream));
+      posted = fast;
     } else {  // apply + refine in ONE persistent launch (k_step)
       st = prepare_apply(g, count);
       if (st != IGK_OK) return st;
       ApplyArgs aa = make_apply_args(g, dm, count);
       RefineArgs ra = make_refine_args(g, 1);
+      const bool fast = notice_begin(g);
       void* args[] = {(void*)&g->d, (void*)&aa, (void*)&ra};
       CK(cudaEventRecord(g->ev[0], g->stream));
       CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
+      g->d.seq = 0;
       g->launches++;
       CK(cudaEventRecord(g->ev[1], g->stream));
+      posted = fast;
     }
-    st = sync_ctl(g, 1);
+    st = posted ? notice_wait(g) : sync_ctl(g, 1);
     if (st != IGK_OK) return st;
     if (count > 0 && g->h_ctl->err_idx == kNoErr && g->h_ctl->err_nomem && attempt < 2) {
       st = make_room(g);  // the kernel stopped before any mutation: grow / compact, then re-run
@@ -932,7 +983,7 @@ igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, 
 }
 
 static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
-  cudaEventElapsedTime(&g->ms_refine, g->ev[0], g->ev[1]);
+  if (!g->ms_pending) cudaEventElapsedTime(&g->ms_refine, g->ev[0], g->ev[1]);
   g->epochA = next_epoch(g);
   const long long* so = g->h_ctl->st_out;
   if (stats) {
@@ -1190,6 +1241,12 @@ igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_acti
 
 igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms) {
   if (!g) return IGK_ESTATE;
+  if (g->ms_pending) {  // fast path: the step returned before its end event completed
+    igk_graph* gm = const_cast<igk_graph*>(g);
+    cudaEventSynchronize(gm->ev[1]);
+    cudaEventElapsedTime(&gm->ms_refine, gm->ev[0], gm->ev[1]);
+    gm->ms_pending = 0;
+  }
   if (refine_ms) *refine_ms = g->ms_refine;
   if (apply_ms) *apply_ms = g->ms_apply;
   if (recount_ms) *recount_ms = g->ms_recount;
@@ -1231,6 +1288,8 @@ void igk_destroy(igk_graph* g) {
   if (g->d_rec_in) cudaFree(g->d_rec_in);
   if (g->h_rec) cudaFreeHost(g->h_rec);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
+  if (g->h_map) cudaFreeHost(g->h_map);
+  if (g->h_flag) cudaFreeHost(g->h_flag);
   for (auto& e : g->ev)
     if (e) cudaEventDestroy(e);
   delete g;

@@ -1567,6 +1567,7 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
   sh.mode = kModeFull;
   sh.nranks = 1;
   refine_body<false>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh);
+  publish(d);
 }
 
 // sharded refine: one launch per mode (pre | round gain | round finish | post)

@@ -18,6 +18,7 @@ __global__ void __launch_bounds__(kThreads) k_step(Dev d, ApplyArgs aa, RefineAr
   StepSmem& sm = *reinterpret_cast<StepSmem*>(smem_raw);
   if (!apply_body(d, aa, grid, sm.ap)) {
     if (blockIdx.x == 0 && threadIdx.x == 0) d.ctl->refine_skipped = 1;
+    publish(d);
     return;
   }
   grid.sync();  // the refine starts from the complete applied state
@@ -25,6 +26,7 @@ __global__ void __launch_bounds__(kThreads) k_step(Dev d, ApplyArgs aa, RefineAr
   sh.mode = kModeFull;
   sh.nranks = 1;
   refine_body<false>(d, ra, grid, sm.rf, sh);
+  publish(d);
 }
 
 }  // namespace igk

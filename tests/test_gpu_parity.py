@@ -242,15 +242,18 @@ def test_edge_cases():
         Q.compare_state(f"k254 it{it}")
 
 
+@pytest.mark.parametrize("check", [True, False], ids=["check", "notice"])
 @pytest.mark.parametrize("split", ["fused", "split"])
-def test_fused_step_api(split, monkeypatch):
+def test_fused_step_api(split, check, monkeypatch):
     """igk_step (apply + refine in one call) == oracle; an invalid batch is
     rejected atomically and the refine is skipped.  "split" forces the
     large-batch launch pair (k_apply at full occupancy + k_refine) that
-    igk_step uses from kSplitB modifiers on."""
+    igk_step uses from kSplitB modifiers on.  "notice" (check mode off) runs
+    the fast completion path: the kernel posts its outputs to host-mapped
+    memory and the host polls a flag instead of copying + synchronising."""
     if split == "split":
         monkeypatch.setenv("IGK_SPLIT_B", "1")  # read when the handle is created
-    cfg, g, part, P = _cfg_pair("C1", 1)
+    cfg, g, part, P = _cfg_pair("C1", 1, check=check)
     P.refine("settle")
     S = gi.Stream(g, gi.stream_seed(gi.graph_seed(1)) + 1)
     for it in range(8):
