@@ -314,13 +314,14 @@ def main():
             h_batches.append(hb)
         torch.cuda.synchronize()
         evs = [torch.cuda.Event(enable_timing=True) for _ in range(len(h_batches) + 1)]
-        aff_e = 0
+        aff_e, rounds_e = 0, 0
         slab0 = G.store_stats()["slab_cap"]
         evs[0].record(stream)
         for j, b in enumerate(h_batches):
             _, st, _ = G.step(b)  # igk_step: H2D DMA from pinned host memory, apply + refine
             G.cut()               # D2H read of the step's result
             aff_e += st["affected"]
+            rounds_e += st["rounds"]
             evs[j + 1].record(stream)
         torch.cuda.synchronize()
         te = evs[0].elapsed_time(evs[-1])
@@ -330,6 +331,9 @@ def main():
                "h2d_bytes_per_step": int(np.mean([b.nbytes for b in h_batches])),
                "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches),
                "ms_p50": float(np.median(per)), "ms_max": float(np.max(per)),
+               # the e2e steps are the iterations AFTER the device-timed ones (the graph keeps
+               # changing): their work is reported so the two legs can be compared
+               "affected_per_step": aff_e / len(h_batches), "rounds_per_step": rounds_e / len(h_batches),
                "store_compacted": G.store_stats()["slab_cap"] != slab0}
 
     # ---- S9 cut/weight reduction (full store scan, HBM-bound): own roofline
