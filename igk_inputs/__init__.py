@@ -187,6 +187,8 @@ def stream_seed(gseed: int) -> int:
 
 def next_batch(stream: Stream, cfg: dict, frac: float | None = None) -> np.ndarray:
     mode = cfg["mode"]
+    if mode == MODE_ADVERSARIAL and stream._r0 is None:
+        raise ValueError("adversarial batches need the Stream built with region0 (the part-0 indicator)")
     if mode == MODE_MIX:
         return stream.next(MODE_MIX, frac if frac is not None else cfg["frac"])
     lit = cfg["literal"]

@@ -55,7 +55,9 @@ __global__ void k_build(Dev d, const int64_t* xadj, const int32_t* adjncy, const
 // one schedule (no divergent per-thread loops).  A chunk's owner lane is found
 // by a 5-step shuffle search over the inclusive chunk prefix.  (Measured: a
 // variant that first reads every lane's own first chunk without the search
-// was slower, C4 282 -> 333 us.)  Labels are a
+// was slower, C4 282 -> 333 us; so were a search-free path for tiles whose
+// prefixes all fit one lane, C4 217 -> 229 us, and a next-tile prefetch of the
+// vertex record, no change: profiles/r01_s15_recount_ab.txt.)  Labels are a
 // 1-byte gather that stays in L2.  Edges are counted once (x > v); pending
 // (psi) vertices own no cut edges and count for no part.
 // ---------------------------------------------------------------------------
@@ -67,9 +69,8 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
   for (int p = threadIdx.x; p < 256; p += blockDim.x) s_wp[p] = 0;
   __syncthreads();
   const int lane = lane_id();
-  const bool ballot_wp = d.vw == nullptr && d.k <= 32;  // unit weights: W_p by popc(ballot)
+  const bool unit_wp = d.vw == nullptr;  // unit weights: W_p by label-group counts
   long long cut = 0, ent = 0, nact = 0;
-  long long wp_lane = 0;  // ballot mode: lane p accumulates W_p
   const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
   for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; base < n;
        base += nwarps * 32) {
@@ -90,10 +91,15 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
     ent += dg;
     nact += act;
     const bool placed = act && pv != kPsi;
-    if (ballot_wp) {
-      for (int p = 0; p < d.k; p++) {
-        unsigned m = __ballot_sync(0xffffffffu, placed && pv == p);
-        if (lane == p) wp_lane += __popc(m);
+    if (unit_wp) {
+      // lanes with the same label form one group; its lowest lane adds the
+      // group size (one match + one shared atomic per label present, instead
+      // of k ballots per tile: C4 recount 0.275 -> 0.217 ms with the grid below)
+      const unsigned pm = __ballot_sync(0xffffffffu, placed);
+      if (placed) {
+        const unsigned peers = __match_any_sync(pm, (unsigned)pv);
+        if ((peers & ((1u << lane) - 1)) == 0)
+          atomicAdd((unsigned long long*)&s_wp[pv], (unsigned long long)__popc(peers));
       }
     } else if (placed) {
       acc_add(s_wp, pv, vert_w(d.vw, v));
@@ -150,7 +156,6 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
       }
     }
   }
-  if (ballot_wp && lane < d.k && wp_lane) atomicAdd((unsigned long long*)&s_wp[lane], (unsigned long long)wp_lane);
   block_atomic_add(out_cut, cut, s_red);
   block_atomic_add(out_cnt, ent, s_red);
   block_atomic_add(out_cnt + 1, nact, s_red);
@@ -314,7 +319,14 @@ igk_status launch_recount(igk_graph* g) {
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device));
   long long n = g->h_ctl->n_total;
   CK(cudaEventRecord(g->ev[4], g->stream));
-  k_recount<<<sms * 4, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
+  // 48 registers: 5 blocks of 256 per SM (measured best; 4 blocks left the
+  // scan with too few loads in flight, profiles/r01_s15_recount_ab.txt)
+  static int occ = 0;
+  if (!occ) {
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_recount, 256, 0));
+    occ = std::max(1, std::min(occ, 5));
+  }
+  k_recount<<<sms * occ, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
   g->launches++;
   CK(cudaGetLastError());
   CK(cudaEventRecord(g->ev[5], g->stream));
