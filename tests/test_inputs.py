@@ -58,3 +58,13 @@ def test_weighted_and_adversarial_streams_valid():
         evicted += stats["evicted"]
         assert O.check_invariants() is None
     assert evicted > 0
+
+
+def test_adversarial_batch_needs_region0():
+    """MODE_ADVERSARIAL draws deletions from part 0; without the region the
+    generator has nothing to draw from, so next_batch refuses (no crash)."""
+    import pytest
+    g = gi.make_graph(2000, 64, 5)
+    S = gi.Stream(g, 3)
+    with pytest.raises(ValueError):
+        gi.next_batch(S, dict(gi.CONFIGS["C5"], literal=dict(nvd=10, nvi=10)))
