@@ -64,6 +64,13 @@ def lib():
         L.ora_num_slots.argtypes = [P]
         L.ora_export_csr.argtypes = [P, i64p, i32p, i32p]
         L.ora_check_invariants.argtypes = [P, C.c_char_p, C.c_int]
+        L.ora_check_invariants_ext.argtypes = [P, C.c_int64, C.c_int, C.c_char_p, C.c_int]
+        L.ora_debug_set_part.argtypes = [P, C.c_int64, C.c_int32]
+        L.ora_debug_set_part_weight.argtypes = [P, C.c_int32, C.c_int64]
+        L.ora_debug_set_total_weight.argtypes = [P, C.c_int64]
+        L.ora_debug_set_frontier.argtypes = [P, C.c_int64, C.c_int]
+        L.ora_debug_add_half_edge.argtypes = [P, C.c_int64, C.c_int32, C.c_int32]
+        L.ora_debug_set_edge_weight.argtypes = [P, C.c_int64, C.c_int32, C.c_int32]
         L.ora_cap.restype = C.c_int64
         L.ora_cap.argtypes = [C.c_int64, C.c_double, C.c_int32]
         L.ora_trace_rounds.restype = C.c_int64
@@ -162,10 +169,33 @@ class Oracle:
         lib().ora_export_csr(self.h, _p(xadj, C.c_int64), _p(adj, C.c_int32), _p(w, C.c_int32))
         return xadj, adj[:m], w[:m]
 
-    def check_invariants(self):
+    def check_invariants(self, reported_cut: int = -1, structure: bool = True):
+        """None if I1-I6 hold, else the first violation ("I6: ...", "I5: ...",
+        order I6, I5, I2, I3, I4, I1).  I1 compares `reported_cut` (e.g. the
+        product's maintained cut) with the oracle's recount; -1 skips it.
+        structure=False skips the O(m log m) adjacency check I6."""
         buf = C.create_string_buffer(256)
-        r = lib().ora_check_invariants(self.h, buf, 256)
+        r = lib().ora_check_invariants_ext(self.h, int(reported_cut), 0 if structure else 1, buf, 256)
         return None if r == 0 else buf.value.decode()
+
+    # TEST-ONLY corruption hooks: build states violating one invariant
+    def debug_set_part(self, v, p):
+        lib().ora_debug_set_part(self.h, int(v), int(p))
+
+    def debug_set_part_weight(self, p, w):
+        lib().ora_debug_set_part_weight(self.h, int(p), int(w))
+
+    def debug_set_total_weight(self, W):
+        lib().ora_debug_set_total_weight(self.h, int(W))
+
+    def debug_set_frontier(self, v, f):
+        lib().ora_debug_set_frontier(self.h, int(v), int(bool(f)))
+
+    def debug_add_half_edge(self, u, x, w=1):
+        lib().ora_debug_add_half_edge(self.h, int(u), int(x), int(w))
+
+    def debug_set_edge_weight(self, u, x, w):
+        lib().ora_debug_set_edge_weight(self.h, int(u), int(x), int(w))
 
     def trace_rounds(self, maxr=1 << 16):
         S = np.zeros(maxr, dtype=np.int64)

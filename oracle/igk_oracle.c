@@ -757,49 +757,145 @@ void ora_export_csr(const ora_graph* g, int64_t* xadj, int32_t* adjncy, int32_t*
   }
 }
 
-/* invariants after a refine (north_star):
- * I1 cut == recount (trivial here: ora_cut is the recount)
- * I2 W_p == recount and sum W_p == W
- * I3 W_p <= c (unless the weighted imbalance flag fired)
- * I4 only vertices that entered Psi moved
- * I5 Psi empty, every active vertex in [0,k)
- * I6 adjacency symmetric, simple, no self loops, no inactive endpoints */
-int ora_check_invariants(const ora_graph* g, char* msg, int msglen) {
+/* invariants after a refine (north_star).  Checked in a
+ * fixed order -- structure first, then labels, weights, balance, frontier,
+ * cut -- and the first violation is reported with its tag:
+ * I6 adjacency symmetric (equal weights both ways), simple, no self loops,
+ *    no inactive endpoints (G = (V, E) undirected, simple)
+ * I5 Psi empty: every active vertex has a part in [0,k) (rounds
+ *    repeat until the pseudo-partition is empty)
+ * I2 W = sum of active vw, every maintained W_p = its recount, sum W_p = W
+ *    (P:48 part weights)
+ * I3 W_p <= c for every part unless the weighted fallback fired
+ * I4 only vertices that entered Psi in the last refine changed part
+ *    (north_star "only frontier vertices moved")
+ * I1 a caller-reported maintained cut equals the recount ora_cut;
+ *    skipped when reported_cut < 0 (the oracle keeps no cut of its own)
+ * I6 runs on sorted copies of every row: O(m log m), so it stays cheap on
+ * 10^4-degree hubs (C4).  The recounts here share nothing with apply/refine. */
+static int cmp_i32(const void* a, const void* b) {
+  int32_t x = *(const int32_t*)a, y = *(const int32_t*)b;
+  return x < y ? -1 : (x > y);
+}
+int ora_check_invariants_ext(const ora_graph* g, int64_t reported_cut, int flags, char* msg, int msglen) {
+  const int64_t n = g->n;
+  /* I6 (skipped with flags & 1: labels/weights only) ------------------ */
+  if (!(flags & 1)) {
+  int64_t* rs = (int64_t*)xcalloc((size_t)n + 1, sizeof(int64_t));
+  for (int64_t v = 0; v < n; v++) rs[v + 1] = rs[v] + g->adj[v].cnt;
+  int32_t* rows = (int32_t*)xcalloc(2 * (size_t)rs[n], sizeof(int32_t));
+  for (int64_t v = 0; v < n; v++) {
+    const ora_adj* L = &g->adj[v];
+    int32_t* r = rows + 2 * rs[v];
+    for (int32_t i = 0; i < L->cnt; i++) {
+      r[2 * i] = L->nb[i];
+      r[2 * i + 1] = L->w[i];
+    }
+    qsort(r, L->cnt, 2 * sizeof(int32_t), cmp_i32);
+  }
+  int bad = 0;
+  for (int64_t v = 0; v < n && !bad; v++) {
+    const int32_t* r = rows + 2 * rs[v];
+    const int64_t d = rs[v + 1] - rs[v];
+    if (!g->active[v]) {
+      if (d) { snprintf(msg, msglen, "I6: deleted %lld has edges", (long long)v); bad = 1; }
+      continue;
+    }
+    for (int64_t i = 0; i < d && !bad; i++) {
+      const int32_t x = r[2 * i];
+      if (x == v || x < 0 || x >= n || !g->active[x]) {
+        snprintf(msg, msglen, "I6: bad neighbour %d of %lld", x, (long long)v);
+        bad = 1;
+        break;
+      }
+      if (i > 0 && r[2 * i - 2] == x) {
+        snprintf(msg, msglen, "I6: duplicate edge %lld-%d", (long long)v, x);
+        bad = 1;
+        break;
+      }
+      const int32_t* rx = rows + 2 * rs[x];
+      int64_t lo = 0, hi = rs[x + 1] - rs[x];
+      while (lo < hi) { /* binary search for v in the sorted row of x */
+        int64_t mid = (lo + hi) / 2;
+        if (rx[2 * mid] < v) lo = mid + 1; else hi = mid;
+      }
+      if (lo >= rs[x + 1] - rs[x] || rx[2 * lo] != v || rx[2 * lo + 1] != r[2 * i + 1]) {
+        snprintf(msg, msglen, "I6: asymmetric edge %lld-%d", (long long)v, x);
+        bad = 1;
+      }
+    }
+  }
+  free(rows);
+  free(rs);
+  if (bad) return 1;
+  }
+  /* I5 ------------------------------------------------------------- */
+  for (int64_t v = 0; v < n; v++) {
+    if (!g->active[v]) continue;
+    if (g->part[v] < 0 || g->part[v] >= g->k) {
+      snprintf(msg, msglen, "I5: vertex %lld has part %d", (long long)v, g->part[v]);
+      return 1;
+    }
+  }
+  /* I2 ------------------------------------------------------------- */
   int64_t Wp[LIM_K_MAX];
   int64_t W = 0;
   for (int32_t p = 0; p < g->k; p++) Wp[p] = 0;
-  for (int64_t v = 0; v < g->n; v++) {
-    if (!g->active[v]) {
-      if (g->adj[v].cnt) { snprintf(msg, msglen, "I6: deleted %lld has edges", (long long)v); return 1; }
-      continue;
-    }
+  for (int64_t v = 0; v < n; v++) {
+    if (!g->active[v]) continue;
     W += g->vw[v];
-    if (g->part[v] < 0 || g->part[v] >= g->k) { snprintf(msg, msglen, "I5: vertex %lld has part %d", (long long)v, g->part[v]); return 1; }
     Wp[g->part[v]] += g->vw[v];
-    if (!g->inF[v] && g->prev_part[v] != g->part[v] && g->prev_part[v] >= 0) {
-      snprintf(msg, msglen, "I4: vertex %lld moved outside the frontier", (long long)v);
-      return 1;
-    }
-    const ora_adj* L = &g->adj[v];
-    for (int32_t i = 0; i < L->cnt; i++) {
-      int32_t x = L->nb[i];
-      if (x == v || x < 0 || x >= g->n || !g->active[x]) { snprintf(msg, msglen, "I6: bad neighbour %d of %lld", x, (long long)v); return 1; }
-      int32_t j = adj_find(&g->adj[x], (int32_t)v);
-      if (j < 0 || g->adj[x].w[j] != L->w[i]) { snprintf(msg, msglen, "I6: asymmetric edge %lld-%d", (long long)v, x); return 1; }
-      for (int32_t t = i + 1; t < L->cnt; t++)
-        if (L->nb[t] == x) { snprintf(msg, msglen, "I6: duplicate edge %lld-%d", (long long)v, x); return 1; }
-    }
   }
   if (W != g->W) { snprintf(msg, msglen, "I2: W mismatch"); return 1; }
   int64_t s = 0;
-  int64_t c = cap_of(g->W, g->e_ppm, g->k);
   for (int32_t p = 0; p < g->k; p++) {
     s += g->Wp[p];
     if (Wp[p] != g->Wp[p]) { snprintf(msg, msglen, "I2: W_%d mismatch", p); return 1; }
-    if (g->Wp[p] > c && !g->last_imbalanced) { snprintf(msg, msglen, "I3: W_%d=%lld > cap %lld", p, (long long)g->Wp[p], (long long)c); return 1; }
   }
   if (s != g->W) { snprintf(msg, msglen, "I2: sum W_p != W"); return 1; }
+  /* I3 ------------------------------------------------------------- */
+  const int64_t c = cap_of(g->W, g->e_ppm, g->k);
+  for (int32_t p = 0; p < g->k; p++)
+    if (g->Wp[p] > c && !g->last_imbalanced) {
+      snprintf(msg, msglen, "I3: W_%d=%lld > cap %lld", p, (long long)g->Wp[p], (long long)c);
+      return 1;
+    }
+  /* I4 ------------------------------------------------------------- */
+  for (int64_t v = 0; v < n; v++) {
+    if (!g->active[v]) continue;
+    if (!g->inF[v] && g->prev_part[v] >= 0 && g->prev_part[v] != g->part[v]) {
+      snprintf(msg, msglen, "I4: vertex %lld moved outside the frontier", (long long)v);
+      return 1;
+    }
+  }
+  /* I1 ------------------------------------------------------------- */
+  if (reported_cut >= 0) {
+    int64_t rc = ora_cut(g);
+    if (rc != reported_cut) {
+      snprintf(msg, msglen, "I1: maintained cut %lld != recount %lld", (long long)reported_cut, (long long)rc);
+      return 1;
+    }
+  }
   return 0;
+}
+int ora_check_invariants(const ora_graph* g, char* msg, int msglen) {
+  return ora_check_invariants_ext(g, -1, 0, msg, msglen);
+}
+
+/* ------------------------------------------------------------------ */
+/* TEST-ONLY corruption hooks: they write one field of the state so that */
+/* tests can build states that violate exactly one invariant and check    */
+/* that ora_check_invariants_ext names it.  They are never called by      */
+/* apply/refine and carry none of the method's arithmetic.                */
+/* ------------------------------------------------------------------ */
+void ora_debug_set_part(ora_graph* g, int64_t v, int32_t p) { g->part[v] = p < 0 ? PSI : p; }
+void ora_debug_set_part_weight(ora_graph* g, int32_t p, int64_t w) { g->Wp[p] = w; }
+void ora_debug_set_total_weight(ora_graph* g, int64_t W) { g->W = W; }
+void ora_debug_set_frontier(ora_graph* g, int64_t v, int f) { g->inF[v] = (uint8_t)(f != 0); }
+void ora_debug_add_half_edge(ora_graph* g, int64_t u, int32_t x, int32_t w) { adj_push(&g->adj[u], x, w); }
+void ora_debug_set_edge_weight(ora_graph* g, int64_t u, int32_t x, int32_t w) {
+  int32_t i = adj_find(&g->adj[u], x);
+  if (i >= 0) g->adj[u].w[i] = w;
 }
 
 int64_t ora_trace_rounds(const ora_graph* g, int64_t* S, int64_t* L, int64_t maxr) {

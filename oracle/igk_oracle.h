@@ -81,8 +81,22 @@ int64_t ora_cap_value(const ora_graph* g);
 /* symmetric CSR of the current graph over all IDs, rows sorted ascending */
 int64_t ora_num_slots(const ora_graph* g);
 void ora_export_csr(const ora_graph* g, int64_t* xadj, int32_t* adjncy, int32_t* adjwgt);
-/* invariants I1-I6; returns 0 if all hold, else writes msg */
+/* invariants I1-I6; returns 0 if all hold, else writes msg
+ * (tagged "I6: ...", "I5: ...", ...: the first violation in the order
+ * I6, I5, I2, I3, I4, I1).  I1 compares reported_cut (e.g. the maintained
+ * cut of the product) with the recount; reported_cut < 0 skips I1.
+ * flags & 1 skips the O(m log m) structural check I6. */
+int ora_check_invariants_ext(const ora_graph* g, int64_t reported_cut, int flags, char* msg, int msglen);
 int ora_check_invariants(const ora_graph* g, char* msg, int msglen);
+
+/* TEST-ONLY corruption hooks (pins of the invariant checker): each writes
+ * one field of the state; p < 0 in set_part means the pseudo label */
+void ora_debug_set_part(ora_graph* g, int64_t v, int32_t p);
+void ora_debug_set_part_weight(ora_graph* g, int32_t p, int64_t w);
+void ora_debug_set_total_weight(ora_graph* g, int64_t W);
+void ora_debug_set_frontier(ora_graph* g, int64_t v, int f);
+void ora_debug_add_half_edge(ora_graph* g, int64_t u, int32_t x, int32_t w);
+void ora_debug_set_edge_weight(ora_graph* g, int64_t u, int32_t x, int32_t w);
 
 /* step-level hooks used by the pinning tests (tests/test_oracle_*.py) */
 int64_t ora_cap(int64_t W, double epsilon, int32_t k);

@@ -12,10 +12,27 @@ COMMON = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evi
 
 
 class Pair:
-    def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, check=True, **kw):
+    """inv_every: run the oracle's invariant checker (I1-I5, with the GPU's
+    maintained cut as the I1 operand) after every inv_every-th refine; the
+    O(m log m) adjacency check I6 runs every struct_every-th refine."""
+
+    def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, check=True, inv_every=1,
+                 struct_every=1, **kw):
         self.O = oracle.Oracle(xadj, adjncy, k, eps, part, vwgt, adjwgt)
         self.G = igk.IGKGraph(xadj, adjncy, k, eps, part, vwgt, adjwgt, check=check, **kw)
         self.k = k
+        self.inv_every, self.struct_every = inv_every, struct_every
+        self.n_refines = 0
+
+    def invariants(self, gpu_cut, where=""):
+        """north_star invariants after a refine, on the oracle's state, with
+        the GPU's maintained cut checked against the oracle's recount (I1)."""
+        self.n_refines += 1
+        if not self.inv_every or self.n_refines % self.inv_every:
+            return
+        structure = bool(self.struct_every) and self.n_refines % self.struct_every == 0
+        msg = self.O.check_invariants(gpu_cut, structure=structure)
+        assert msg is None, f"{where}: invariant violated: {msg}"
 
     def compare_state(self, where="", full_csr=False):
         po, pg = self.O.partition(), self.G.partition()
@@ -48,6 +65,7 @@ class Pair:
         assert so == sg, where
         diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
         assert not diff, f"{where}: stats differ (oracle, gpu): {diff}"
+        self.invariants(stg["cut"], where)
         return sto, stg
 
     def refine_global(self, where=""):
@@ -56,6 +74,7 @@ class Pair:
         assert so == sg, where
         diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
         assert not diff, f"{where}: global refine stats differ (oracle, gpu): {diff}"
+        self.invariants(stg["cut"], where)
         return sto, stg
 
 

@@ -141,6 +141,9 @@ def _run_case(seed):
             off += S[r]
         part = O.partition()
         assert {u: int(part[u]) for u in range(len(part))} == {u: (ref["part"][u] if active1[u] else -1) for u in ref["part"]}
+        # maintained W_p and W (apply, commits, rounds) == a recount from the labels
+        assert list(O.part_weights()) == [sum(vw[u] for u in range(len(part)) if part[u] == p) for p in range(k)]
+        assert O.total_weight() == sum(vw[u] for u in range(len(part)) if part[u] >= 0)
         assert O.cut() == stats["cut"] == refsem.cut_of(adj1, {u: int(part[u]) for u in range(len(part))})
         assert bool(stats["imbalanced"]) == ref["imbalanced"]
         assert O.check_invariants() is None
