@@ -137,9 +137,37 @@ def refine_bytes(st, weighted=False):
     return st["adj_entries_scanned"] * per_entry + touched * 16
 
 
+def host_cpu():
+    model = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return model, os.cpu_count()
+
+
+class pinned_to_one_core:
+    """taskset-equivalent: run the block on ONE host core (the oracle is
+    single-threaded by construction; pinning makes 'cores: 1' literal)."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.core = max(self.old)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *a):
+        os.sched_setaffinity(0, self.old)
+
+
 def cpu_baseline(g, part, k, eps, batches, gpu_cuts, iters):
     import oracle
     n_it = min(iters, len(batches))
+    model, ncpu = host_cpu()
+    pin = pinned_to_one_core().__enter__()
     t0 = time.perf_counter()
     O = oracle.Oracle(g.xadj, g.adjncy, k, eps, part)
     O.refine()
@@ -153,9 +181,11 @@ def cpu_baseline(g, part, k, eps, batches, gpu_cuts, iters):
         aff += st["affected"]
         if i < len(gpu_cuts) and gpu_cuts[i] != st["cut"]:
             cut_ok = False
+    pin.__exit__()
     return {"value": aff / tt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "host_cpu": model, "host_nproc": ncpu, "taskset_core": pin.core,
             "sample": f"first {n_it} iterations of the same workload (apply+refine, single-threaded, "
-                      f"{tt:.1f}s; setup {t_setup:.1f}s excluded)",
+                      f"pinned to core {pin.core} of {ncpu}; {tt:.1f}s; setup {t_setup:.1f}s excluded)",
             "ms_per_iteration": 1e3 * tt / n_it,
             "parity_cut_checked_iters": min(n_it, len(gpu_cuts)), "parity_cut_match": cut_ok}
 
@@ -210,19 +240,23 @@ def run_reference(args, rank, world):
         O.apply(batches[i])
         O.refine()
     aff, tt = 0, 0.0
-    for i in range(args.warmup, args.warmup + args.steps):
-        t = time.perf_counter()
-        O.apply(batches[i])
-        _, st = O.refine()
-        tt += time.perf_counter() - t
-        aff += st["affected"]
+    model, ncpu = host_cpu()
+    with pinned_to_one_core() as pin:
+        for i in range(args.warmup, args.warmup + args.steps):
+            t = time.perf_counter()
+            O.apply(batches[i])
+            _, st = O.refine()
+            tt += time.perf_counter() - t
+            aff += st["affected"]
     v = aff / tt
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tt / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic", "config": {"workload": desc, "n": g.n, "k": k},
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"{args.steps} timed iterations after {args.warmup} warm-up"},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "host_cpu": model,
+                             "host_nproc": ncpu, "taskset_core": pin.core,
+                             "sample": f"{args.steps} timed iterations after {args.warmup} warm-up, "
+                                       f"pinned to core {pin.core} of {ncpu}"},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -266,6 +300,7 @@ def main():
         G.apply_device(dev_batches[i].data_ptr(), len(b))  # replicated apply
         return G.refine_sharded(comm)[1]  # owner-split round gain + per-round record all-gather
 
+    deg_start = round(2.0 * g.m / g.n, 3)
     for i in range(W):
         gpu_cuts.append(one_step(i, batches[i])["cut"])
     torch.cuda.synchronize()
@@ -307,19 +342,26 @@ def main():
         # the caller's batches live in page-locked host memory (DMA'd straight
         # to the device by igk_step); filling them is the caller's own work
         h_batches = []
+        # the step's result returns to the caller as the partition DELTA
+        # (igk_partition_delta: every vertex whose part changed, P:23's
+        # IGP-in-the-loop client), into a page-locked buffer
+        dcap = 1 << 22
+        h_delta = torch.empty((dcap, 2), dtype=torch.int32, pin_memory=True).numpy()
         G.step(batches[W + K])  # untimed warm-up of the host-batch path (first call sizes its device buffer)
+        G.partition_delta(h_delta)
         for b in batches[W + K + 1:]:
             hb = torch.empty(b.shape, dtype=torch.int32, pin_memory=True).numpy()
             hb[...] = b
             h_batches.append(hb)
         torch.cuda.synchronize()
         evs = [torch.cuda.Event(enable_timing=True) for _ in range(len(h_batches) + 1)]
-        aff_e, rounds_e = 0, 0
+        aff_e, rounds_e, dbytes = 0, 0, 0
         slab0 = G.store_stats()["slab_cap"]
         evs[0].record(stream)
         for j, b in enumerate(h_batches):
-            _, st, _ = G.step(b)  # igk_step: H2D DMA from pinned host memory, apply + refine
-            G.cut()               # D2H read of the step's result
+            _, st, _ = G.step(b)               # igk_step: H2D DMA from pinned host memory, apply + refine
+            dl = G.partition_delta(h_delta)    # D2H of the step's result: (vertex, new part) pairs
+            dbytes += dl.nbytes
             aff_e += st["affected"]
             rounds_e += st["rounds"]
             evs[j + 1].record(stream)
@@ -329,7 +371,10 @@ def main():
         te, aff_e = benchdist.reduce_time_and_work(te, aff_e, dist, "cuda")
         e2e = {"value": aff_e / (te / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": int(np.mean([b.nbytes for b in h_batches])),
-               "d2h_bytes_per_step": 8, "ms_per_step": te / len(h_batches),
+               "d2h_bytes_per_step": int(dbytes / len(h_batches)),
+               "d2h": "partition delta (igk_partition_delta: vertex, new part pairs); the step's ~200-byte "
+                      "status head arrives through host-mapped memory",
+               "ms_per_step": te / len(h_batches),
                "ms_p50": float(np.median(per)), "ms_max": float(np.max(per)),
                # the e2e steps are the iterations AFTER the device-timed ones (the graph keeps
                # changing): their work is reported so the two legs can be compared
@@ -347,10 +392,14 @@ def main():
             G.recount()
             t9.append(G.last_ms()["recount"])
         ss = G.store_stats()
-        b9 = ss["adj_entries"] * 5 + ss["n_total"] * 14  # 4 B ID + 1 B label per entry; 8+4+1+1 B per vertex
+        # algorithmic bytes (SURVEY 8(d) 2m*5 B + 16 n, made exact): every LIVE
+        # entry's 4-byte ID, the 1-byte label of the neighbour for the half
+        # of the entries that own the edge (x > v), and per ACTIVE vertex its
+        # 16-byte record + 1-byte label
+        b9 = ss["adj_entries"] * 4 + ss["adj_entries"] // 2 + ss["n_active"] * 17
         a9 = b9 / (float(np.median(t9)) / 1e3) / 1e9
         s9 = {"kernel": "k_recount", "bound": "hbm", "achieved": a9, "unit": "GB/s", "bytes_per_launch": b9,
-              "launch_ms": float(np.median(t9)), "adj_entries": ss["adj_entries"]}
+              "launch_ms": float(np.median(t9)), "adj_entries": ss["adj_entries"], "n_active": ss["n_active"]}
 
     if rank != 0:
         if dist:
@@ -377,7 +426,12 @@ def main():
         "config": {"workload": desc, "n": g.n, "k": k,
                    "parallelism": ("sharded" if args.shard else "replicas") if world > 1 else "single",
                    "l2": "flushed between iterations (256 MiB write)" if flush is not None else "not flushed",
-                   "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]]))},
+                   "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]])),
+                   # the stream is edge-conserving: average degree at the start of
+                   # the run and after the last generated batch
+                   "avg_degree_start": deg_start, "avg_degree_end": round(S.avg_degree, 3),
+                   "affected_def": "|A \\ psi| + |Psi0|: placed vertices touched by the batch + pending inserts "
+                                   "(R2-expanded and R3-evicted vertices are not counted: conservative)"},
         "gpu_launches": launches,
         "roofline": {"kernel": kname, "bound": "hbm", "achieved": achieved, "peak": peak,
                      "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,

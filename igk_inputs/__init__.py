@@ -62,6 +62,8 @@ def lib():
         L.gen_stream_n_active.argtypes = [P]
         L.gen_stream_region_size.restype = C.c_int64
         L.gen_stream_region_size.argtypes = [P]
+        L.gen_stream_n_edges.restype = C.c_int64
+        L.gen_stream_n_edges.argtypes = [P]
         L.gen_stream_free.argtypes = [P]
         _lib = L
     return _lib
@@ -131,6 +133,7 @@ class Stream:
         self._keep = (g.xadj, g.adjncy, g.adjwgt)
         r0 = None if region0 is None else np.ascontiguousarray(region0, dtype=np.int32)
         self._r0 = r0
+        self._free = L.gen_stream_free  # kept: module globals may be gone at interpreter exit
         self.h = L.gen_stream_create(g.n, g.xadj.ctypes.data, g.adjncy.ctypes.data,
                                      None if g.adjwgt is None else g.adjwgt.ctypes.data,
                                      None if r0 is None else r0.ctypes.data, seed, int(weighted))
@@ -138,7 +141,7 @@ class Stream:
     def __del__(self):
         h = getattr(self, "h", None)
         if h:
-            lib().gen_stream_free(h)
+            self._free(h)
             self.h = None
 
     def next(self, mode: int = MODE_MIX, frac: float = 0.01, nvd: int = 0, nvi: int = 0,
@@ -156,6 +159,15 @@ class Stream:
     @property
     def n_active(self) -> int:
         return int(lib().gen_stream_n_active(self.h))
+
+    @property
+    def n_edges(self) -> int:
+        """undirected edges of the current graph (the generator's mirror)"""
+        return int(lib().gen_stream_n_edges(self.h))
+
+    @property
+    def avg_degree(self) -> float:
+        return 2.0 * self.n_edges / max(self.n_active, 1)
 
     @property
     def region_size(self) -> int:

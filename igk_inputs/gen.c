@@ -244,6 +244,7 @@ typedef struct {
   int64_t bcap;
   int32_t* out;    /* current batch, 4 int32 per modifier */
   int64_t ocnt, ocap;
+  int64_t m;       /* undirected edges in the mirror */
 } gstream;
 
 static void gs_grow(gstream* s, int64_t need) {
@@ -268,9 +269,11 @@ gstream* gen_stream_create(int64_t n, const int64_t* xadj, const int32_t* adjncy
   s->n = n;
   for (int64_t u = 0; u < n; u++) {
     for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) dpush(&s->A[u], adjncy[j], adjwgt ? adjwgt[j] : 1);
+    s->m += xadj[u + 1] - xadj[u];
     ms_add(&s->act, (int32_t)u);
     if (region0 && region0[u]) ms_add(&s->r0, (int32_t)u);
   }
+  s->m /= 2;
   return s;
 }
 
@@ -315,11 +318,18 @@ int64_t gen_stream_next(gstream* s, int mode, double frac, int64_t nvd, int64_t 
   s->ocnt = 0;
   s->stamp++;
   if (mode == MODE_MIX) {
-    int64_t B = llround(frac * (double)s->act.cnt / 1.8);
+    /* edge-conserving mix: B0 base modifiers, 10% VI, 10% VD,
+     * 40% ED, and EI = the ED count PLUS the edges the batch's vertex
+     * deletions remove, so the edge count (and, with VI = VD, the average
+     * degree ~4 of the north_star's inputs) stays level over thousands of
+     * iterations.  A base modifier touches 2.6 vertices on average (VI, VD
+     * one each; ED and the doubled EI two each), so B0 = f n / 2.6 keeps
+     * the batch at ~f n touched vertices (SURVEY 8(d)'s B = f n / 1.8 for
+     * the draining 10/10/40/40 mix). */
+    int64_t B = llround(frac * (double)s->act.cnt / 2.6);
     if (B < 10) B = 10;
-    nvi = llround(0.1 * B); nvd = llround(0.1 * B); ned = llround(0.4 * B); nei = B - nvi - nvd - ned;
+    nvi = llround(0.1 * B); nvd = llround(0.1 * B); ned = llround(0.4 * B); nei = ned;
   }
-  bk_reset(s, ned + nei + 3 * nvi + 16);
   const int32_t st = s->stamp; /* mark[v] == st: deleted in this batch */
   const int64_t n0 = s->n;
   mset* pool = (mode == MODE_ADVERSARIAL) ? &s->r0 : &s->act;
@@ -332,6 +342,16 @@ int64_t gen_stream_next(gstream* s, int mode, double frac, int64_t nvd, int64_t 
     out_push(s, K_VD, u, 0, 0);
     got++;
   }
+  if (mode == MODE_MIX) { /* + the edges incident to the deleted vertices (each once) */
+    for (int64_t i = 0; i < s->ocnt; i++) {
+      const int32_t u = s->out[4 * i + 1];
+      for (int32_t j = 0; j < s->A[u].cnt; j++) {
+        const int32_t x = s->A[u].nb[j];
+        if (s->mark[x] != st || x > u) nei++;
+      }
+    }
+  }
+  bk_reset(s, ned + nei + 3 * nvi + 16);
   /* edge deletions: random active vertex with edges, random neighbour */
   if (mode != MODE_ADVERSARIAL) {
     got = 0;
@@ -404,13 +424,14 @@ int64_t gen_stream_next(gstream* s, int mode, double frac, int64_t nvd, int64_t 
   /* mirror update in S1 phase order: ED, VD, VI, EI */
   for (int64_t i = 0; i < s->ocnt; i++) {
     int32_t* o = s->out + 4 * i;
-    if (o[0] == K_ED) { dremove(&s->A[o[1]], o[2]); dremove(&s->A[o[2]], o[1]); }
+    if (o[0] == K_ED) { dremove(&s->A[o[1]], o[2]); dremove(&s->A[o[2]], o[1]); s->m--; }
   }
   for (int64_t i = 0; i < s->ocnt; i++) {
     int32_t* o = s->out + 4 * i;
     if (o[0] != K_VD) continue;
     int32_t u = o[1];
     for (int32_t j = 0; j < s->A[u].cnt; j++) dremove(&s->A[s->A[u].nb[j]], u);
+    s->m -= s->A[u].cnt;
     s->A[u].cnt = 0;
     ms_del(&s->act, u);
     ms_del(&s->r0, u);
@@ -422,7 +443,7 @@ int64_t gen_stream_next(gstream* s, int mode, double frac, int64_t nvd, int64_t 
   s->n = n0 + nvi;
   for (int64_t i = 0; i < s->ocnt; i++) {
     int32_t* o = s->out + 4 * i;
-    if (o[0] == K_EI) { dpush(&s->A[o[1]], o[2], o[3]); dpush(&s->A[o[2]], o[1], o[3]); }
+    if (o[0] == K_EI) { dpush(&s->A[o[1]], o[2], o[3]); dpush(&s->A[o[2]], o[1], o[3]); s->m++; }
   }
   return s->ocnt;
 }
@@ -430,6 +451,7 @@ void gen_stream_copy(const gstream* s, int32_t* out) { memcpy(out, s->out, sizeo
 int64_t gen_stream_n_total(const gstream* s) { return s->n; }
 int64_t gen_stream_n_active(const gstream* s) { return s->act.cnt; }
 int64_t gen_stream_region_size(const gstream* s) { return s->r0.cnt; }
+int64_t gen_stream_n_edges(const gstream* s) { return s->m; }
 void gen_stream_free(gstream* s) {
   if (!s) return;
   for (int64_t i = 0; i < s->ncap; i++) { free(s->A[i].nb); free(s->A[i].w); }

@@ -166,26 +166,46 @@ typedef struct {
 } igk_comm;
 igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_stats* stats);
 
-/* out[v] for v < n_total: part in [0,k), -1 = deleted, -2 = pending (in the
- * pseudo-partition between apply and refine).  cap_len too small ->
- * IGK_EINVAL with *n_total still set. */
+/* The k-way partition (V_1..V_k; P:50 the part of every vertex).
+ * out[v] for v < n_total: part in [0,k), -1 = deleted, -2 = pending (in the
+ * pseudo-partition between apply and refine).  out is a HOST buffer of
+ * cap_len entries; cap_len too small -> IGK_EINVAL with *n_total still set
+ * (call with out == NULL to query the size).  One device gather + one D2H. */
 igk_status igk_partition(const igk_graph* g, int32_t* out, int64_t cap_len, int64_t* n_total);
+/* The partition CHANGES of the last igk_refine / igk_refine_global /
+ * igk_step: (vertex, new part) int32 pairs, one per vertex whose part now
+ * differs from its part before that refine -- the frontier vertices that
+ * moved (only they can, invariant I4) and every vertex inserted
+ * since the previous refine (its first placement, Alg. 3 L2-5).  Vertices
+ * deleted by the batch are not listed (the caller issued those deletions).
+ * This is what an IGP-in-the-loop client consumes each iteration
+ * instead of the whole vector.  pairs: HOST buffer of 2 * cap int32 (pair
+ * order unspecified); *count = number of pairs.  cap < count -> IGK_EINVAL
+ * with *count set (pairs == NULL queries the count).  The list is built on
+ * the device by the refine kernel; this call is one D2H of 8 * count bytes
+ * (page-locked `pairs` are DMA'd directly). */
+igk_status igk_partition_delta(const igk_graph* g, int32_t* pairs, int64_t cap, int64_t* count);
 /* cut size, maintained incrementally; edges with a pending endpoint
  * are not counted. */
 igk_status igk_cut_size(const igk_graph* g, int64_t* out);
 /* part weights W_p, k entries */
 igk_status igk_part_weights(const igk_graph* g, int64_t* out_k);
+/* |V| bookkeeping (P:48 V; vertex_status): *n_total = IDs in use
+ * (deleted IDs are never reused), *n_active = active vertices (a device
+ * reduction over the labels, one 8-byte read back).  Either may be NULL. */
 igk_status igk_num_vertices(const igk_graph* g, int64_t* n_total, int64_t* n_active);
 /* Recount cut and W_p from scratch with the cut/weight reduction kernel
  * (S9, HBM-bound full store scan).  out_wp may be NULL. */
 igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp);
 /* Debug/test: current graph as a symmetric CSR over all IDs (deleted rows
- * empty; row order unspecified).  Size query: call with xadj == NULL to get
- * *n_total and *n_slots. */
+ * empty; order inside a row unspecified).  Size query: call with xadj ==
+ * NULL to get *n_total and *n_slots.  Built on the device (live-degree scan
+ * + row gather kernel) and read back in one copy per output array. */
 igk_status igk_export_csr(const igk_graph* g, int64_t* xadj, int64_t xadj_len, int32_t* adjncy,
                           int32_t* adjwgt, int64_t adj_len, int64_t* n_total, int64_t* n_slots);
-/* store occupancy: IDs in use, active vertices and adjacency entries as of
- * the last igk_recount, slab bump pointer and capacity (entries) */
+/* store occupancy: IDs in use, active vertices and live (directed)
+ * adjacency entries (= 2m) as of the last igk_recount, slab bump pointer
+ * and capacity (entries) */
 igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_active, int64_t* adj_entries,
                            int64_t* slab_top, int64_t* slab_cap);
 /* Store maintenance (NEXT-4): rewrite the adjacency slab densely (drops
@@ -196,6 +216,34 @@ igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_acti
 igk_status igk_compact(igk_graph* g);
 /* number of kernels this handle has launched so far (instrumentation) */
 int64_t igk_kernel_launches(const igk_graph* g);
+/* instrumentation: how often each rarely-taken code path ran since
+ * igk_create, so tests can show every path the full-size inputs need was
+ * exercised.  out[i] for i < returned count (<= cap), index = IGK_PATH_*. */
+enum {
+  IGK_PATH_HUB_FILTER = 0,  /* filter of a hub (degree > 1024) by a whole CTA           */
+  IGK_PATH_HUB_COMMIT,      /* commit of a hub candidate by a whole CTA                 */
+  IGK_PATH_HUB_GAIN,        /* round gain of a pending hub by a whole CTA               */
+  IGK_PATH_TIE_CTA,         /* cutoff round: an overflowing part's tie group in one CTA */
+  IGK_PATH_TIE_GRID,        /* cutoff round: grid-wide radix passes (fallback)          */
+  IGK_PATH_KEY_EXACT,       /* cutoff threshold digit with #nbr < 255 (ID key)          */
+  IGK_PATH_KEY64,           /* cutoff threshold digit with #nbr >= 255 (64-bit key)     */
+  IGK_PATH_FORCED_L0,       /* L = 0: first sorted move forced (reading Q8)             */
+  IGK_PATH_WFALLBACK,       /* E(u) empty: lightest part + imbalance flag (Q8)          */
+  IGK_PATH_R3,              /* balance restoration ran                                   */
+  IGK_PATH_R3_KEY64,        /* restoration threshold in a clamped loss digit             */
+  IGK_PATH_RELOC,           /* prefixes relocated on overflow                            */
+  IGK_PATH_VDEL_WARP,       /* vertex deletions, warp per 8-entry item                   */
+  IGK_PATH_VDEL_THREAD,     /* vertex deletions, thread per 8-entry item                 */
+  IGK_PATH_WARP_GAIN,       /* round gains in the warp bucket (degree 17..1024)          */
+  IGK_PATH_RESERVED15,
+  IGK_PATH_COMPACTION = 16, /* slab compactions (host)                                   */
+  IGK_PATH_VERTEX_GROWTH,   /* vertex-array growths (host)                               */
+  IGK_PATH_SPLIT_STEP,      /* igk_step as k_apply + k_refine (large batch)              */
+  IGK_PATH_FUSED_STEP,      /* igk_step as one k_step                                    */
+  IGK_PATH_NOTICE_FALLBACK, /* step completion notice missed: copy + sync fallback       */
+  IGK_PATH_N
+};
+int32_t igk_debug_paths(const igk_graph* g, int64_t* out, int32_t cap);
 /* device-side duration (ms) of the last igk_refine / apply / recount kernel,
  * measured with CUDA events on the handle's stream */
 igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms);

@@ -107,11 +107,12 @@ class Oracle:
                               _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(st))
         if not self.h:
             raise ValueError(f"ora_create rejected the input (status {st.value})")
+        self._destroy = L.ora_destroy  # kept: module globals may be gone at interpreter exit
 
     def __del__(self):
         h = getattr(self, "h", None)
         if h:
-            lib().ora_destroy(h)
+            self._destroy(h)
             self.h = None
 
     def apply(self, mods):

@@ -26,9 +26,16 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine", "igk_refine_global",
            "igk_step", "igk_step_device", "igk_refine_sharded",
-           "igk_partition", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
+           "igk_partition", "igk_partition_delta", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
+           "igk_debug_paths",
            "igk_last_error", "igk_destroy"]
+
+
+# igk_debug_paths counters (include/igk.h IGK_PATH_*)
+PATHS = ["hub_filter", "hub_commit", "hub_gain", "tie_cta", "tie_grid", "key_exact", "key64", "forced_l0",
+         "wfallback", "r3", "r3_key64", "reloc", "vdel_warp", "vdel_thread", "warp_gain", "reserved15",
+         "compaction", "vertex_growth", "split_step", "fused_step", "notice_fallback"]
 
 
 class Options(C.Structure):
@@ -136,6 +143,10 @@ def lib():
         L.igk_refine_sharded.argtypes = [P, C.POINTER(Comm), C.POINTER(Stats)]
         L.igk_partition.restype = C.c_int
         L.igk_partition.argtypes = [P, i32p, i64, i64p]
+        L.igk_partition_delta.restype = C.c_int
+        L.igk_partition_delta.argtypes = [P, P, i64, i64p]
+        L.igk_debug_paths.restype = C.c_int32
+        L.igk_debug_paths.argtypes = [P, i64p, C.c_int32]
         L.igk_cut_size.restype = C.c_int
         L.igk_cut_size.argtypes = [P, i64p]
         L.igk_part_weights.restype = C.c_int
@@ -187,12 +198,13 @@ class IGKGraph:
                          _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(h))
         if s != OK:
             raise IGKError(s, "igk_create failed")
+        self._destroy = L.igk_destroy  # kept: module globals may be gone at interpreter exit
         self.h = h
         self.k = int(k)
 
     def close(self):
         if getattr(self, "h", None):
-            lib().igk_destroy(self.h)
+            self._destroy(self.h)
             self.h = None
 
     __del__ = close
@@ -269,6 +281,26 @@ class IGKGraph:
         if s != OK:
             raise IGKError(s, self._err())
         return out[: nt.value]
+
+    def partition_delta(self, out: "np.ndarray | None" = None):
+        """(count, 2) int32 array of (vertex, new part) of the last refine / step
+        (igk_partition_delta).  `out`: optional (cap, 2) int32 buffer to fill
+        (page-locked memory is DMA'd directly); returns a view of it."""
+        cnt = C.c_int64(0)
+        L = lib()
+        if out is None:
+            L.igk_partition_delta(self.h, None, 0, C.byref(cnt))
+            out = np.empty((max(cnt.value, 1), 2), dtype=np.int32)
+        s = L.igk_partition_delta(self.h, C.c_void_p(out.ctypes.data), len(out), C.byref(cnt))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return out[: cnt.value]
+
+    def debug_paths(self):
+        """{path name: count} of the device / host path counters (igk_debug_paths)."""
+        out = np.zeros(32, np.int64)
+        n = lib().igk_debug_paths(self.h, _p(out, C.c_int64), 32)
+        return {PATHS[i]: int(out[i]) for i in range(min(n, len(PATHS)))}
 
     def cut(self):
         c = C.c_int64(0)

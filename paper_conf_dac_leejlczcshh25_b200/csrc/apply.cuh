@@ -357,7 +357,10 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     if (m.x == kVertDel && m.y >= 0 && m.y < n0) d.vcnt[m.y] = 0;
   }
   if (failed) {  // uniform: every CTA read the same error words
-    if (tid == 0) ctl->slab_top = ctl->slab_top0;
+    if (tid == 0) {
+      ctl->slab_need = ctl->slab_top - ctl->slab_top0;  // what the batch asked for: sizes the compaction
+      ctl->slab_top = ctl->slab_top0;
+    }
     return false;
   }
 
@@ -411,6 +414,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   // thread per item, all of its loads in flight together (measured: C2
   // 0.2047 vs 0.2096 ms, C4 0.780 vs 0.808 ms for the other choice).
   const int nvd = ldv(&ctl->nvdch);
+  if (tid == 0 && nvd) path_hit(ctl, nvd <= nwarp ? PA_VDEL_WARP : PA_VDEL_THREAD);
   if (nvd <= nwarp) {
     for (long long t = gwarp; t < nvd; t += nwarp) {
       const int2 ch = __ldcg(d.vdch + t);
@@ -495,6 +499,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       d.active[id] = 1;
       if (d.vw) d.vw[id] = m.w;
       d.part[id] = kPsi;  // Alg. 3 L2-5: straight to the pseudo-partition
+      d.oldp[id] = kPsi;  // no part before: its first placement is a label change (delta list)
       if (__ldcg(d.markG + id) != a.epG) {
         d.vr[id].deg = 0;
         d.capv[id] = 0;
@@ -537,6 +542,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     return wr;
   };
   const int nrl = ldv(&ctl->nreloc);
+  if (tid == 0 && nrl) path_hit(ctl, PA_RELOC, nrl);
   for (long long t = gwarp; t < nrl; t += nwarp) {  // growing prefixes move to their new slots
     int x = __ldcg(d.rlist + t);
     long long pk = __ldcg(d.reloc + x);

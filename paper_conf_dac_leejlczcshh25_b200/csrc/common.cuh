@@ -39,6 +39,28 @@ enum StatIdx {
   ST_N
 };
 
+// Device path counters (igk_debug_paths): how often each rarely-taken code
+// path ran since igk_create -- so the tests can show that every path the
+// full-size inputs need was exercised (and bit-exact).  Order = igk.h IGK_PATH_*.
+enum PathIdx {
+  PA_HUB_FILTER = 0,  // filter of a hub (degree > kBlockDeg) by a whole CTA
+  PA_HUB_COMMIT,      // commit of a hub candidate by a whole CTA
+  PA_HUB_GAIN,        // round gain of a pending hub by a whole CTA
+  PA_TIE_CTA,         // cutoff round: an overflowing part's tie group finished in one CTA
+  PA_TIE_GRID,        // cutoff round: grid-wide radix passes over the tie groups (fallback)
+  PA_KEY_EXACT,       // cutoff round threshold in an exact-key digit (#nbr < 255): 32-bit ID key
+  PA_KEY64,           // cutoff round threshold in digit 0 (#nbr >= 255): 64-bit (#nbr, ID) key
+  PA_FORCED_L0,       // L = 0: the first sorted move forced (reading Q8)
+  PA_WFALLBACK,       // E(u) empty: move to the lightest part with the imbalance flag (Q8)
+  PA_R3,              // balance restoration ran (some W_p > cap)
+  PA_R3_KEY64,        // restoration threshold in a clamped (non-exact) loss digit
+  PA_RELOC,           // prefixes relocated on overflow (apply M3)
+  PA_VDEL_WARP,       // vertex deletions: one warp per 8-entry item
+  PA_VDEL_THREAD,     // vertex deletions: one thread per 8-entry item
+  PA_WARP_GAIN,       // rounds that ran the warp bucket of the gain (degree 17..1024)
+  PA_N_DEV = 16
+};
+
 struct Ctl {
   // ---- outputs read back after every call (kept first: lean D2H copy) ----
   long long n_total;   // vertex IDs in use
@@ -55,6 +77,9 @@ struct Ctl {
   int rs_cur;          // sharded refine: round state between host-driven launches
   long long rs_rounds, rs_rounds_all, rs_applied, rs_deferred;
   int rs_pending;      // pending vertices left for the next sharded round
+  long long slab_need; // slots the last rejected batch asked for (capacity failure: sizes the compaction)
+  int n_delta;         // (vertex, part) pairs in the delta list of the last refine
+  int n_delta_pad;
   // ---- device-side state ----
   long long Wp[256];   // part weights
   long long tot3[3][256];  // per round (mod 3): weight of selected moves per target part
@@ -78,7 +103,11 @@ struct Ctl {
   unsigned long long tph[128];  // %globaltimer after each phase (CTA 0)
   int idph[128];                // phase ids
   int ndone;                    // CTAs finished (publish: the last one posts the notice)
+  long long paths[PA_N_DEV];    // device path counters (cumulative)
 };
+__device__ __forceinline__ void path_hit(Ctl* ctl, int which, long long v = 1) {
+  atomicAdd((unsigned long long*)&ctl->paths[which], (unsigned long long)v);
+}
 
 // ---------------------------------------------------------------------------
 // all device pointers of one handle, passed by value to every kernel
@@ -148,6 +177,7 @@ struct Dev {
   int64_t hmask;
   int32_t* blkcnt;            // per-block counts for chunked scans
   int32_t* newid;             // per modifier: new vertex ID of a VERTEX_INSERT
+  int2* delta;                // (vertex, new part) of every label change of the last refine
   unsigned long long* dbg;    // optional per-CTA barrier arrival stamps [128][grid]
   Ctl* ctl;
   Ctl* hmap;                  // host-mapped copy of the output head (igk_step fast path)
@@ -161,11 +191,20 @@ struct Dev {
 __device__ __forceinline__ long long ldv(const long long* p) { return *(volatile const long long*)p; }
 __device__ __forceinline__ int ldv(const int* p) { return *(volatile const int*)p; }
 __device__ __forceinline__ uint8_t ld_part(const uint8_t* p, int64_t i) { return __ldcg(p + i); }
+// Loads of the store (adjacency, weights, vertex records) in the apply /
+// refine kernels.  The fused k_step writes that data in its apply half and
+// reads it in its refine half, so the non-coherent read-only path (__ldg,
+// ld.global.nc: data must not change during the kernel) is never used for
+// it: every such load goes through L2 (ld.global.cg).
+template <typename T>
+__device__ __forceinline__ T ldro(const T* p) {
+  return __ldcg(p);
+}
 
-// one 16-byte load of a vertex record's (offset, prefix length): read-only
-// path (__ldg) and L2-coherent path (__ldcg, for fields written in-kernel)
+// one 16-byte load of a vertex record's (offset, prefix length) through L2
+// (written in-kernel by the apply half of k_step, see ldro)
 __device__ __forceinline__ void vr_ld(const Dev& d, int64_t u, long long& o, int& dg) {
-  const longlong2 r = __ldg(reinterpret_cast<const longlong2*>(d.vr + u));
+  const longlong2 r = __ldcg(reinterpret_cast<const longlong2*>(d.vr + u));
   o = r.x;
   dg = (int)(unsigned)(unsigned long long)r.y;
 }
@@ -325,8 +364,8 @@ __device__ __forceinline__ bool stamp_insert(uint32_t* mark, int64_t v, uint32_t
   return atomicExch(mark + v, epoch) != epoch;
 }
 
-__device__ __forceinline__ int edge_w(const int32_t* adjw, int64_t j) { return adjw ? __ldg(adjw + j) : 1; }
-__device__ __forceinline__ int vert_w(const int32_t* vw, int64_t v) { return vw ? __ldg(vw + v) : 1; }
+__device__ __forceinline__ int edge_w(const int32_t* adjw, int64_t j) { return adjw ? ldro(adjw + j) : 1; }
+__device__ __forceinline__ int vert_w(const int32_t* vw, int64_t v) { return vw ? ldro(vw + v) : 1; }
 
 // cap(W) = max(floor(W (1e6 + e) / (1e6 k)), ceil(W / k))  (reading Q4)
 __host__ __device__ __forceinline__ long long cap_of(long long W, long long e_ppm, int k) {

@@ -4,6 +4,7 @@
 // persistent cooperative launch per call.  This file holds the handle, the
 // store build (S0), the cut/weight reduction (S9) and the exports.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <atomic>
@@ -19,6 +20,7 @@
 #include "common.cuh"
 #include "refine.cuh"
 #include "step.cuh"
+#include <cub/cub.cuh>
 
 using namespace igk;
 
@@ -77,18 +79,22 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
     const long long v = base + lane;
     bool act = false;
     uint8_t pv = kPsi;
-    int dg = 0;
+    int dg = 0, ld = 0;
     long long o = 0;
     if (v < n) {
       pv = __ldg(d.part + v);
       act = pv != kDel;  // the label doubles as the active flag
-      vr_ld(d, v, o, dg);
+      const longlong2 r = __ldg(reinterpret_cast<const longlong2*>(d.vr + v));  // one 16-byte record
+      o = r.x;
+      dg = (int)(unsigned)(unsigned long long)r.y;  // prefix length incl. tombstones
+      ld = (int)(r.y >> 32);                         // live degree
     }
     if (!act) {
       pv = kPsi;
       dg = 0;
+      ld = 0;
     }
-    ent += dg;
+    ent += ld;  // live adjacency entries (algorithmic bytes of the scan)
     nact += act;
     const bool placed = act && pv != kPsi;
     if (unit_wp) {
@@ -198,6 +204,43 @@ __global__ void k_compact_twins(long long used, const int32_t* nadj, int32_t* nt
     if (nadj[s] >= 0) ntwin[s] = fwd[ntwin[s]];
 }
 
+// igk_num_vertices: active vertices (the label doubles as the active flag)
+__global__ void k_count_active(Dev d, long long n, long long* out) {
+  long long c = 0;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    c += d.part[v] != kDel;
+  c = warp_sum(c);
+  if (lane_id() == 0 && c) atomicAdd((unsigned long long*)out, (unsigned long long)c);
+}
+// igk_export_csr: live degree of every ID (deleted rows are empty, I6)
+__global__ void k_export_deg(Dev d, long long n, long long* ldeg) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    ldeg[v] = d.part[v] != kDel ? d.vr[v].ldeg : 0;
+}
+// igk_export_csr: the live entries of every prefix (tombstones dropped, slot
+// order kept) gathered into one dense CSR on the device -- one warp per row
+__global__ void k_export_rows(Dev d, long long n, const long long* xoff, int32_t* oadj, int32_t* ow) {
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long v = gw; v < n; v += nw) {
+    if (d.part[v] == kDel) continue;
+    const long long o = d.vr[v].off, base = xoff[v];
+    const int dg = d.vr[v].deg;
+    int wr = 0;
+    for (int b = 0; b < dg; b += 32) {
+      const int j = b + lane_id();
+      const int y = j < dg ? d.adj[o + j] : -1;
+      const unsigned keep = __ballot_sync(0xffffffffu, y >= 0);
+      if (y >= 0) {
+        const long long pos = base + wr + __popc(keep & ((1u << lane_id()) - 1u));
+        oadj[pos] = y;
+        ow[pos] = d.adjw ? d.adjw[o + j] : 1;
+      }
+      wr += __popc(keep);
+    }
+  }
+}
+
 __global__ void k_export_part(Dev d, long long n, int32_t* out) {
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
     uint8_t p = d.part[v];
@@ -210,6 +253,11 @@ __global__ void k_export_part(Dev d, long long n, int32_t* out) {
 // ---------------------------------------------------------------------------
 struct igk_graph {
   int device = 0;
+  int recount_blocks = 0;    // k_recount grid (occupancy-derived at create)
+  long long n_grow = 0;      // vertex-array growths (host path counter)
+  long long n_split = 0;     // igk_step launches as k_apply + k_refine (batch >= split_b)
+  long long n_fused = 0;     // igk_step launches as one k_step
+  long long n_notice_fallback = 0;  // fast-path steps that fell back to the copy + sync
   cudaStream_t stream = nullptr;
   bool poisoned = false;
   std::string err;
@@ -251,6 +299,27 @@ struct igk_graph {
 };
 
 namespace {
+
+// Every entry point runs on the handle's device and restores the caller's
+// current device on return (the ABI allows handles on several GPUs).
+struct DevGuard {
+  int prev = -1;
+  explicit DevGuard(int dev) {
+    int cur = -1;
+    if (cudaGetDevice(&cur) == cudaSuccess && cur != dev && cudaSetDevice(dev) == cudaSuccess) prev = cur;
+  }
+  ~DevGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+// NVTX range around each entry point (visible in nsys / ncu timelines)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+#define ENTRY(g, name)             \
+  DevGuard igk_dg_((g)->device);   \
+  NvtxRange igk_nv_(name)
 
 igk_status fail(igk_graph* g, igk_status s, const std::string& msg) {
   if (g) g->err = msg;
@@ -303,9 +372,8 @@ static cudaError_t vr_get(void* dst, const VRec* vr, size_t field, size_t elem, 
   return cudaMemcpy2DAsync(dst, elem, (const char*)vr + field, sizeof(VRec), elem, (size_t)n, kind, s);
 }
 
-int coop_grid(const void* fn, size_t smem, int want_per_sm) {
-  int dev = 0, sms = 0, occ = 0;
-  cudaGetDevice(&dev);
+int coop_grid(const void* fn, size_t smem, int want_per_sm, int dev) {
+  int sms = 0, occ = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kThreads, smem);
   if (occ < 1) occ = 1;
@@ -315,18 +383,9 @@ int coop_grid(const void* fn, size_t smem, int want_per_sm) {
 
 igk_status launch_recount(igk_graph* g) {
   CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 259, g->stream));
-  int sms = 0;
-  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device));
   long long n = g->h_ctl->n_total;
   CK(cudaEventRecord(g->ev[4], g->stream));
-  // 48 registers: 5 blocks of 256 per SM (measured best; 4 blocks left the
-  // scan with too few loads in flight, profiles/r01_s15_recount_ab.txt)
-  static int occ = 0;
-  if (!occ) {
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_recount, 256, 0));
-    occ = std::max(1, std::min(occ, 5));
-  }
-  k_recount<<<sms * occ, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
+  k_recount<<<g->recount_blocks, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
   g->launches++;
   CK(cudaGetLastError());
   CK(cudaEventRecord(g->ev[5], g->stream));
@@ -382,7 +441,7 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
       {(void**)&d.reloc, 8, 0},    {(void**)&d.tgt, 1, 0},     {(void**)&d.gain, 4, 0},   {(void**)&d.pw, 4, 0},
       {(void**)&d.meta, 4, 0},     {(void**)&d.metav, 4, 0},   {(void**)&d.oldp, 1, 0},   {(void**)&d.hubA, 4, 0},
       {(void**)&d.hubC, 4, 0},     {(void**)&d.hubN, 4, 0},    {(void**)&d.hubC2, 4, 0},  {(void**)&d.hubP, 4, 0},
-      {(void**)&g->d_out, 4, 0},
+      {(void**)&g->d_out, 4, 0},   {(void**)&d.delta, 8, 0},
   };
   for (auto& a : arrs)
     if (!regrow(g, a.p, a.elem, o, n, a.fill)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
@@ -395,19 +454,23 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
   while ((1ll << ib) < d.n_cap) ib++;
   d.idbits = ib;
   CK(cudaStreamSynchronize(g->stream));
+  g->n_grow++;
   return IGK_OK;
 }
 
-// compact the slab into fresh arrays (capacity >= min_cap); live entries only
-igk_status compact_slab(igk_graph* g, long long min_cap) {
+// compact the slab into fresh arrays; live entries only.  The new capacity
+// keeps at least half of it free AND room for `extra` more slots (the demand
+// of the batch whose validation ran out of slots), so one compaction always
+// suffices for that batch.
+igk_status compact_slab(igk_graph* g, long long extra) {
   Dev& d = g->d;
   const long long n = g->h_ctl->n_total;
   std::vector<int32_t> ldeg((size_t)std::max<long long>(n, 1));
   std::vector<uint8_t> act((size_t)std::max<long long>(n, 1));
   if (n) {
     CK(vr_get(ldeg.data(), d.vr, offsetof(VRec, ldeg), 4, n, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaMemcpyAsync(act.data(), d.active, n, cudaMemcpyDeviceToHost, g->stream));
     CK(cudaStreamSynchronize(g->stream));
-    CK(cudaMemcpy(act.data(), d.active, n, cudaMemcpyDeviceToHost));
   }
   std::vector<int64_t> noff((size_t)std::max<long long>(n, 1));
   std::vector<int32_t> ncap((size_t)std::max<long long>(n, 1));
@@ -420,8 +483,8 @@ igk_status compact_slab(igk_graph* g, long long min_cap) {
     ncap[v] = (int32_t)c;
     used += c;
   }
-  long long cap = std::max<long long>(d.slot_cap, min_cap);
-  while (cap < 2 * used + (1ll << 20)) cap *= 2;  // keep at least half free after compaction
+  long long cap = d.slot_cap;
+  while (cap < 2 * used + (1ll << 20) || cap < used + extra + (1ll << 20)) cap *= 2;  // half free + the batch
   cap = std::min<long long>(cap, (1ll << 31) - 2);
   if (used > cap) return fail(g, IGK_ENOMEM, "adjacency slab cannot hold the graph");
   int32_t *nadj = nullptr, *nadjw = nullptr, *ntwin = nullptr, *fwd = nullptr;
@@ -468,7 +531,8 @@ igk_status compact_slab(igk_graph* g, long long min_cap) {
     return fail(g, IGK_ENOMEM, "slab compaction: allocation failed");
   d.slot_cap = cap;
   g->h_ctl->slab_top = used;
-  CK(cudaMemcpy(&d.ctl->slab_top, &used, 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpyAsync(&d.ctl->slab_top, &g->h_ctl->slab_top, 8, cudaMemcpyHostToDevice, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
   g->compactions++;
   return IGK_OK;
 }
@@ -526,9 +590,21 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   g->vw_unit = vwgt == nullptr;
   g->ew_unit = adjwgt == nullptr;
   g->check = o.check_invariants;
-  if (cudaSetDevice(g->device) != cudaSuccess) {
-    delete g;
-    return IGK_ECUDA;
+  DevGuard dev_guard(g->device);
+  NvtxRange nv("igk_create");
+  {
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != g->device) {
+      delete g;
+      return IGK_ECUDA;
+    }
+  }
+  {  // k_recount: 48 registers, 5 blocks of 256 per SM (measured best:
+     // profiles/r01_s15_recount_ab.txt), computed per handle and device
+    int sms = 0, occ = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_recount, 256, 0);
+    g->recount_blocks = sms * std::max(1, std::min(occ, 5));
   }
   Dev& d = g->d;
   d.k = k;
@@ -575,7 +651,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.rlist, N) && dalloc(g, &d.r3list, N) && dalloc(g, &d.reloc, N) &&
             dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) && dalloc(g, &d.metav, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
-            dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) &&
+            dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) && dalloc(g, &d.delta, N) &&
             dalloc(g, &g->d_red, 259);
   if (!ok) {
     igk_destroy(g);
@@ -629,19 +705,22 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   std::vector<uint8_t> part8((size_t)std::max<int64_t>(n, 1)), act((size_t)std::max<int64_t>(n, 1), 1);
   for (int64_t u = 0; u < n; u++) part8[u] = (uint8_t)init_part[u];
   cudaError_t e = cudaSuccess;
+  // every upload is ordered on the handle's stream after the zero-fills
+  // above (the stream may be a non-blocking one)
+  const auto H2D = cudaMemcpyHostToDevice;
   if (n > 0) {
-    e = cudaMemcpy(d_xadj, xadj, (n + 1) * 8, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess && m2) e = cudaMemcpy(d_adjncy, adjncy, m2 * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess && m2 && d_adjwgt) e = cudaMemcpy(d_adjwgt, adjwgt, m2 * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, off), off.data(), 8, n, cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess && used) e = cudaMemcpy(d.twin, twin_h.data(), used * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, deg), deg.data(), 4, n, cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, ldeg), deg.data(), 4, n, cudaMemcpyHostToDevice, s);
+    e = cudaMemcpyAsync(d_xadj, xadj, (n + 1) * 8, H2D, s);
+    if (e == cudaSuccess && m2) e = cudaMemcpyAsync(d_adjncy, adjncy, m2 * 4, H2D, s);
+    if (e == cudaSuccess && m2 && d_adjwgt) e = cudaMemcpyAsync(d_adjwgt, adjwgt, m2 * 4, H2D, s);
+    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, off), off.data(), 8, n, H2D, s);
+    if (e == cudaSuccess && used) e = cudaMemcpyAsync(d.twin, twin_h.data(), used * 4, H2D, s);
+    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, deg), deg.data(), 4, n, H2D, s);
+    if (e == cudaSuccess) e = vr_put(d.vr, offsetof(VRec, ldeg), deg.data(), 4, n, H2D, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(d.capv, capv.data(), n * 4, H2D, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(d.part, part8.data(), n, H2D, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(d.active, act.data(), n, H2D, s);
+    if (e == cudaSuccess && d.vw) e = cudaMemcpyAsync(d.vw, vwgt, n * 4, H2D, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    if (e == cudaSuccess) e = cudaMemcpy(d.capv, capv.data(), n * 4, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(d.part, part8.data(), n, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(d.active, act.data(), n, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess && d.vw) e = cudaMemcpy(d.vw, vwgt, n * 4, cudaMemcpyHostToDevice);
   }
   if (e == cudaSuccess && n > 0) {
     k_build<<<1184, 256, 0, s>>>(d, d_xadj, d_adjncy, d_adjwgt, n);
@@ -669,13 +748,15 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     return IGK_ECUDA;
   }
   long long red[257];
-  if (cudaMemcpy(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost) != cudaSuccess) {
+  if (cudaMemcpyAsync(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess) {
     igk_destroy(g);
     return IGK_ECUDA;
   }
   g->h_ctl->cut = red[0];
   for (int p = 0; p < k; p++) g->h_ctl->Wp[p] = red[1 + p];
-  if (cudaMemcpy(d.ctl, g->h_ctl, sizeof(Ctl), cudaMemcpyHostToDevice) != cudaSuccess) {
+  if (cudaMemcpyAsync(d.ctl, g->h_ctl, sizeof(Ctl), cudaMemcpyHostToDevice, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess) {
     igk_destroy(g);
     return IGK_ECUDA;
   }
@@ -686,7 +767,8 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
       igk_destroy(g);
       return IGK_ENOMEM;
     }
-    cudaMemset(d.dbg, 0, 128 * 4096 * 8);
+    cudaMemsetAsync(d.dbg, 0, 128 * 4096 * 8, s);
+    cudaStreamSynchronize(s);
   }
   // persistent grids
   g->smem_refine = sizeof(RefSmem);
@@ -694,12 +776,14 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   cudaFuncSetAttribute(k_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
   cudaFuncSetAttribute(k_refine_sh, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
   cudaFuncSetAttribute(k_step, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_step);
-  g->grid_apply = coop_grid((const void*)k_apply, 0, o.blocks_per_sm);
-  g->grid_refine = coop_grid((const void*)k_refine, g->smem_refine, o.blocks_per_sm);
-  g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_step, g->smem_step, o.blocks_per_sm));
-  g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_refine_sh, g->smem_refine, o.blocks_per_sm));
+  const int dv = g->device;
+  g->grid_apply = coop_grid((const void*)k_apply, 0, o.blocks_per_sm, dv);
+  g->grid_refine = coop_grid((const void*)k_refine, g->smem_refine, o.blocks_per_sm, dv);
+  g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_step, g->smem_step, o.blocks_per_sm, dv));
+  g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_refine_sh, g->smem_refine, o.blocks_per_sm, dv));
   if (g->grid_apply > 4096) g->grid_apply = 4096;
-  g->grid_apply_wide = std::min(4096, coop_grid((const void*)k_apply, 0, 64));
+  g->grid_apply_wide = std::min(4096, coop_grid((const void*)k_apply, 0, 64, dv));
+
   g->split_b = kSplitB;
   if (const char* e = getenv("IGK_SPLIT_B")) g->split_b = atoll(e);
   g->epochA = next_epoch(g);
@@ -821,7 +905,9 @@ static igk_status make_room(igk_graph* g) {
     if (need > kNMax) return fail(g, IGK_ENOMEM, "vertex ID space (2^30) exhausted");
     st = grow_vertex_capacity(g, std::min<long long>(kNMax, std::max<long long>(2 * g->d.n_cap, need + 65536)));
   }
-  if (st == IGK_OK && (why & 2)) st = compact_slab(g, 0);
+  // the batch's own slot demand (recorded by the rejected validation) sizes
+  // the compaction, so one compaction suffices for it
+  if (st == IGK_OK && (why & 2)) st = compact_slab(g, g->h_ctl->slab_need);
   return st;
 }
 
@@ -866,7 +952,10 @@ static igk_status notice_wait(igk_graph* g) {
       cudaError_t e = cudaStreamQuery(g->stream);
       if (e == cudaErrorNotReady) continue;
       if (e != cudaSuccess) CK(e);
-      if (*f != g->seq) return sync_ctl(g, 1);
+      if (*f != g->seq) {
+        g->n_notice_fallback++;
+        return sync_ctl(g, 1);
+      }
     }
   }
   std::atomic_thread_fence(std::memory_order_acquire);
@@ -905,6 +994,7 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
       CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, a2, g->smem_refine, g->stream));
       g->d.seq = 0;
       g->launches += 2;
+      g->n_split++;
       CK(cudaEventRecord(g->ev[1], g->stream));
       posted = fast;
     } else {  // apply + refine in ONE persistent launch (k_step)
@@ -918,6 +1008,7 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
       CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
       g->d.seq = 0;
       g->launches++;
+      g->n_fused++;
       CK(cudaEventRecord(g->ev[1], g->stream));
       posted = fast;
     }
@@ -980,6 +1071,7 @@ static igk_status stage_batch(igk_graph* g, const igk_modifier* mods, int64_t co
 igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t count, int64_t* first_new_id,
                                int64_t* bad_index) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_apply_modifiers");
   if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
   if (count == 0) return apply_dev(g, nullptr, 0, first_new_id, bad_index);
   igk_status st = stage_batch(g, mods, count);
@@ -990,6 +1082,7 @@ igk_status igk_apply_modifiers(igk_graph* g, const igk_modifier* mods, int64_t c
 igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, int64_t count,
                                       int64_t* first_new_id, int64_t* bad_index) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_apply_modifiers_device");
   if (count < 0 || (count > 0 && !d_mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
   return apply_dev(g, (const int4*)d_mods, count, first_new_id, bad_index);
 }
@@ -1032,6 +1125,7 @@ static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
 
 igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_refine");
   igk_status st = launch_refine(g, 0);
   if (st != IGK_OK) return st;
   st = sync_ctl(g, 1);
@@ -1041,6 +1135,7 @@ igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
 
 igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_refine_global");
   igk_status st = launch_refine(g, 0, 1);  // boundary scan + refine: one launch
   if (st != IGK_OK) return st;
   st = sync_ctl(g, 1);
@@ -1050,6 +1145,7 @@ igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats) {
 
 igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_refine_sharded");
   if (!comm || !comm->allgather || comm->nranks < 1 || comm->rank < 0 || comm->rank >= comm->nranks)
     return fail(g, IGK_EINVAL, "bad communicator");
   RefineArgs ra = make_refine_args(g, 0);
@@ -1108,6 +1204,7 @@ igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_sta
 igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_refine_stats* stats,
                     int64_t* first_new_id, int64_t* bad_index) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_step");
   if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
   if (count > 0) {
     igk_status st = stage_batch(g, mods, count);
@@ -1119,6 +1216,7 @@ igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_r
 igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,
                            int64_t* first_new_id, int64_t* bad_index) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_step_device");
   if (count < 0 || (count > 0 && !d_mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
   return step_dev(g, (const int4*)d_mods, count, stats, first_new_id, bad_index);
 }
@@ -1126,6 +1224,7 @@ igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t cou
 igk_status igk_partition(const igk_graph* gc, int32_t* out, int64_t cap_len, int64_t* n_total) {
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_partition");
   long long n = g->h_ctl->n_total;
   if (n_total) *n_total = n;
   if (!out || cap_len < n) return fail(g, IGK_EINVAL, "output buffer too small");
@@ -1138,10 +1237,24 @@ igk_status igk_partition(const igk_graph* gc, int32_t* out, int64_t cap_len, int
   return IGK_OK;
 }
 
+igk_status igk_partition_delta(const igk_graph* gc, int32_t* pairs, int64_t cap, int64_t* count) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_partition_delta");
+  const long long nd = g->h_ctl->n_delta;  // in the output head read back by the last refine / step
+  if (count) *count = nd;
+  if (nd == 0) return IGK_OK;
+  if (!pairs || cap < nd) return fail(g, IGK_EINVAL, "delta buffer too small");
+  CK(cudaMemcpyAsync(pairs, g->d.delta, nd * 8, cudaMemcpyDeviceToHost, g->stream));  // one D2H
+  CK(cudaStreamSynchronize(g->stream));
+  return IGK_OK;
+}
+
 igk_status igk_cut_size(const igk_graph* gc, int64_t* out) {
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned) return IGK_ESTATE;
   if (!out) return IGK_EINVAL;
+  ENTRY(g, "igk_cut_size");
   CK(cudaMemcpyAsync(&g->h_ctl->cut, &g->d.ctl->cut, 8, cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
   *out = g->h_ctl->cut;
@@ -1152,6 +1265,7 @@ igk_status igk_part_weights(const igk_graph* gc, int64_t* out_k) {
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned) return IGK_ESTATE;
   if (!out_k) return IGK_EINVAL;
+  ENTRY(g, "igk_part_weights");
   CK(cudaMemcpyAsync(g->h_ctl->Wp, g->d.ctl->Wp, 8 * g->d.k, cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
   for (int p = 0; p < g->d.k; p++) out_k[p] = g->h_ctl->Wp[p];
@@ -1161,13 +1275,19 @@ igk_status igk_part_weights(const igk_graph* gc, int64_t* out_k) {
 igk_status igk_num_vertices(const igk_graph* gc, int64_t* n_total, int64_t* n_active) {
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_num_vertices");
   if (n_total) *n_total = g->h_ctl->n_total;
-  if (n_active) {
+  if (n_active) {  // device reduction over the labels, one 8-byte read back
     long long n = g->h_ctl->n_total;
-    std::vector<uint8_t> act((size_t)std::max<long long>(n, 1));
-    if (n) CK(cudaMemcpy(act.data(), g->d.active, n, cudaMemcpyDeviceToHost));
+    CK(cudaMemsetAsync(g->d_red + 258, 0, 8, g->stream));
+    if (n) {
+      k_count_active<<<592, 256, 0, g->stream>>>(g->d, n, g->d_red + 258);
+      g->launches++;
+      CK(cudaGetLastError());
+    }
     long long c = 0;
-    for (long long v = 0; v < n; v++) c += act[v];
+    CK(cudaMemcpyAsync(&c, g->d_red + 258, 8, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
     *n_active = c;
   }
   return IGK_OK;
@@ -1175,6 +1295,7 @@ igk_status igk_num_vertices(const igk_graph* gc, int64_t* n_total, int64_t* n_ac
 
 igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_recount");
   igk_status st = launch_recount(g);
   if (st != IGK_OK) return st;
   long long red[259];
@@ -1193,48 +1314,93 @@ igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, 
                           int64_t adj_len, int64_t* n_total, int64_t* n_slots) {
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned) return IGK_ESTATE;
-  long long n = g->h_ctl->n_total;
-  std::vector<int64_t> off((size_t)std::max<long long>(n, 1));
-  std::vector<int32_t> deg((size_t)std::max<long long>(n, 1)), ldeg((size_t)std::max<long long>(n, 1));
-  if (n) {
-    CK(vr_get(off.data(), g->d.vr, offsetof(VRec, off), 8, n, cudaMemcpyDeviceToHost, g->stream));
-    CK(vr_get(deg.data(), g->d.vr, offsetof(VRec, deg), 4, n, cudaMemcpyDeviceToHost, g->stream));
-    CK(vr_get(ldeg.data(), g->d.vr, offsetof(VRec, ldeg), 4, n, cudaMemcpyDeviceToHost, g->stream));
-    CK(cudaStreamSynchronize(g->stream));
+  ENTRY(g, "igk_export_csr");
+  const long long n = g->h_ctl->n_total;
+  // live degree of every ID -> exclusive prefix sum (CUB) -> row gather
+  // kernel: the whole CSR is built on the device and read back in three
+  // copies (xadj, adjncy, adjwgt)
+  long long *d_deg = nullptr, *d_off = nullptr;
+  void* tmp = nullptr;
+  size_t tmp_bytes = 0;
+  int32_t *d_adj = nullptr, *d_w = nullptr;
+  auto cleanup = [&]() {
+    cudaFree(d_deg);
+    cudaFree(d_off);
+    cudaFree(tmp);
+    cudaFree(d_adj);
+    cudaFree(d_w);
+  };
+  const long long nn = std::max<long long>(n, 1);
+  if (cudaMalloc(&d_deg, (nn + 1) * 8) != cudaSuccess || cudaMalloc(&d_off, (nn + 1) * 8) != cudaSuccess) {
+    cleanup();
+    return fail(g, IGK_ENOMEM, "export: allocation failed");
   }
+  cudaMemsetAsync(d_deg, 0, (nn + 1) * 8, g->stream);
+  if (n) k_export_deg<<<592, 256, 0, g->stream>>>(g->d, n, d_deg);
+  cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, d_deg, d_off, n + 1, g->stream);
+  if (cudaMalloc(&tmp, std::max<size_t>(tmp_bytes, 1)) != cudaSuccess) {
+    cleanup();
+    return fail(g, IGK_ENOMEM, "export: allocation failed");
+  }
+  cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, d_deg, d_off, n + 1, g->stream);
+  g->launches += n ? 2 : 1;
   long long tot = 0;
-  for (long long v = 0; v < n; v++) tot += ldeg[v];
+  if (cudaMemcpyAsync(&tot, d_off + n, 8, cudaMemcpyDeviceToHost, g->stream) != cudaSuccess ||
+      cudaStreamSynchronize(g->stream) != cudaSuccess) {
+    cleanup();
+    CK(cudaGetLastError());
+    return fail(g, IGK_ECUDA, "export failed");
+  }
   if (n_total) *n_total = n;
   if (n_slots) *n_slots = tot;
-  if (!xadj) return IGK_OK;
-  if (xadj_len < n + 1 || adj_len < tot || !adjncy) return fail(g, IGK_EINVAL, "export buffers too small");
-  xadj[0] = 0;
-  long long pos = 0;
-  std::vector<int32_t> row, roww;
-  for (long long v = 0; v < n; v++) {
-    if (deg[v]) {  // copy the prefix, drop tombstones (-1)
-      row.resize(deg[v]);
-      roww.assign(deg[v], 1);
-      CK(cudaMemcpy(row.data(), g->d.adj + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
-      if (g->d.adjw) CK(cudaMemcpy(roww.data(), g->d.adjw + off[v], deg[v] * 4, cudaMemcpyDeviceToHost));
-      for (int i = 0; i < deg[v]; i++) {
-        if (row[i] < 0) continue;
-        if (pos >= adj_len) return fail(g, IGK_ESTATE, "export: live degree mismatch");
-        adjncy[pos] = row[i];
-        if (adjwgt) adjwgt[pos] = roww[i];
-        pos++;
-      }
-    }
-    xadj[v + 1] = pos;
+  if (!xadj) {
+    cleanup();
+    return IGK_OK;
   }
-  if (pos != tot) return fail(g, IGK_ESTATE, "export: live degree mismatch");
+  if (xadj_len < n + 1 || adj_len < tot || !adjncy) {
+    cleanup();
+    return fail(g, IGK_EINVAL, "export buffers too small");
+  }
+  if (cudaMalloc(&d_adj, std::max<long long>(tot, 1) * 4) != cudaSuccess ||
+      cudaMalloc(&d_w, std::max<long long>(tot, 1) * 4) != cudaSuccess) {
+    cleanup();
+    return fail(g, IGK_ENOMEM, "export: allocation failed");
+  }
+  if (n) {
+    k_export_rows<<<1184, 256, 0, g->stream>>>(g->d, n, d_off, d_adj, d_w);
+    g->launches++;
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaMemcpyAsync(xadj, d_off, (n + 1) * 8, cudaMemcpyDeviceToHost, g->stream);
+  if (e == cudaSuccess && tot) e = cudaMemcpyAsync(adjncy, d_adj, tot * 4, cudaMemcpyDeviceToHost, g->stream);
+  if (e == cudaSuccess && tot && adjwgt) e = cudaMemcpyAsync(adjwgt, d_w, tot * 4, cudaMemcpyDeviceToHost, g->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(g->stream);
+  cleanup();
+  CK(e);
   return IGK_OK;
+}
+
+int32_t igk_debug_paths(const igk_graph* gc, int64_t* out, int32_t cap) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned || !out) return 0;
+  ENTRY(g, "igk_debug_paths");
+  long long dev[PA_N_DEV];
+  if (cudaMemcpyAsync(dev, g->d.ctl->paths, sizeof(dev), cudaMemcpyDeviceToHost, g->stream) != cudaSuccess ||
+      cudaStreamSynchronize(g->stream) != cudaSuccess)
+    return 0;
+  const long long host[] = {g->compactions, g->n_grow, g->n_split, g->n_fused, g->n_notice_fallback};
+  int32_t n = 0;
+  for (int i = 0; i < PA_N_DEV && n < cap; i++) out[n++] = dev[i];
+  for (long long h : host)
+    if (n < cap) out[n++] = h;
+  return n;
 }
 
 int64_t igk_kernel_launches(const igk_graph* g) { return g ? g->launches : 0; }
 
 igk_status igk_compact(igk_graph* g) {
   if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_compact");
   igk_status st = sync_ctl(g, -1);
   if (st != IGK_OK) return st;
   return compact_slab(g, 0);
@@ -1253,6 +1419,7 @@ igk_status igk_store_stats(const igk_graph* g, int64_t* n_total, int64_t* n_acti
 
 igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms) {
   if (!g) return IGK_ESTATE;
+  DevGuard dev_guard(g->device);
   if (g->ms_pending) {  // fast path: the step returned before its end event completed
     igk_graph* gm = const_cast<igk_graph*>(g);
     cudaEventSynchronize(gm->ev[1]);
@@ -1289,6 +1456,7 @@ const char* igk_last_error(const igk_graph* g) { return g ? g->err.c_str() : "nu
 
 void igk_destroy(igk_graph* g) {
   if (!g) return;
+  DevGuard dev_guard(g->device);
   cudaStreamSynchronize(g->stream);
   for (void* p : g->allocs) cudaFree(p);
   if (g->d.hkeys) cudaFree(g->d.hkeys);

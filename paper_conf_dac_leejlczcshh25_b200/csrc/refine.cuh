@@ -60,8 +60,8 @@ __device__ __forceinline__ void nbrs_thread(const Dev& d, int u, F f) {
     uint8_t q[kTC];
 #pragma unroll
     for (int t = 0; t < kTC; t++) {
-      x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
-      w[t] = (i + t < dg && d.adjw) ? __ldg(d.adjw + o + i + t) : 1;
+      x[t] = (i + t < dg) ? ldro(d.adj + o + i + t) : -1;
+      w[t] = (i + t < dg && d.adjw) ? ldro(d.adjw + o + i + t) : 1;
     }
 #pragma unroll
     for (int t = 0; t < kTC; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
@@ -82,7 +82,7 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
 #pragma unroll
   for (int t = 0; t < C; t++) {
     unsigned mk = x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN;
-    dgx[t] = x[t] >= 0 ? __ldg(&d.vr[x[t]].deg) : 0;
+    dgx[t] = x[t] >= 0 ? ldro(&d.vr[x[t]].deg) : 0;
     want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC;  // C1 members are pseudo on sigma2
   }
   unsigned old[C];
@@ -111,7 +111,7 @@ __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t e
     int x[kTC];
     uint8_t q[kTC];
 #pragma unroll
-    for (int t = 0; t < kTC; t++) x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
+    for (int t = 0; t < kTC; t++) x[t] = (i + t < dg) ? ldro(d.adj + o + i + t) : -1;
 #pragma unroll
     for (int t = 0; t < kTC; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
     mark_chunk<kTC>(d, x, q, epN, epC);
@@ -127,7 +127,7 @@ __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN
 #pragma unroll
     for (int t = 0; t < 8; t++) {
       int i = b + t * 32 + lane_id();
-      x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
+      x[t] = i < dg ? ldro(d.adj + o + i) : -1;
     }
 #pragma unroll
     for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
@@ -146,8 +146,8 @@ __device__ __forceinline__ void nbrs_warp(const Dev& d, int u, F f) {
 #pragma unroll
     for (int t = 0; t < 8; t++) {
       int i = b + t * 32 + lane_id();
-      x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
-      w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+      x[t] = i < dg ? ldro(d.adj + o + i) : -1;
+      w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
     }
 #pragma unroll
     for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
@@ -170,7 +170,7 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
   for (long long r0 = 0; r0 < n; r0 += per_round) {
     long long i = r0 + (long long)lane_id() * nw + gw;
     int u = i < n ? get(i) : -1;
-    int dg = u >= 0 ? __ldg(&d.vr[u].deg) : 0;
+    int dg = u >= 0 ? ldro(&d.vr[u].deg) : 0;
     bool heavy = dg > kThreadDeg;
     if (u >= 0 && !heavy) tf(u, i);
     unsigned hm = __ballot_sync(0xffffffffu, heavy);
@@ -181,44 +181,6 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
       wf(uu, r0 + (long long)src * nw + gw);
     }
   }
-}
-
-// Scoped variants: kBlock = true restricts the work to the calling CTA (used
-// by CTA 0 alone for the last, small rounds; barriers become __syncthreads).
-template <bool kBlock, class Get, class TF, class WF>
-__device__ __forceinline__ void foreach_vertex_s(const Dev& d, long long n, Get get, TF tf, WF wf) {
-  if (!kBlock) {
-    foreach_vertex(d, n, get, tf, wf);
-    return;
-  }
-  const long long nw = blockDim.x >> 5, gw = threadIdx.x >> 5;
-  for (long long r0 = 0; r0 < n; r0 += nw * 32) {
-    long long i = r0 + (long long)lane_id() * nw + gw;
-    int u = i < n ? get(i) : -1;
-    int dg = u >= 0 ? __ldg(&d.vr[u].deg) : 0;
-    bool heavy = dg > kThreadDeg;
-    if (u >= 0 && !heavy) tf(u, i);
-    unsigned hm = __ballot_sync(0xffffffffu, heavy);
-    while (hm) {
-      int src = __ffs(hm) - 1;
-      hm &= hm - 1;
-      int uu = __shfl_sync(0xffffffffu, u, src);
-      wf(uu, r0 + (long long)src * nw + gw);
-    }
-  }
-}
-template <bool kBlock, class F>
-__device__ __forceinline__ void rr_for_s(long long n, F f) {
-  if (!kBlock) {
-    rr_for(n, f);
-    return;
-  }
-  for (long long i = threadIdx.x; i < n; i += blockDim.x) f(i);
-}
-template <bool kBlock>
-__device__ __forceinline__ void scope_sync(cg::grid_group& grid) {
-  if (kBlock) __syncthreads();
-  else grid.sync();
 }
 
 // ---------------------------------------------------------------------------
@@ -318,14 +280,14 @@ __device__ void sel_digit0(const Dev& d, SelSmem& sm, ExactFn is_exact, int exac
   __syncthreads();
 }
 
-template <bool kBlock, class Items>
+template <class Items>
 __device__ void sel_accumulate(const Dev& d, SelSmem& sm, int pass, long long nitems, Items items) {
   long long* hb = d.histR + (long long)(pass % 3) * 256 * kDigits;
   long long* hz = d.histR + (long long)((pass + 1) % 3) * 256 * kDigits;
-  rr_for_s<kBlock>((long long)d.k * kDigits, [&](long long t) {
+  rr_for((long long)d.k * kDigits, [&](long long t) {
     if (sm.active[t / kDigits]) hz[t] = 0;
   });
-  rr_for_s<kBlock>(nitems, [&](long long j) {
+  rr_for(nitems, [&](long long j) {
     int p, d0;
     unsigned long long R;
     long long w;
@@ -363,30 +325,29 @@ __device__ void sel_choose(const Dev& d, SelSmem& sm, int pass) {
   __syncthreads();
 }
 
-template <bool kBlock = false, class Items>
+template <class Items>
 __device__ void sel_passes(const Dev& d, SelSmem& sm, cg::grid_group& grid, long long nitems, Items items) {
   int pass = 0;
   while (sm.nactive > 0) {
-    sel_accumulate<kBlock>(d, sm, pass, nitems, items);
-    if (!kBlock) arrive_stamp(d.dbg, 300 + pass - 200);
-    scope_sync<kBlock>(grid);
+    sel_accumulate(d, sm, pass, nitems, items);
+    arrive_stamp(d.dbg, 300 + pass - 200);
+    grid.sync();
     stamp_phase(d.ctl, 300 + pass);
     sel_choose(d, sm, pass);
     pass++;
   }
-  if (pass > 0) scope_sync<kBlock>(grid);  // every CTA finished reading before anyone clears
+  if (pass > 0) grid.sync();  // every CTA finished reading before anyone clears
 }
 
-template <bool kBlock = false, class ExactFn, class Items>
+template <class ExactFn, class Items>
 __device__ void weighted_select(const Dev& d, SelSmem& sm, cg::grid_group& grid, ExactFn is_exact,
                                 int exact_shift, long long nitems, Items items) {
   sel_digit0(d, sm, is_exact, exact_shift);
-  sel_passes<kBlock>(d, sm, grid, nitems, items);
+  sel_passes(d, sm, grid, nitems, items);
 }
 
-template <bool kBlock = false>
 __device__ void sel_clear(const Dev& d, const SelSmem& sm) {
-  rr_for_s<kBlock>((long long)d.k * kDigits, [&](long long t) {
+  rr_for((long long)d.k * kDigits, [&](long long t) {
     if (!sm.used[t / kDigits]) return;
     d.hist0[t] = 0;
     d.histR[t] = 0;
@@ -519,8 +480,8 @@ __device__ __forceinline__ void nbrs_block(const Dev& d, int u, F f) {
 #pragma unroll
     for (int t = 0; t < 4; t++) {
       int i = b + t * (int)blockDim.x + (int)threadIdx.x;
-      x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
-      w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+      x[t] = i < dg ? ldro(d.adj + o + i) : -1;
+      w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
     }
 #pragma unroll
     for (int t = 0; t < 4; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
@@ -544,8 +505,9 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
     });
     block_sum2(s, in, ex);
     if (threadIdx.x == 0) {
+      path_hit(d.ctl, PA_HUB_FILTER);
       counted++;
-      scanned += __ldg(&d.vr[u].deg);
+      scanned += ldro(&d.vr[u].deg);
       if (ex > in) {
         d.markT[u] = ep;
         d.oldp[u] = pu;
@@ -572,7 +534,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
       if (q == pu) in += w; else ex += w;
       return true;
     });
-    scanned += __ldg(&d.vr[u].deg);
+    scanned += ldro(&d.vr[u].deg);
     bool c = ex > in;
     if (c) {  // stamp + snapshot label: the commit reads it while labels change
       d.markT[u] = ep;
@@ -594,7 +556,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     ex = warp_sum(ex);
     if (lane_id() == 0) {
       counted++;
-      scanned += __ldg(&d.vr[u].deg);
+      scanned += ldro(&d.vr[u].deg);
       if (ex > in) {
         d.markT[u] = ep;
         d.oldp[u] = pu;
@@ -632,8 +594,8 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
       unsigned mk[kTC];
 #pragma unroll
       for (int t = 0; t < kTC; t++) {
-        x[t] = (i + t < dg) ? __ldg(d.adj + o + i + t) : -1;
-        w[t] = (i + t < dg && d.adjw) ? __ldg(d.adjw + o + i + t) : 1;
+        x[t] = (i + t < dg) ? ldro(d.adj + o + i + t) : -1;
+        w[t] = (i + t < dg && d.adjw) ? ldro(d.adjw + o + i + t) : 1;
       }
       uint8_t op[kTC];
 #pragma unroll
@@ -668,8 +630,8 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
 #pragma unroll
       for (int t = 0; t < 8; t++) {
         int i = b + t * 32 + lane_id();
-        x[t] = i < dg ? __ldg(d.adj + o + i) : -1;
-        w[t] = (i < dg && d.adjw) ? __ldg(d.adjw + o + i) : 1;
+        x[t] = i < dg ? ldro(d.adj + o + i) : -1;
+        w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
       }
       uint8_t op[8];
 #pragma unroll
@@ -724,7 +686,8 @@ __device__ void hub_commit(const Dev& d, RefSmem& s, const RefineArgs& a, const 
     });
     block_sum2(s, del, dummy);
     if (threadIdx.x == 0) {
-      scanned += __ldg(&d.vr[u].deg);
+      path_hit(ctl, PA_HUB_COMMIT);
+      scanned += ldro(&d.vr[u].deg);
       cut_acc -= del;
       atomic_add_ll(&ctl->Wp[pu], -(long long)vert_w(d.vw, u));
       d.part[u] = kPsi;
@@ -745,16 +708,14 @@ __device__ __forceinline__ bool better(long long ca, int pa, long long cb, int p
 }
 
 // ---------------------------------------------------------------------------
-// R4 rounds (Alg. 4) until the pseudo-partition is empty.
-// kBlock = false: all CTAs with grid barriers (the only mode in use);
-// kBlock = true: the calling CTA alone with __syncthreads barriers.
+// R4 rounds (Alg. 4) until the pseudo-partition is empty,
+// all CTAs with grid barriers.
 // ---------------------------------------------------------------------------
-constexpr int kSmallPsi = 0;  // > 0: hand tails of <= kSmallPsi pending vertices to kBlock mode
 struct RoundState {
   int cur = 0;
   long long rounds = 0, rounds_all = 0, applied_tot = 0, deferred_tot = 0;
 };
-template <bool kBlock, bool kSh>
+template <bool kSh>
 __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::grid_group& grid, long long c,
                            int exact_shift_id, RoundState& rs, long long& scanned, long long& cut_acc,
                            const ShardArgs& sh_in) {
@@ -776,13 +737,13 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
   const int nhp = ldv(&ctl->nhubP);  // final after F3: hubs pending in the rounds
   auto round_sync = [&](int id) {  // per-round arrival slots 20 + 2r (gain), 21 + 2r (apply)
     const bool per_round = (id == 208 || id == 209) && rounds_all < 40;
-    if (!kBlock) arrive_stamp(d.dbg, per_round ? 20 + 2 * (int)rounds_all + (id - 208) : id % 100);
-    scope_sync<kBlock>(grid);
-    stamp_phase(ctl, kBlock ? id + 20 : id);
+    arrive_stamp(d.dbg, per_round ? 20 + 2 * (int)rounds_all + (id - 208) : id % 100);
+    grid.sync();
+    stamp_phase(ctl, id);
   };
   while (true) {
     const int np = ldv(&ctl->npsi[cur]);
-    if (np == 0 || (!kBlock && np <= kSmallPsi)) break;
+    if (np == 0) break;
     const int nxt = cur == 1 ? 2 : 1;
     const int32_t* plist = d.psi[cur];
     int32_t* pnext = d.psi[nxt];
@@ -805,7 +766,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     // -- gain: selection + best part, one adjacency pass per vertex
     long long sel_cnt = 0;
     if (!kSh || sh.mode != kModeFinish) {  // (the finish kernel of a sharded round skips to the install)
-    rr_for_s<kBlock>(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
+    rr_for(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
     auto emit_move = [&](long long j, int u, int best, long long g, long long pwv, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
       d.tgt[u] = (uint8_t)best;
@@ -815,7 +776,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       long long w = vert_w(d.vw, u);
       atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
       atomic_add_ll(&ctl->tot3[r3][best], w);
-      if (imbal) ctl->st[ST_IMBAL] = 1;
+      if (imbal) {
+        ctl->st[ST_IMBAL] = 1;
+        path_hit(ctl, PA_WFALLBACK);
+      }
       if (sharded)
         sh.out[atomicAdd(&ctl->nrec, 1)] =
             make_int4(u, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)), (int)g,
@@ -830,7 +794,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       long long w = vert_w(d.vw, u);
       atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
       atomic_add_ll(&ctl->tot3[r3][best], w);
-      if (imbal) ctl->st[ST_IMBAL] = 1;
+      if (imbal) {
+        ctl->st[ST_IMBAL] = 1;
+        path_hit(ctl, PA_WFALLBACK);
+      }
       if (sharded)
         sh.out[atomicAdd(&ctl->nrec, 1)] =
             make_int4(u, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)), (int)g,
@@ -860,39 +827,50 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       }
       return u;
     };
+    // thread bucket (degree <= kThreadDeg, one load round trip): the whole
+    // prefix sits in registers (static indices only -- no local-memory
+    // tally); conn(u, p) for each neighbour's label p is a register-only
+    // sum over the <= 16 slots, so every candidate part is evaluated
+    // exactly as the warp / CTA buckets do it (reading Q6).
     auto tf = [&](int u, long long j) {
       const long long vwu = vert_w(d.vw, u);
-      scanned += __ldg(&d.vr[u].deg);
-      int qs[kThreadDeg];
-      int ws[kThreadDeg];
-      int m = 0;
+      long long o;
+      int dg;
+      vr_ld(d, u, o, dg);
+      scanned += dg;
+      int x[kThreadDeg], w[kThreadDeg];
+      uint8_t q[kThreadDeg];
+#pragma unroll
+      for (int t = 0; t < kThreadDeg; t++) {
+        x[t] = t < dg ? ldro(d.adj + o + t) : -1;
+        w[t] = (t < dg && d.adjw) ? ldro(d.adjw + o + t) : 1;
+      }
+#pragma unroll
+      for (int t = 0; t < kThreadDeg; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : kDel;  // tombstone: no part
       bool sel = true;
       long long pwv = 0;
-      nbrs_thread(d, u, [&](int x, int w, uint8_t q) {
-        if (q == kPsi) {
-          if (x < u) sel = false;  // a smaller-ID pseudo neighbour moves first (Alg. 4 L8)
-          return sel;
-        }
-        qs[m] = q;
-        ws[m] = w;
-        m++;
-        pwv += w;
-        return true;
-      });
+#pragma unroll
+      for (int t = 0; t < kThreadDeg; t++) {
+        if (q[t] == kPsi && x[t] < u) sel = false;  // a smaller-ID pseudo neighbour moves first (Alg. 4 L8)
+        if (q[t] < kDel) pwv += w[t];
+      }
       if (!sel) {
         d.meta[j] = 0;
         return;
       }
+      auto conn_of = [&](int p) {
+        int cc = 0;
+#pragma unroll
+        for (int t = 0; t < kThreadDeg; t++) cc += q[t] == p ? w[t] : 0;
+        return (long long)cc;
+      };
       int best = -1;
       long long bc = -1;
-      for (int i = 0; i < m; i++) {
-        int p = qs[i];
-        bool seen = false;
-        for (int t = 0; t < i; t++) seen |= qs[t] == p;
-        if (seen) continue;
-        long long cc = 0;
-        for (int t = i; t < m; t++) cc += qs[t] == p ? ws[t] : 0;
-        if (s.Wr[p] + vwu > c) continue;
+#pragma unroll
+      for (int t = 0; t < kThreadDeg; t++) {
+        const int p = q[t];
+        if (p >= kDel || s.Wr[p] + vwu > c) continue;  // tombstone / pseudo / ineligible (Q3)
+        const long long cc = conn_of(p);
         if (better(cc, p, bc, best, s.Wr)) {
           best = p;
           bc = cc;
@@ -904,7 +882,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         bc = 0;
         if (s.Wr[best] + vwu > c) {
           imbal = true;
-          for (int t = 0; t < m; t++) bc += qs[t] == best ? ws[t] : 0;
+          bc = conn_of(best);
         }
       }
       sel_cnt++;
@@ -913,7 +891,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     auto wf = [&](int u, long long j) {
       const long long vwu = vert_w(d.vw, u);
       int* wc = s.wconn[warp_id()];
-      if (lane_id() == 0) scanned += __ldg(&d.vr[u].deg);
+      if (lane_id() == 0) {
+        scanned += ldro(&d.vr[u].deg);
+        path_hit(ctl, PA_WARP_GAIN);
+      }
       bool lb = false;
       long long pwv = 0;
       nbrs_warp(d, u, [&](int x, int w, uint8_t q) {
@@ -966,8 +947,8 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         }
       }
     };
-    foreach_vertex_s<kBlock>(d, np, get, tf, wf);
-    if (!kBlock) {  // hubs in the pseudo-partition: one CTA each
+    foreach_vertex(d, np, get, tf, wf);
+    {  // hubs in the pseudo-partition: one CTA each
       int* conn = s.wconn[0];
       for (int h = blockIdx.x; h < nhp; h += gridDim.x) {
         const int u = __ldcg(d.hubP + h);
@@ -1022,6 +1003,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         }
         __syncthreads();
         if (threadIdx.x == 0) {
+          path_hit(ctl, PA_HUB_GAIN);
           if (blocked) {
             d.metav[u] = 0;
           } else {
@@ -1041,7 +1023,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
               imbal = true;
             }
             sel_cnt++;
-            scanned += __ldg(&d.vr[u].deg);
+            scanned += ldro(&d.vr[u].deg);
             emit_move_v(u, best, bc, pwv, imbal);
           }
         }
@@ -1059,7 +1041,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     if (kSh && sh.mode == kModeGain) return;  // the host all-gathers the move records
     if (kSh && sh.mode == kModeFinish) {
       // install the other ranks' moves of this round (per vertex, metav)
-      rr_for_s<kBlock>(sh.nrecs, [&](long long r) {
+      rr_for(sh.nrecs, [&](long long r) {
         const int4 e = sh.recs[r];
         const int u = e.x;
         if (IGK_OWNED(sh, u)) return;
@@ -1101,7 +1083,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     sel_digit0(d, s.sel, [](int d0) { return d0 != 0; }, exact_shift_id);
     if (s.sel.nactive > 0) {
       // tie groups (moves of an overflowing part with its threshold digit 0)
-      rr_for_s<kBlock>(np, [&](long long j) {
+      rr_for(np, [&](long long j) {
         int p, d0;
         unsigned long long R;
         long long w;
@@ -1115,11 +1097,21 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       round_sync(212);
       const int ntie = ldv(&ctl->ntie);
       bool local_ok = true;
+      int nexact = 0, n64 = 0;
       for (int p = 0; p < k; p++)
-        if (s.sel.active[p]) local_ok &= s.sel.exact[p] && ldv(&ctl->tiecnt[p]) <= kTieMax;
+        if (s.sel.active[p]) {
+          local_ok &= s.sel.exact[p] && ldv(&ctl->tiecnt[p]) <= kTieMax;
+          nexact += s.sel.exact[p] != 0;
+          n64 += s.sel.exact[p] == 0;
+        }
+      if (tid == 0) {
+        if (nexact) path_hit(ctl, PA_KEY_EXACT, nexact);
+        if (n64) path_hit(ctl, PA_KEY64, n64);
+        if (!local_ok) path_hit(ctl, PA_TIE_GRID);
+      }
       if (local_ok) {
         // one CTA per overflowing part finishes its select in shared memory
-        for (int p = kBlock ? 0 : (int)blockIdx.x; p < k; p += kBlock ? 1 : (int)gridDim.x) {
+        for (int p = blockIdx.x; p < k; p += gridDim.x) {
           if (!s.sel.active[p]) continue;
           if (threadIdx.x == 0) s.tie_n = 0;
           __syncthreads();
@@ -1133,7 +1125,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
           }
           __syncthreads();
           unsigned key = block_select_ids(s, s.tie_n, s.sel.base[p], s.sel.T[p]);
-          if (threadIdx.x == 0) ctl->kres[p] = key;
+          if (threadIdx.x == 0) {
+            ctl->kres[p] = key;
+            path_hit(ctl, PA_TIE_CTA);
+          }
           __syncthreads();
         }
         round_sync(213);
@@ -1154,7 +1149,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
                                    (unsigned)e.x;
           return true;
         };
-        sel_passes<kBlock>(d, s.sel, grid, ntie, tie_items);
+        sel_passes(d, s.sel, grid, ntie, tie_items);
       }
     }
     int kd = 1 << 30;
@@ -1167,7 +1162,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     }
     // -- apply the prefix (moves with key < K*); the rest stay pseudo
     long long app = 0;
-    rr_for_s<kBlock>(np, [&](long long j) {
+    rr_for(np, [&](long long j) {
       int u = __ldcg(plist + j);
       if (u < 0) return;
       unsigned m = __ldcg(d.meta + j);
@@ -1196,17 +1191,17 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       long long sa = warp_sum(app);
       if (lane_id() == 0 && sa) atomicAdd(&ctl->applied3[r3], (int)sa);
     }
-    rr_for_s<kBlock>((long long)k * kDigits, [&](long long t) { d.hist0[t] = 0; });
-    rr_for_s<kBlock>(k, [&](long long p) { ctl->tiecnt[p] = 0; });
+    rr_for((long long)k * kDigits, [&](long long t) { d.hist0[t] = 0; });
+    rr_for(k, [&](long long p) { ctl->tiecnt[p] = 0; });
     if (tid == 0) ctl->ntie = 0;
-    sel_clear<kBlock>(d, s.sel);
+    sel_clear(d, s.sel);
     round_sync(209);
     const int napp = ldv(&ctl->applied3[r3]), nsel = ldv(&ctl->selected3[r3]);
     if (napp == 0 && nsel > 0) {
       // L = 0: force the first move (reading Q8); it is the threshold item K*
       const int uf = (int)(kr & 0xffffffffu);
       const int nn = ldv(&ctl->npsi[nxt]);
-      rr_for_s<kBlock>(nn, [&](long long j) {
+      rr_for(nn, [&](long long j) {
         if (__ldcg(pnext + j) == uf) pnext[j] = -1;
       });
       if (tid == 0) {
@@ -1215,6 +1210,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         atomic_add_ll(&ctl->Wp[p], vert_w(d.vw, uf));
         atomic_add_ll(&ctl->cut, (long long)__ldcg(d.pw + uf) - __ldcg(d.gain + uf));
         ctl->st[ST_IMBAL] = 1;
+        path_hit(ctl, PA_FORCED_L0);
       }
       round_sync(210);
     }
@@ -1262,8 +1258,8 @@ __device__ __forceinline__ void boundary_mark(const Dev& d, uint32_t epA) {
     if (placed && !heavy) {
       const int4* a4 = reinterpret_cast<const int4*>(d.adj + o);
       for (int i = 0; i < dg && !bnd; i += 8) {  // two int4 per round trip, then 8 label gathers
-        int4 a0 = __ldg(a4 + (i >> 2));
-        int4 a1 = (i + 4 < dg) ? __ldg(a4 + (i >> 2) + 1) : make_int4(-1, -1, -1, -1);
+        int4 a0 = ldro(a4 + (i >> 2));
+        int4 a1 = (i + 4 < dg) ? ldro(a4 + (i >> 2) + 1) : make_int4(-1, -1, -1, -1);
         const int xs[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
         uint8_t qs[8];
 #pragma unroll
@@ -1285,7 +1281,7 @@ __device__ __forceinline__ void boundary_mark(const Dev& d, uint32_t epA) {
 #pragma unroll
         for (int t = 0; t < 8; t++) {
           int i = b + 32 * t + lane;
-          x[t] = i < hd ? __ldg(d.adj + ho + i) : -1;
+          x[t] = i < hd ? ldro(d.adj + ho + i) : -1;
         }
         bool e = false;
 #pragma unroll
@@ -1309,7 +1305,10 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     if (tid == 0) ctl->refine_skipped = 1;  // uniform exit: nothing was modified
     return;
   }
-  if (tid == 0) ctl->refine_skipped = 0;
+  if (tid == 0) {
+    ctl->refine_skipped = 0;
+    ctl->n_delta = 0;  // appended only after the last round (many barriers later)
+  }
   const long long c = cap_of(ldv(&ctl->W), a.e_ppm, k);
   const int exact_shift_id = ((d.idbits + 7) / 8) * 8 - 8;
 
@@ -1336,7 +1335,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     rs.rounds_all = ldv(&ctl->rs_rounds_all);
     rs.applied_tot = ldv(&ctl->rs_applied);
     rs.deferred_tot = ldv(&ctl->rs_deferred);
-    run_rounds<false, kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
+    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
     flush_partial();
     grid.sync();  // every CTA read the round state before it is written back
     if (tid == 0 && sh.mode == kModeFinish) {
@@ -1381,11 +1380,11 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       return ld_part(d.part, u) == kPsi ? u : -1;  // C1 joins beyond np0
     };
     auto mt = [&](int u, long long) {
-      scanned += __ldg(&d.vr[u].deg);
+      scanned += ldro(&d.vr[u].deg);
       mark_nbrs_thread(d, u, a.epN, a.epC1);
     };
     auto mw = [&](int u, long long) {
-      if (lane_id() == 0) scanned += __ldg(&d.vr[u].deg);
+      if (lane_id() == 0) scanned += ldro(&d.vr[u].deg);
       mark_nbrs_warp(d, u, a.epN, a.epC1);
     };
     foreach_vertex(d, np0, get, mt, mw);
@@ -1420,6 +1419,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     bool any = false;
     for (int p = 0; p < k; p++) any |= ldv(&ctl->Wp[p]) > c;
     if (any) {
+      if (tid == 0) path_hit(ctl, PA_R3);
       for (int p = threadIdx.x; p < k; p += blockDim.x) {
         long long wp = ldv(&ctl->Wp[p]);
         s.sel.used[p] = wp > c;
@@ -1445,7 +1445,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
           if (q == pv) in += w; else ex += w;
           return true;
         });
-        scanned += __ldg(&d.vr[v].deg);
+        scanned += ldro(&d.vr[v].deg);
         emit(v, pv, in - ex);
       };
       auto wf = [&](int v, long long) {
@@ -1457,7 +1457,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         in = warp_sum(in);
         ex = warp_sum(ex);
         if (lane_id() == 0) {
-          scanned += __ldg(&d.vr[v].deg);
+          scanned += ldro(&d.vr[v].deg);
           emit(v, pv, in - ex);
         }
       };
@@ -1475,6 +1475,11 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         return true;
       };
       weighted_select(d, s.sel, grid, [](int d0) { return d0 != 0 && d0 != 255; }, exact_shift_id, nr3, items);
+      if (tid == 0) {
+        int n64 = 0;
+        for (int p = 0; p < k; p++) n64 += s.sel.used[p] && s.sel.found[p] && (s.sel.d0[p] == 0 || s.sel.d0[p] == 255);
+        if (n64) path_hit(ctl, PA_R3_KEY64, n64);
+      }
       // evict every item with key <= the threshold of its part
       rr_for(nr3, [&](long long j) {
         int p, d0;
@@ -1519,9 +1524,22 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     rs.applied_tot = ldv(&ctl->rs_applied);
     rs.deferred_tot = ldv(&ctl->rs_deferred);
   } else {
-    run_rounds<false, kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
+    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
   }
   const long long rounds = rs.rounds, applied_tot = rs.applied_tot, deferred_tot = rs.deferred_tot;
+
+  // delta list for the caller (igk_partition_delta): every vertex of the
+  // frontier F (it holds all that can have moved, I4) whose label now
+  // differs from its label before the refine; inserted vertices (oldp = psi)
+  // are listed with their first placement.  The labels are final after the
+  // last round's barrier.
+  rr_for(ldv(&ctl->npsi[0]), [&](long long i) {
+    const int u = __ldcg(d.psi[0] + i);
+    const uint8_t p = u >= 0 ? ld_part(d.part, u) : kDel;
+    const bool ch = p != kDel && p != kPsi && p != __ldcg(d.oldp + u);
+    const int slot = agg_append(&ctl->n_delta, ch);
+    if (ch) d.delta[slot] = make_int2(u, (int)p);
+  });
 
   block_atomic_add(&ctl->cut, cut_acc, s.red);
   block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);

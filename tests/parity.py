@@ -59,22 +59,40 @@ class Pair:
             assert so[2] == sg[2], f"{where}: bad index oracle {so[2]} gpu {sg[2]}"
         return so[0]
 
+    def check_delta(self, pre, where=""):
+        """igk_partition_delta == the oracle's label changes of the last
+        refine: every vertex whose part now differs from its label before the
+        refine (pending / inserted vertices included), deleted ones excluded."""
+        post = self.O.partition()
+        old = np.full(len(post), -2, np.int32)
+        old[: len(pre)] = pre
+        idx = np.nonzero((post >= 0) & (post != old))[0]
+        d = self.G.partition_delta()
+        got = d[np.argsort(d[:, 0], kind="stable")] if len(d) else d.reshape(0, 2)
+        exp = np.stack([idx, post[idx]], axis=1).astype(np.int32)
+        assert got.shape == exp.shape and np.array_equal(got, exp), \
+            f"{where}: delta differs ({len(got)} gpu pairs vs {len(exp)} expected)"
+
     def refine(self, where=""):
+        pre = self.O.partition()
         so, sto = self.O.refine()
         sg, stg = self.G.refine()
         assert so == sg, where
         diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
         assert not diff, f"{where}: stats differ (oracle, gpu): {diff}"
         self.invariants(stg["cut"], where)
+        self.check_delta(pre, where)
         return sto, stg
 
     def refine_global(self, where=""):
+        pre = self.O.partition()
         so, sto = self.O.refine_global()
         sg, stg = self.G.refine_global()
         assert so == sg, where
         diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
         assert not diff, f"{where}: global refine stats differ (oracle, gpu): {diff}"
         self.invariants(stg["cut"], where)
+        self.check_delta(pre, where)
         return sto, stg
 
 

@@ -68,3 +68,14 @@ def test_gpu_free_import_fails_loudly_without_library(tmp_path, monkeypatch):
     monkeypatch.setattr(igk, "_lib", None)
     with pytest.raises(ImportError):
         igk.lib()
+
+
+def test_no_read_only_path_loads_in_the_fused_kernels():
+    """k_step runs apply_body and refine_body in ONE launch: the refine reads
+    adjacency / records the apply just wrote, so no load in those sources may
+    use the non-coherent read-only path (__ldg / ld.global.nc), which
+    requires data to stay unchanged for the whole kernel."""
+    csrc = os.path.join(PKG, "csrc")
+    for f in ("common.cuh", "apply.cuh", "refine.cuh", "step.cuh"):
+        code = "\n".join(l.split("//")[0] for l in open(os.path.join(csrc, f)).read().splitlines())
+        assert "__ldg(" not in code and "ld.global.nc" not in code, f

@@ -273,11 +273,13 @@ def test_fused_step_api(split, check, monkeypatch):
     for it in range(8):
         b = gi.next_batch(S, cfg)
         assert P.O.apply(b)[0] == 0
+        pre = P.O.partition()
         so, sto = P.O.refine()
         sg, stg, bad = P.G.step(b)
         assert sg == so and bad == -1
         assert all(sto[f] == stg[f] for f in COMMON)
         P.invariants(stg["cut"], f"step it{it}")
+        P.check_delta(pre, f"step it{it}")
         P.compare_state(f"step it{it}")
         if it == 3:
             before = (P.G.partition().tobytes(), P.G.cut())
@@ -313,12 +315,14 @@ def test_c4_full_size_step_split_launch():
         b = gi.next_batch(S, cfg)
         assert len(b) >= 131072
         assert P.O.apply(b)[0] == 0
+        pre = P.O.partition()
         so, sto = P.O.refine()
         sg, stg, bad = P.G.step(b)
         assert sg == so and bad == -1
         diff = {f: (sto[f], stg[f]) for f in COMMON if sto[f] != stg[f]}
         assert not diff, diff
         P.invariants(stg["cut"], f"C4 step it{it}")
+        P.check_delta(pre, f"C4 step it{it}")
         P.compare_state(f"C4 step it{it}")
 
 

@@ -1,0 +1,90 @@
+"""Store maintenance and robustness through the C ABI (GPU).
+
+* export -> create resume (NEXT-4, "preallocated" store): a graph
+  exported with igk_export_csr / igk_partition after many iterations and
+  re-created with igk_create (deleted IDs kept as isolated vertices, then
+  deleted again) continues the SAME modifier stream bit-identically to the
+  original handle, which itself stays bit-exact with the oracle.
+* sticky CUDA errors: a kernel fault returns IGK_ECUDA once and poisons the
+  handle; every later call returns IGK_ESTATE (include/igk.h conventions).
+  Run in a subprocess: the fault kills that process's CUDA context.
+"""
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import igk_inputs as gi
+import paper_conf_dac_leejlczcshh25_b200 as igk
+from tests.parity import Pair
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_export_create_resume_continues_identically():
+    cfg = gi.CONFIGS["C1"]
+    g = gi.make_graph(20_000, 64, gi.graph_seed(1) + 77)
+    part, _ = gi.metis_partition(g, 4)
+    P = Pair(g.xadj, g.adjncy, 4, cfg["eps"], part, check=True)
+    P.refine("settle")
+    S = gi.Stream(g, 4321)
+    for it in range(8):
+        assert P.apply(S.next(gi.MODE_MIX, 0.02), f"it{it}") == 0
+        P.refine(f"it{it}")
+    P.compare_state("before export", full_csr=True)
+    # export the device state (checkpoint) and re-create a handle from it
+    xadj, adj, w = P.G.export_csr(sort_rows=False)
+    lab = P.G.partition()
+    dead = np.nonzero(lab == -1)[0]
+    init = np.where(lab >= 0, lab, 0).astype(np.int32)
+    G2 = igk.IGKGraph(xadj, adj, 4, cfg["eps"], init, check=True)
+    if len(dead):
+        s, _, _ = G2.apply(np.stack([np.ones(len(dead)), dead, np.zeros(len(dead)), np.zeros(len(dead))], 1)
+                           .astype(np.int32))
+        assert s == 0
+        G2.refine()
+    assert np.array_equal(G2.partition(), lab) and G2.cut() == P.G.cut()
+    assert np.array_equal(G2.part_weights(), P.G.part_weights())
+    # continue the same stream on both
+    for it in range(8, 16):
+        b = S.next(gi.MODE_MIX, 0.02)
+        assert P.apply(b, f"it{it}") == 0
+        _, stg = P.refine(f"it{it}")
+        s2, _, _ = G2.apply(b)
+        assert s2 == 0
+        _, st2 = G2.refine()
+        assert np.array_equal(G2.partition(), P.G.partition()), it
+        assert st2["cut"] == stg["cut"] and st2["rounds"] == stg["rounds"], it
+    x1, a1, w1 = P.G.export_csr()
+    x2, a2, w2 = G2.export_csr()
+    assert np.array_equal(x1, x2) and np.array_equal(a1, a2) and np.array_equal(w1, w2)
+
+
+_STICKY = r"""
+import ctypes as C, numpy as np, sys
+sys.path.insert(0, sys.argv[1])
+import igk_inputs as gi
+import paper_conf_dac_leejlczcshh25_b200 as igk
+g = gi.make_graph(2000, 16, 3)
+G = igk.IGKGraph(g.xadj, g.adjncy, 2, 0.1, gi.block_partition(g.n, 2))
+L = igk.lib()
+bad = C.c_int64(-1)
+s = L.igk_apply_modifiers_device(G.h, C.c_void_p(0x1000), 4096, None, C.byref(bad))   # not device memory
+assert s == igk.ECUDA, s
+msg = L.igk_last_error(G.h).decode()
+assert msg, msg
+st = igk.Stats()
+assert L.igk_refine(G.h, C.byref(st)) == igk.ESTATE
+assert L.igk_partition(G.h, None, 0, None) == igk.ESTATE
+m = np.zeros((1, 4), np.int32)
+assert L.igk_step(G.h, m.ctypes.data, 1, None, None, None) == igk.ESTATE
+print("STICKY_OK", msg)
+"""
+
+
+def test_cuda_error_is_sticky():
+    r = subprocess.run([sys.executable, "-c", _STICKY, ROOT], capture_output=True, text=True, timeout=300)
+    assert "STICKY_OK" in r.stdout, r.stdout + r.stderr
