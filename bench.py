@@ -190,6 +190,58 @@ def cpu_baseline(g, part, k, eps, batches, gpu_cuts, iters):
             "parity_cut_checked_iters": min(n_it, len(gpu_cuts)), "parity_cut_match": cut_ok}
 
 
+PH_NAMES = {220: "boundary", 201: "F0_filter", 202: "F1_commit_expand", 203: "F2_filter", 204: "F3_commit",
+            205: "R3_restore", 206: "R3_restore", 207: "R3_restore", 208: "round_gain", 209: "round_move",
+            210: "round_move", 212: "round_move", 213: "round_move", 211: "epilogue"}
+
+
+def phase_profile(G, batches_dev, peak):
+    """Per-phase roofline of the refine (verdict r1 item 3):
+    profile mode records a %globaltimer stamp after every grid barrier and,
+    per phase, the adjacency entries scanned and list items processed.
+    Algorithmic bytes of a phase = 5 B per scanned entry (4 B neighbour ID +
+    1 B label gather) + 16 B per list item (its vertex record / list entry);
+    time = the phase's stamp interval (barrier included).  Run AFTER the timed
+    region on further iterations of the same stream (profile mode replaces
+    the step's completion notice by a full control-block copy)."""
+    G.set_profile(True)
+    acc = {}
+    for ptr, cnt in batches_dev:
+        G.step_device(ptr, cnt)
+        st = G.phase_times(1)
+        work = G.phase_work()
+        prev = st[0][1] if st else 0
+        for pid, t in st[1:]:
+            name = PH_NAMES.get(pid)  # sub-phase stamps (select passes) merge into the next named one
+            if name:
+                a = acc.setdefault(name, {"ns": 0, "scanned": 0, "items": 0})
+                a["ns"] += t - prev
+                prev = t
+        for name, (sc, it) in work.items():
+            a = acc.setdefault(name, {"ns": 0, "scanned": 0, "items": 0})
+            a["scanned"] += sc
+            a["items"] += it
+    G.set_profile(False)
+    n = max(len(batches_dev), 1)
+    out = {}
+    for name, a in acc.items():
+        if a["ns"] == 0 and a["scanned"] == 0:
+            continue
+        by = 5 * a["scanned"] + 16 * a["items"]
+        us = a["ns"] / 1e3 / n
+        gbs = by / n / (a["ns"] / n) if a["ns"] else 0.0  # bytes per ns = GB/s
+        out[name] = {"us": round(us, 2), "bytes": int(by / n), "gbs": round(gbs, 2), "frac": gbs / peak}
+    gm = [out[x] for x in ("round_gain", "round_move") if x in out]
+    gain_move = None
+    if gm:
+        by = sum(x["bytes"] for x in gm)
+        us = sum(x["us"] for x in gm)
+        gain_move = {"bytes": by, "us": round(us, 2), "gbs": by / (us * 1e3) if us else 0.0,
+                     "frac": (by / (us * 1e3)) / peak if us else 0.0}
+    return {"iterations": n, "phases": out, "gain_move": gain_move,
+            "bytes_rule": "5 B per scanned adjacency entry + 16 B per list item; time = stamp interval"}
+
+
 def full_repartition(G, k, igk_cut, ms_per_step):
     """The metric's "cut vs full repartition": METIS k-way
     (default options, ufactor 30 = the same 3% imbalance) from scratch on the
@@ -283,7 +335,8 @@ def main():
     g, part, metis_cut, S, cfg, k, desc = workload(args, rank)
     W, K = args.warmup, args.steps
     e2e_steps = 0 if (args.profile or args.shard) else K
-    batches = [gi.next_batch(S, cfg) for _ in range(W + K + e2e_steps + (1 if e2e_steps else 0))]
+    n_prof = 0 if (args.profile or args.shard) else 5
+    batches = [gi.next_batch(S, cfg) for _ in range(W + K + e2e_steps + (1 if e2e_steps else 0) + n_prof)]
     stream = torch.cuda.current_stream()
     G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part, device=local, stream=stream.cuda_stream)
     G.refine()  # settle the METIS partition (untimed)
@@ -349,7 +402,7 @@ def main():
         h_delta = torch.empty((dcap, 2), dtype=torch.int32, pin_memory=True).numpy()
         G.step(batches[W + K])  # untimed warm-up of the host-batch path (first call sizes its device buffer)
         G.partition_delta(h_delta)
-        for b in batches[W + K + 1:]:
+        for b in batches[W + K + 1: len(batches) - n_prof]:
             hb = torch.empty(b.shape, dtype=torch.int32, pin_memory=True).numpy()
             hb[...] = b
             h_batches.append(hb)
@@ -380,6 +433,12 @@ def main():
                # changing): their work is reported so the two legs can be compared
                "affected_per_step": aff_e / len(h_batches), "rounds_per_step": rounds_e / len(h_batches),
                "store_compacted": G.store_stats()["slab_cap"] != slab0}
+
+    # ---- per-phase roofline (profile mode, after the timed legs)
+    phases = None
+    if n_prof:
+        pb = [torch.from_numpy(b).cuda() for b in batches[len(batches) - n_prof:]]
+        phases = phase_profile(G, [(t.data_ptr(), len(t)) for t in pb], peaks()[0])
 
     # ---- S9 cut/weight reduction (full store scan, HBM-bound): own roofline
     s9 = None
@@ -450,6 +509,8 @@ def main():
     }
     if e2e:
         line["e2e"] = e2e
+    if phases:
+        line["phases"] = phases
     if not args.no_repartition and not args.profile:
         line["full_repartition"] = full_repartition(G, k, G.cut(), t_ms / K)
     if not args.no_cpu_baseline and not args.profile:

@@ -244,6 +244,18 @@ enum {
   IGK_PATH_N
 };
 int32_t igk_debug_paths(const igk_graph* g, int64_t* out, int32_t cap);
+/* instrumentation: profile mode on/off.  On: every refine records the
+ * %globaltimer phase stamps (igk_debug_phase_times) and, per phase, the
+ * adjacency entries scanned and the list items processed
+ * (igk_debug_phase_work), for per-phase roofline accounting; the step's
+ * fast completion notice is replaced by a full control-block copy. */
+igk_status igk_debug_set_profile(igk_graph* g, int32_t on);
+/* per-phase work of the last refine in profile mode, index = phase:
+ * 0 boundary scan (igk_refine_global), 1 F0 R1 filter, 2 F1 commit C1 +
+ * expansion marks, 3 F2 R2 filter, 4 F3 commit C2, 5 R3 restoration,
+ * 6 round gain (all rounds), 7 round prefix select + move (all rounds).
+ * Returns the number of phases written (<= cap). */
+int32_t igk_debug_phase_work(const igk_graph* g, int64_t* scanned, int64_t* items, int32_t cap);
 /* device-side duration (ms) of the last igk_refine / apply / recount kernel,
  * measured with CUDA events on the handle's stream */
 igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply_ms, float* recount_ms);

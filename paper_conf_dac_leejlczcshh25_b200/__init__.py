@@ -28,7 +28,7 @@ SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "i
            "igk_step", "igk_step_device", "igk_refine_sharded",
            "igk_partition", "igk_partition_delta", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
-           "igk_debug_paths",
+           "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work",
            "igk_last_error", "igk_destroy"]
 
 
@@ -147,6 +147,10 @@ def lib():
         L.igk_partition_delta.argtypes = [P, P, i64, i64p]
         L.igk_debug_paths.restype = C.c_int32
         L.igk_debug_paths.argtypes = [P, i64p, C.c_int32]
+        L.igk_debug_set_profile.restype = C.c_int
+        L.igk_debug_set_profile.argtypes = [P, C.c_int32]
+        L.igk_debug_phase_work.restype = C.c_int32
+        L.igk_debug_phase_work.argtypes = [P, i64p, i64p, C.c_int32]
         L.igk_cut_size.restype = C.c_int
         L.igk_cut_size.argtypes = [P, i64p]
         L.igk_part_weights.restype = C.c_int
@@ -295,6 +299,22 @@ class IGKGraph:
         if s != OK:
             raise IGKError(s, self._err())
         return out[: cnt.value]
+
+    PHASES = ["boundary", "F0_filter", "F1_commit_expand", "F2_filter", "F3_commit", "R3_restore",
+              "round_gain", "round_move"]
+
+    def set_profile(self, on: bool = True):
+        """profile mode: phase stamps + per-phase work counters on every refine"""
+        s = lib().igk_debug_set_profile(self.h, int(bool(on)))
+        if s != OK:
+            raise IGKError(s, self._err())
+
+    def phase_work(self):
+        """{phase: (adjacency entries scanned, list items)} of the last refine (profile mode)"""
+        sc = np.zeros(8, np.int64)
+        it = np.zeros(8, np.int64)
+        n = lib().igk_debug_phase_work(self.h, _p(sc, C.c_int64), _p(it, C.c_int64), 8)
+        return {self.PHASES[i]: (int(sc[i]), int(it[i])) for i in range(n)}
 
     def debug_paths(self):
         """{path name: count} of the device / host path counters (igk_debug_paths)."""

@@ -104,7 +104,11 @@ struct Ctl {
   int idph[128];                // phase ids
   int ndone;                    // CTAs finished (publish: the last one posts the notice)
   long long paths[PA_N_DEV];    // device path counters (cumulative)
+  long long phscan[8];          // profile mode: adjacency entries scanned per refine phase (PH_*)
+  long long phitems[8];         // profile mode: list items (vertices) processed per refine phase
 };
+// refine phases of the per-phase work counters (igk_debug_phase_work)
+enum PhaseIdx { PH_BOUNDARY = 0, PH_F0, PH_F1, PH_F2, PH_F3, PH_R3, PH_GAIN, PH_MOVE, PH_N };
 __device__ __forceinline__ void path_hit(Ctl* ctl, int which, long long v = 1) {
   atomicAdd((unsigned long long*)&ctl->paths[which], (unsigned long long)v);
 }

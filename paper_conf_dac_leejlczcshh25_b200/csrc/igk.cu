@@ -278,6 +278,7 @@ struct igk_graph {
   long long newid_cap = 0;
   int check = 0;
   int debug_phases = 0;
+  int prof = 0;  // profile mode (igk_debug_set_profile): phase stamps + per-phase work counters
   int4* d_rec_out = nullptr;  // sharded rounds: this rank's move records
   int4* d_rec_in = nullptr;   //                 all ranks' records
   int4* h_rec = nullptr;      //                 pinned host staging (out, then in)
@@ -873,6 +874,9 @@ static RefineArgs make_refine_args(igk_graph* g, int after_apply, int global) {
   a.epA = g->epochA;
   a.after_apply = after_apply;
   a.global = global;
+  a.prof = g->prof;
+  if (g->prof)  // per-phase counters of THIS refine (ordered before its launch on the stream)
+    cudaMemsetAsync(&g->d.ctl->phscan[0], 0, sizeof(long long) * 16, g->stream);
   return a;
 }
 
@@ -1378,6 +1382,29 @@ igk_status igk_export_csr(const igk_graph* gc, int64_t* xadj, int64_t xadj_len, 
   cleanup();
   CK(e);
   return IGK_OK;
+}
+
+igk_status igk_debug_set_profile(igk_graph* g, int32_t on) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  g->prof = on != 0;
+  g->debug_phases = on != 0 || getenv("IGK_DEBUG_PHASES") != nullptr || getenv("IGK_DEBUG_ARRIVALS") != nullptr;
+  return IGK_OK;
+}
+
+int32_t igk_debug_phase_work(const igk_graph* gc, int64_t* scanned, int64_t* items, int32_t cap) {
+  igk_graph* g = const_cast<igk_graph*>(gc);
+  if (!g || g->poisoned) return 0;
+  ENTRY(g, "igk_debug_phase_work");
+  long long buf[16];
+  if (cudaMemcpyAsync(buf, &g->d.ctl->phscan[0], sizeof(buf), cudaMemcpyDeviceToHost, g->stream) != cudaSuccess ||
+      cudaStreamSynchronize(g->stream) != cudaSuccess)
+    return 0;
+  const int n = std::min<int>(cap, PH_N);
+  for (int i = 0; i < n; i++) {
+    if (scanned) scanned[i] = buf[i];
+    if (items) items[i] = buf[8 + i];
+  }
+  return n;
 }
 
 int32_t igk_debug_paths(const igk_graph* gc, int64_t* out, int32_t cap) {

@@ -28,7 +28,23 @@ struct RefineArgs {
   uint32_t epA;     // stamp of the affected set (hubs in A carry markH == epA)
   int after_apply;  // fused step: skip (leave the state untouched) if the batch was rejected
   int global;       // NEXT-1: the partition boundary joins A before F0 (igk_refine_global)
+  int prof;         // profile mode: per-phase work counters (Ctl::phscan / phitems)
 };
+
+// profile mode: the adjacency entries this thread scanned since the last
+// flush go to the phase's counter (block reduction + one atomic per CTA)
+struct PhaseWork {
+  long long mark = 0;
+};
+#define PHASE_FLUSH(ph, items)                                                 \
+  do {                                                                         \
+    if (a.prof) {                                                              \
+      block_atomic_add(&d.ctl->phscan[ph], scanned - pw_.mark, s.red);         \
+      pw_.mark = scanned;                                                      \
+      if (blockIdx.x == 0 && threadIdx.x == 0 && (items))                      \
+        atomic_add_ll(&d.ctl->phitems[ph], (long long)(items));                \
+    }                                                                          \
+  } while (0)
 
 // Sharded refine: every rank holds the replicated store and
 // state; the round gain is split by owner (u mod nranks) and the selected
@@ -718,7 +734,7 @@ struct RoundState {
 template <bool kSh>
 __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::grid_group& grid, long long c,
                            int exact_shift_id, RoundState& rs, long long& scanned, long long& cut_acc,
-                           const ShardArgs& sh_in) {
+                           const ShardArgs& sh_in, PhaseWork& pw_) {
   // kSh = false: the single-GPU kernels, all sharding code compiled out
   ShardArgs sh = sh_in;
   if (!kSh) {
@@ -1058,6 +1074,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         if ((unsigned)e.y & (1u << 30)) ctl->st[ST_IMBAL] = 1;
       });
     }
+    PHASE_FLUSH(PH_GAIN, np);
     round_sync(208);
 
     // -- balanced prefix: T_p = c - W_p + 1; K* = min over parts of the first
@@ -1195,6 +1212,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     rr_for(k, [&](long long p) { ctl->tiecnt[p] = 0; });
     if (tid == 0) ctl->ntie = 0;
     sel_clear(d, s.sel);
+    PHASE_FLUSH(PH_MOVE, np);
     round_sync(209);
     const int napp = ldv(&ctl->applied3[r3]), nsel = ldv(&ctl->selected3[r3]);
     if (napp == 0 && nsel > 0) {
@@ -1324,6 +1342,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   stamp_phase(ctl, 200);
   arrive_stamp(d.dbg, 0);
   long long scanned = 0, counted = 0, cnt_ins = 0, cut_acc = 0;
+  PhaseWork pw_;
   auto flush_partial = [&]() {  // split (sharded) modes: per-kernel accumulators to the control block
     block_atomic_add(&ctl->cut, cut_acc, s.red);
     block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
@@ -1335,7 +1354,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     rs.rounds_all = ldv(&ctl->rs_rounds_all);
     rs.applied_tot = ldv(&ctl->rs_applied);
     rs.deferred_tot = ldv(&ctl->rs_deferred);
-    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
+    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh, pw_);
     flush_partial();
     grid.sync();  // every CTA read the round state before it is written back
     if (tid == 0 && sh.mode == kModeFinish) {
@@ -1351,6 +1370,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   if (!kSh || sh.mode != kModePost) {
   if (!kSh && a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
     boundary_mark(d, a.epA);
+    PHASE_FLUSH(PH_BOUNDARY, ldv(&ctl->n_total));
     GRID_SYNC_STAMPED(ctl, 220);
   }
   // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
@@ -1366,6 +1386,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
   block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
   block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
+  PHASE_FLUSH(PH_F0, nA + nhA + np0);
   GRID_SYNC_STAMPED(ctl, 201);
 
   // ---- F1: commit C1 + R2 expansion marks -----------------------------------
@@ -1389,6 +1410,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     };
     foreach_vertex(d, np0, get, mt, mw);
     flush_acc(s, ctl->Wp, k);
+    PHASE_FLUSH(PH_F1, nc + nhC + np0);
   }
   GRID_SYNC_STAMPED(ctl, 202);
 
@@ -1401,6 +1423,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     hub_filter(d, s, d.hubN, nhN, a.epC2, &ctl->nhubC2, d.hubC2, scanned, cntN);
     block_atomic_add(&ctl->st[ST_EXPANDED], cntN, s.red);
     if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
+    PHASE_FLUSH(PH_F2, nN + nhN);
   }
   GRID_SYNC_STAMPED(ctl, 203);
 
@@ -1411,6 +1434,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     commit(d, s, a, nc, d.cand2, a.epC2, false, scanned, cut_acc);
     hub_commit(d, s, a, d.hubC2, nhC2, a.epC2, false, scanned, cut_acc);
     flush_acc(s, ctl->Wp, k);
+    PHASE_FLUSH(PH_F3, nc + nhC2);
   }
   GRID_SYNC_STAMPED(ctl, 204);
 
@@ -1462,6 +1486,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         }
       };
       foreach_vertex(d, ntot, get, tf, wf);
+      PHASE_FLUSH(PH_R3, ntot);
       GRID_SYNC_STAMPED(ctl, 205);
       const int nr3 = ldv(&ctl->nr3);
       auto items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
@@ -1500,6 +1525,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       const int nc = ldv(&ctl->ncand);
       commit(d, s, a, nc, d.cand, a.epE, false, scanned, cut_acc);
       flush_acc(s, ctl->Wp, k);
+      PHASE_FLUSH(PH_R3, nc + nr3);
       if (tid == 0) ctl->st[ST_EVICTED] = nc;
       for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
       GRID_SYNC_STAMPED(ctl, 207);
@@ -1524,7 +1550,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     rs.applied_tot = ldv(&ctl->rs_applied);
     rs.deferred_tot = ldv(&ctl->rs_deferred);
   } else {
-    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh);
+    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh, pw_);
   }
   const long long rounds = rs.rounds, applied_tot = rs.applied_tot, deferred_tot = rs.deferred_tot;
 
