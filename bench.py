@@ -14,8 +14,11 @@ ms_per_step = device ms per incremental iteration (apply + refine)
 e2e         = same metric through the public C ABI with HOST batches (H2D of the
               batch + D2H of the cut inside the timed region)
 --impl reference = the CPU oracle (oracle/) timed on this host (the slow arm).
-Multi-GPU: "replicas" -- each rank refines its own independent graph instance
-(no data-path collective), weak scaling, max over ranks.
+Multi-GPU: by default ONE C4 graph vertex-range sharded
+over the N ranks (igk_options.nranks/rank/nccl_id: the library's own NCCL
+communicator; fixed-size all-reduces of candidate bitmaps and per-round move
+records), strong scaling, device time max over ranks; --replicas runs N
+independent instances (weak scaling).
 """
 from __future__ import annotations
 
@@ -46,7 +49,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2")
+    ap.add_argument("--config", default=None,
+                    help="workload (default: C2 at N=1; C4 vertex-range sharded at N>1)")
     ap.add_argument("--k", type=int, default=0)
     ap.add_argument("--frac", type=float, default=0.0)
     ap.add_argument("--n", type=int, default=0)
@@ -56,8 +60,10 @@ def parse():
     ap.add_argument("--no-repartition", action="store_true", help="skip the METIS full-repartition comparison")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
     ap.add_argument("--shard", action="store_true",
-                    help="N>1: ONE graph, round gain split over the ranks (igk_refine_sharded, strong scaling) "
-                         "instead of independent replicas")
+                    help="ONE graph vertex-range sharded over the ranks (the default at N>1; strong scaling; "
+                         "at N=1 the sharded protocol runs on one rank over an NCCL loopback communicator)")
+    ap.add_argument("--replicas", action="store_true",
+                    help="N>1: independent graph instances per rank (weak scaling) instead of sharding")
     return ap.parse_args()
 
 
@@ -316,6 +322,10 @@ def run_reference(args, rank, world):
 def main():
     args = parse()
     rank, world, local = benchdist.env_ranks()
+    if world > 1 and not args.replicas:
+        args.shard = True
+    if args.config is None:
+        args.config = "C4" if (args.shard and world > 1) else "C2"
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
@@ -334,24 +344,28 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     g, part, metis_cut, S, cfg, k, desc = workload(args, rank)
     W, K = args.warmup, args.steps
-    e2e_steps = 0 if (args.profile or args.shard) else K
+    e2e_steps = 0 if args.profile else K
     n_prof = 0 if (args.profile or args.shard) else 5
     batches = [gi.next_batch(S, cfg) for _ in range(W + K + e2e_steps + (1 if e2e_steps else 0) + n_prof)]
     stream = torch.cuda.current_stream()
-    G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part, device=local, stream=stream.cuda_stream)
-    G.refine()  # settle the METIS partition (untimed)
+    shard_kw = {}
+    if args.shard:  # every rank: the same graph, its own vertex range; the library's NCCL communicator
+        if one_gpu_test:
+            shard_kw = dict(nranks=world, rank=rank, comm=igk.TorchComm())
+        else:
+            uid = [igk.nccl_unique_id() if rank == 0 else None]
+            if dist:
+                dist.broadcast_object_list(uid, src=0)
+            shard_kw = dict(nranks=world, rank=rank, nccl_id=uid[0])
+    G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part, device=local, stream=stream.cuda_stream, **shard_kw)
+    G.refine()  # settle the METIS partition (untimed; collective when sharded)
     dev_batches = [torch.from_numpy(b).cuda() for b in batches[: W + K]]
     flush = None if args.no_flush else torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     gpu_cuts = []
     st_buf = igk.Stats()
-    comm = igk.TorchComm() if (args.shard and dist) else None
-
-    def one_step(i, b):
-        if comm is None:
-            G.step_device(dev_batches[i].data_ptr(), len(b), st_buf)  # igk_step_device: apply + refine
-            return {f: int(getattr(st_buf, f)) for f in igk.STATS}
-        G.apply_device(dev_batches[i].data_ptr(), len(b))  # replicated apply
-        return G.refine_sharded(comm)[1]  # owner-split round gain + per-round record all-gather
+    def one_step(i, b):  # igk_step_device: apply + refine (collective on a sharded handle)
+        G.step_device(dev_batches[i].data_ptr(), len(b), st_buf)
+        return {f: int(getattr(st_buf, f)) for f in igk.STATS}
 
     deg_start = round(2.0 * g.m / g.n, 3)
     for i in range(W):
@@ -372,7 +386,7 @@ def main():
         st = one_step(W + i, b)
         ev[i][1].record(stream)
         ms = G.last_ms()
-        refine_ms += ms["refine"]  # igk_step: ONE fused kernel (k_step = apply + refine)
+        refine_ms += ms["refine"] + ms["apply"]  # igk_step: ONE fused k_step (apply_ms 0); sharded: both halves
         apply_ms += ms["apply"]
         aff += st["affected"]
         rbytes += refine_bytes(st) + 16 * len(b)  # + the batch itself
@@ -385,7 +399,7 @@ def main():
     launches = G.kernel_launches() - l0
     t_ms = sum(a.elapsed_time(b) for a, b in ev)
     t_ms, aff_all = benchdist.reduce_time_and_work(t_ms, aff, dist, "cuda")
-    if comm is not None:
+    if args.shard:
         aff_all = aff  # one shared graph: the work is not multiplied by the ranks
     value = aff_all / (t_ms / 1e3)
 
@@ -469,8 +483,10 @@ def main():
         s9.update(peak=peak, peak_kind=peak_kind, frac=s9["achieved"] / peak)
     achieved = rbytes / (refine_ms / 1e3) / 1e9 if refine_ms > 0 else 0.0
     # batches of >= kSplitB modifiers run as k_apply + k_refine (2 launches per step)
-    split = launches >= 2 * K and comm is None
+    split = launches >= 2 * K and not args.shard
     kname = "k_apply+k_refine (split launch, one step)" if split else "k_step (apply+refine fused)"
+    if args.shard:
+        kname = "k_apply x2 + k_refine_sh x(5 + 2 R) (sharded step)"
     traffic = None
     try:
         tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
@@ -511,7 +527,7 @@ def main():
         line["e2e"] = e2e
     if phases:
         line["phases"] = phases
-    if not args.no_repartition and not args.profile:
+    if not args.no_repartition and not args.profile and not args.shard:
         line["full_repartition"] = full_repartition(G, k, G.cut(), t_ms / K)
     if not args.no_cpu_baseline and not args.profile:
         line["cpu_baseline"] = cpu_baseline(g, part, k, cfg["eps"], batches, gpu_cuts, args.cpu_iters)

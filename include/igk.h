@@ -37,7 +37,7 @@ typedef enum {
   IGK_EINVAL = 1,       /* invalid argument or invalid modifier batch (state unchanged) */
   IGK_ENOMEM = 2,       /* vertex or adjacency capacity exhausted / allocation failed   */
   IGK_ECUDA = 3,        /* CUDA error; the handle is poisoned                            */
-  IGK_ENCCL = 4,        /* reserved for the sharded build                                */
+  IGK_ENCCL = 4,        /* a collective of a sharded handle failed; the handle is poisoned */
   IGK_ESTATE = 5,       /* handle poisoned by an earlier CUDA error, or NULL handle      */
   IGK_WIMBALANCED = 6   /* result valid, but a weighted corner case left W_p > cap (Q8)  */
 } igk_status;
@@ -59,6 +59,16 @@ typedef struct {
   int32_t kind, u, v, w;
 } igk_modifier;
 
+/* Host-side collective for sharded handles without NCCL (tests: gloo over
+ * torch.distributed; also any MPI-like transport).  allreduce: in-place
+ * all-reduce over all ranks of `count` elements at `buf` (HOST memory);
+ * dtype 0 = int64, 1 = uint32; op 0 = sum, 1 = min, 2 = max; returns 0 on
+ * success.  Every rank calls it in the same order with the same count. */
+typedef struct {
+  void* ctx;
+  int32_t (*allreduce)(void* ctx, void* buf, int64_t count, int32_t dtype, int32_t op);
+} igk_comm;
+
 typedef struct {
   int device;              /* CUDA device ordinal                                         */
   void* stream;            /* cudaStream_t; NULL = default stream                          */
@@ -68,6 +78,23 @@ typedef struct {
   int32_t validate;        /* reserved: batches are always validated                       */
   int32_t check_invariants;/* 1 = recount cut/W_p after every refine and compare (slow)    */
   int32_t blocks_per_sm;   /* persistent-kernel CTAs per SM (0 = auto)                     */
+  /* Vertex-range sharding.  nranks > 1: this
+   * handle is rank `rank` of a sharded graph, one process per GPU, all
+   * ranks calling every entry point in the same order with the same
+   * arguments (collective calls).  Rank r owns the IDs [r B, (r+1) B) of the
+   * created graph (B = ceil(n / nranks)) and every r-th inserted ID, stores
+   * the adjacency of its vertices plus the entries of other vertices that
+   * point at them (ghost prefixes), and keeps labels, weights, W_p
+   * replicated.  Each refine exchanges fixed-size all-reduces: the candidate
+   * bitmaps of R1/R2, the restoration keys, and per round the move records
+   * of the selected vertices -- results are bit-identical to one
+   * GPU and to the oracle.  The transport is NCCL (nccl_id: an ncclUniqueId
+   * of 128 bytes from igk_nccl_unique_id, shared by all ranks; the library
+   * creates its communicator on `device`) or the host callback `comm`. */
+  int32_t nranks;          /* 0 or 1 = one GPU                                            */
+  int32_t rank;
+  const void* nccl_id;     /* ncclUniqueId (128 bytes) or NULL                            */
+  const igk_comm* comm;    /* host-callback transport (used when nccl_id == NULL)         */
 } igk_options;
 
 typedef struct {
@@ -135,7 +162,7 @@ igk_status igk_refine(igk_graph* g, igk_refine_stats* stats);
  * called periodically to undo the cut drift of many incremental iterations
  * (P:322).  Same arguments, stats and return codes as igk_refine;
  * stats->affected counts the boundary as affected. */
-igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats);
+igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats);  /* one GPU only (EINVAL when sharded) */
 
 /* One incremental iteration: igk_apply_modifiers + igk_refine fused (both
  * kernels launched back to back, one host synchronisation).  If the batch is
@@ -147,24 +174,10 @@ igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_r
 igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,
                            int64_t* first_new_id, int64_t* bad_index);
 
-/* Vertex-range sharded refinement across nranks processes (one per GPU).
- * Every rank holds the replicated store and state (it applies the same
- * batches); the per-round gain (the adjacency scans of the pending vertices,
- * Alg. 4 L1-23) is split by owner = vertex ID mod nranks, and each round the
- * selected moves are exchanged as 16-byte records {u, meta, #nbr, placed
- * weight} through `allgather`; every rank then computes the same balanced
- * prefix and applies all moves.  Results are identical to
- * igk_refine on one GPU (and to the oracle).
- * allgather(ctx, send, nsend, recv, recv_cap): collective over the ranks;
- * send/recv are HOST buffers of 16-byte records (recv may alias send); must
- * write the concatenation of all ranks' records in rank order to recv and
- * return their total count (<= recv_cap), or -1 on failure (-> IGK_ENCCL). */
-typedef struct {
-  int32_t nranks, rank;
-  void* ctx;
-  int64_t (*allgather)(void* ctx, const void* send, int64_t nsend, void* recv, int64_t recv_cap);
-} igk_comm;
-igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_stats* stats);
+/* NCCL unique id for sharded handles (call on ONE rank, share the 128
+ * bytes with the others, pass as igk_options.nccl_id).  NCCL is loaded at
+ * run time (libnccl.so.2); IGK_ENCCL if it is unavailable. */
+igk_status igk_nccl_unique_id(void* out, int64_t len);
 
 /* The k-way partition (V_1..V_k; P:50 the part of every vertex).
  * out[v] for v < n_total: part in [0,k), -1 = deleted, -2 = pending (in the

@@ -25,7 +25,7 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine", "igk_refine_global",
-           "igk_step", "igk_step_device", "igk_refine_sharded",
+           "igk_step", "igk_step_device", "igk_nccl_unique_id",
            "igk_partition", "igk_partition_delta", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
            "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work",
@@ -38,67 +38,57 @@ PATHS = ["hub_filter", "hub_commit", "hub_gain", "tie_cta", "tie_grid", "key_exa
          "compaction", "vertex_growth", "split_step", "fused_step", "notice_fallback"]
 
 
+ALLREDUCE_FN = C.CFUNCTYPE(C.c_int32, C.c_void_p, C.c_void_p, C.c_int64, C.c_int32, C.c_int32)
+
+
+class Comm(C.Structure):
+    """igk_comm: host-callback collective of sharded handles (include/igk.h)"""
+    _fields_ = [("ctx", C.c_void_p), ("allreduce", ALLREDUCE_FN)]
+
+
 class Options(C.Structure):
     _fields_ = [("device", C.c_int), ("stream", C.c_void_p), ("max_vertices", C.c_int64),
                 ("max_slots", C.c_int64), ("slack_min", C.c_int32), ("validate", C.c_int32),
-                ("check_invariants", C.c_int32), ("blocks_per_sm", C.c_int32)]
+                ("check_invariants", C.c_int32), ("blocks_per_sm", C.c_int32),
+                ("nranks", C.c_int32), ("rank", C.c_int32), ("nccl_id", C.c_void_p),
+                ("comm", C.POINTER(Comm))]
 
 
 class Stats(C.Structure):
     _fields_ = [(s, C.c_int64) for s in STATS]
 
 
-ALLGATHER_FN = C.CFUNCTYPE(C.c_int64, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64)
-
-
-class Comm(C.Structure):
-    _fields_ = [("nranks", C.c_int32), ("rank", C.c_int32), ("ctx", C.c_void_p), ("allgather", ALLGATHER_FN)]
-
-
 class TorchComm:
-    """igk_comm over torch.distributed: the per-round all-gather of 16-byte
-    move records (igk_refine_sharded).  gloo moves host tensors; NCCL moves
-    device tensors.  Plumbing only: the records are produced and consumed by
-    the CUDA kernels."""
+    """igk_comm over torch.distributed (host tensors: the gloo backend), for
+    sharded handles without NCCL -- the tests' transport (several ranks on
+    one GPU).  Plumbing only: the library hands it host buffers of fixed
+    size (candidate bitmaps, restoration keys, move records, scalars) to
+    all-reduce; every value is produced and consumed by the CUDA kernels."""
+
+    _DT = {0: ("int64", 8), 1: ("uint32", 4)}
 
     def __init__(self, group=None):
         import torch.distributed as dist
         self.dist, self.group = dist, group
         self.nranks = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
-        self.backend = dist.get_backend(group)
         self.calls = 0
-        self._cb = ALLGATHER_FN(self._allgather)
-        self.struct = Comm(self.nranks, self.rank, None, self._cb)
+        self._cb = ALLREDUCE_FN(self._allreduce)
+        self.struct = Comm(None, self._cb)
 
-    def gather_records(self, recs: np.ndarray) -> np.ndarray:
-        """all ranks' (n_i, 4) int32 record arrays, concatenated in rank order"""
-        import torch
-        dev = torch.device("cuda", torch.cuda.current_device()) if self.backend == "nccl" else torch.device("cpu")
-        cnt = torch.tensor([len(recs)], dtype=torch.int64, device=dev)
-        cnts = [torch.zeros_like(cnt) for _ in range(self.nranks)]
-        self.dist.all_gather(cnts, cnt, group=self.group)
-        counts = [int(c.item()) for c in cnts]
-        mx = max(max(counts), 1)
-        buf = np.zeros((mx, 4), np.int32)
-        buf[: len(recs)] = recs
-        t = torch.from_numpy(buf).to(dev)
-        outs = [torch.empty_like(t) for _ in range(self.nranks)]
-        self.dist.all_gather(outs, t, group=self.group)
-        self.calls += 1
-        return np.concatenate([o.cpu().numpy()[:c] for o, c in zip(outs, counts)]).reshape(-1, 4)
-
-    def _allgather(self, ctx, send, nsend, recv, cap):
+    def _allreduce(self, ctx, buf, count, dtype, op):
         try:
-            recs = np.empty((nsend, 4), np.int32)
-            if nsend:
-                C.memmove(recs.ctypes.data, send, nsend * 16)
-            out = self.gather_records(recs)
-            if len(out) > cap:
-                return -1
-            if len(out):
-                C.memmove(recv, np.ascontiguousarray(out).ctypes.data, len(out) * 16)
-            return len(out)
+            import torch
+            name, size = self._DT[dtype]
+            arr = np.ctypeslib.as_array((C.c_uint8 * (count * size)).from_address(buf)).view(name)
+            # gloo has no uint32: reduce the bit patterns as int64 (values < 2^32, at most one
+            # non-zero contribution per element for SUM, or a MIN / MAX of non-negative values)
+            t = torch.from_numpy(arr.astype(np.int64))
+            red = {0: self.dist.ReduceOp.SUM, 1: self.dist.ReduceOp.MIN, 2: self.dist.ReduceOp.MAX}[op]
+            self.dist.all_reduce(t, op=red, group=self.group)
+            arr[:] = t.numpy().astype(name)
+            self.calls += 1
+            return 0
         except Exception:  # never let an exception cross the C ABI
             import traceback
             traceback.print_exc()
@@ -139,8 +129,8 @@ def lib():
         L.igk_step.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
         L.igk_step_device.restype = C.c_int
         L.igk_step_device.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
-        L.igk_refine_sharded.restype = C.c_int
-        L.igk_refine_sharded.argtypes = [P, C.POINTER(Comm), C.POINTER(Stats)]
+        L.igk_nccl_unique_id.restype = C.c_int
+        L.igk_nccl_unique_id.argtypes = [P, i64]
         L.igk_partition.restype = C.c_int
         L.igk_partition.argtypes = [P, i32p, i64, i64p]
         L.igk_partition_delta.restype = C.c_int
@@ -185,18 +175,35 @@ def _p(a, ct):
     return None if a is None else a.ctypes.data_as(C.POINTER(ct))
 
 
+def nccl_unique_id() -> bytes:
+    """ncclUniqueId (128 bytes) for sharded handles: create on one rank, share."""
+    buf = C.create_string_buffer(128)
+    s = lib().igk_nccl_unique_id(buf, 128)
+    if s != OK:
+        raise IGKError(s, "igk_nccl_unique_id failed (NCCL not loadable?)")
+    return buf.raw
+
+
 class IGKGraph:
     """One GPU-resident graph + k-way partition (igk_create)."""
 
     def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, device=0, stream=None,
-                 max_vertices=0, max_slots=0, slack_min=0, check=False, blocks_per_sm=0):
+                 max_vertices=0, max_slots=0, slack_min=0, check=False, blocks_per_sm=0,
+                 nranks=1, rank=0, nccl_id: bytes | None = None, comm: "TorchComm | None" = None):
+        """nranks > 1: rank `rank` of a vertex-range sharded graph (collective
+        calls; every rank passes the same graph and batches).  Transport: NCCL
+        from `nccl_id` (nccl_unique_id() on one rank, shared), else `comm`."""
         L = lib()
         xadj = np.ascontiguousarray(xadj, dtype=np.int64)
         adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
         part = np.ascontiguousarray(part, dtype=np.int32)
         vwgt = None if vwgt is None else np.ascontiguousarray(vwgt, dtype=np.int32)
         adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
-        o = Options(device, stream or None, max_vertices, max_slots, slack_min, 1, int(check), blocks_per_sm)
+        self._id = None if nccl_id is None else C.create_string_buffer(bytes(nccl_id), 128)
+        self._comm = comm  # keeps the callback alive as long as the handle
+        o = Options(device, stream or None, max_vertices, max_slots, slack_min, 1, int(check), blocks_per_sm,
+                    int(nranks), int(rank), None if self._id is None else C.cast(self._id, C.c_void_p),
+                    None if comm is None else C.pointer(comm.struct))
         h = C.c_void_p()
         s = L.igk_create(C.byref(o), len(xadj) - 1, _p(xadj, C.c_int64), _p(adjncy, C.c_int32),
                          _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(h))
@@ -239,14 +246,6 @@ class IGKGraph:
         """igk_refine_global: the partition boundary (adj_ext != 0) joins A, then refine."""
         st = Stats()
         s = lib().igk_refine_global(self.h, C.byref(st))
-        if s not in (OK, WIMBALANCED):
-            raise IGKError(s, self._err())
-        return s, {f: int(getattr(st, f)) for f in STATS}
-
-    def refine_sharded(self, comm: "TorchComm"):
-        """igk_refine_sharded: round gain split by owner, move records all-gathered."""
-        st = Stats()
-        s = lib().igk_refine_sharded(self.h, C.byref(comm.struct), C.byref(st))
         if s not in (OK, WIMBALANCED):
             raise IGKError(s, self._err())
         return s, {f: int(getattr(st, f)) for f in STATS}

@@ -28,7 +28,16 @@ struct ApplyArgs {
   long long n0;  // n_total before the batch
   uint32_t epD, epT, epG, epA;
   int vw_unit, ew_unit;
+  int phases;  // bit 0: V1 + V2 (validate, allocate); bit 1: M12..M4 (mutate).  Sharded handles
+               // run them as two launches with the all-reduced verdict in between; else 3.
 };
+
+// Sharded store (common.cuh Dev::nranks): an edge modifier is applied on the
+// ranks that own one of its endpoints (both directions are stored there);
+// vertex modifiers everywhere (labels, weights, W, W_p are replicated).  The
+// cut is a per-rank partial: an edge event is counted by owner(m.y), the
+// edges of a deleted vertex by owner(u).
+__device__ __forceinline__ bool rel_edge(const Dev& d, const int4& m) { return own(d, m.y) || own(d, m.z); }
 
 __device__ __forceinline__ unsigned long long edge_key(int u, int v) {
   unsigned a = (unsigned)min(u, v), b = (unsigned)max(u, v);
@@ -161,6 +170,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   if (tid == 0) ctl->nph = 0;
   stamp_phase(ctl, 100);
   arrive_stamp(d.dbg, 0);
+  if (a.phases & 1) {
   // ---- V1: counts, duplicate hash, per-vertex counters ---------------------
   {
     int cnt = 0;
@@ -191,7 +201,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
         }
         s = (s + 1) & d.hmask;
       }
-      if (m.x == kEdgeIns) {
+      if (m.x == kEdgeIns && rel_edge(d, m)) {
         if (m.y < d.n_cap) atomicAdd(d.icnt + m.y, 1);
         if (m.z < d.n_cap) atomicAdd(d.icnt + m.z, 1);
       }
@@ -293,8 +303,9 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     auto exists = [&]() {  // search the shorter prefix
       return dgy <= dgz ? thread_find(d.adj, ofy, dgy, m.z) >= 0 : thread_find(d.adj, ofz, dgz, m.y) >= 0;
     };
+    const bool rel = !edge || rel_edge(d, m);  // the existence / degree checks belong to the endpoint owners
     if (m.x == kEdgeDel) {
-      ok = m.y != m.z && live_y && live_z && dup_free() && exists();
+      ok = m.y != m.z && live_y && live_z && dup_free() && (!rel || exists());
     } else if (m.x == kVertDel) {
       ok = yo && acty && vcy == 1;
       if (ok) {  // kVdC-entry work chunks of this deletion
@@ -308,17 +319,17 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       ok = m.y != m.z && (live_y || is_new(m.y)) && (live_z || is_new(m.z));
       ok = ok && (a.ew_unit ? (m.w == 1) : (m.w >= 1 && m.w <= kEwMax));
       ok = ok && dup_free();
-      if (ok && live_y && live_z) ok = !exists();
+      if (ok && live_y && live_z && rel) ok = !exists();
       if (ok) {
         long long du = (m.y < n0 ? ldy : 0) + icy;
         long long dv = (m.z < n0 ? ldz : 0) + icz;
-        ok = du <= kDegMax && dv <= kDegMax;
+        ok = (du <= kDegMax || !own(d, m.y)) && (dv <= kDegMax || !own(d, m.z));
       }
     } else {
       ok = false;
     }
     if (!ok) atomicMin((long long*)&ctl->err_idx, i);
-    if (m.x == kEdgeIns) {  // slots for every endpoint an insertion touches (first touch)
+    if (m.x == kEdgeIns && rel) {  // slots for every endpoint an insertion touches (first touch)
       int ends[2] = {m.y, m.z};
       for (int e = 0; e < 2; e++) {
         int x = ends[e];
@@ -343,9 +354,21 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     }
   });
   GRID_SYNC_STAMPED(ctl, 102);
+  if (tid == 0 && d.sharded) {  // this rank's verdict, all-reduced (MIN, MAX) before the mutation launch
+    ctl->sh_err[0] = ctl->err_idx;
+    ctl->sh_err[1] = ctl->err_nomem;
+  }
+  }  // V1 + V2
+  if (!(a.phases & 2)) return true;
+  const long long n_ins = ldv(&ctl->n_ins);
 
   // ---- scratch reset (hash, counters) on both the failure and success paths ---
-  const bool failed = ldv(&ctl->err_idx) != kNoErr || ldv(&ctl->err_nomem) != 0;
+  long long e_idx = ldv(&ctl->err_idx), e_mem = ldv(&ctl->err_nomem);
+  if (d.sharded) {  // the global verdict: every rank rejects or applies the batch alike
+    e_idx = ldv(&ctl->sh_err[0]);
+    e_mem = ldv(&ctl->sh_err[1]);
+  }
+  const bool failed = e_idx != kNoErr || e_mem != 0;  // (the host reads sh_err on sharded handles)
   for (long long i = tid; i <= d.hmask; i += nthr) {
     d.hkeys[i] = ~0ull;
     d.hcnt[i] = 0;
@@ -370,7 +393,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   // 32 entries is done by the whole warp (ballot loop)
   rr_for_warp(B, [&](long long i, bool valid) {
     int4 m = valid ? a.mods[i] : make_int4(-1, 0, 0, 0);
-    const bool ed = m.x == kEdgeDel;
+    const bool ed = m.x == kEdgeDel && rel_edge(d, m);
     // search the shorter prefix; the twin gives the reverse slot
     int a0 = m.y, b0 = m.z;
     long long oa = 0;
@@ -402,7 +425,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       atomicSub(&d.vr[m.y].ldeg, 1);
       atomicSub(&d.vr[m.z].ldeg, 1);
       uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
-      if (pu != kPsi && pv != kPsi && pu != pv) cut_acc -= w;
+      if (pu != kPsi && pv != kPsi && pu != pv && own(d, m.y)) cut_acc -= w;
       mark_affected(d, m.y, a.epA, du);
       mark_affected(d, m.z, a.epA, dv);
     }
@@ -434,7 +457,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       }
       if (x >= 0) {
         const uint8_t px = ld_part(d.part, x);
-        if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < x)) cut_acc -= w;
+        if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < x) && own(d, u)) cut_acc -= w;
       }
       if (x >= 0 && !xdel) mark_affected(d, x, a.epA, dx);
       if (ch.y == 0 && lane_id() == 0) {
@@ -468,7 +491,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     for (int e = 0; e < kVdC; e++) {
       if (x[e] < 0) continue;
       uint8_t px = ld_part(d.part, x[e]);
-      if (pu != kPsi && px != kPsi && pu != px && (!xdel[e] || u < x[e])) cut_acc -= w[e];
+      if (pu != kPsi && px != kPsi && pu != px && (!xdel[e] || u < x[e]) && own(d, u)) cut_acc -= w[e];
       if (!xdel[e]) {  // the twin is u's entry in x's prefix
         d.adj[tw[e]] = -1;
         atomicSub(&d.vr[x[e]].ldeg, 1);
@@ -566,7 +589,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   // ---- M4: edge insertions (Alg. 1): append to the dense prefixes ----------
   rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
-    if (m.x != kEdgeIns) return;
+    if (m.x != kEdgeIns || !rel_edge(d, m)) return;
     int pu_pos = atomicAdd(&d.vr[m.y].deg, 1);
     int pv_pos = atomicAdd(&d.vr[m.z].deg, 1);
     atomicAdd(&d.vr[m.y].ldeg, 1);
@@ -581,7 +604,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       d.adjw[sv] = m.w;
     }
     uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
-    if (pu != kPsi && pv != kPsi && pu != pv) cut_acc += m.w;
+    if (pu != kPsi && pv != kPsi && pu != pv && own(d, m.y)) cut_acc += m.w;
     mark_affected(d, m.y, a.epA, pu_pos + 1);
     mark_affected(d, m.z, a.epA, pv_pos + 1);
   });

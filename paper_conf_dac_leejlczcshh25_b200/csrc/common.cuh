@@ -79,7 +79,10 @@ struct Ctl {
   int rs_pending;      // pending vertices left for the next sharded round
   long long slab_need; // slots the last rejected batch asked for (capacity failure: sizes the compaction)
   int n_delta;         // (vertex, part) pairs in the delta list of the last refine
-  int n_delta_pad;
+  int sh_flag;         // sharded refine: restoration (R3) needed after kShF3
+  int sh_np;           // sharded refine: pending vertices after F3 / R3 (length of the canonical list)
+  int sh_pad;
+  long long sh_err[2]; // sharded apply: [0] lowest invalid index, [1] capacity flags (all-reduced MIN / MAX)
   // ---- device-side state ----
   long long Wp[256];   // part weights
   long long tot3[3][256];  // per round (mod 3): weight of selected moves per target part
@@ -131,6 +134,18 @@ struct Dev {
   int64_t slot_cap;  // slab capacity (entries)
   int32_t slack_min;
   int32_t idbits;    // bits to hold any vertex ID < n_cap
+  // vertex-range sharding: rank `rank` of `nranks` owns the IDs
+  // [rank * sh_blk, (rank + 1) * sh_blk) of the created graph and the inserted
+  // IDs n with (n - sh_n0) % nranks == rank.  It stores the adjacency of its
+  // own vertices in full and, for every other vertex, the "ghost" prefix of
+  // its neighbours that this rank owns, so both directions of every edge it
+  // touches are local (twins stay valid).  nranks == 1: one GPU owns all.
+  int32_t nranks, rank;
+  int32_t sharded;   // the sharded protocol runs (nranks > 1, or a transport given for one rank)
+  int64_t sh_n0, sh_blk;
+  uint64_t* bm;      // sharded refine: candidate bitmap (n_cap bits), all-reduced (sum of disjoint bits = OR)
+  uint32_t* lossbuf; // sharded R3: (int - ext) + 2^31 of owned restoration candidates, 0 = none; all-reduced
+  int4* recs;        // sharded rounds: one move record per position of the canonical pending list
   // graph store (S0)
   VRec* vr;          // per-vertex record: prefix offset, length, live degree (one sector)
   int32_t* capv;     // capacity
@@ -192,6 +207,13 @@ struct Dev {
 // ---------------------------------------------------------------------------
 // helpers
 // ---------------------------------------------------------------------------
+// the rank owning vertex v (its full adjacency lives there); any v on one GPU
+__host__ __device__ __forceinline__ bool own(const Dev& d, long long v) {
+  if (d.nranks <= 1) return true;
+  if (v < 0) return false;
+  const long long r = v < d.sh_n0 ? v / d.sh_blk : (v - d.sh_n0) % d.nranks;
+  return r == d.rank;
+}
 __device__ __forceinline__ long long ldv(const long long* p) { return *(volatile const long long*)p; }
 __device__ __forceinline__ int ldv(const int* p) { return *(volatile const int*)p; }
 __device__ __forceinline__ uint8_t ld_part(const uint8_t* p, int64_t i) { return __ldcg(p + i); }

@@ -4,6 +4,8 @@
 // persistent cooperative launch per call.  This file holds the handle, the
 // store build (S0), the cut/weight reduction (S9) and the exports.
 #include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>  // types only: NCCL is loaded at run time (nccl_api), not linked
 #include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
@@ -12,12 +14,14 @@
 #include <cstddef>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
 #include <vector>
 
 #include "../../include/igk.h"
 #include "apply.cuh"
 #include "common.cuh"
+#include "recount.cuh"
 #include "refine.cuh"
 #include "step.cuh"
 #include <cub/cub.cuh>
@@ -94,7 +98,7 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
       dg = 0;
       ld = 0;
     }
-    ent += ld;  // live adjacency entries (algorithmic bytes of the scan)
+    ent += own(d, v) ? ld : 0;  // live adjacency entries (algorithmic bytes of the scan)
     nact += act;
     const bool placed = act && pv != kPsi;
     if (unit_wp) {
@@ -110,7 +114,7 @@ __global__ void __launch_bounds__(256) k_recount(Dev d, long long n, long long* 
     } else if (placed) {
       acc_add(s_wp, pv, vert_w(d.vw, v));
     }
-    if (!placed) dg = 0;  // pending vertices own no cut edges
+    if (!placed || !own(d, v)) dg = 0;  // pending vertices own no cut edges; sharded: the owner of the smaller endpoint counts
     // inclusive prefix of the tile's chunk counts
     int incl = (dg + 3) >> 2;
 #pragma unroll
@@ -254,10 +258,23 @@ __global__ void k_export_part(Dev d, long long n, int32_t* out) {
 struct igk_graph {
   int device = 0;
   int recount_blocks = 0;    // k_recount grid (occupancy-derived at create)
+  int recount_tma_blocks = 0;  // k_recount_tma grid (unit edge weights)
+  int recount_tma = 1;       // S9 kernel: TMA-pipelined (1) or direct gathers (0; IGK_RECOUNT=gather)
   long long n_grow = 0;      // vertex-array growths (host path counter)
   long long n_split = 0;     // igk_step launches as k_apply + k_refine (batch >= split_b)
   long long n_fused = 0;     // igk_step launches as one k_step
   long long n_notice_fallback = 0;  // fast-path steps that fell back to the copy + sync
+  // sharding (igk_options.nranks > 1)
+  int nranks = 1, rank = 0;
+  bool sharded = false;        // the sharded protocol (nranks > 1, or a transport given for one rank)
+  igk_comm comm{};             // host-callback transport (when no NCCL communicator)
+  void* nccl = nullptr;        // ncclComm_t created from igk_options.nccl_id
+  void* xp_host = nullptr;     // pinned staging of the callback transport
+  size_t xp_host_cap = 0;
+  long long* d_xp = nullptr;   // 8-word device scratch for host-value all-reduces
+  long long cut_total = 0;     // sharded: the global cut (sum of the ranks' partial cuts)
+  void* sort_tmp = nullptr;    // sharded: CUB radix-sort scratch (canonical pending list)
+  size_t sort_tmp_cap = 0;
   cudaStream_t stream = nullptr;
   bool poisoned = false;
   std::string err;
@@ -279,10 +296,6 @@ struct igk_graph {
   int check = 0;
   int debug_phases = 0;
   int prof = 0;  // profile mode (igk_debug_set_profile): phase stamps + per-phase work counters
-  int4* d_rec_out = nullptr;  // sharded rounds: this rank's move records
-  int4* d_rec_in = nullptr;   //                 all ranks' records
-  int4* h_rec = nullptr;      //                 pinned host staging (out, then in)
-  long long rec_cap = 0;
   long long compactions = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
@@ -382,11 +395,91 @@ int coop_grid(const void* fn, size_t smem, int want_per_sm, int dev) {
   return sms * per;
 }
 
+// ---------------------------------------------------------------------------
+// collectives of sharded handles: NCCL (loaded at run time) or the host
+// callback of igk_options.comm.  Every all-reduce is in place on DEVICE
+// memory, ordered on the handle's stream.
+// ---------------------------------------------------------------------------
+struct NcclApi {
+  decltype(&ncclGetUniqueId) get_unique_id = nullptr;
+  decltype(&ncclCommInitRank) init_rank = nullptr;
+  decltype(&ncclAllReduce) all_reduce = nullptr;
+  decltype(&ncclCommDestroy) destroy = nullptr;
+  decltype(&ncclGetErrorString) error_string = nullptr;
+};
+const NcclApi* nccl_api() {
+  static NcclApi api;
+  static bool ok = false;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);  // the copy torch already loaded, if any
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+    api.get_unique_id = (decltype(api.get_unique_id))dlsym(h, "ncclGetUniqueId");
+    api.init_rank = (decltype(api.init_rank))dlsym(h, "ncclCommInitRank");
+    api.all_reduce = (decltype(api.all_reduce))dlsym(h, "ncclAllReduce");
+    api.destroy = (decltype(api.destroy))dlsym(h, "ncclCommDestroy");
+    api.error_string = (decltype(api.error_string))dlsym(h, "ncclGetErrorString");
+    ok = api.get_unique_id && api.init_rank && api.all_reduce && api.destroy && api.error_string;
+  });
+  return ok ? &api : nullptr;
+}
+
+enum { XP_I64 = 0, XP_U32 = 1 };
+enum { XP_SUM = 0, XP_MIN = 1, XP_MAX = 2 };
+igk_status xp_allreduce(igk_graph* g, void* dptr, long long count, int dtype, int op) {
+  if (!g->sharded || count <= 0) return IGK_OK;
+  const size_t bytes = (size_t)count * (dtype == XP_I64 ? 8 : 4);
+  if (g->nccl) {
+    const NcclApi* api = nccl_api();
+    const ncclRedOp_t rop = op == XP_SUM ? ncclSum : (op == XP_MIN ? ncclMin : ncclMax);
+    ncclResult_t r = api->all_reduce(dptr, dptr, (size_t)count, dtype == XP_I64 ? ncclInt64 : ncclUint32, rop,
+                                     (ncclComm_t)g->nccl, g->stream);
+    if (r != ncclSuccess) {
+      g->poisoned = true;
+      return fail(g, IGK_ENCCL, std::string("ncclAllReduce: ") + api->error_string(r));
+    }
+    return IGK_OK;
+  }
+  if (bytes > g->xp_host_cap) {
+    if (g->xp_host) cudaFreeHost(g->xp_host);
+    g->xp_host = nullptr;
+    g->xp_host_cap = 0;
+    size_t cap = 1 << 16;
+    while (cap < bytes) cap <<= 1;
+    CK(cudaMallocHost(&g->xp_host, cap));
+    g->xp_host_cap = cap;
+  }
+  CK(cudaMemcpyAsync(g->xp_host, dptr, bytes, cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  if (g->comm.allreduce(g->comm.ctx, g->xp_host, count, dtype, op) != 0) {
+    g->poisoned = true;
+    return fail(g, IGK_ENCCL, "all-reduce callback failed");
+  }
+  CK(cudaMemcpyAsync(dptr, g->xp_host, bytes, cudaMemcpyHostToDevice, g->stream));
+  return IGK_OK;
+}
+// all-reduce (sum) of host values through the device scratch
+igk_status xp_sum_host(igk_graph* g, long long* vals, int n) {
+  if (!g->sharded) return IGK_OK;
+  CK(cudaMemcpyAsync(g->d_xp, vals, n * 8, cudaMemcpyHostToDevice, g->stream));
+  igk_status st = xp_allreduce(g, g->d_xp, n, XP_I64, XP_SUM);
+  if (st != IGK_OK) return st;
+  CK(cudaMemcpyAsync(vals, g->d_xp, n * 8, cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  return IGK_OK;
+}
+
 igk_status launch_recount(igk_graph* g) {
   CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 259, g->stream));
   long long n = g->h_ctl->n_total;
   CK(cudaEventRecord(g->ev[4], g->stream));
-  k_recount<<<g->recount_blocks, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
+  if (g->recount_tma && !g->d.adjw)
+    k_recount_tma<<<g->recount_tma_blocks, kRcT, sizeof(RcSmem), g->stream>>>(g->d, n, g->d_red, g->d_red + 1,
+                                                                             g->d_red + 257);
+  else
+    k_recount<<<g->recount_blocks, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
   g->launches++;
   CK(cudaGetLastError());
   CK(cudaEventRecord(g->ev[5], g->stream));
@@ -447,6 +540,9 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
   for (auto& a : arrs)
     if (!regrow(g, a.p, a.elem, o, n, a.fill)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
   if (d.vw && !regrow(g, (void**)&d.vw, 4, o, n, 0)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
+  if (d.bm && (!regrow(g, (void**)&d.bm, 8, o / 64 + 2, n / 64 + 2, 0) || !regrow(g, (void**)&d.lossbuf, 4, o, n, 0) ||
+               !regrow(g, (void**)&d.recs, 16, o, n, 0)))
+    return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
   const size_t vdo = o + (size_t)(d.slot_cap / kVdC) + 1024, vdn = n + (size_t)(d.slot_cap / kVdC) + 1024;
   if (!regrow(g, (void**)&d.vdch, 8, 0, vdn, 0)) return fail(g, IGK_ENOMEM, "vertex capacity growth failed");
   (void)vdo;
@@ -538,6 +634,37 @@ igk_status compact_slab(igk_graph* g, long long extra) {
   return IGK_OK;
 }
 
+// CSR checks (no self loops, no duplicates, IDs in range, weights in
+// range, symmetric with equal weights) and the twin of every entry: the
+// position of u in row x for the entry u -> x
+bool csr_twins(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t* adjwgt,
+               std::vector<int32_t>& twin_pos) {
+  const long long m2 = n > 0 ? xadj[n] : 0;
+  std::vector<std::pair<int32_t, int32_t>> rows((size_t)m2);
+  for (int64_t u = 0; u < n; u++) {
+    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+      int32_t x = adjncy[j], w = adjwgt ? adjwgt[j] : 1;
+      if (x < 0 || x >= n || x == u || w < 1 || w > kEwMax) return false;
+      rows[j] = {x, (int32_t)(j - xadj[u])};
+    }
+    std::sort(rows.begin() + xadj[u], rows.begin() + xadj[u + 1]);
+    for (int64_t j = xadj[u] + 1; j < xadj[u + 1]; j++)
+      if (rows[j].first == rows[j - 1].first) return false;
+  }
+  twin_pos.assign((size_t)std::max<long long>(m2, 1), 0);
+  for (int64_t u = 0; u < n; u++) {
+    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
+      int32_t x = adjncy[j];
+      auto b = rows.begin() + xadj[x], e = rows.begin() + xadj[x + 1];
+      auto it = std::lower_bound(b, e, std::make_pair((int32_t)u, INT32_MIN));
+      if (it == e || it->first != u) return false;
+      if (adjwgt && adjwgt[xadj[x] + it->second] != adjwgt[j]) return false;
+      twin_pos[j] = it->second;
+    }
+  }
+  return true;
+}
+
 }  // namespace
 
 extern "C" {
@@ -551,40 +678,47 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   if (n > 0 && (!xadj || !init_part || (xadj[n] > 0 && !adjncy))) return IGK_EINVAL;
   igk_options o{};
   if (opt) o = *opt;
+  const int nranks = o.nranks > 1 ? o.nranks : 1;
+  const bool sharded = nranks > 1 || o.nccl_id || o.comm;  // one rank + a transport: the protocol on one GPU
+  if (sharded && (o.rank < 0 || o.rank >= nranks || (!o.nccl_id && (!o.comm || !o.comm->allreduce))))
+    return IGK_EINVAL;
   // ---- host-side validation of the CSR (create-time plumbing) ----
-  const long long m2 = n > 0 ? xadj[n] : 0;
   if (n > 0 && xadj[0] != 0) return IGK_EINVAL;
   for (int64_t u = 0; u < n; u++) {
     if (xadj[u + 1] < xadj[u] || xadj[u + 1] - xadj[u] > kDegMax) return IGK_EINVAL;
     if (init_part[u] < 0 || init_part[u] >= k) return IGK_EINVAL;
     if (vwgt && (vwgt[u] < 1 || vwgt[u] > kVwMax)) return IGK_EINVAL;
   }
-  // rows sorted by neighbour (neighbour, position in row): duplicate check,
-  // symmetry check with equal weights, and the twin of every entry
-  std::vector<std::pair<int32_t, int32_t>> rows((size_t)m2);
-  for (int64_t u = 0; u < n; u++) {
-    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
-      int32_t x = adjncy[j], w = adjwgt ? adjwgt[j] : 1;
-      if (x < 0 || x >= n || x == u || w < 1 || w > kEwMax) return IGK_EINVAL;
-      rows[j] = {x, (int32_t)(j - xadj[u])};
+  std::vector<int32_t> twin_pos;
+  if (!csr_twins(n, xadj, adjncy, adjwgt, twin_pos)) return IGK_EINVAL;
+  // sharded: keep the entries u -> x with owner(u) == rank or owner(x) ==
+  // rank (own vertices in full + the ghost prefixes pointing at them); the
+  // condition is symmetric, so the kept CSR is again symmetric
+  std::vector<int64_t> fx;
+  std::vector<int32_t> fa, fw;
+  const long long sh_blk = nranks > 1 ? std::max<long long>(1, (n + nranks - 1) / nranks) : 1;
+  if (nranks > 1) {
+    auto owns = [&](long long v) { return v / sh_blk == o.rank; };
+    fx.assign((size_t)n + 1, 0);
+    for (int64_t u = 0; u < n; u++) {
+      for (int64_t j = xadj[u]; j < xadj[u + 1]; j++)
+        if (owns(u) || owns(adjncy[j])) {
+          fa.push_back(adjncy[j]);
+          if (adjwgt) fw.push_back(adjwgt[j]);
+        }
+      fx[u + 1] = (int64_t)fa.size();
     }
-    std::sort(rows.begin() + xadj[u], rows.begin() + xadj[u + 1]);
-    for (int64_t j = xadj[u] + 1; j < xadj[u + 1]; j++)
-      if (rows[j].first == rows[j - 1].first) return IGK_EINVAL;
+    xadj = fx.data();
+    adjncy = fa.data();
+    if (adjwgt) adjwgt = fw.data();
+    if (!csr_twins(n, xadj, adjncy, adjwgt, twin_pos)) return IGK_EINVAL;
   }
-  std::vector<int32_t> twin_pos((size_t)std::max<long long>(m2, 1));  // position of u in row x
-  for (int64_t u = 0; u < n; u++) {
-    for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
-      int32_t x = adjncy[j];
-      auto b = rows.begin() + xadj[x], e = rows.begin() + xadj[x + 1];
-      auto it = std::lower_bound(b, e, std::make_pair((int32_t)u, INT32_MIN));
-      if (it == e || it->first != u) return IGK_EINVAL;
-      if (adjwgt && adjwgt[xadj[x] + it->second] != adjwgt[j]) return IGK_EINVAL;
-      twin_pos[j] = it->second;
-    }
-  }
-  std::vector<std::pair<int32_t, int32_t>>().swap(rows);
+  const long long m2 = n > 0 ? xadj[n] : 0;
   igk_graph* g = new igk_graph();
+  g->nranks = nranks;
+  g->rank = nranks > 1 ? o.rank : 0;
+  g->sharded = sharded;
+  if (sharded && !o.nccl_id) g->comm = *o.comm;
   g->device = o.device;
   g->stream = (cudaStream_t)o.stream;
   g->e_ppm = llround(epsilon * 1e6);
@@ -606,6 +740,12 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_recount, 256, 0);
     g->recount_blocks = sms * std::max(1, std::min(occ, 5));
+    cudaFuncSetAttribute(k_recount_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(RcSmem));
+    occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_recount_tma, kRcT, sizeof(RcSmem));
+    g->recount_tma_blocks = sms * std::max(1, occ);
+    const char* rc = getenv("IGK_RECOUNT");
+    g->recount_tma = !(rc && std::strcmp(rc, "gather") == 0);
   }
   Dev& d = g->d;
   d.k = k;
@@ -618,6 +758,11 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   int ib = 1;
   while ((1ll << ib) < d.n_cap) ib++;
   d.idbits = ib;
+  d.nranks = nranks;
+  d.rank = g->rank;
+  d.sharded = sharded;
+  d.sh_n0 = n;
+  d.sh_blk = sh_blk;
   // slack capacities and offsets (prefix sum on the host at create time)
   std::vector<int64_t> off((size_t)std::max<int64_t>(n, 1));
   std::vector<int32_t> deg((size_t)std::max<int64_t>(n, 1)), capv((size_t)std::max<int64_t>(n, 1));
@@ -653,10 +798,26 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) && dalloc(g, &d.metav, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) && dalloc(g, &d.delta, N) &&
-            dalloc(g, &g->d_red, 259);
+            dalloc(g, &g->d_red, 259) && dalloc(g, &g->d_xp, 8);
+  if (ok && sharded)  // sharded exchange buffers (bitmap words, restoration keys, round records)
+    ok = dalloc(g, &d.bm, N / 64 + 2) && dalloc(g, &d.lossbuf, N) && dalloc(g, &d.recs, N);
   if (!ok) {
     igk_destroy(g);
     return IGK_ENOMEM;
+  }
+  if (sharded) {
+    cudaMemsetAsync(d.bm, 0, (N / 64 + 2) * 8, g->stream);
+    if (o.nccl_id) {  // the library's own communicator over NVLink / NVSwitch
+      const NcclApi* api = nccl_api();
+      ncclUniqueId id;
+      std::memcpy(&id, o.nccl_id, sizeof id);
+      ncclComm_t comm = nullptr;
+      if (!api || api->init_rank(&comm, nranks, id, g->rank) != ncclSuccess) {
+        igk_destroy(g);
+        return IGK_ENCCL;
+      }
+      g->nccl = comm;
+    }
   }
   if (cudaMallocHost(&g->h_ctl, sizeof(Ctl)) != cudaSuccess ||
       cudaHostAlloc(&g->h_map, sizeof(Ctl), cudaHostAllocMapped) != cudaSuccess ||
@@ -754,7 +915,12 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     igk_destroy(g);
     return IGK_ECUDA;
   }
-  g->h_ctl->cut = red[0];
+  g->h_ctl->cut = red[0];  // sharded: this rank's partial (edges whose smaller endpoint it owns)
+  g->cut_total = red[0];
+  if (sharded && xp_sum_host(g, &g->cut_total, 1) != IGK_OK) {
+    igk_destroy(g);
+    return IGK_ENCCL;
+  }
   for (int p = 0; p < k; p++) g->h_ctl->Wp[p] = red[1 + p];
   if (cudaMemcpyAsync(d.ctl, g->h_ctl, sizeof(Ctl), cudaMemcpyHostToDevice, s) != cudaSuccess ||
       cudaStreamSynchronize(s) != cudaSuccess) {
@@ -860,6 +1026,7 @@ static ApplyArgs make_apply_args(igk_graph* g, const int4* dm, int64_t count) {
   a.epA = g->epochA;
   a.vw_unit = g->vw_unit;
   a.ew_unit = g->ew_unit;
+  a.phases = 3;
   return a;
 }
 
@@ -899,6 +1066,75 @@ static igk_status launch_refine(igk_graph* g, int after_apply, int global = 0) {
 
 static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats);
 
+// sharded refine (collective; refine.cuh RefineMode): F0 | bitmap | F1+F2 |
+// bitmap | F3 (+ R3 keys | keys | R3) | canonical pending list | per round:
+// gain | records | finish | post.  All-reduces are fixed-size sums of
+// disjoint contributions; the host synchronises after F3 / R3 (restoration
+// decision, pending count) and after every round (pending count).
+static igk_status refine_sharded(igk_graph* g, igk_refine_stats* stats) {
+  RefineArgs ra = make_refine_args(g, 0);
+  ShardArgs sh{};
+  Dev& d = g->d;
+  const long long nw = (g->h_ctl->n_total + 63) / 64;
+  CK(cudaEventRecord(g->ev[0], g->stream));
+  CK(cudaMemsetAsync(d.bm, 0, (size_t)std::max<long long>(nw, 1) * 8, g->stream));
+  igk_status st = IGK_OK;
+  auto launch = [&](int mode) {
+    sh.mode = mode;
+    return launch_refine_sh(g, ra, sh);
+  };
+  if ((st = launch(kShF0)) != IGK_OK) return st;
+  if ((st = xp_allreduce(g, d.bm, nw, XP_I64, XP_SUM)) != IGK_OK) return st;  // C1 (disjoint bits: OR)
+  if ((st = launch(kShF1)) != IGK_OK) return st;
+  if ((st = xp_allreduce(g, d.bm, nw, XP_I64, XP_SUM)) != IGK_OK) return st;  // C2
+  if ((st = launch(kShF3)) != IGK_OK) return st;
+  if ((st = sync_ctl(g, -1)) != IGK_OK) return st;
+  if (g->h_ctl->sh_flag) {  // restoration: the owners' keys, then the replicated select
+    if ((st = xp_allreduce(g, d.lossbuf, g->h_ctl->n_total, XP_U32, XP_SUM)) != IGK_OK) return st;
+    if ((st = launch(kShR3)) != IGK_OK) return st;
+    if ((st = sync_ctl(g, -1)) != IGK_OK) return st;
+  }
+  const long long np = g->h_ctl->sh_np;
+  if (np > 0) {  // the canonical pending list: psi[0] sorted by ID into psi[1]
+    size_t need = 0;
+    cub::DeviceRadixSort::SortKeys(nullptr, need, (const uint32_t*)d.psi[0], (uint32_t*)d.psi[1], (int)np, 0,
+                                   d.idbits, g->stream);
+    if (need > g->sort_tmp_cap) {
+      if (g->sort_tmp) cudaFree(g->sort_tmp);
+      g->sort_tmp = nullptr;
+      g->sort_tmp_cap = 0;
+      CK(cudaMalloc(&g->sort_tmp, need));
+      g->sort_tmp_cap = need;
+    }
+    CK(cub::DeviceRadixSort::SortKeys(g->sort_tmp, need, (const uint32_t*)d.psi[0], (uint32_t*)d.psi[1], (int)np,
+                                      0, d.idbits, g->stream));
+    g->launches++;
+    sh.np = np;
+    for (long long r = 0; r <= np; r++) {  // <= |Psi| rounds (the minimum-ID pending vertex always moves)
+      CK(cudaMemsetAsync(d.recs, 0, (size_t)np * 16, g->stream));
+      if ((st = launch(kShGain)) != IGK_OK) return st;
+      if ((st = xp_allreduce(g, d.recs, 4 * np, XP_U32, XP_SUM)) != IGK_OK) return st;  // records
+      if ((st = launch(kShFinish)) != IGK_OK) return st;
+      if ((st = sync_ctl(g, -1)) != IGK_OK) return st;
+      if (g->h_ctl->rs_pending == 0) break;
+    }
+  }
+  if ((st = launch(kShPost)) != IGK_OK) return st;
+  CK(cudaEventRecord(g->ev[1], g->stream));
+  if ((st = sync_ctl(g, 1)) != IGK_OK) return st;
+  // the per-rank sums: affected / inserted / expanded / scanned (replicated
+  // parts added by rank 0 only) and the partial cut
+  long long* so = g->h_ctl->st_out;
+  long long v[5] = {so[ST_AFFECTED], so[ST_INSERTED], so[ST_EXPANDED], so[ST_SCANNED], so[ST_CUT]};
+  if ((st = xp_sum_host(g, v, 5)) != IGK_OK) return st;
+  so[ST_AFFECTED] = v[0];
+  so[ST_INSERTED] = v[1];
+  so[ST_EXPANDED] = v[2];
+  so[ST_SCANNED] = v[3];
+  so[ST_CUT] = g->cut_total = v[4];
+  return finish_refine(g, stats);
+}
+
 // after a capacity failure (detected in validation: nothing was mutated),
 // grow the vertex arrays and/or compact the slab so the batch can be re-run
 static igk_status make_room(igk_graph* g) {
@@ -915,10 +1151,47 @@ static igk_status make_room(igk_graph* g) {
   return st;
 }
 
+// sharded apply (collective): validation launch, the verdict all-reduced
+// (lowest invalid index: MIN; capacity flags: MAX) on the stream, mutation
+// launch -- every rank rejects or applies the batch alike; a capacity
+// shortfall on any rank makes every rank grow / compact and re-run it
+static igk_status apply_dev_sharded(igk_graph* g, const int4* dm, int64_t count, int64_t* bad_index) {
+  for (int attempt = 0;; attempt++) {
+    igk_status st = prepare_apply(g, count);
+    if (st != IGK_OK) return st;
+    ApplyArgs a = make_apply_args(g, dm, count);
+    void* args[] = {(void*)&g->d, (void*)&a};
+    CK(cudaEventRecord(g->ev[2], g->stream));
+    a.phases = 1;
+    CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply, kThreads, args, 0, g->stream));
+    st = xp_allreduce(g, &g->d.ctl->sh_err[0], 1, XP_I64, XP_MIN);
+    if (st == IGK_OK) st = xp_allreduce(g, &g->d.ctl->sh_err[1], 1, XP_I64, XP_MAX);
+    if (st != IGK_OK) return st;
+    a.phases = 2;
+    CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply, kThreads, args, 0, g->stream));
+    g->launches += 2;
+    CK(cudaEventRecord(g->ev[3], g->stream));
+    st = sync_ctl(g, 0);
+    if (st != IGK_OK) return st;
+    g->h_ctl->err_idx = g->h_ctl->sh_err[0];  // the global verdict
+    g->h_ctl->err_nomem = (int)g->h_ctl->sh_err[1];
+    if (g->h_ctl->err_idx == kNoErr && g->h_ctl->err_nomem && attempt < 2) {
+      st = make_room(g);
+      if (st != IGK_OK) return st;
+      continue;
+    }
+    st = finish_apply(g, bad_index);
+    if (st != IGK_OK) return st;
+    g->cut_total = g->h_ctl->cut;  // the ranks' partial cuts -> the global cut
+    return xp_sum_host(g, &g->cut_total, 1);
+  }
+}
+
 static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t* first_new_id, int64_t* bad_index) {
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   if (count == 0) return IGK_OK;
+  if (g->sharded) return apply_dev_sharded(g, dm, count, bad_index);
   for (int attempt = 0;; attempt++) {
     igk_status st = launch_apply(g, dm, count);
     if (st != IGK_OK) return st;
@@ -973,6 +1246,11 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   igk_status st;
+  if (g->sharded) {  // sharded: the collective apply, then the collective refine
+    st = apply_dev(g, dm, count, first_new_id, bad_index);
+    if (st != IGK_OK) return st;
+    return refine_sharded(g, stats);
+  }
   for (int attempt = 0;; attempt++) {
     bool posted = false;  // this launch posts a host-mapped completion notice
     if (count == 0) {
@@ -1112,12 +1390,12 @@ static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
     stats->adj_entries_scanned = so[ST_SCANNED];
   }
   const bool imbal = so[ST_IMBAL] != 0;
-  if (g->check) {  // invariant I1/I2: maintained cut and W_p equal a recount
+  if (g->check) {  // invariant I1/I2: maintained cut and W_p equal a recount (sharded: collective)
     int64_t cut = 0;
     int64_t wp[256];
     igk_status st = igk_recount(g, &cut, wp);
     if (st != IGK_OK) return st;
-    bool bad = cut != g->h_ctl->cut;
+    bool bad = cut != (g->sharded ? g->cut_total : g->h_ctl->cut);
     for (int p = 0; p < g->d.k; p++) bad |= wp[p] != g->h_ctl->Wp[p];
     if (bad) {
       g->poisoned = true;
@@ -1130,6 +1408,7 @@ static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
 igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
   ENTRY(g, "igk_refine");
+  if (g->sharded) return refine_sharded(g, stats);
   igk_status st = launch_refine(g, 0);
   if (st != IGK_OK) return st;
   st = sync_ctl(g, 1);
@@ -1140,66 +1419,9 @@ igk_status igk_refine(igk_graph* g, igk_refine_stats* stats) {
 igk_status igk_refine_global(igk_graph* g, igk_refine_stats* stats) {
   if (!g || g->poisoned) return IGK_ESTATE;
   ENTRY(g, "igk_refine_global");
+  if (g->sharded) return fail(g, IGK_EINVAL, "igk_refine_global: single-GPU handles only");
   igk_status st = launch_refine(g, 0, 1);  // boundary scan + refine: one launch
   if (st != IGK_OK) return st;
-  st = sync_ctl(g, 1);
-  if (st != IGK_OK) return st;
-  return finish_refine(g, stats);
-}
-
-igk_status igk_refine_sharded(igk_graph* g, const igk_comm* comm, igk_refine_stats* stats) {
-  if (!g || g->poisoned) return IGK_ESTATE;
-  ENTRY(g, "igk_refine_sharded");
-  if (!comm || !comm->allgather || comm->nranks < 1 || comm->rank < 0 || comm->rank >= comm->nranks)
-    return fail(g, IGK_EINVAL, "bad communicator");
-  RefineArgs ra = make_refine_args(g, 0);
-  ShardArgs sh{};
-  sh.nranks = comm->nranks;
-  sh.rank = comm->rank;
-  sh.mode = kModePre;  // F0..R3 replicated on every rank
-  CK(cudaEventRecord(g->ev[0], g->stream));
-  igk_status st = launch_refine_sh(g, ra, sh);
-  if (st == IGK_OK) st = sync_ctl(g, -1);
-  while (st == IGK_OK && g->h_ctl->rs_pending > 0) {
-    const long long np = g->h_ctl->rs_pending;
-    if (np > g->rec_cap) {  // records of one round <= pending vertices
-      cudaFree(g->d_rec_out);
-      cudaFree(g->d_rec_in);
-      if (g->h_rec) cudaFreeHost(g->h_rec);
-      g->d_rec_out = g->d_rec_in = g->h_rec = nullptr;
-      g->rec_cap = 0;
-      long long cap = grow_cap(np);
-      if (cudaMalloc(&g->d_rec_out, cap * 16) != cudaSuccess || cudaMalloc(&g->d_rec_in, cap * 16) != cudaSuccess ||
-          cudaMallocHost(&g->h_rec, cap * 16) != cudaSuccess)
-        return fail(g, IGK_ENOMEM, "record buffers");
-      g->rec_cap = cap;
-    }
-    CK(cudaMemsetAsync(&g->d.ctl->nrec, 0, sizeof(int), g->stream));
-    sh.mode = kModeGain;  // this rank's share of the round gain
-    sh.out = g->d_rec_out;
-    st = launch_refine_sh(g, ra, sh);
-    if (st == IGK_OK) st = sync_ctl(g, -1);
-    if (st != IGK_OK) break;
-    const long long nout = g->h_ctl->nrec;
-    if (nout) CK(cudaMemcpy(g->h_rec, g->d_rec_out, nout * 16, cudaMemcpyDeviceToHost));
-    // the exchange: all-gather of the move records (host buffers, in place)
-    const long long tot = comm->allgather(comm->ctx, g->h_rec, nout, g->h_rec, g->rec_cap);
-    if (tot < 0 || tot > g->rec_cap) {
-      g->poisoned = true;
-      return fail(g, IGK_ENCCL, "all-gather of move records failed");
-    }
-    if (tot) CK(cudaMemcpyAsync(g->d_rec_in, g->h_rec, tot * 16, cudaMemcpyHostToDevice, g->stream));
-    sh.mode = kModeFinish;  // install remote moves, balanced prefix, apply (replicated)
-    sh.recs = g->d_rec_in;
-    sh.nrecs = tot;
-    st = launch_refine_sh(g, ra, sh);
-    if (st == IGK_OK) st = sync_ctl(g, -1);
-  }
-  if (st != IGK_OK) return st;
-  sh.mode = kModePost;
-  st = launch_refine_sh(g, ra, sh);
-  if (st != IGK_OK) return st;
-  CK(cudaEventRecord(g->ev[1], g->stream));
   st = sync_ctl(g, 1);
   if (st != IGK_OK) return st;
   return finish_refine(g, stats);
@@ -1259,6 +1481,10 @@ igk_status igk_cut_size(const igk_graph* gc, int64_t* out) {
   if (!g || g->poisoned) return IGK_ESTATE;
   if (!out) return IGK_EINVAL;
   ENTRY(g, "igk_cut_size");
+  if (g->sharded) {  // the global cut, all-reduced at the end of every collective call
+    *out = g->cut_total;
+    return IGK_OK;
+  }
   CK(cudaMemcpyAsync(&g->h_ctl->cut, &g->d.ctl->cut, 8, cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
   *out = g->h_ctl->cut;
@@ -1306,6 +1532,13 @@ igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp) {
   CK(cudaMemcpyAsync(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
   cudaEventElapsedTime(&g->ms_recount, g->ev[4], g->ev[5]);
+  if (g->sharded) {  // collective: the partial cuts / entry counts of the ranks summed
+    long long v[2] = {red[0], red[257]};
+    st = xp_sum_host(g, v, 2);
+    if (st != IGK_OK) return st;
+    red[0] = v[0];
+    red[257] = v[1];
+  }
   g->last_entries = red[257];
   g->last_active = red[258];
   if (out_cut) *out_cut = red[0];
@@ -1407,6 +1640,16 @@ int32_t igk_debug_phase_work(const igk_graph* gc, int64_t* scanned, int64_t* ite
   return n;
 }
 
+igk_status igk_nccl_unique_id(void* out, int64_t len) {
+  if (!out || len < (int64_t)sizeof(ncclUniqueId)) return IGK_EINVAL;
+  const NcclApi* api = nccl_api();
+  if (!api) return IGK_ENCCL;
+  ncclUniqueId id;
+  if (api->get_unique_id(&id) != ncclSuccess) return IGK_ENCCL;
+  std::memcpy(out, &id, sizeof id);
+  return IGK_OK;
+}
+
 int32_t igk_debug_paths(const igk_graph* gc, int64_t* out, int32_t cap) {
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned || !out) return 0;
@@ -1485,15 +1728,15 @@ void igk_destroy(igk_graph* g) {
   if (!g) return;
   DevGuard dev_guard(g->device);
   cudaStreamSynchronize(g->stream);
+  if (g->nccl && nccl_api()) nccl_api()->destroy((ncclComm_t)g->nccl);
+  if (g->xp_host) cudaFreeHost(g->xp_host);
+  if (g->sort_tmp) cudaFree(g->sort_tmp);
   for (void* p : g->allocs) cudaFree(p);
   if (g->d.hkeys) cudaFree(g->d.hkeys);
   if (g->d.hcnt) cudaFree(g->d.hcnt);
   if (g->d.newid) cudaFree(g->d.newid);
   if (g->d_mods) cudaFree(g->d_mods);
   if (g->h_stage) cudaFreeHost(g->h_stage);
-  if (g->d_rec_out) cudaFree(g->d_rec_out);
-  if (g->d_rec_in) cudaFree(g->d_rec_in);
-  if (g->h_rec) cudaFreeHost(g->h_rec);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
   if (g->h_map) cudaFreeHost(g->h_map);
   if (g->h_flag) cudaFreeHost(g->h_flag);

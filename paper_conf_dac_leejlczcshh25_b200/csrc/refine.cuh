@@ -46,19 +46,32 @@ struct PhaseWork {
     }                                                                          \
   } while (0)
 
-// Sharded refine: every rank holds the replicated store and
-// state; the round gain is split by owner (u mod nranks) and the selected
-// moves are all-gathered as 16-byte records {u, meta | imbal << 30, gain, pw}.
-enum RefineMode { kModeFull = 0, kModePre = 1, kModeGain = 2, kModeFinish = 3, kModePost = 4 };
+// Sharded refine: vertex-range owners (common.cuh own()) hold
+// the full adjacency of their vertices plus ghost prefixes; labels, weights,
+// W_p are replicated.  The refine runs as a sequence of launches with one
+// all-reduce between them (igk.cu refine_sharded):
+//   kShF0     R1 filter of the OWNED affected vertices -> C1 bitmap
+//   [all-reduce C1 bitmap]
+//   kShF1     every rank lists C1 from the bitmap, commits it (W_p, labels:
+//             replicated; cut delta: by the owner), marks the OWNED placed
+//             neighbours of pseudo vertices (N), R2-filters them -> C2 bitmap
+//   [all-reduce C2 bitmap]
+//   kShF3     lists + commits C2; if a part is overweight, the owners write
+//             the (int - ext) key of their vertices of overweight parts
+//   [all-reduce keys]  kShR3  the replicated weighted select + eviction commit
+//   [the pending list is sorted by ID: one canonical order on every rank]
+//   per round: kShGain  owners of selected pending vertices write their move
+//             record at the vertex's position of the canonical list
+//   [all-reduce records]  kShFinish  every rank installs all records, takes
+//             the same balanced prefix and applies it
+//   kShPost   epilogue (stats, delta list)
+// Every all-reduce is a SUM of disjoint contributions (each vertex has one
+// owner), i.e. a fixed-size OR / gather -- no size exchange is needed.
+enum RefineMode { kModeFull = 0, kShF0, kShF1, kShF3, kShR3, kShGain, kShFinish, kShPost };
 struct ShardArgs {
-  int mode;            // RefineMode
-  int nranks, rank;    // owner(u) = u mod nranks
-  const int4* recs;    // kModeFinish: all ranks' move records of this round
-  long long nrecs;
-  int4* out;           // kModeGain: this rank's move records (count in ctl->nrec)
+  int mode;       // RefineMode
+  long long np;   // kShGain / kShFinish: length of the canonical pending list (d.psi[1])
 };
-__device__ __forceinline__ bool owned(const ShardArgs& sh, int u) { return sh.nranks <= 1 || u % sh.nranks == sh.rank; }
-#define IGK_OWNED(sh, u) (!kSh || owned(sh, u))
 
 // ---------------------------------------------------------------------------
 // neighbour iteration with several loads in flight
@@ -99,7 +112,8 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
   for (int t = 0; t < C; t++) {
     unsigned mk = x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN;
     dgx[t] = x[t] >= 0 ? ldro(&d.vr[x[t]].deg) : 0;
-    want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC;  // C1 members are pseudo on sigma2
+    // C1 members are pseudo on sigma2; sharded: each rank lists its own vertices
+    want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC && own(d, x[t]);
   }
   unsigned old[C];
 #pragma unroll
@@ -510,7 +524,7 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
   for (int h = blockIdx.x; h < nh; h += gridDim.x) {
     const int u = __ldcg(hubs + h);
     const uint8_t pu = ld_part(d.part, u);  // deleted vertices carry kDel (== !active)
-    if (pu == kDel || pu == kPsi) continue;  // uniform over the CTA
+    if (pu == kDel || pu == kPsi || !own(d, u)) continue;  // uniform over the CTA (sharded: owners filter)
     long long in = 0, ex = 0;
     nbrs_block(d, u, [&](const int* x, const int* w, const uint8_t* q) {
 #pragma unroll
@@ -543,7 +557,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     const uint8_t pu = ld_part(d.part, u);
     const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
-    if (!act || hub || pu == kPsi) return;
+    if (!act || hub || pu == kPsi || !own(d, u)) return;  // sharded: the owner filters
     counted++;
     long long in = 0, ex = 0;
     nbrs_thread(d, u, [&](int, int w, uint8_t q) {
@@ -563,7 +577,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     const uint8_t pu = ld_part(d.part, u);
     const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
-    if (!act || hub || pu == kPsi) return;
+    if (!act || hub || pu == kPsi || !own(d, u)) return;  // sharded: the owner filters
     long long in = 0, ex = 0;
     nbrs_warp(d, u, [&](int, int w, uint8_t q) {
       if (q == pu) in += w; else ex += w;
@@ -629,7 +643,7 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
       }
       if (expand) mark_chunk<kTC>(d, x, q, a.epN, ep);
     }
-    cut_acc -= del;
+    if (own(d, u)) cut_acc -= del;  // sharded: the owner (full prefix) keeps the cut delta
     finish(u, pu);
   };
   auto wf = [&](int u, long long) {
@@ -667,7 +681,7 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     }
     del = warp_sum(del);
     if (lane_id() == 0) {
-      cut_acc -= del;
+      if (own(d, u)) cut_acc -= del;
       finish(u, pu);
     }
   };
@@ -704,7 +718,7 @@ __device__ void hub_commit(const Dev& d, RefSmem& s, const RefineArgs& a, const 
     if (threadIdx.x == 0) {
       path_hit(ctl, PA_HUB_COMMIT);
       scanned += ldro(&d.vr[u].deg);
-      cut_acc -= del;
+      if (own(d, u)) cut_acc -= del;
       atomic_add_ll(&ctl->Wp[pu], -(long long)vert_w(d.vw, u));
       d.part[u] = kPsi;
       d.psi[0][atomicAdd(&ctl->npsi[0], 1)] = u;
@@ -735,13 +749,14 @@ template <bool kSh>
 __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::grid_group& grid, long long c,
                            int exact_shift_id, RoundState& rs, long long& scanned, long long& cut_acc,
                            const ShardArgs& sh_in, PhaseWork& pw_) {
-  // kSh = false: the single-GPU kernels, all sharding code compiled out
+  // kSh = false: the single-GPU kernels, all sharding code compiled out.
+  // kSh: ONE round per launch, on the canonical pending list d.psi[1] (sorted
+  // by ID, the same on every rank, positions fixed for all rounds): kShGain
+  // writes the owned moves' records d.recs[j]; kShFinish installs every
+  // rank's records (all-reduced) and takes + applies the balanced prefix.
   ShardArgs sh = sh_in;
-  if (!kSh) {
-    sh.mode = kModeFull;
-    sh.nranks = 1;
-  }
-  const bool sharded = kSh && (sh.mode == kModeGain || sh.mode == kModeFinish);
+  if (!kSh) sh.mode = kModeFull;
+  const bool sh_gain = kSh && sh.mode == kShGain, sh_fin = kSh && sh.mode == kShFinish;
   Ctl* ctl = d.ctl;
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -758,10 +773,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     stamp_phase(ctl, id);
   };
   while (true) {
-    const int np = ldv(&ctl->npsi[cur]);
+    const int np = kSh ? (int)sh.np : ldv(&ctl->npsi[cur]);
     if (np == 0) break;
     const int nxt = cur == 1 ? 2 : 1;
-    const int32_t* plist = d.psi[cur];
+    const int32_t* plist = kSh ? d.psi[1] : d.psi[cur];
     int32_t* pnext = d.psi[nxt];
     const int r3 = (int)(rounds_all % 3), r3n = (int)((rounds_all + 1) % 3);
     // round-start snapshot of W_p (Q14) and the lightest part (zero-conn choice)
@@ -774,17 +789,23 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       s.best0 = b;
     }
     __syncthreads();
-    if (tid == 0 && (!kSh || sh.mode != kModeFinish)) {
+    if (tid == 0 && !sh_gain) {
       ctl->npsi[nxt] = 0;
       ctl->applied3[r3n] = 0;
       ctl->selected3[r3n] = 0;
+      if (kSh) ctl->rs_pending = 0;  // counted by the apply below (after barrier 208)
     }
     // -- gain: selection + best part, one adjacency pass per vertex
     long long sel_cnt = 0;
-    if (!kSh || sh.mode != kModeFinish) {  // (the finish kernel of a sharded round skips to the install)
-    rr_for(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
+    if (!sh_fin) {  // (the finish launch of a sharded round starts at the install)
+    if (!kSh) rr_for(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });
     auto emit_move = [&](long long j, int u, int best, long long g, long long pwv, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
+      if (kSh) {  // the record at the vertex's canonical position; installed by every rank in kShFinish
+        d.recs[j] = make_int4(u + 1, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)),
+                              (int)g, (int)pwv);
+        return;
+      }
       d.tgt[u] = (uint8_t)best;
       d.gain[u] = (int)g;
       d.pw[u] = (int)pwv;
@@ -796,10 +817,6 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         ctl->st[ST_IMBAL] = 1;
         path_hit(ctl, PA_WFALLBACK);
       }
-      if (sharded)
-        sh.out[atomicAdd(&ctl->nrec, 1)] =
-            make_int4(u, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)), (int)g,
-                      (int)pwv);
     };
     auto emit_move_v = [&](int u, int best, long long g, long long pwv, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
@@ -814,10 +831,6 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         ctl->st[ST_IMBAL] = 1;
         path_hit(ctl, PA_WFALLBACK);
       }
-      if (sharded)
-        sh.out[atomicAdd(&ctl->nrec, 1)] =
-            make_int4(u, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)), (int)g,
-                      (int)pwv);
     };
     auto get = [&](long long i) {
       int u = __ldcg(plist + i);
@@ -827,14 +840,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       }
       const uint8_t pu = ld_part(d.part, u);
       const bool act = pu != kDel;  // the label doubles as the active flag
+      if (kSh) return (act && pu == kPsi && own(d, u)) ? u : -1;  // hubs: warp path; others' vertices: their owners
       const bool hub = __ldcg(d.markH + u) == a.epF;
       if (!act || pu != kPsi) {
         d.meta[i] = 0;
-        return -1;
-      }
-      if (!IGK_OWNED(sh, u)) {  // another rank's vertex: its record arrives per vertex (metav)
-        d.meta[i] = kMetaHub;
-        if (!hub) d.metav[u] = 0;
         return -1;
       }
       if (hub) {  // CTA-cooperative below; its record is kept per vertex in metav
@@ -871,7 +880,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         if (q[t] < kDel) pwv += w[t];
       }
       if (!sel) {
-        d.meta[j] = 0;
+        if (!kSh) d.meta[j] = 0;
         return;
       }
       auto conn_of = [&](int p) {
@@ -956,7 +965,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       __syncwarp();
       if (lane_id() == 0) {
         if (blocked) {
-          d.meta[j] = 0;
+          if (!kSh) d.meta[j] = 0;
         } else {
           sel_cnt++;
           emit_move(j, u, best, bc, pwv, imbal);
@@ -964,15 +973,11 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       }
     };
     foreach_vertex(d, np, get, tf, wf);
-    {  // hubs in the pseudo-partition: one CTA each
+    if (!kSh) {  // hubs in the pseudo-partition: one CTA each
       int* conn = s.wconn[0];
       for (int h = blockIdx.x; h < nhp; h += gridDim.x) {
         const int u = __ldcg(d.hubP + h);
         if (ld_part(d.part, u) != kPsi) continue;  // uniform: placed earlier (or deleted)
-        if (!IGK_OWNED(sh, u)) {  // another rank's hub: its record arrives in the finish
-          if (threadIdx.x == 0) d.metav[u] = 0;
-          continue;
-        }
         const long long vwu = vert_w(d.vw, u);
         __syncthreads();
         for (int p = threadIdx.x; p < 256; p += blockDim.x) conn[p] = 0;
@@ -1049,29 +1054,37 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         __syncthreads();
       }
     }
-    {
+    if (!kSh) {
       long long sc = warp_sum(sel_cnt);
       if (lane_id() == 0 && sc) atomicAdd(&ctl->selected3[r3], (int)sc);
     }
     }  // gain
-    if (kSh && sh.mode == kModeGain) return;  // the host all-gathers the move records
-    if (kSh && sh.mode == kModeFinish) {
-      // install the other ranks' moves of this round (per vertex, metav)
-      rr_for(sh.nrecs, [&](long long r) {
-        const int4 e = sh.recs[r];
-        const int u = e.x;
-        if (IGK_OWNED(sh, u)) return;
+    if (sh_gain) return;  // the host all-reduces the move records
+    if (sh_fin) {
+      // install every rank's move of this round (records all-reduced: at most
+      // one rank wrote each position) exactly as the single-GPU gain does;
+      // tot3[r3] was zeroed by the previous finish (or the last epilogue)
+      rr_for(np, [&](long long j) {
+        const int4 e = __ldcg(d.recs + j);
+        if (e.x == 0) {
+          d.meta[j] = 0;
+          return;
+        }
+        const int u = e.x - 1;
         const unsigned m = (unsigned)e.y & ~(1u << 30);
         const int best = (int)(m & 255u), d0 = (int)((m >> 8) & 255u);
         d.tgt[u] = (uint8_t)best;
         d.gain[u] = e.z;
         d.pw[u] = e.w;
-        d.metav[u] = m;
+        d.meta[j] = m;
         const long long w = vert_w(d.vw, u);
         atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
         atomic_add_ll(&ctl->tot3[r3][best], w);
         atomicAdd(&ctl->selected3[r3], 1);
-        if ((unsigned)e.y & (1u << 30)) ctl->st[ST_IMBAL] = 1;
+        if ((unsigned)e.y & (1u << 30)) {
+          ctl->st[ST_IMBAL] = 1;
+          path_hit(ctl, PA_WFALLBACK);
+        }
       });
     }
     PHASE_FLUSH(PH_GAIN, np);
@@ -1194,11 +1207,16 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
           keep = false;
           d.part[u] = (uint8_t)p;
           acc_add(s.acc, p, w);
-          cut_acc += (long long)__ldcg(d.pw + u) - __ldcg(d.gain + u);  // independent set: exact
+          if (!kSh || own(d, u))  // sharded: the owner keeps this delta in its partial cut
+            cut_acc += (long long)__ldcg(d.pw + u) - __ldcg(d.gain + u);  // independent set: exact
           app++;
         }
       } else if (ld_part(d.part, u) != kPsi) {
-        keep = false;  // stale entry (deleted before this refine)
+        keep = false;  // stale entry (deleted before this refine / placed in an earlier round)
+      }
+      if (kSh) {  // canonical list: positions stay; count what is left pending
+        agg_append(&ctl->rs_pending, keep);
+        return;
       }
       int slot = agg_append(&ctl->npsi[nxt], keep);
       if (keep) pnext[slot] = u;
@@ -1210,6 +1228,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     }
     rr_for((long long)k * kDigits, [&](long long t) { d.hist0[t] = 0; });
     rr_for(k, [&](long long p) { ctl->tiecnt[p] = 0; });
+    if (kSh) rr_for(k, [&](long long p) { ctl->tot3[r3n][p] = 0; });  // the next finish accumulates there
     if (tid == 0) ctl->ntie = 0;
     sel_clear(d, s.sel);
     PHASE_FLUSH(PH_MOVE, np);
@@ -1218,15 +1237,18 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     if (napp == 0 && nsel > 0) {
       // L = 0: force the first move (reading Q8); it is the threshold item K*
       const int uf = (int)(kr & 0xffffffffu);
-      const int nn = ldv(&ctl->npsi[nxt]);
-      rr_for(nn, [&](long long j) {
-        if (__ldcg(pnext + j) == uf) pnext[j] = -1;
-      });
+      if (!kSh) {
+        const int nn = ldv(&ctl->npsi[nxt]);
+        rr_for(nn, [&](long long j) {
+          if (__ldcg(pnext + j) == uf) pnext[j] = -1;
+        });
+      }
       if (tid == 0) {
         int p = __ldcg(d.tgt + uf);
         d.part[uf] = (uint8_t)p;
         atomic_add_ll(&ctl->Wp[p], vert_w(d.vw, uf));
-        atomic_add_ll(&ctl->cut, (long long)__ldcg(d.pw + uf) - __ldcg(d.gain + uf));
+        if (kSh) ctl->rs_pending -= 1;
+        if (!kSh || own(d, uf)) atomic_add_ll(&ctl->cut, (long long)__ldcg(d.pw + uf) - __ldcg(d.gain + uf));
         ctl->st[ST_IMBAL] = 1;
         path_hit(ctl, PA_FORCED_L0);
       }
@@ -1242,7 +1264,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     __syncthreads();
     cur = nxt;
     rounds_all++;
-    if (kSh && sh.mode == kModeFinish) return;  // one round per sharded finish launch
+    if (sh_fin) return;  // one round per sharded finish launch
   }
 
 }
@@ -1312,20 +1334,50 @@ __device__ __forceinline__ void boundary_mark(const Dev& d, uint32_t epA) {
   }
 }
 
+// Sharded refine helpers.  Every set bit u of the all-reduced candidate
+// bitmap joins the replicated candidate list: stamped `ep`, its label saved,
+// hubs (by their LOCAL prefix length: the commit walks the local prefix)
+// listed apart.  sh_publish sets the bits of this rank's candidates.
+__device__ void sh_extract(const Dev& d, long long nwords, uint32_t ep, int* ncand, int32_t* cand, int* nhub,
+                           int32_t* hubs) {
+  rr_for(nwords, [&](long long w) {
+    unsigned long long b = __ldcg(d.bm + w);
+    while (b) {
+      const int bit = __ffsll((long long)b) - 1;
+      b &= b - 1;
+      const int u = (int)(w * 64 + bit);
+      d.markT[u] = ep;
+      d.oldp[u] = ld_part(d.part, u);
+      if (ldro(&d.vr[u].deg) > kBlockDeg) hubs[atomicAdd(nhub, 1)] = u;
+      else cand[atomicAdd(ncand, 1)] = u;
+    }
+  });
+}
+__device__ void sh_publish(const Dev& d, int n, const int32_t* cand, int nh, const int32_t* hubs) {
+  rr_for(n + nh, [&](long long i) {
+    const int u = i < n ? __ldcg(cand + i) : __ldcg(hubs + (i - n));
+    atomicOr((unsigned long long*)d.bm + (u >> 6), 1ull << (u & 63));
+  });
+}
+__device__ void sh_clear_bm(const Dev& d, long long nwords) {
+  rr_for(nwords, [&](long long w) { d.bm[w] = 0; });
+}
+
 template <bool kSh>
 __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s,
                                             const ShardArgs& sh) {
   Ctl* ctl = d.ctl;
   const int k = d.k;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  const long long nthr = (long long)gridDim.x * blockDim.x;
-  if (a.after_apply && (ldv(&ctl->err_idx) != kNoErr || ldv(&ctl->err_nomem) != 0)) {
+  const int mode = kSh ? sh.mode : (int)kModeFull;
+  if (!kSh && a.after_apply && (ldv(&ctl->err_idx) != kNoErr || ldv(&ctl->err_nomem) != 0)) {
     if (tid == 0) ctl->refine_skipped = 1;  // uniform exit: nothing was modified
     return;
   }
-  if (tid == 0) {
+  if (tid == 0 && (mode == kModeFull || mode == kShF0)) {
     ctl->refine_skipped = 0;
     ctl->n_delta = 0;  // appended only after the last round (many barriers later)
+    if (kSh) ctl->rs_rounds = ctl->rs_rounds_all = ctl->rs_applied = ctl->rs_deferred = 0;
   }
   const long long c = cap_of(ldv(&ctl->W), a.e_ppm, k);
   const int exact_shift_id = ((d.idbits + 7) / 8) * 8 - 8;
@@ -1343,151 +1395,34 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   arrive_stamp(d.dbg, 0);
   long long scanned = 0, counted = 0, cnt_ins = 0, cut_acc = 0;
   PhaseWork pw_;
-  auto flush_partial = [&]() {  // split (sharded) modes: per-kernel accumulators to the control block
+  auto flush_partial = [&]() {  // sharded launches: per-kernel accumulators to the control block
     block_atomic_add(&ctl->cut, cut_acc, s.red);
     block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
   };
-  if (kSh && (sh.mode == kModeGain || sh.mode == kModeFinish)) {  // one sharded round
-    RoundState rs;
-    rs.cur = ldv(&ctl->rs_cur);
-    rs.rounds = ldv(&ctl->rs_rounds);
-    rs.rounds_all = ldv(&ctl->rs_rounds_all);
-    rs.applied_tot = ldv(&ctl->rs_applied);
-    rs.deferred_tot = ldv(&ctl->rs_deferred);
-    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh, pw_);
-    flush_partial();
-    grid.sync();  // every CTA read the round state before it is written back
-    if (tid == 0 && sh.mode == kModeFinish) {
-      ctl->rs_pending = ctl->npsi[rs.cur];
-      ctl->rs_cur = rs.cur;
-      ctl->rs_rounds = rs.rounds;
-      ctl->rs_rounds_all = rs.rounds_all;
-      ctl->rs_applied = rs.applied_tot;
-      ctl->rs_deferred = rs.deferred_tot;
-    }
-    return;
-  }
-  if (!kSh || sh.mode != kModePost) {
-  if (!kSh && a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
-    boundary_mark(d, a.epA);
-    PHASE_FLUSH(PH_BOUNDARY, ldv(&ctl->n_total));
-    GRID_SYNC_STAMPED(ctl, 220);
-  }
-  // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
-  const int nA = ldv(&ctl->nA);
-  const int np0 = ldv(&ctl->npsi[0]);
-  const int nhA = ldv(&ctl->nhubA);
-  rr_for(np0, [&](long long i) {
-    int u = __ldcg(d.psi[0] + i);
-    if (ld_part(d.part, u) == kPsi) cnt_ins++;
-  });
-  filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
-              counted, a.epA);  // hubs of A: CTA-cooperative below
-  hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
-  block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
-  block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
-  PHASE_FLUSH(PH_F0, nA + nhA + np0);
-  GRID_SYNC_STAMPED(ctl, 201);
-
-  // ---- F1: commit C1 + R2 expansion marks -----------------------------------
-  {
-    const int nc = ldv(&ctl->ncand), nhC = ldv(&ctl->nhubC);
-    if (tid == 0) ctl->st[ST_FILTERED_IN] = nc + nhC;
-    commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
-    hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
-    // neighbours of the pseudo vertices pending since apply
-    auto get = [&](long long i) {
-      int u = __ldcg(d.psi[0] + i);
-      return ld_part(d.part, u) == kPsi ? u : -1;  // C1 joins beyond np0
-    };
-    auto mt = [&](int u, long long) {
-      scanned += ldro(&d.vr[u].deg);
-      mark_nbrs_thread(d, u, a.epN, a.epC1);
-    };
-    auto mw = [&](int u, long long) {
-      if (lane_id() == 0) scanned += ldro(&d.vr[u].deg);
-      mark_nbrs_warp(d, u, a.epN, a.epC1);
-    };
-    foreach_vertex(d, np0, get, mt, mw);
-    flush_acc(s, ctl->Wp, k);
-    PHASE_FLUSH(PH_F1, nc + nhC + np0);
-  }
-  GRID_SYNC_STAMPED(ctl, 202);
-
-  // ---- F2: R2 filter on sigma2 ------------------------------------------------
-  {
-    const int nN = ldv(&ctl->nN), nhN = ldv(&ctl->nhubN);
-    long long cntN = 0;
-    filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, &ctl->ncand2, d.cand2, a.epC2, scanned,
-                cntN);
-    hub_filter(d, s, d.hubN, nhN, a.epC2, &ctl->nhubC2, d.hubC2, scanned, cntN);
-    block_atomic_add(&ctl->st[ST_EXPANDED], cntN, s.red);
-    if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
-    PHASE_FLUSH(PH_F2, nN + nhN);
-  }
-  GRID_SYNC_STAMPED(ctl, 203);
-
-  // ---- F3: commit C2 --------------------------------------------------------------
-  {
-    const int nc = ldv(&ctl->ncand2), nhC2 = ldv(&ctl->nhubC2);
-    if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc + nhC2;
-    commit(d, s, a, nc, d.cand2, a.epC2, false, scanned, cut_acc);
-    hub_commit(d, s, a, d.hubC2, nhC2, a.epC2, false, scanned, cut_acc);
-    flush_acc(s, ctl->Wp, k);
-    PHASE_FLUSH(PH_F3, nc + nhC2);
-  }
-  GRID_SYNC_STAMPED(ctl, 204);
-
+  const long long nwords = kSh ? (ldv(&ctl->n_total) + 63) / 64 : 0;
   // ---- R3: balance restoration (reading Q9) ----------------------------------------
-  {
+  // the (int - ext, id) keys of every vertex of an overweight part on sigma3,
+  // then the weighted select of each part's eviction threshold + commit
+  auto r3_setup = [&]() {
     bool any = false;
     for (int p = 0; p < k; p++) any |= ldv(&ctl->Wp[p]) > c;
     if (any) {
-      if (tid == 0) path_hit(ctl, PA_R3);
       for (int p = threadIdx.x; p < k; p += blockDim.x) {
         long long wp = ldv(&ctl->Wp[p]);
         s.sel.used[p] = wp > c;
         s.sel.T[p] = wp - c;
       }
-      __syncthreads();
-      // keys (int - ext, id) of every vertex of an overweight part on sigma3
-      const long long ntot = ldv(&ctl->n_total);
-      auto get = [&](long long v) {
-        uint8_t p = ld_part(d.part, v);
-        return (p != kDel && p != kPsi && s.sel.used[p]) ? (int)v : -1;
-      };
-      auto emit = [&](int v, uint8_t p, long long loss) {
-        int d0 = (int)max(0ll, min(255ll, loss + 128));
-        atomic_add_ll(d.hist0 + (long long)p * kDigits + d0, vert_w(d.vw, v));
-        int slot = atomicAdd(&ctl->nr3, 1);
-        d.r3list[slot] = make_int2(v, (int)loss);
-      };
-      auto tf = [&](int v, long long) {
-        const uint8_t pv = ld_part(d.part, v);
-        long long in = 0, ex = 0;
-        nbrs_thread(d, v, [&](int, int w, uint8_t q) {
-          if (q == pv) in += w; else ex += w;
-          return true;
-        });
-        scanned += ldro(&d.vr[v].deg);
-        emit(v, pv, in - ex);
-      };
-      auto wf = [&](int v, long long) {
-        const uint8_t pv = ld_part(d.part, v);
-        long long in = 0, ex = 0;
-        nbrs_warp(d, v, [&](int, int w, uint8_t q) {
-          if (q == pv) in += w; else ex += w;
-        });
-        in = warp_sum(in);
-        ex = warp_sum(ex);
-        if (lane_id() == 0) {
-          scanned += ldro(&d.vr[v].deg);
-          emit(v, pv, in - ex);
-        }
-      };
-      foreach_vertex(d, ntot, get, tf, wf);
-      PHASE_FLUSH(PH_R3, ntot);
-      GRID_SYNC_STAMPED(ctl, 205);
+    }
+    __syncthreads();
+    return any;
+  };
+  auto r3_emit = [&](int v, uint8_t p, long long loss) {
+    int d0 = (int)max(0ll, min(255ll, loss + 128));
+    atomic_add_ll(d.hist0 + (long long)p * kDigits + d0, vert_w(d.vw, v));
+    int slot = atomicAdd(&ctl->nr3, 1);
+    d.r3list[slot] = make_int2(v, (int)loss);
+  };
+  auto r3_select_evict_commit = [&]() {
       const int nr3 = ldv(&ctl->nr3);
       auto items = [&](long long j, int& p, int& d0, unsigned long long& R, long long& w) {
         int2 e = __ldcg(d.r3list + j);
@@ -1529,23 +1464,212 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       if (tid == 0) ctl->st[ST_EVICTED] = nc;
       for (int p = threadIdx.x; p < 256; p += blockDim.x) s.sel.used[p] = 0;
       GRID_SYNC_STAMPED(ctl, 207);
-    }
-  }
-
-  if (kSh && sh.mode == kModePre) {  // sharded: the host drives the rounds
+  };
+  if (kSh && (mode == kShGain || mode == kShFinish)) {  // one sharded round
+    RoundState rs;
+    rs.cur = 1;
+    rs.rounds = ldv(&ctl->rs_rounds);
+    rs.rounds_all = ldv(&ctl->rs_rounds_all);
+    rs.applied_tot = ldv(&ctl->rs_applied);
+    rs.deferred_tot = ldv(&ctl->rs_deferred);
+    run_rounds<kSh>(d, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh, pw_);
     flush_partial();
-    if (tid == 0) {
-      ctl->rs_cur = 0;
-      ctl->rs_rounds = ctl->rs_rounds_all = ctl->rs_applied = ctl->rs_deferred = 0;
-      ctl->rs_pending = ctl->npsi[0];
+    grid.sync();  // every CTA read the round state before it is written back
+    if (tid == 0 && mode == kShFinish) {
+      ctl->rs_rounds = rs.rounds;
+      ctl->rs_rounds_all = rs.rounds_all;
+      ctl->rs_applied = rs.applied_tot;
+      ctl->rs_deferred = rs.deferred_tot;
     }
     return;
   }
-  }  // pre-round phases
+  if (mode == kModeFull || mode == kShF0) {
+  if (!kSh && a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
+    boundary_mark(d, a.epA);
+    PHASE_FLUSH(PH_BOUNDARY, ldv(&ctl->n_total));
+    GRID_SYNC_STAMPED(ctl, 220);
+  }
+  // ---- F0: pending set joins F; R1 filter over A on sigma1 -----------------
+  const int nA = ldv(&ctl->nA);
+  const int np0 = ldv(&ctl->npsi[0]);
+  const int nhA = ldv(&ctl->nhubA);
+  rr_for(np0, [&](long long i) {
+    int u = __ldcg(d.psi[0] + i);
+    if (ld_part(d.part, u) == kPsi) cnt_ins++;
+  });
+  filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
+              counted, a.epA);  // hubs of A: CTA-cooperative below
+  hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
+  if (kSh && d.rank != 0) cnt_ins = 0;  // replicated count: summed over the ranks, so rank 0 adds it
+  block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
+  block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
+  PHASE_FLUSH(PH_F0, nA + nhA + np0);
+  if (kSh) {  // this rank's C1 -> the bitmap (all-reduced by the host)
+    grid.sync();
+    sh_publish(d, ldv(&ctl->ncand), d.cand, ldv(&ctl->nhubC), d.hubC);
+    flush_partial();
+    return;
+  }
+  GRID_SYNC_STAMPED(ctl, 201);
+  }
+
+  // ---- F1: commit C1 + R2 expansion marks -----------------------------------
+  if (mode == kModeFull || mode == kShF1) {
+  if (kSh) {  // C1 = every rank's candidates (all-reduced bitmap)
+    if (tid == 0) {
+      ctl->ncand = 0;
+      ctl->nhubC = 0;
+    }
+    grid.sync();
+    sh_extract(d, nwords, a.epC1, &ctl->ncand, d.cand, &ctl->nhubC, d.hubC);
+    grid.sync();
+    sh_clear_bm(d, nwords);
+  }
+  {
+    const int np0 = ldv(&ctl->npsi[0]);  // pending since apply (C1 joins beyond)
+    const int nc = ldv(&ctl->ncand), nhC = ldv(&ctl->nhubC);
+    if (tid == 0) ctl->st[ST_FILTERED_IN] = nc + nhC;
+    commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
+    hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
+    // neighbours of the pseudo vertices pending since apply
+    auto get = [&](long long i) {
+      int u = __ldcg(d.psi[0] + i);
+      return ld_part(d.part, u) == kPsi ? u : -1;  // C1 joins beyond np0
+    };
+    auto mt = [&](int u, long long) {
+      scanned += ldro(&d.vr[u].deg);
+      mark_nbrs_thread(d, u, a.epN, a.epC1);
+    };
+    auto mw = [&](int u, long long) {
+      if (lane_id() == 0) scanned += ldro(&d.vr[u].deg);
+      mark_nbrs_warp(d, u, a.epN, a.epC1);
+    };
+    foreach_vertex(d, np0, get, mt, mw);
+    flush_acc(s, ctl->Wp, k);
+    PHASE_FLUSH(PH_F1, nc + nhC + np0);
+  }
+  GRID_SYNC_STAMPED(ctl, 202);
+
+  // ---- F2: R2 filter on sigma2 ------------------------------------------------
+  {
+    const int nN = ldv(&ctl->nN), nhN = ldv(&ctl->nhubN);
+    long long cntN = 0;
+    filter_pass(d, nN, [&](long long i) { return __ldcg(d.Nlist + i); }, &ctl->ncand2, d.cand2, a.epC2, scanned,
+                cntN);
+    hub_filter(d, s, d.hubN, nhN, a.epC2, &ctl->nhubC2, d.hubC2, scanned, cntN);
+    block_atomic_add(&ctl->st[ST_EXPANDED], cntN, s.red);
+    if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
+    PHASE_FLUSH(PH_F2, nN + nhN);
+  }
+  if (kSh) {  // this rank's C2 -> the bitmap
+    grid.sync();
+    sh_publish(d, ldv(&ctl->ncand2), d.cand2, ldv(&ctl->nhubC2), d.hubC2);
+    flush_partial();
+    return;
+  }
+  GRID_SYNC_STAMPED(ctl, 203);
+  }
+
+  // ---- F3: commit C2 --------------------------------------------------------------
+  if (mode == kModeFull || mode == kShF3) {
+  if (kSh) {  // C2 = every rank's candidates
+    if (tid == 0) {
+      ctl->ncand2 = 0;
+      ctl->nhubC2 = 0;
+    }
+    grid.sync();
+    sh_extract(d, nwords, a.epC2, &ctl->ncand2, d.cand2, &ctl->nhubC2, d.hubC2);
+    grid.sync();
+    sh_clear_bm(d, nwords);
+  }
+  {
+    const int nc = ldv(&ctl->ncand2), nhC2 = ldv(&ctl->nhubC2);
+    if (tid == 0) ctl->st[ST_EXPANDED_IN] = nc + nhC2;
+    commit(d, s, a, nc, d.cand2, a.epC2, false, scanned, cut_acc);
+    hub_commit(d, s, a, d.hubC2, nhC2, a.epC2, false, scanned, cut_acc);
+    flush_acc(s, ctl->Wp, k);
+    PHASE_FLUSH(PH_F3, nc + nhC2);
+  }
+  GRID_SYNC_STAMPED(ctl, 204);
+
+  // ---- R3: balance restoration (reading Q9), helpers above -------------------------
+  if (mode == kModeFull || mode == kShF3) {
+    const bool any = r3_setup();
+    if (kSh && tid == 0) ctl->sh_flag = any;
+    if (any) {
+      if (tid == 0) path_hit(ctl, PA_R3);
+      const long long ntot = ldv(&ctl->n_total);
+      if (kSh) {  // only owners know a key: 0 everywhere else (the host all-reduces the array)
+        rr_for(ntot, [&](long long v) {
+          const uint8_t p = ld_part(d.part, v);
+          if (p == kDel || p == kPsi || !s.sel.used[p] || !own(d, v)) d.lossbuf[v] = 0;
+        });
+      }
+      auto emit = [&](int v, uint8_t p, long long loss) {
+        if (kSh) d.lossbuf[v] = (uint32_t)(loss + 0x80000000ll);  // |loss| < 2^31 (limits: 255 * 2^23)
+        else r3_emit(v, p, loss);
+      };
+
+      // keys (int - ext, id) of every vertex of an overweight part on sigma3
+      auto get = [&](long long v) {
+        uint8_t p = ld_part(d.part, v);
+        return (p != kDel && p != kPsi && s.sel.used[p] && own(d, v)) ? (int)v : -1;
+      };
+      auto tf = [&](int v, long long) {
+        const uint8_t pv = ld_part(d.part, v);
+        long long in = 0, ex = 0;
+        nbrs_thread(d, v, [&](int, int w, uint8_t q) {
+          if (q == pv) in += w; else ex += w;
+          return true;
+        });
+        scanned += ldro(&d.vr[v].deg);
+        emit(v, pv, in - ex);
+      };
+      auto wf = [&](int v, long long) {
+        const uint8_t pv = ld_part(d.part, v);
+        long long in = 0, ex = 0;
+        nbrs_warp(d, v, [&](int, int w, uint8_t q) {
+          if (q == pv) in += w; else ex += w;
+        });
+        in = warp_sum(in);
+        ex = warp_sum(ex);
+        if (lane_id() == 0) {
+          scanned += ldro(&d.vr[v].deg);
+          emit(v, pv, in - ex);
+        }
+      };
+      foreach_vertex(d, ntot, get, tf, wf);
+      PHASE_FLUSH(PH_R3, ntot);
+      if (!kSh) {
+        GRID_SYNC_STAMPED(ctl, 205);
+        r3_select_evict_commit();
+      }
+    }
+    if (kSh) {
+      if (tid == 0) ctl->sh_np = ldv(&ctl->npsi[0]);  // every commit is behind barrier 204
+      flush_partial();
+      return;
+    }
+  }
+  }
+  if (kSh && mode == kShR3) {  // every rank: the all-reduced keys -> the replicated select + commit
+    r3_setup();
+    const long long ntot = ldv(&ctl->n_total);
+    rr_for(ntot, [&](long long v) {
+      const uint32_t e = __ldcg(d.lossbuf + v);
+      if (e) r3_emit((int)v, ld_part(d.part, v), (long long)e - 0x80000000ll);
+    });
+    GRID_SYNC_STAMPED(ctl, 205);
+    r3_select_evict_commit();
+    if (tid == 0) ctl->sh_np = ldv(&ctl->npsi[0]);  // the eviction commit is behind barrier 207
+    flush_partial();
+    return;
+  }
+
   // ---- R4: rounds (Alg. 4), grid-wide (a CTA-local variant for small tails
   //      measured slower: the rounds are load-latency bound, not barrier bound)
   RoundState rs;
-  if (kSh && sh.mode == kModePost) {
+  if (kSh && sh.mode == kShPost) {
     rs.rounds = ldv(&ctl->rs_rounds);
     rs.applied_tot = ldv(&ctl->rs_applied);
     rs.deferred_tot = ldv(&ctl->rs_deferred);
@@ -1609,12 +1733,11 @@ __global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   ShardArgs sh{};
   sh.mode = kModeFull;
-  sh.nranks = 1;
   refine_body<false>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh);
   publish(d);
 }
 
-// sharded refine: one launch per mode (pre | round gain | round finish | post)
+// sharded refine: one launch per mode (RefineMode kSh*), driven by igk.cu refine_sharded
 __global__ void __launch_bounds__(kThreads) k_refine_sh(Dev d, RefineArgs a, ShardArgs sh) {
   cg::grid_group grid = cg::this_grid();
   extern __shared__ __align__(16) unsigned char smem_raw[];

@@ -24,7 +24,6 @@ __global__ void __launch_bounds__(kThreads) k_step(Dev d, ApplyArgs aa, RefineAr
   grid.sync();  // the refine starts from the complete applied state
   ShardArgs sh{};
   sh.mode = kModeFull;
-  sh.nranks = 1;
   refine_body<false>(d, ra, grid, sm.rf, sh);
   publish(d);
 }
