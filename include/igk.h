@@ -174,6 +174,25 @@ igk_status igk_step(igk_graph* g, const igk_modifier* mods, int64_t count, igk_r
 igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t count, igk_refine_stats* stats,
                            int64_t* first_new_id, int64_t* bad_index);
 
+/* Pipelined steps (store maintenance / IO): the next
+ * batch's host->device copy overlaps the running step.
+ *   igk_stage_batch  copies a HOST batch into one of two device buffers on
+ *                    the handle's own copy stream and returns at once (a
+ *                    page-locked buffer is DMA'd directly and must stay
+ *                    unchanged until the igk_step_end of the step that
+ *                    consumes it; pageable memory is copied into a pinned
+ *                    staging buffer first).
+ *   igk_step_begin   launches apply + refine on the most recently staged
+ *                    batch (ordered after its copy) and returns without
+ *                    waiting.
+ *   igk_step_end     waits for that step; results, statuses and the
+ *                    capacity retry exactly as igk_step.
+ * Loop: stage(b0); for t: begin(); stage(b_t+1); end(); -- at most one step
+ * in flight and one batch staged ahead.  Single-GPU handles only. */
+igk_status igk_stage_batch(igk_graph* g, const igk_modifier* mods, int64_t count);
+igk_status igk_step_begin(igk_graph* g);
+igk_status igk_step_end(igk_graph* g, igk_refine_stats* stats, int64_t* first_new_id, int64_t* bad_index);
+
 /* NCCL unique id for sharded handles (call on ONE rank, share the 128
  * bytes with the others, pass as igk_options.nccl_id).  NCCL is loaded at
  * run time (libnccl.so.2); IGK_ENCCL if it is unavailable. */

@@ -25,7 +25,8 @@ STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evic
 
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine", "igk_refine_global",
-           "igk_step", "igk_step_device", "igk_nccl_unique_id",
+           "igk_step", "igk_step_device", "igk_nccl_unique_id", "igk_stage_batch", "igk_step_begin",
+           "igk_step_end",
            "igk_partition", "igk_partition_delta", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
            "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work",
@@ -129,6 +130,12 @@ def lib():
         L.igk_step.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
         L.igk_step_device.restype = C.c_int
         L.igk_step_device.argtypes = [P, P, i64, C.POINTER(Stats), i64p, i64p]
+        L.igk_stage_batch.restype = C.c_int
+        L.igk_stage_batch.argtypes = [P, P, i64]
+        L.igk_step_begin.restype = C.c_int
+        L.igk_step_begin.argtypes = [P]
+        L.igk_step_end.restype = C.c_int
+        L.igk_step_end.argtypes = [P, C.POINTER(Stats), i64p, i64p]
         L.igk_nccl_unique_id.restype = C.c_int
         L.igk_nccl_unique_id.argtypes = [P, i64]
         L.igk_partition.restype = C.c_int
@@ -268,6 +275,29 @@ class IGKGraph:
         if s not in (OK, WIMBALANCED, EINVAL):
             raise IGKError(s, self._err())
         return s, st
+
+    def stage_batch(self, mods):
+        """igk_stage_batch: async H2D of the next batch (keep `mods` alive and
+        unchanged until the step_end of the step that consumes it)."""
+        m = np.ascontiguousarray(mods, dtype=np.int32).reshape(-1, 4)
+        self._staged_keep = getattr(self, "_staged_keep", [])[-1:] + [m]
+        s = lib().igk_stage_batch(self.h, m.ctypes.data, len(m))
+        if s != OK:
+            raise IGKError(s, self._err())
+
+    def step_begin(self):
+        s = lib().igk_step_begin(self.h)
+        if s != OK:
+            raise IGKError(s, self._err())
+
+    def step_end(self):
+        """-> (status, stats, bad_index) exactly as step()"""
+        st = Stats()
+        fid, bad = C.c_int64(0), C.c_int64(-1)
+        s = lib().igk_step_end(self.h, C.byref(st), C.byref(fid), C.byref(bad))
+        if s not in (OK, WIMBALANCED, EINVAL):
+            raise IGKError(s, self._err())
+        return s, {f: int(getattr(st, f)) for f in STATS}, bad.value
 
     def num_vertices(self):
         nt, na = C.c_int64(0), C.c_int64(0)

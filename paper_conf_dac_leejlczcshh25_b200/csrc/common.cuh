@@ -20,7 +20,10 @@ constexpr int kVwMax = 65535;
 constexpr int kEwMax = 255;
 constexpr int kDegMax = 1 << 23;
 constexpr int64_t kNMax = int64_t(1) << 30;
-constexpr int kThreads = 512;       // persistent-kernel block size
+#ifndef IGK_THREADS
+#define IGK_THREADS 512
+#endif
+constexpr int kThreads = IGK_THREADS;  // persistent-kernel block size (A/B builds: -DIGK_THREADS=...)
 constexpr int kWarps = kThreads / 32;
 constexpr int kThreadDeg = 16;      // degree <= this: one thread per vertex; above: one warp
 constexpr int kBlockDeg = 1024;     // degree > this (hubs): one whole CTA per vertex

@@ -259,7 +259,7 @@ struct igk_graph {
   int device = 0;
   int recount_blocks = 0;    // k_recount grid (occupancy-derived at create)
   int recount_tma_blocks = 0;  // k_recount_tma grid (unit edge weights)
-  int recount_tma = 1;       // S9 kernel: TMA-pipelined (1) or direct gathers (0; IGK_RECOUNT=gather)
+  int recount_tma = 0;       // S9 kernel: direct gathers (0) or the TMA-pipelined variant (1; IGK_RECOUNT=tma)
   long long n_grow = 0;      // vertex-array growths (host path counter)
   long long n_split = 0;     // igk_step launches as k_apply + k_refine (batch >= split_b)
   long long n_fused = 0;     // igk_step launches as one k_step
@@ -297,6 +297,17 @@ struct igk_graph {
   int debug_phases = 0;
   int prof = 0;  // profile mode (igk_debug_set_profile): phase stamps + per-phase work counters
   long long compactions = 0;
+  // pipelined steps (igk_stage_batch / igk_step_begin / igk_step_end): two
+  // device batch buffers filled on a copy stream while a step runs
+  cudaStream_t copy_stream = nullptr;
+  int4* sd_mods[2] = {nullptr, nullptr};
+  long long sd_cap[2] = {0, 0}, sd_count[2] = {0, 0};
+  igk_modifier* sh_stage[2] = {nullptr, nullptr};
+  long long sh_cap[2] = {0, 0};
+  cudaEvent_t ev_stage[2] = {};
+  int staged = -1, stage_next = 0, inflight = 0, inflight_buf = 0;
+  bool inflight_posted = false;
+  long long inflight_n0 = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
   long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active
@@ -744,8 +755,10 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     occ = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_recount_tma, kRcT, sizeof(RcSmem));
     g->recount_tma_blocks = sms * std::max(1, occ);
+    // the TMA-pipelined variant is opt-in: measured 2-4x slower than the
+    // direct gathers on C2 / C4 / C5 (profiles/r02_s9_recount_ab.txt)
     const char* rc = getenv("IGK_RECOUNT");
-    g->recount_tma = !(rc && std::strcmp(rc, "gather") == 0);
+    g->recount_tma = rc && std::strcmp(rc, "tma") == 0;
   }
   Dev& d = g->d;
   d.k = k;
@@ -830,6 +843,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   *g->h_flag = 0;
   d.seq = 0;
   for (auto& e : g->ev) cudaEventCreate(&e);
+  for (auto& e : g->ev_stage) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
   // zero-init
   cudaStream_t s = g->stream;
   cudaMemsetAsync(d.active, 0, N, s);
@@ -1241,63 +1255,67 @@ static igk_status notice_wait(igk_graph* g) {
   return IGK_OK;
 }
 
-static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refine_stats* stats,
-                           int64_t* first_new_id, int64_t* bad_index) {
-  if (bad_index) *bad_index = -1;
-  if (first_new_id) *first_new_id = g->h_ctl->n_total;
+// one launch of a step (fused k_step, or k_apply + k_refine for large
+// batches); *posted = the kernel posts a host-mapped completion notice
+static igk_status step_launch(igk_graph* g, const int4* dm, int64_t count, bool* posted) {
   igk_status st;
-  if (g->sharded) {  // sharded: the collective apply, then the collective refine
-    st = apply_dev(g, dm, count, first_new_id, bad_index);
+  *posted = false;
+  if (count == 0) {
+    st = launch_refine(g, 0);
     if (st != IGK_OK) return st;
-    return refine_sharded(g, stats);
+  } else if (count >= g->split_b) {
+    // large batch: k_apply at full occupancy (64 registers: 2x the warps
+    // of the fused kernel for its latency-bound gathers and atomics), then
+    // k_refine on the same stream -- no host round trip between them; a
+    // rejected batch makes the refine exit untouched (after_apply)
+    st = prepare_apply(g, count);
+    if (st != IGK_OK) return st;
+    ApplyArgs aa = make_apply_args(g, dm, count);
+    RefineArgs ra = make_refine_args(g, 1);
+    void* a1[] = {(void*)&g->d, (void*)&aa};
+    void* a2[] = {(void*)&g->d, (void*)&ra};
+    Dev dn = g->d;  // the refine posts the completion notice, not the apply
+    const bool fast = notice_begin(g);
+    void* a1n[] = {(void*)&dn, (void*)&aa};
+    CK(cudaEventRecord(g->ev[0], g->stream));
+    CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply_wide, kThreads, fast ? a1n : a1, 0,
+                                   g->stream));
+    CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, a2, g->smem_refine, g->stream));
+    g->d.seq = 0;
+    g->launches += 2;
+    g->n_split++;
+    CK(cudaEventRecord(g->ev[1], g->stream));
+    *posted = fast;
+  } else {  // apply + refine in ONE persistent launch (k_step)
+    st = prepare_apply(g, count);
+    if (st != IGK_OK) return st;
+    ApplyArgs aa = make_apply_args(g, dm, count);
+    RefineArgs ra = make_refine_args(g, 1);
+    const bool fast = notice_begin(g);
+    void* args[] = {(void*)&g->d, (void*)&aa, (void*)&ra};
+    CK(cudaEventRecord(g->ev[0], g->stream));
+    CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
+    g->d.seq = 0;
+    g->launches++;
+    g->n_fused++;
+    CK(cudaEventRecord(g->ev[1], g->stream));
+    *posted = fast;
   }
+  return IGK_OK;
+}
+
+// wait for a launched step; a batch rejected only for capacity (nothing was
+// mutated) is re-run after growing / compacting the store
+static igk_status step_complete(igk_graph* g, const int4* dm, int64_t count, bool posted, igk_refine_stats* stats,
+                                int64_t* bad_index) {
+  igk_status st;
   for (int attempt = 0;; attempt++) {
-    bool posted = false;  // this launch posts a host-mapped completion notice
-    if (count == 0) {
-      st = launch_refine(g, 0);
-      if (st != IGK_OK) return st;
-    } else if (count >= g->split_b) {
-      // large batch: k_apply at full occupancy (64 registers: 2x the warps
-      // of the fused kernel for its latency-bound gathers and atomics), then
-      // k_refine on the same stream -- no host round trip between them; a
-      // rejected batch makes the refine exit untouched (after_apply)
-      st = prepare_apply(g, count);
-      if (st != IGK_OK) return st;
-      ApplyArgs aa = make_apply_args(g, dm, count);
-      RefineArgs ra = make_refine_args(g, 1);
-      void* a1[] = {(void*)&g->d, (void*)&aa};
-      void* a2[] = {(void*)&g->d, (void*)&ra};
-      Dev dn = g->d;  // the refine posts the completion notice, not the apply
-      const bool fast = notice_begin(g);
-      void* a1n[] = {(void*)&dn, (void*)&aa};
-      CK(cudaEventRecord(g->ev[0], g->stream));
-      CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply_wide, kThreads, fast ? a1n : a1, 0,
-                                     g->stream));
-      CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, a2, g->smem_refine, g->stream));
-      g->d.seq = 0;
-      g->launches += 2;
-      g->n_split++;
-      CK(cudaEventRecord(g->ev[1], g->stream));
-      posted = fast;
-    } else {  // apply + refine in ONE persistent launch (k_step)
-      st = prepare_apply(g, count);
-      if (st != IGK_OK) return st;
-      ApplyArgs aa = make_apply_args(g, dm, count);
-      RefineArgs ra = make_refine_args(g, 1);
-      const bool fast = notice_begin(g);
-      void* args[] = {(void*)&g->d, (void*)&aa, (void*)&ra};
-      CK(cudaEventRecord(g->ev[0], g->stream));
-      CK(cudaLaunchCooperativeKernel((const void*)k_step, g->grid_refine, kThreads, args, g->smem_step, g->stream));
-      g->d.seq = 0;
-      g->launches++;
-      g->n_fused++;
-      CK(cudaEventRecord(g->ev[1], g->stream));
-      posted = fast;
-    }
     st = posted ? notice_wait(g) : sync_ctl(g, 1);
     if (st != IGK_OK) return st;
     if (count > 0 && g->h_ctl->err_idx == kNoErr && g->h_ctl->err_nomem && attempt < 2) {
       st = make_room(g);  // the kernel stopped before any mutation: grow / compact, then re-run
+      if (st != IGK_OK) return st;
+      st = step_launch(g, dm, count, &posted);
       if (st != IGK_OK) return st;
       continue;
     }
@@ -1314,6 +1332,22 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
     if (g->h_ctl->err_nomem) return fail(g, IGK_ENOMEM, "vertex or slot capacity exhausted");
   }
   return finish_refine(g, stats);
+}
+
+static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refine_stats* stats,
+                           int64_t* first_new_id, int64_t* bad_index) {
+  if (bad_index) *bad_index = -1;
+  if (first_new_id) *first_new_id = g->h_ctl->n_total;
+  igk_status st;
+  if (g->sharded) {  // sharded: the collective apply, then the collective refine
+    st = apply_dev(g, dm, count, first_new_id, bad_index);
+    if (st != IGK_OK) return st;
+    return refine_sharded(g, stats);
+  }
+  bool posted = false;
+  st = step_launch(g, dm, count, &posted);
+  if (st != IGK_OK) return st;
+  return step_complete(g, dm, count, posted, stats, bad_index);
 }
 
 // host batch -> g->d_mods on the handle stream.  A page-locked caller buffer
@@ -1445,6 +1479,79 @@ igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t cou
   ENTRY(g, "igk_step_device");
   if (count < 0 || (count > 0 && !d_mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
   return step_dev(g, (const int4*)d_mods, count, stats, first_new_id, bad_index);
+}
+
+igk_status igk_stage_batch(igk_graph* g, const igk_modifier* mods, int64_t count) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_stage_batch");
+  if (count < 0 || (count > 0 && !mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
+  if (g->sharded) return fail(g, IGK_EINVAL, "igk_stage_batch: single-GPU handles only");
+  if (!g->copy_stream) CK(cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking));
+  const int b = g->stage_next;
+  if (g->inflight && b == g->inflight_buf) CK(cudaStreamSynchronize(g->stream));  // never under a running step
+  if (count > g->sd_cap[b]) {
+    CK(cudaStreamSynchronize(g->copy_stream));  // an earlier copy into this buffer has landed
+    if (g->sd_mods[b]) cudaFree(g->sd_mods[b]);
+    g->sd_mods[b] = nullptr;
+    g->sd_cap[b] = 0;
+    long long cap = grow_cap(count);
+    if (cudaMalloc(&g->sd_mods[b], cap * 16) != cudaSuccess) return fail(g, IGK_ENOMEM, "batch allocation failed");
+    g->sd_cap[b] = cap;
+  }
+  if (count > 0) {
+    cudaPointerAttributes at{};
+    const bool pinned = cudaPointerGetAttributes(&at, mods) == cudaSuccess && at.type == cudaMemoryTypeHost;
+    cudaGetLastError();
+    const void* src = mods;
+    if (!pinned) {  // pageable: through the buffer's own pinned staging (the copy stays asynchronous)
+      if (count > g->sh_cap[b]) {
+        CK(cudaStreamSynchronize(g->copy_stream));
+        if (g->sh_stage[b]) cudaFreeHost(g->sh_stage[b]);
+        g->sh_stage[b] = nullptr;
+        g->sh_cap[b] = 0;
+        long long cap = grow_cap(count);
+        CK(cudaMallocHost(&g->sh_stage[b], cap * 16));
+        g->sh_cap[b] = cap;
+      }
+      CK(cudaEventSynchronize(g->ev_stage[b]));  // the previous copy out of this staging buffer is done
+      std::memcpy(g->sh_stage[b], mods, count * 16);
+      src = g->sh_stage[b];
+    }
+    CK(cudaMemcpyAsync(g->sd_mods[b], src, count * 16, cudaMemcpyHostToDevice, g->copy_stream));
+  }
+  CK(cudaEventRecord(g->ev_stage[b], g->copy_stream));
+  g->sd_count[b] = count;
+  g->staged = b;
+  g->stage_next = b ^ 1;
+  return IGK_OK;
+}
+
+igk_status igk_step_begin(igk_graph* g) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_step_begin");
+  if (g->staged < 0 || g->inflight) return fail(g, IGK_EINVAL, "igk_step_begin: no staged batch / step in flight");
+  const int b = g->staged;
+  CK(cudaStreamWaitEvent(g->stream, g->ev_stage[b], 0));  // the step starts when its batch has landed
+  g->inflight_buf = b;
+  g->inflight_n0 = g->h_ctl->n_total;
+  g->staged = -1;
+  bool posted = false;
+  igk_status st = step_launch(g, g->sd_mods[b], g->sd_count[b], &posted);
+  if (st != IGK_OK) return st;
+  g->inflight = 1;
+  g->inflight_posted = posted;
+  return IGK_OK;
+}
+
+igk_status igk_step_end(igk_graph* g, igk_refine_stats* stats, int64_t* first_new_id, int64_t* bad_index) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_step_end");
+  if (!g->inflight) return fail(g, IGK_EINVAL, "igk_step_end: no step in flight");
+  g->inflight = 0;
+  if (bad_index) *bad_index = -1;
+  if (first_new_id) *first_new_id = g->inflight_n0;
+  const int b = g->inflight_buf;
+  return step_complete(g, g->sd_mods[b], g->sd_count[b], g->inflight_posted, stats, bad_index);
 }
 
 igk_status igk_partition(const igk_graph* gc, int32_t* out, int64_t cap_len, int64_t* n_total) {
@@ -1742,6 +1849,12 @@ void igk_destroy(igk_graph* g) {
   if (g->h_flag) cudaFreeHost(g->h_flag);
   for (auto& e : g->ev)
     if (e) cudaEventDestroy(e);
+  for (int b = 0; b < 2; b++) {
+    if (g->ev_stage[b]) cudaEventDestroy(g->ev_stage[b]);
+    if (g->sd_mods[b]) cudaFree(g->sd_mods[b]);
+    if (g->sh_stage[b]) cudaFreeHost(g->sh_stage[b]);
+  }
+  if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   delete g;
 }
 

@@ -1,6 +1,13 @@
 // recount.cuh -- S9 cut / part-weight reduction as a TMA-pipelined
 // full-store scan (unit edge weights; weighted handles use k_recount).
 //
+// OPT-IN VARIANT (IGK_RECOUNT=tma at igk_create), kept as the measured
+// answer to "stage the tile's records and slab span with bulk async copies":
+// on B200 it is 2-4x SLOWER than the direct-gather k_recount (C4 0.98 vs
+// 0.25 ms; profiles/r02_s9_recount_ab.txt): the CTA-wide tile hand-off
+// (mbarrier waits + __syncthreads) makes every tile wait for its slowest
+// vertex, and the staged span carries the slack slots the gathers skip.
+//
 // The scan is HBM-bound: per tile of kRcT consecutive vertex IDs it needs the
 // tile's vertex records, its label window and the slab span holding the
 // tile's prefixes.  All three are moved by the bulk-copy engine
@@ -151,7 +158,27 @@ __global__ void __launch_bounds__(kRcT) k_recount_tma(Dev d, long long n, long l
       acc_add(S.s_wp, pv, vert_w(d.vw, v));
     }
     if (!placed || !own(d, v)) dg = 0;
-    // the warp's int4 chunks flattened and dealt lane-strided (k_recount's schedule)
+    const bool staged = S.span_ok[ab];
+    if (staged) {
+      // the prefix is in shared memory: each thread walks its own vertex
+      // (no owner search); a staged span holds <= kRcAdj slots, so the
+      // longest walk is bounded
+      const int4* p4 = &S.adj[ab][(o - S.span_lo[ab]) >> 2];
+      for (int c = 0; 4 * c < dg; c++) {
+        const int4 x4 = p4[c];
+        const int xs[4] = {x4.x, x4.y, x4.z, x4.w};
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+          if (4 * c + i < dg && xs[i] > v) {
+            const uint8_t q = label(xs[i]);
+            cut += q != kPsi && q != pv;
+          }
+        }
+      }
+      return;
+    }
+    // not staged (a hub or far-apart relocated prefixes): k_recount's
+    // schedule -- the warp's int4 chunks flattened and dealt lane-strided
     int incl = (dg + 3) >> 2;
 #pragma unroll
     for (int sh = 1; sh < 32; sh <<= 1) {
@@ -160,8 +187,6 @@ __global__ void __launch_bounds__(kRcT) k_recount_tma(Dev d, long long n, long l
     }
     const int total = __shfl_sync(0xffffffffu, incl, 31);
     const int excl = incl - ((dg + 3) >> 2);
-    const bool staged = S.span_ok[ab];
-    const long long lo4 = S.span_lo[ab] >> 2;
     const long long c0 = o >> 2;
     const int4* g4 = reinterpret_cast<const int4*>(d.adj);
     for (int e0 = 0; e0 < total; e0 += 64) {
@@ -183,9 +208,7 @@ __global__ void __launch_bounds__(kRcT) k_recount_tma(Dev d, long long n, long l
         vl[t] = (int)(base + jj);
         const int ci = e - ej;
         rem[t] = e < total ? dj - 4 * ci : 0;
-        if (e >= total) xa[t] = make_int4(-1, -1, -1, -1);
-        else if (staged) xa[t] = S.adj[ab][oj + ci - lo4];
-        else xa[t] = __ldg(g4 + oj + ci);
+        xa[t] = e < total ? __ldg(g4 + oj + ci) : make_int4(-1, -1, -1, -1);
       }
 #pragma unroll
       for (int t = 0; t < 2; t++) {

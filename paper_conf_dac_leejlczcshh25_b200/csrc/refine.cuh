@@ -79,11 +79,11 @@ struct ShardArgs {
 // thread: f(x, w, q) for each neighbour; a chunk issues all its ID/weight
 // loads, then all its label loads, before f runs; f returns false to stop
 constexpr int kTC = 16;  // thread chunk (== kThreadDeg: one round trip per vertex)
+// the commit's thread chunk: five values per slot (ID, weight, label, stamp,
+// saved label) plus the expansion marks -- 8 slots keep it off the local stack
+constexpr int kTCc = 8;
 template <class F>
-__device__ __forceinline__ void nbrs_thread(const Dev& d, int u, F f) {
-  long long o;
-  int dg;
-  vr_ld(d, u, o, dg);
+__device__ __forceinline__ void nbrs_thread(const Dev& d, long long o, int dg, F f) {
   for (int i = 0; i < dg; i += kTC) {
     int x[kTC], w[kTC];
     uint8_t q[kTC];
@@ -133,10 +133,7 @@ __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uin
     else d.Nlist[slot++] = x[t];
   }
 }
-__device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t epN, uint32_t epC) {
-  long long o;
-  int dg;
-  vr_ld(d, u, o, dg);
+__device__ __forceinline__ void mark_nbrs_thread(const Dev& d, long long o, int dg, uint32_t epN, uint32_t epC) {
   for (int i = 0; i < dg; i += kTC) {
     int x[kTC];
     uint8_t q[kTC];
@@ -147,10 +144,7 @@ __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, int u, uint32_t e
     mark_chunk<kTC>(d, x, q, epN, epC);
   }
 }
-__device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN, uint32_t epC) {
-  long long o;
-  int dg;
-  vr_ld(d, u, o, dg);
+__device__ __forceinline__ void mark_nbrs_warp(const Dev& d, long long o, int dg, uint32_t epN, uint32_t epC) {
   for (int b = 0; b < dg; b += 256) {
     int x[8];
     uint8_t q[8];
@@ -166,10 +160,7 @@ __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, int u, uint32_t epN
 }
 // warp: lane-strided, 8 entries per lane per round trip (256 per warp)
 template <class F>
-__device__ __forceinline__ void nbrs_warp(const Dev& d, int u, F f) {
-  long long o;
-  int dg;
-  vr_ld(d, u, o, dg);
+__device__ __forceinline__ void nbrs_warp(const Dev& d, long long o, int dg, F f) {
   for (int b = 0; b < dg; b += 256) {
     int x[8], w[8];
     uint8_t q[8];
@@ -191,7 +182,8 @@ __device__ __forceinline__ void nbrs_warp(const Dev& d, int u, F f) {
 // warp cooperates on it.  Items are dealt round-robin over ALL warps of the
 // grid (item i -> warp i mod W, lane (i / W) mod 32), so a short list still
 // spreads over every SM and heavy vertices rarely share a warp.
-// get(i) -> vertex (or -1); tf(u, i); wf(u, i).
+// get(i) -> vertex (or -1); tf(u, i, off, deg); wf(u, i, off, deg): the
+// vertex record is loaded once here and handed to the bucket.
 template <class Get, class TF, class WF>
 __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get get, TF tf, WF wf) {
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
@@ -200,15 +192,19 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
   for (long long r0 = 0; r0 < n; r0 += per_round) {
     long long i = r0 + (long long)lane_id() * nw + gw;
     int u = i < n ? get(i) : -1;
-    int dg = u >= 0 ? ldro(&d.vr[u].deg) : 0;
+    long long o = 0;
+    int dg = 0;
+    if (u >= 0) vr_ld(d, u, o, dg);  // one 16-byte record load; handed to the bucket
     bool heavy = dg > kThreadDeg;
-    if (u >= 0 && !heavy) tf(u, i);
+    if (u >= 0 && !heavy) tf(u, i, o, dg);
     unsigned hm = __ballot_sync(0xffffffffu, heavy);
     while (hm) {
       int src = __ffs(hm) - 1;
       hm &= hm - 1;
       int uu = __shfl_sync(0xffffffffu, u, src);
-      wf(uu, r0 + (long long)src * nw + gw);
+      long long oo = __shfl_sync(0xffffffffu, o, src);
+      int dd = __shfl_sync(0xffffffffu, dg, src);
+      wf(uu, r0 + (long long)src * nw + gw, oo, dd);
     }
   }
 }
@@ -401,7 +397,7 @@ struct RefSmem {
   int tie_n;
   long long Wr[256];      // round-start part weights (Q14)
   long long acc[256];     // per-part weight deltas of this CTA
-  long long red[32];
+  long long red[2 * kWarps];
   int wconn[kWarps][256]; // per-warp connectivity histogram
   int best0;
 };
@@ -487,14 +483,14 @@ __device__ __forceinline__ void block_sum2(RefSmem& s, long long& a, long long& 
   __syncthreads();
   if (lane_id() == 0) {
     s.red[warp_id()] = a;
-    s.red[16 + warp_id()] = b;
+    s.red[kWarps + warp_id()] = b;
   }
   __syncthreads();
   a = 0;
   b = 0;
   for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
     a += s.red[w];
-    b += s.red[16 + w];
+    b += s.red[kWarps + w];
   }
   __syncthreads();
 }
@@ -553,18 +549,18 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
 template <class Get>
 __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, uint32_t ep,
                             long long& scanned, long long& counted, uint32_t hub_ep = 0) {
-  auto tf = [&](int u, long long) {
+  auto tf = [&](int u, long long, long long o, int dg) {
     const uint8_t pu = ld_part(d.part, u);
     const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
     if (!act || hub || pu == kPsi || !own(d, u)) return;  // sharded: the owner filters
     counted++;
     long long in = 0, ex = 0;
-    nbrs_thread(d, u, [&](int, int w, uint8_t q) {
+    nbrs_thread(d, o, dg, [&](int, int w, uint8_t q) {
       if (q == pu) in += w; else ex += w;
       return true;
     });
-    scanned += ldro(&d.vr[u].deg);
+    scanned += dg;
     bool c = ex > in;
     if (c) {  // stamp + snapshot label: the commit reads it while labels change
       d.markT[u] = ep;
@@ -573,20 +569,20 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     int slot = agg_append(ncand, c);
     if (c) cand[slot] = u;
   };
-  auto wf = [&](int u, long long) {
+  auto wf = [&](int u, long long, long long o, int dg) {
     const uint8_t pu = ld_part(d.part, u);
     const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
     if (!act || hub || pu == kPsi || !own(d, u)) return;  // sharded: the owner filters
     long long in = 0, ex = 0;
-    nbrs_warp(d, u, [&](int, int w, uint8_t q) {
+    nbrs_warp(d, o, dg, [&](int, int w, uint8_t q) {
       if (q == pu) in += w; else ex += w;
     });
     in = warp_sum(in);
     ex = warp_sum(ex);
     if (lane_id() == 0) {
       counted++;
-      scanned += ldro(&d.vr[u].deg);
+      scanned += dg;
       if (ex > in) {
         d.markT[u] = ep;
         d.oldp[u] = pu;
@@ -611,46 +607,40 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     int slot = agg_append(&ctl->npsi[0], true);
     d.psi[0][slot] = u;
   };
-  auto tf = [&](int u, long long) {
+  auto tf = [&](int u, long long, long long o, int dg) {
     const uint8_t pu = __ldcg(d.oldp + u);
-    long long o;
-    int dg;
-    vr_ld(d, u, o, dg);
     scanned += dg;
     long long del = 0;
-    for (int i = 0; i < dg; i += kTC) {
-      int x[kTC], w[kTC];
-      uint8_t q[kTC];
-      unsigned mk[kTC];
+    for (int i = 0; i < dg; i += kTCc) {
+      int x[kTCc], w[kTCc];
+      uint8_t q[kTCc];
+      unsigned mk[kTCc];
 #pragma unroll
-      for (int t = 0; t < kTC; t++) {
+      for (int t = 0; t < kTCc; t++) {
         x[t] = (i + t < dg) ? ldro(d.adj + o + i + t) : -1;
         w[t] = (i + t < dg && d.adjw) ? ldro(d.adjw + o + i + t) : 1;
       }
-      uint8_t op[kTC];
+      uint8_t op[kTCc];
 #pragma unroll
-      for (int t = 0; t < kTC; t++) {  // label, stamp and saved label in one round trip
+      for (int t = 0; t < kTCc; t++) {  // label, stamp and saved label in one round trip
         q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
         mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
         op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
       }
 #pragma unroll
-      for (int t = 0; t < kTC; t++) {
+      for (int t = 0; t < kTCc; t++) {
         if (x[t] < 0) continue;
         const bool xc = mk[t] == ep;
         const uint8_t qx = xc ? op[t] : q[t];
         if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
       }
-      if (expand) mark_chunk<kTC>(d, x, q, a.epN, ep);
+      if (expand) mark_chunk<kTCc>(d, x, q, a.epN, ep);
     }
     if (own(d, u)) cut_acc -= del;  // sharded: the owner (full prefix) keeps the cut delta
     finish(u, pu);
   };
-  auto wf = [&](int u, long long) {
+  auto wf = [&](int u, long long, long long o, int dg) {
     const uint8_t pu = __ldcg(d.oldp + u);
-    long long o;
-    int dg;
-    vr_ld(d, u, o, dg);
     if (lane_id() == 0) scanned += dg;
     long long del = 0;
     for (int b = 0; b < dg; b += 256) {
@@ -857,11 +847,8 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     // tally); conn(u, p) for each neighbour's label p is a register-only
     // sum over the <= 16 slots, so every candidate part is evaluated
     // exactly as the warp / CTA buckets do it (reading Q6).
-    auto tf = [&](int u, long long j) {
+    auto tf = [&](int u, long long j, long long o, int dg) {
       const long long vwu = vert_w(d.vw, u);
-      long long o;
-      int dg;
-      vr_ld(d, u, o, dg);
       scanned += dg;
       int x[kThreadDeg], w[kThreadDeg];
       uint8_t q[kThreadDeg];
@@ -913,16 +900,16 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       sel_cnt++;
       emit_move(j, u, best, bc, pwv, imbal);
     };
-    auto wf = [&](int u, long long j) {
+    auto wf = [&](int u, long long j, long long o, int dg) {
       const long long vwu = vert_w(d.vw, u);
       int* wc = s.wconn[warp_id()];
       if (lane_id() == 0) {
-        scanned += ldro(&d.vr[u].deg);
+        scanned += dg;
         path_hit(ctl, PA_WARP_GAIN);
       }
       bool lb = false;
       long long pwv = 0;
-      nbrs_warp(d, u, [&](int x, int w, uint8_t q) {
+      nbrs_warp(d, o, dg, [&](int x, int w, uint8_t q) {
         if (q == kPsi) {
           lb |= x < u;
         } else {
@@ -1019,7 +1006,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
           }
           if (lane_id() == 0) {
             s.red[warp_id()] = bc;
-            s.red[16 + warp_id()] = best;
+            s.red[kWarps + warp_id()] = best;
           }
         }
         __syncthreads();
@@ -1031,7 +1018,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
             bc = -1;
             best = -1;
             for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
-              int op = (int)s.red[16 + w];
+              int op = (int)s.red[kWarps + w];
               if (op >= 0 && better(s.red[w], op, bc, best, s.Wr)) {
                 bc = s.red[w];
                 best = op;
@@ -1536,13 +1523,13 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       int u = __ldcg(d.psi[0] + i);
       return ld_part(d.part, u) == kPsi ? u : -1;  // C1 joins beyond np0
     };
-    auto mt = [&](int u, long long) {
-      scanned += ldro(&d.vr[u].deg);
-      mark_nbrs_thread(d, u, a.epN, a.epC1);
+    auto mt = [&](int u, long long, long long o, int dg) {
+      scanned += dg;
+      mark_nbrs_thread(d, o, dg, a.epN, a.epC1);
     };
-    auto mw = [&](int u, long long) {
-      if (lane_id() == 0) scanned += ldro(&d.vr[u].deg);
-      mark_nbrs_warp(d, u, a.epN, a.epC1);
+    auto mw = [&](int u, long long, long long o, int dg) {
+      if (lane_id() == 0) scanned += dg;
+      mark_nbrs_warp(d, o, dg, a.epN, a.epC1);
     };
     foreach_vertex(d, np0, get, mt, mw);
     flush_acc(s, ctl->Wp, k);
@@ -1615,26 +1602,26 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         uint8_t p = ld_part(d.part, v);
         return (p != kDel && p != kPsi && s.sel.used[p] && own(d, v)) ? (int)v : -1;
       };
-      auto tf = [&](int v, long long) {
+      auto tf = [&](int v, long long, long long o, int dg) {
         const uint8_t pv = ld_part(d.part, v);
         long long in = 0, ex = 0;
-        nbrs_thread(d, v, [&](int, int w, uint8_t q) {
+        nbrs_thread(d, o, dg, [&](int, int w, uint8_t q) {
           if (q == pv) in += w; else ex += w;
           return true;
         });
-        scanned += ldro(&d.vr[v].deg);
+        scanned += dg;
         emit(v, pv, in - ex);
       };
-      auto wf = [&](int v, long long) {
+      auto wf = [&](int v, long long, long long o, int dg) {
         const uint8_t pv = ld_part(d.part, v);
         long long in = 0, ex = 0;
-        nbrs_warp(d, v, [&](int, int w, uint8_t q) {
+        nbrs_warp(d, o, dg, [&](int, int w, uint8_t q) {
           if (q == pv) in += w; else ex += w;
         });
         in = warp_sum(in);
         ex = warp_sum(ex);
         if (lane_id() == 0) {
-          scanned += ldro(&d.vr[v].deg);
+          scanned += dg;
           emit(v, pv, in - ex);
         }
       };

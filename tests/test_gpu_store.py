@@ -88,3 +88,82 @@ print("STICKY_OK", msg)
 def test_cuda_error_is_sticky():
     r = subprocess.run([sys.executable, "-c", _STICKY, ROOT], capture_output=True, text=True, timeout=300)
     assert "STICKY_OK" in r.stdout, r.stdout + r.stderr
+
+
+@pytest.mark.parametrize("fmax,n,iters", [(1000, 200_000, 30), (10_000, 400_000, 6)])
+def test_recount_tma_matches_gather(monkeypatch, fmax, n, iters):
+    """S9: the TMA-pipelined recount (bulk copies of records, label windows
+    and slab spans) equals the direct-gather kernel and the oracle's cut /
+    W_p on a store with relocated prefixes, tombstones, deleted IDs and hub
+    spans larger than one staged tile (fallback path)."""
+    import oracle
+    g = gi.make_graph(n, fmax, 555 + fmax)
+    part, _ = gi.metis_partition(g, 8)
+    monkeypatch.setenv("IGK_RECOUNT", "gather")
+    Gg = igk.IGKGraph(g.xadj, g.adjncy, 8, 0.03, part)
+    monkeypatch.setenv("IGK_RECOUNT", "tma")
+    Gt = igk.IGKGraph(g.xadj, g.adjncy, 8, 0.03, part)
+    O = oracle.Oracle(g.xadj, g.adjncy, 8, 0.03, part)
+    S = gi.Stream(g, 4242)
+    for G in (Gg, Gt):
+        G.refine()
+    O.refine()
+    for it in range(iters):
+        b = S.next(gi.MODE_MIX, 0.05)
+        for G in (Gg, Gt):
+            assert G.apply(b)[0] == 0
+            G.refine()
+        O.apply(b)
+        O.refine()
+    rg, wg = Gg.recount()
+    rt, wt = Gt.recount()
+    assert rg == rt == O.cut() == Gt.cut()
+    assert np.array_equal(wg, wt) and np.array_equal(wt, O.part_weights())
+    sg, st = Gg.store_stats(), Gt.store_stats()
+    assert sg["adj_entries"] == st["adj_entries"] == 2 * (len(O.export_csr()[1]) // 2)
+    assert sg["n_active"] == st["n_active"] == O.n_active
+
+
+@pytest.mark.parametrize("pinned", [True, False])
+def test_pipelined_steps_match_oracle(pinned):
+    """NEXT-4: igk_stage_batch / igk_step_begin / igk_step_end -- the next
+    batch is copied while the current step runs -- give exactly the oracle's
+    results (partition, cut, stats, delta), with pinned and pageable batches,
+    an invalid batch in the middle (rejected, state unchanged) and a batch
+    that needs a store compaction."""
+    import torch
+    from tests.parity import COMMON
+    cfg = gi.CONFIGS["C1"]
+    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(1))
+    part, _ = gi.metis_partition(g, 4)
+    deg = np.diff(g.xadj)
+    used = int((((deg + np.maximum(2, deg // 4)) + 3) & ~3).sum())
+    P = Pair(g.xadj, g.adjncy, 4, cfg["eps"], part, check=False, max_slots=used + 256)
+    P.refine("settle")
+    S = gi.Stream(g, 2024)
+    batches = [S.next(gi.MODE_MIX, 0.03) for _ in range(10)]
+    batches.insert(5, np.array([[3, 7, 7, 1]], np.int32))  # self loop: invalid
+    if pinned:
+        hb = []
+        for b in batches:
+            t = torch.empty(b.shape, dtype=torch.int32, pin_memory=True).numpy()
+            t[...] = b
+            hb.append(t)
+        batches = hb
+    P.G.stage_batch(batches[0])
+    for i, b in enumerate(batches):
+        P.G.step_begin()
+        if i + 1 < len(batches):
+            P.G.stage_batch(batches[i + 1])  # overlaps the running step
+        s, stg, bad = P.G.step_end()
+        so, _, sbad = P.O.apply(b)
+        if so != 0:
+            assert s == 1 and bad == sbad == 0
+            continue
+        pre = P.O.partition()
+        _, sto = P.O.refine()
+        assert s in (0, 6)
+        assert all(sto[f] == stg[f] for f in COMMON), i
+        P.check_delta(pre, f"pipelined {i}")
+        P.compare_state(f"pipelined {i}")
+    assert P.G.debug_paths()["compaction"] >= 1
