@@ -607,6 +607,7 @@ igk_status compact_slab(igk_graph* g, long long extra) {
     return fail(g, IGK_ENOMEM, "slab compaction: allocation failed");
   }
   CK(cudaMemsetAsync(nadj, 0xff, cap * 4, g->stream));
+  if (nadjw) CK(cudaMemsetAsync(nadjw, 0, cap * 4, g->stream));
   if (n) CK(cudaMemcpyAsync(d_noff, noff.data(), n * 8, cudaMemcpyHostToDevice, g->stream));
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
@@ -859,6 +860,10 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   cudaMemsetAsync(d.vcnt, 0, N * 4, s);
   cudaMemsetAsync(d.icnt, 0, N * 4, s);
   cudaMemsetAsync(d.hist0, 0, 256 * kDigits * 8, s);
+  // the slab: every slot a tombstone until written (the recount reads whole
+  // int4 chunks of a prefix; the slack slots it masks are then initialised)
+  cudaMemsetAsync(d.adj, 0xff, (size_t)d.slot_cap * 4, s);
+  if (d.adjw) cudaMemsetAsync(d.adjw, 0, (size_t)d.slot_cap * 4, s);
   cudaMemsetAsync(d.histR, 0, 3 * 256 * kDigits * 8, s);
   cudaMemsetAsync(d.ctl, 0, sizeof(Ctl), s);
   // upload

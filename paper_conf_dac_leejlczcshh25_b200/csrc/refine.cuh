@@ -182,10 +182,13 @@ __device__ __forceinline__ void nbrs_warp(const Dev& d, long long o, int dg, F f
 // warp cooperates on it.  Items are dealt round-robin over ALL warps of the
 // grid (item i -> warp i mod W, lane (i / W) mod 32), so a short list still
 // spreads over every SM and heavy vertices rarely share a warp.
-// get(i) -> vertex (or -1); tf(u, i, off, deg); wf(u, i, off, deg): the
-// vertex record is loaded once here and handed to the bucket.
-template <class Get, class TF, class WF>
-__device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get get, TF tf, WF wf) {
+// get(i) -> list entry (vertex or -1); pre(u, i) -> the per-vertex word the
+// bucket needs (its label, saved label, ...) or -1 to skip the vertex;
+// tf(u, i, off, deg, pv) / wf(u, i, off, deg, pv).  The vertex record and
+// pre's loads do not depend on each other, so they are issued together: one
+// dependent round trip per item before the adjacency loads.
+template <class Get, class Pre, class TF, class WF>
+__device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get get, Pre pre, TF tf, WF wf) {
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long per_round = nw * 32;
@@ -193,10 +196,14 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
     long long i = r0 + (long long)lane_id() * nw + gw;
     int u = i < n ? get(i) : -1;
     long long o = 0;
-    int dg = 0;
-    if (u >= 0) vr_ld(d, u, o, dg);  // one 16-byte record load; handed to the bucket
-    bool heavy = dg > kThreadDeg;
-    if (u >= 0 && !heavy) tf(u, i, o, dg);
+    int dg = 0, pv = -1;
+    if (u >= 0) {
+      vr_ld(d, u, o, dg);  // one 16-byte record load; handed to the bucket
+      pv = pre(u, i);
+    }
+    const bool ok = pv >= 0;
+    const bool heavy = ok && dg > kThreadDeg;
+    if (ok && !heavy) tf(u, i, o, dg, pv);
     unsigned hm = __ballot_sync(0xffffffffu, heavy);
     while (hm) {
       int src = __ffs(hm) - 1;
@@ -204,7 +211,8 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
       int uu = __shfl_sync(0xffffffffu, u, src);
       long long oo = __shfl_sync(0xffffffffu, o, src);
       int dd = __shfl_sync(0xffffffffu, dg, src);
-      wf(uu, r0 + (long long)src * nw + gw, oo, dd);
+      int pp = __shfl_sync(0xffffffffu, pv, src);
+      wf(uu, r0 + (long long)src * nw + gw, oo, dd, pp);
     }
   }
 }
@@ -461,6 +469,7 @@ __device__ unsigned block_select_ids(RefSmem& s, int cnt, long long base, long l
         int src = __ffs(m) - 1;
         int dd = __shfl_sync(0xffffffffu, cd, src);
         long long bb = __shfl_sync(0xffffffffu, cb, src);
+        __syncwarp();  // every lane's read of tie_base precedes lane 0's update (racecheck: WAR)
         if (l == 0) {
           s.tie_prefix |= (unsigned long long)dd << shift;
           s.tie_base = bb;
@@ -549,11 +558,15 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
 template <class Get>
 __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, uint32_t ep,
                             long long& scanned, long long& counted, uint32_t hub_ep = 0) {
-  auto tf = [&](int u, long long, long long o, int dg) {
+  // the label doubles as the active flag; hubs of A go to the CTA pass;
+  // sharded: the owner filters
+  auto pre = [&](int u, long long) -> int {
     const uint8_t pu = ld_part(d.part, u);
-    const bool act = pu != kDel;  // the label doubles as the active flag
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
-    if (!act || hub || pu == kPsi || !own(d, u)) return;  // sharded: the owner filters
+    return (pu == kDel || hub || pu == kPsi || !own(d, u)) ? -1 : (int)pu;
+  };
+  auto tf = [&](int u, long long, long long o, int dg, int pvv) {
+    const uint8_t pu = (uint8_t)pvv;
     counted++;
     long long in = 0, ex = 0;
     nbrs_thread(d, o, dg, [&](int, int w, uint8_t q) {
@@ -569,11 +582,8 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
     int slot = agg_append(ncand, c);
     if (c) cand[slot] = u;
   };
-  auto wf = [&](int u, long long, long long o, int dg) {
-    const uint8_t pu = ld_part(d.part, u);
-    const bool act = pu != kDel;  // the label doubles as the active flag
-    const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
-    if (!act || hub || pu == kPsi || !own(d, u)) return;  // sharded: the owner filters
+  auto wf = [&](int u, long long, long long o, int dg, int pvv) {
+    const uint8_t pu = (uint8_t)pvv;
     long long in = 0, ex = 0;
     nbrs_warp(d, o, dg, [&](int, int w, uint8_t q) {
       if (q == pu) in += w; else ex += w;
@@ -590,7 +600,7 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
       }
     }
   };
-  foreach_vertex(d, n, get, tf, wf);
+  foreach_vertex(d, n, get, pre, tf, wf);
 }
 
 // deferred commit to the pseudo-partition (Alg. 3 L25-26) of the candidates
@@ -607,8 +617,9 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     int slot = agg_append(&ctl->npsi[0], true);
     d.psi[0][slot] = u;
   };
-  auto tf = [&](int u, long long, long long o, int dg) {
-    const uint8_t pu = __ldcg(d.oldp + u);
+  auto pre = [&](int u, long long) -> int { return __ldcg(d.oldp + u); };
+  auto tf = [&](int u, long long, long long o, int dg, int pvv) {
+    const uint8_t pu = (uint8_t)pvv;
     scanned += dg;
     long long del = 0;
     for (int i = 0; i < dg; i += kTCc) {
@@ -639,8 +650,8 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     if (own(d, u)) cut_acc -= del;  // sharded: the owner (full prefix) keeps the cut delta
     finish(u, pu);
   };
-  auto wf = [&](int u, long long, long long o, int dg) {
-    const uint8_t pu = __ldcg(d.oldp + u);
+  auto wf = [&](int u, long long, long long o, int dg, int pvv) {
+    const uint8_t pu = (uint8_t)pvv;
     if (lane_id() == 0) scanned += dg;
     long long del = 0;
     for (int b = 0; b < dg; b += 256) {
@@ -675,7 +686,7 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
       finish(u, pu);
     }
   };
-  foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, tf, wf);
+  foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, pre, tf, wf);
 }
 
 // commit of hub candidates by a whole CTA each (same arithmetic as commit());
@@ -824,13 +835,13 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     };
     auto get = [&](long long i) {
       int u = __ldcg(plist + i);
-      if (u < 0) {
-        d.meta[i] = 0;
-        return -1;
-      }
+      if (u < 0 && !kSh) d.meta[i] = 0;
+      return u;
+    };
+    auto pre = [&](int u, long long i) -> int {  // issued together with the vertex record
       const uint8_t pu = ld_part(d.part, u);
       const bool act = pu != kDel;  // the label doubles as the active flag
-      if (kSh) return (act && pu == kPsi && own(d, u)) ? u : -1;  // hubs: warp path; others' vertices: their owners
+      if (kSh) return (act && pu == kPsi && own(d, u)) ? (int)pu : -1;  // hubs: warp path; others: their owners
       const bool hub = __ldcg(d.markH + u) == a.epF;
       if (!act || pu != kPsi) {
         d.meta[i] = 0;
@@ -840,14 +851,14 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         d.meta[i] = kMetaHub;
         return -1;
       }
-      return u;
+      return (int)pu;
     };
     // thread bucket (degree <= kThreadDeg, one load round trip): the whole
     // prefix sits in registers (static indices only -- no local-memory
     // tally); conn(u, p) for each neighbour's label p is a register-only
     // sum over the <= 16 slots, so every candidate part is evaluated
     // exactly as the warp / CTA buckets do it (reading Q6).
-    auto tf = [&](int u, long long j, long long o, int dg) {
+    auto tf = [&](int u, long long j, long long o, int dg, int) {
       const long long vwu = vert_w(d.vw, u);
       scanned += dg;
       int x[kThreadDeg], w[kThreadDeg];
@@ -900,7 +911,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       sel_cnt++;
       emit_move(j, u, best, bc, pwv, imbal);
     };
-    auto wf = [&](int u, long long j, long long o, int dg) {
+    auto wf = [&](int u, long long j, long long o, int dg, int) {
       const long long vwu = vert_w(d.vw, u);
       int* wc = s.wconn[warp_id()];
       if (lane_id() == 0) {
@@ -959,7 +970,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         }
       }
     };
-    foreach_vertex(d, np, get, tf, wf);
+    foreach_vertex(d, np, get, pre, tf, wf);
     if (!kSh) {  // hubs in the pseudo-partition: one CTA each
       int* conn = s.wconn[0];
       for (int h = blockIdx.x; h < nhp; h += gridDim.x) {
@@ -1519,19 +1530,17 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
     hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
     // neighbours of the pseudo vertices pending since apply
-    auto get = [&](long long i) {
-      int u = __ldcg(d.psi[0] + i);
-      return ld_part(d.part, u) == kPsi ? u : -1;  // C1 joins beyond np0
-    };
-    auto mt = [&](int u, long long, long long o, int dg) {
+    auto get = [&](long long i) { return __ldcg(d.psi[0] + i); };  // C1 joins beyond np0
+    auto pre = [&](int u, long long) -> int { return ld_part(d.part, u) == kPsi ? (int)kPsi : -1; };
+    auto mt = [&](int u, long long, long long o, int dg, int) {
       scanned += dg;
       mark_nbrs_thread(d, o, dg, a.epN, a.epC1);
     };
-    auto mw = [&](int u, long long, long long o, int dg) {
+    auto mw = [&](int u, long long, long long o, int dg, int) {
       if (lane_id() == 0) scanned += dg;
       mark_nbrs_warp(d, o, dg, a.epN, a.epC1);
     };
-    foreach_vertex(d, np0, get, mt, mw);
+    foreach_vertex(d, np0, get, pre, mt, mw);
     flush_acc(s, ctl->Wp, k);
     PHASE_FLUSH(PH_F1, nc + nhC + np0);
   }
@@ -1602,8 +1611,9 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         uint8_t p = ld_part(d.part, v);
         return (p != kDel && p != kPsi && s.sel.used[p] && own(d, v)) ? (int)v : -1;
       };
-      auto tf = [&](int v, long long, long long o, int dg) {
-        const uint8_t pv = ld_part(d.part, v);
+      auto pre = [&](int v, long long) -> int { return ld_part(d.part, v); };  // an L1/L2 hit: get read it
+      auto tf = [&](int v, long long, long long o, int dg, int pvv) {
+        const uint8_t pv = (uint8_t)pvv;
         long long in = 0, ex = 0;
         nbrs_thread(d, o, dg, [&](int, int w, uint8_t q) {
           if (q == pv) in += w; else ex += w;
@@ -1612,8 +1622,8 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
         scanned += dg;
         emit(v, pv, in - ex);
       };
-      auto wf = [&](int v, long long, long long o, int dg) {
-        const uint8_t pv = ld_part(d.part, v);
+      auto wf = [&](int v, long long, long long o, int dg, int pvv) {
+        const uint8_t pv = (uint8_t)pvv;
         long long in = 0, ex = 0;
         nbrs_warp(d, o, dg, [&](int, int w, uint8_t q) {
           if (q == pv) in += w; else ex += w;
@@ -1625,7 +1635,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
           emit(v, pv, in - ex);
         }
       };
-      foreach_vertex(d, ntot, get, tf, wf);
+      foreach_vertex(d, ntot, get, pre, tf, wf);
       PHASE_FLUSH(PH_R3, ntot);
       if (!kSh) {
         GRID_SYNC_STAMPED(ctl, 205);
