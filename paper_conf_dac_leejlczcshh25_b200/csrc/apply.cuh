@@ -310,7 +310,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       ok = yo && acty && vcy == 1;
       if (ok) {  // kVdC-entry work chunks of this deletion
         int nch = max(1, (dgy + kVdC - 1) / kVdC);
-        int s = atomicAdd(&ctl->nvdch, nch);
+        int s = agg_alloc(&ctl->nvdch, nch);
         for (int c = 0; c < nch; c++) d.vdch[s + c] = make_int2(m.y, c);
       }
     } else if (m.x == kVertIns) {
@@ -341,13 +341,20 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
         long long need = (x < n0 ? __ldcg(&d.vr[x].deg) : 0) + __ldcg(d.icnt + x);
         long long have = x < n0 ? __ldcg(d.capv + x) : 0;
         long long pk = -1;
-        if (need > have) {
-          long long nc = need + max((long long)d.slack_min, need / 4);
-          nc = (nc + 3) & ~3ll;
-          long long no = atomicAdd((unsigned long long*)&ctl->slab_top, (unsigned long long)nc);
-          if (no + nc > d.slot_cap) atomicOr(&ctl->err_nomem, 2);  // 2: adjacency slab exhausted
-          pk = (no << 24) | nc;
-          d.rlist[atomicAdd(&ctl->nreloc, 1)] = x;  // M3 / M4 walk only the moving prefixes
+        const bool mv = need > have;
+        unsigned long long nc = 0;
+        if (mv) {
+          nc = (unsigned long long)(need + max((long long)d.slack_min, need / 4));
+          nc = (nc + 3) & ~3ull;
+        }
+        // one slab reservation and one relocation-list slot per warp, not per
+        // vertex (C4: ~10^5 relocations per batch on one counter)
+        const long long no = (long long)agg_alloc((unsigned long long*)&ctl->slab_top, nc);
+        const int rs = agg_append(&ctl->nreloc, mv);
+        if (mv) {
+          if (no + (long long)nc > d.slot_cap) atomicOr(&ctl->err_nomem, 2);  // 2: adjacency slab exhausted
+          pk = (no << 24) | (long long)nc;
+          d.rlist[rs] = x;  // M3 / M4 walk only the moving prefixes
         }
         d.reloc[x] = pk;
       }

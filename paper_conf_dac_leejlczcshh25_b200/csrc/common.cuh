@@ -363,6 +363,27 @@ __device__ __forceinline__ int agg_append(int* ctr, bool pred) {
   return pred ? base + __popc(m & ((1u << lane) - 1u)) : -1;
 }
 
+// warp-aggregated bump allocation: the converged lanes' amounts v (0 =
+// none) are summed, ONE atomicAdd reserves the total, each lane gets its
+// exclusive offset.  Replaces per-lane atomics on one hot counter.
+template <typename T>
+__device__ __forceinline__ T agg_alloc(T* ctr, T v) {
+  const unsigned act = __activemask();
+  const int lane = lane_id();
+  T total = 0, excl = 0;
+  for (unsigned m = act; m; m &= m - 1) {
+    const int src = __ffs(m) - 1;
+    const T vv = __shfl_sync(act, v, src);
+    if (src < lane) excl += vv;
+    total += vv;
+  }
+  const int leader = __ffs(act) - 1;
+  T base = 0;
+  if (lane == leader && total) base = atomicAdd(ctr, total);
+  base = __shfl_sync(act, base, leader);
+  return base + excl;
+}
+
 template <typename T>
 __device__ __forceinline__ T warp_sum(T v) {
 #pragma unroll

@@ -863,6 +863,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   // the slab: every slot a tombstone until written (the recount reads whole
   // int4 chunks of a prefix; the slack slots it masks are then initialised)
   cudaMemsetAsync(d.adj, 0xff, (size_t)d.slot_cap * 4, s);
+  cudaMemsetAsync(d.oldp, kPsi, N, s);  // saved labels: read (masked) for every neighbour by the commit
   if (d.adjw) cudaMemsetAsync(d.adjw, 0, (size_t)d.slot_cap * 4, s);
   cudaMemsetAsync(d.histR, 0, 3 * 256 * kDigits * 8, s);
   cudaMemsetAsync(d.ctl, 0, sizeof(Ctl), s);

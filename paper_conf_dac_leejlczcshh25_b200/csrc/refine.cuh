@@ -812,8 +812,10 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       d.pw[u] = (int)pwv;
       d.meta[j] = 0x80000000u | ((unsigned)d0 << 8) | (unsigned)best;  // j: list position
       long long w = vert_w(d.vw, u);
-      atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
-      atomic_add_ll(&ctl->tot3[r3][best], w);
+      // lanes with the same (part, digit) / part combine first: one global
+      // atomic per distinct key per warp (the round's hot histogram cells)
+      acc_add(d.hist0, best * kDigits + d0, w);
+      acc_add(ctl->tot3[r3], best, w);
       if (imbal) {
         ctl->st[ST_IMBAL] = 1;
         path_hit(ctl, PA_WFALLBACK);
@@ -1076,8 +1078,8 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         d.pw[u] = e.w;
         d.meta[j] = m;
         const long long w = vert_w(d.vw, u);
-        atomic_add_ll(d.hist0 + (long long)best * kDigits + d0, w);
-        atomic_add_ll(&ctl->tot3[r3][best], w);
+        acc_add(d.hist0, best * kDigits + d0, w);
+        acc_add(ctl->tot3[r3], best, w);
         atomicAdd(&ctl->selected3[r3], 1);
         if ((unsigned)e.y & (1u << 30)) {
           ctl->st[ST_IMBAL] = 1;
