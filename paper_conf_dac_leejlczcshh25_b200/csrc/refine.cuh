@@ -178,6 +178,28 @@ __device__ __forceinline__ void nbrs_warp(const Dev& d, long long o, int dg, F f
   }
 }
 
+// nbrs_warp with an early exit after each 256-entry chunk once any lane's
+// stop() holds (the round gain of a blocked vertex)
+template <class F, class S>
+__device__ __forceinline__ void nbrs_warp_until(const Dev& d, long long o, int dg, F f, S stop) {
+  for (int b = 0; b < dg; b += 256) {
+    int x[8], w[8];
+    uint8_t q[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      int i = b + t * 32 + lane_id();
+      x[t] = i < dg ? ldro(d.adj + o + i) : -1;
+      w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
+    }
+#pragma unroll
+    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+#pragma unroll
+    for (int t = 0; t < 8; t++)
+      if (x[t] >= 0) f(x[t], w[t], q[t]);
+    if (__any_sync(0xffffffffu, stop())) return;
+  }
+}
+
 // Iterate a vertex list: degree <= kThreadDeg -> one thread, else the whole
 // warp cooperates on it.  Items are dealt round-robin over ALL warps of the
 // grid (item i -> warp i mod W, lane (i / W) mod 32), so a short list still
@@ -521,6 +543,29 @@ __device__ __forceinline__ void nbrs_block(const Dev& d, int u, F f) {
 #pragma unroll
     for (int t = 0; t < 4; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
     f(x, w, q);
+  }
+}
+// CTA-strided walk with an early exit: after each chunk the CTA stops as soon
+// as any thread's f returned true (used by the round gain: one smaller-ID
+// pseudo neighbour blocks the hub, the rest of its 10^3-10^4 entries need
+// not be read)
+template <class F>
+__device__ __forceinline__ void nbrs_block_until(const Dev& d, int u, F f) {
+  long long o;
+  int dg;
+  vr_ld(d, u, o, dg);
+  for (int b = 0; b < dg; b += 8 * (int)blockDim.x) {
+    int x[8], w[8];
+    uint8_t q[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+      int i = b + t * (int)blockDim.x + (int)threadIdx.x;
+      x[t] = i < dg ? ldro(d.adj + o + i) : -1;
+      w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
+    }
+#pragma unroll
+    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    if (__syncthreads_or(f(x, w, q))) return;
   }
 }
 // hub filter (Alg. 3 L8-24) by a whole CTA; candidates go to `hout`
@@ -922,14 +967,17 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
       }
       bool lb = false;
       long long pwv = 0;
-      nbrs_warp(d, o, dg, [&](int x, int w, uint8_t q) {
-        if (q == kPsi) {
-          lb |= x < u;
-        } else {
-          atomicAdd(wc + q, w);
-          pwv += w;
-        }
-      });
+      nbrs_warp_until(
+          d, o, dg,
+          [&](int x, int w, uint8_t q) {
+            if (q == kPsi) {
+              lb |= x < u;
+            } else {
+              atomicAdd(wc + q, w);
+              pwv += w;
+            }
+          },
+          [&]() { return lb; });  // blocked (Alg. 4 L8-10): the rest of the prefix is not needed
       const bool blocked = __any_sync(0xffffffffu, lb);
       pwv = warp_sum(pwv);
       __syncwarp();
@@ -984,9 +1032,9 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
         __syncthreads();
         bool lb = false;
         long long pwv = 0, dummy = 0;
-        nbrs_block(d, u, [&](const int* x, const int* w, const uint8_t* q) {
+        nbrs_block_until(d, u, [&](const int* x, const int* w, const uint8_t* q) {
 #pragma unroll
-          for (int t = 0; t < 4; t++) {
+          for (int t = 0; t < 8; t++) {
             if (x[t] < 0) continue;
             if (q[t] == kPsi) {
               lb |= x[t] < u;
@@ -995,6 +1043,7 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
               pwv += w[t];
             }
           }
+          return lb;  // blocked (Alg. 4 L8-10): the rest of the prefix is not needed
         });
         const bool blocked = __syncthreads_or(lb);
         block_sum2(s, pwv, dummy);
