@@ -62,6 +62,9 @@ def parse():
     ap.add_argument("--shard", action="store_true",
                     help="ONE graph vertex-range sharded over the ranks (the default at N>1; strong scaling; "
                          "at N=1 the sharded protocol runs on one rank over an NCCL loopback communicator)")
+    ap.add_argument("--p2p", action="store_true",
+                    help="sharded: all rounds of a refine in one persistent kernel per rank, move records "
+                         "stored into peer memory + device barrier (NEXT-3) instead of per-round all-reduces")
     ap.add_argument("--replicas", action="store_true",
                     help="N>1: independent graph instances per rank (weak scaling) instead of sharding")
     return ap.parse_args()
@@ -357,6 +360,7 @@ def main():
             if dist:
                 dist.broadcast_object_list(uid, src=0)
             shard_kw = dict(nranks=world, rank=rank, nccl_id=uid[0])
+        shard_kw["p2p"] = args.p2p
     G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part, device=local, stream=stream.cuda_stream, **shard_kw)
     G.refine()  # settle the METIS partition (untimed; collective when sharded)
     dev_batches = [torch.from_numpy(b).cuda() for b in batches[: W + K]]
@@ -502,7 +506,8 @@ def main():
     split = launches >= 2 * K and not args.shard
     kname = "k_apply+k_refine (split launch, one step)" if split else "k_step (apply+refine fused)"
     if args.shard:
-        kname = "k_apply x2 + k_refine_sh x(5 + 2 R) (sharded step)"
+        kname = ("k_apply x2 + k_refine_sh x5 + k_rounds_p2p (sharded step, persistent P2P rounds)" if args.p2p
+                 else "k_apply x2 + k_refine_sh x(5 + 2 R) (sharded step)")
     traffic = None
     try:
         tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
@@ -515,7 +520,8 @@ def main():
         "vs_baseline": None,
         "dtype": "int32", "data": "synthetic",
         "config": {"workload": desc, "n": g.n, "k": k,
-                   "parallelism": ("sharded" if args.shard else "replicas") if world > 1 else "single",
+                   "parallelism": (("sharded" + ("+p2p" if args.p2p else "")) if args.shard else "replicas")
+                   if (world > 1 or args.shard) else "single",
                    "l2": "flushed between iterations (256 MiB write)" if flush is not None else "not flushed",
                    "batch_modifiers": int(np.mean([len(b) for b in batches[W:W + K]])),
                    # the stream is edge-conserving: average degree at the start of

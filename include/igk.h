@@ -95,6 +95,18 @@ typedef struct {
   int32_t rank;
   const void* nccl_id;     /* ncclUniqueId (128 bytes) or NULL                            */
   const igk_comm* comm;    /* host-callback transport (used when nccl_id == NULL)         */
+  /* NEXT-3 (sharded handles): p2p = 1 runs all rounds of a refine in ONE
+   * persistent kernel per rank that stores the move records straight into
+   * every rank's buffer (peer memory: NVLink P2P between GPUs -- CUDA IPC
+   * across processes, direct pointers inside one process -- or the same
+   * device) and synchronises the ranks with a device-side barrier, instead
+   * of a host round trip + all-reduce per round.  Set up collectively at
+   * create (the buffers' addresses / IPC handles are exchanged through the
+   * transport).  ranks_per_device > 1 when several ranks share one GPU
+   * (tests): each rank's persistent kernel then takes that fraction of the
+   * SMs so all of them are resident at once. */
+  int32_t p2p;
+  int32_t ranks_per_device;
 } igk_options;
 
 typedef struct {
@@ -300,6 +312,7 @@ int32_t igk_debug_phase_times(const igk_graph* g, int32_t which, int32_t* ids, i
  * igk_create): per-CTA %globaltimer arrival stamps at barrier slot s of the
  * last kernel, out[s * grid + cta], 128 slots; returns the grid size. */
 int32_t igk_debug_arrivals(const igk_graph* g, int32_t which, int64_t* out, int32_t cap);
+/* the last failure of g; with g == NULL: why this thread's last igk_create failed */
 const char* igk_last_error(const igk_graph* g);
 void igk_destroy(igk_graph* g);
 

@@ -52,7 +52,7 @@ class Options(C.Structure):
                 ("max_slots", C.c_int64), ("slack_min", C.c_int32), ("validate", C.c_int32),
                 ("check_invariants", C.c_int32), ("blocks_per_sm", C.c_int32),
                 ("nranks", C.c_int32), ("rank", C.c_int32), ("nccl_id", C.c_void_p),
-                ("comm", C.POINTER(Comm))]
+                ("comm", C.POINTER(Comm)), ("p2p", C.c_int32), ("ranks_per_device", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -196,7 +196,7 @@ class IGKGraph:
 
     def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, device=0, stream=None,
                  max_vertices=0, max_slots=0, slack_min=0, check=False, blocks_per_sm=0,
-                 nranks=1, rank=0, nccl_id: bytes | None = None, comm: "TorchComm | None" = None):
+                 nranks=1, rank=0, nccl_id: bytes | None = None, comm=None, p2p=False, ranks_per_device=1):
         """nranks > 1: rank `rank` of a vertex-range sharded graph (collective
         calls; every rank passes the same graph and batches).  Transport: NCCL
         from `nccl_id` (nccl_unique_id() on one rank, shared), else `comm`."""
@@ -210,12 +210,12 @@ class IGKGraph:
         self._comm = comm  # keeps the callback alive as long as the handle
         o = Options(device, stream or None, max_vertices, max_slots, slack_min, 1, int(check), blocks_per_sm,
                     int(nranks), int(rank), None if self._id is None else C.cast(self._id, C.c_void_p),
-                    None if comm is None else C.pointer(comm.struct))
+                    None if comm is None else C.pointer(comm.struct), int(bool(p2p)), int(ranks_per_device))
         h = C.c_void_p()
         s = L.igk_create(C.byref(o), len(xadj) - 1, _p(xadj, C.c_int64), _p(adjncy, C.c_int32),
                          _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(h))
         if s != OK:
-            raise IGKError(s, "igk_create failed")
+            raise IGKError(s, "igk_create failed: " + L.igk_last_error(None).decode())
         self._destroy = L.igk_destroy  # kept: module globals may be gone at interpreter exit
         self.h = h
         self.k = int(k)

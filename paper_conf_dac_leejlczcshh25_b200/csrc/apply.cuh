@@ -122,6 +122,17 @@ __device__ __forceinline__ void mark_affected(const Dev& d, int x, uint32_t epA,
   }
 }
 
+// mark_affected with the stamp already loaded (issued with other loads)
+__device__ __forceinline__ void mark_affected_pre(const Dev& d, int x, uint32_t epA, int dgx, uint32_t stamp) {
+  const bool na = stamp != epA && atomicExch(d.markA + x, epA) != epA;
+  int s2 = agg_append(&d.ctl->nA, na);
+  if (na) d.Alist[s2] = x;
+  if (na && dgx > kBlockDeg) {
+    d.markH[x] = epA;
+    d.hubA[atomicAdd(&d.ctl->nhubA, 1)] = x;
+  }
+}
+
 // mark_affected for C candidates of one thread: every stamp probe and
 // exchange in flight together, one list reservation per thread
 template <int C>
@@ -597,11 +608,17 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
   rr_for(B, [&](long long i) {
     int4 m = a.mods[i];
     if (m.x != kEdgeIns || !rel_edge(d, m)) return;
+    // everything that does not depend on the slot reservations is loaded
+    // first (offsets are final after M3; labels; the affected stamps), so
+    // the reservations and these loads share one round trip
+    const long long oy = __ldcg(&d.vr[m.y].off), oz = __ldcg(&d.vr[m.z].off);
+    const uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
+    const uint32_t sy = __ldcg(d.markA + m.y), sz = __ldcg(d.markA + m.z);
     int pu_pos = atomicAdd(&d.vr[m.y].deg, 1);
     int pv_pos = atomicAdd(&d.vr[m.z].deg, 1);
     atomicAdd(&d.vr[m.y].ldeg, 1);
     atomicAdd(&d.vr[m.z].ldeg, 1);
-    long long su = __ldcg(&d.vr[m.y].off) + pu_pos, sv = __ldcg(&d.vr[m.z].off) + pv_pos;
+    long long su = oy + pu_pos, sv = oz + pv_pos;
     d.adj[su] = m.z;
     d.adj[sv] = m.y;
     d.twin[su] = (int)sv;
@@ -610,10 +627,9 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       d.adjw[su] = m.w;
       d.adjw[sv] = m.w;
     }
-    uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
     if (pu != kPsi && pv != kPsi && pu != pv && own(d, m.y)) cut_acc += m.w;
-    mark_affected(d, m.y, a.epA, pu_pos + 1);
-    mark_affected(d, m.z, a.epA, pv_pos + 1);
+    mark_affected_pre(d, m.y, a.epA, pu_pos + 1, sy);
+    mark_affected_pre(d, m.z, a.epA, pv_pos + 1, sz);
   });
   // twin fix-ups of moved entries: resolve forward marks of moved partners,
   // then point the partner back at the new slot (idempotent when both moved)

@@ -84,7 +84,7 @@ struct Ctl {
   int n_delta;         // (vertex, part) pairs in the delta list of the last refine
   int sh_flag;         // sharded refine: restoration (R3) needed after kShF3
   int sh_np;           // sharded refine: pending vertices after F3 / R3 (length of the canonical list)
-  int sh_pad;
+  int p2p_err;         // persistent P2P rounds: a peer never reached the device barrier (timeout)
   long long sh_err[2]; // sharded apply: [0] lowest invalid index, [1] capacity flags (all-reduced MIN / MAX)
   // ---- device-side state ----
   long long Wp[256];   // part weights
@@ -149,6 +149,11 @@ struct Dev {
   uint64_t* bm;      // sharded refine: candidate bitmap (n_cap bits), all-reduced (sum of disjoint bits = OR)
   uint32_t* lossbuf; // sharded R3: (int - ext) + 2^31 of owned restoration candidates, 0 = none; all-reduced
   int4* recs;        // sharded rounds: one move record per position of the canonical pending list
+  // NEXT-3 persistent round kernel: the round's record buffer of every rank
+  // (peer memory over NVLink P2P, or the same device); the gain stores each
+  // record into all of them
+  int32_t p2p_n;
+  int4* p2p_recs[8];
   // graph store (S0)
   VRec* vr;          // per-vertex record: prefix offset, length, live degree (one sector)
   int32_t* capv;     // capacity

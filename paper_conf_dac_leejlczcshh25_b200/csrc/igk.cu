@@ -5,6 +5,7 @@
 // store build (S0), the cut/weight reduction (S9) and the exports.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
+#include <unistd.h>
 #include <nccl.h>  // types only: NCCL is loaded at run time (nccl_api), not linked
 #include <nvtx3/nvToolsExt.h>
 
@@ -271,10 +272,21 @@ struct igk_graph {
   void* nccl = nullptr;        // ncclComm_t created from igk_options.nccl_id
   void* xp_host = nullptr;     // pinned staging of the callback transport
   size_t xp_host_cap = 0;
-  long long* d_xp = nullptr;   // 8-word device scratch for host-value all-reduces
+  long long* d_xp = nullptr;   // kXpWords-word device scratch for host-value all-reduces
   long long cut_total = 0;     // sharded: the global cut (sum of the ranks' partial cuts)
   void* sort_tmp = nullptr;    // sharded: CUB radix-sort scratch (canonical pending list)
   size_t sort_tmp_cap = 0;
+  // NEXT-3 persistent P2P rounds (igk_options.p2p)
+  bool p2p = false;
+  int ranks_per_device = 1;
+  int grid_p2p = 0;
+  int4* p2p_mem = nullptr;                 // this rank's two record buffers (2 x n_cap int4)
+  unsigned long long* p2p_bar = nullptr;   // this rank's barrier counter
+  long long p2p_cap = 0;                   // entries per buffer
+  int4* p2p_bufs[8][2] = {};               // every rank's buffers (own, peer or IPC-mapped)
+  unsigned long long* p2p_bars[8] = {};
+  bool p2p_ipc[8] = {};                    // mapped with cudaIpcOpenMemHandle (closed on teardown)
+  long long p2p_rounds = 0;                // rounds run so far (barrier counter base / n)
   cudaStream_t stream = nullptr;
   bool poisoned = false;
   std::string err;
@@ -324,6 +336,8 @@ struct igk_graph {
 };
 
 namespace {
+
+thread_local std::string t_create_err;  // why the last igk_create of this thread failed (igk_last_error(NULL))
 
 // Every entry point runs on the handle's device and restores the caller's
 // current device on return (the ABI allows handles on several GPUs).
@@ -438,6 +452,7 @@ const NcclApi* nccl_api() {
 }
 
 enum { XP_I64 = 0, XP_U32 = 1 };
+constexpr int kXpWords = 512;  // device scratch of host-value all-reduces (p2p blobs: 8 ranks x 40 words)
 enum { XP_SUM = 0, XP_MIN = 1, XP_MAX = 2 };
 igk_status xp_allreduce(igk_graph* g, void* dptr, long long count, int dtype, int op) {
   if (!g->sharded || count <= 0) return IGK_OK;
@@ -474,12 +489,118 @@ igk_status xp_allreduce(igk_graph* g, void* dptr, long long count, int dtype, in
 // all-reduce (sum) of host values through the device scratch
 igk_status xp_sum_host(igk_graph* g, long long* vals, int n) {
   if (!g->sharded) return IGK_OK;
+  if (n > kXpWords) return fail(g, IGK_EINVAL, "xp_sum_host: too many values");
   CK(cudaMemcpyAsync(g->d_xp, vals, n * 8, cudaMemcpyHostToDevice, g->stream));
   igk_status st = xp_allreduce(g, g->d_xp, n, XP_I64, XP_SUM);
   if (st != IGK_OK) return st;
   CK(cudaMemcpyAsync(vals, g->d_xp, n * 8, cudaMemcpyDeviceToHost, g->stream));
   CK(cudaStreamSynchronize(g->stream));
   return IGK_OK;
+}
+
+// NEXT-3 set-up (collective): allocate this rank's record buffers and
+// barrier counter, exchange {pid, device, pointers, IPC handles} through the
+// transport (sum of disjoint rows), map every peer: the same process ->
+// direct pointers (+ peer access across devices), another process -> CUDA
+// IPC.  Re-run after a vertex-capacity growth (the buffers hold n_cap).
+constexpr int kBlob = 40;  // int64 words per rank
+void p2p_teardown(igk_graph* g) {
+  for (int q = 0; q < g->nranks && q < 8; q++) {
+    if (g->p2p_ipc[q]) {
+      cudaIpcCloseMemHandle(g->p2p_bufs[q][0]);
+      cudaIpcCloseMemHandle(g->p2p_bars[q]);
+    }
+    g->p2p_ipc[q] = false;
+    g->p2p_bufs[q][0] = g->p2p_bufs[q][1] = nullptr;
+    g->p2p_bars[q] = nullptr;
+  }
+}
+// the CUB scratch of the canonical pending-list sort, sized for n_cap keys
+// once (at create / growth, both collective): no allocation -- and no
+// implicit device synchronisation -- between the last collective of a
+// refine and its persistent round kernel (ranks may share a GPU)
+igk_status sort_scratch(igk_graph* g) {
+  size_t need = 0;
+  cub::DeviceRadixSort::SortKeys(nullptr, need, (const uint32_t*)g->d.psi[0], (uint32_t*)g->d.psi[1],
+                                 (int)std::min<long long>(g->d.n_cap, INT32_MAX), 0, g->d.idbits, g->stream);
+  if (need <= g->sort_tmp_cap) return IGK_OK;
+  if (g->sort_tmp) cudaFree(g->sort_tmp);
+  g->sort_tmp = nullptr;
+  g->sort_tmp_cap = 0;
+  CK(cudaMalloc(&g->sort_tmp, need));
+  g->sort_tmp_cap = need;
+  return IGK_OK;
+}
+
+igk_status p2p_setup(igk_graph* g) {
+  const int n = g->nranks, me = g->rank;
+  if (n > 8) return fail(g, IGK_EINVAL, "p2p: at most 8 ranks");
+  p2p_teardown(g);
+  long long sync1 = 0;
+  igk_status st = xp_sum_host(g, &sync1, 1);  // every rank closed its mappings of the old buffers
+  if (st != IGK_OK) return st;
+  if (g->p2p_mem) cudaFree(g->p2p_mem);
+  if (g->p2p_bar) cudaFree(g->p2p_bar);
+  g->p2p_mem = nullptr;
+  g->p2p_bar = nullptr;
+  const long long cap = g->d.n_cap;
+  CK(cudaMalloc(&g->p2p_mem, (size_t)cap * 2 * sizeof(int4)));
+  CK(cudaMalloc(&g->p2p_bar, 256));
+  CK(cudaMemsetAsync(g->p2p_mem, 0, (size_t)cap * 2 * sizeof(int4), g->stream));
+  CK(cudaMemsetAsync(g->p2p_bar, 0, 256, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  g->p2p_cap = cap;
+  g->p2p_rounds = 0;
+  std::vector<long long> blob((size_t)n * kBlob, 0);
+  long long* row = &blob[(size_t)me * kBlob];
+  row[0] = (long long)getpid();
+  row[1] = g->device;
+  row[2] = (long long)(uintptr_t)g->p2p_mem;
+  row[3] = (long long)(uintptr_t)g->p2p_bar;
+  cudaIpcMemHandle_t hm{}, hb{};  // for peers in other processes (not needed inside one process)
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+  if (cudaIpcGetMemHandle(&hm, g->p2p_mem) == cudaSuccess && cudaIpcGetMemHandle(&hb, g->p2p_bar) == cudaSuccess) {
+    row[20] = 1;
+    std::memcpy(&row[4], &hm, 64);
+    std::memcpy(&row[12], &hb, 64);
+  }
+  cudaGetLastError();
+  st = xp_sum_host(g, blob.data(), n * kBlob);  // every rank's row (disjoint: the sum is a gather)
+  if (st != IGK_OK) return st;
+  for (int q = 0; q < n; q++) {
+    const long long* r = &blob[(size_t)q * kBlob];
+    int4* mem = nullptr;
+    unsigned long long* bar = nullptr;
+    if (q == me) {
+      mem = g->p2p_mem;
+      bar = g->p2p_bar;
+    } else if (r[0] == (long long)getpid()) {  // same process: the pointers are valid here
+      mem = (int4*)(uintptr_t)r[2];
+      bar = (unsigned long long*)(uintptr_t)r[3];
+      if ((int)r[1] != g->device) {
+        cudaError_t e = cudaDeviceEnablePeerAccess((int)r[1], 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CK(e);
+        cudaGetLastError();
+      }
+    } else {  // another process: CUDA IPC (NVLink peer mapping across GPUs)
+      if (!r[20]) return fail(g, IGK_ENCCL, "p2p: a peer in another process exported no IPC handle");
+      cudaIpcMemHandle_t h1, h2;
+      std::memcpy(&h1, &r[4], 64);
+      std::memcpy(&h2, &r[12], 64);
+      void* p1 = nullptr;
+      void* p2 = nullptr;
+      CK(cudaIpcOpenMemHandle(&p1, h1, cudaIpcMemLazyEnablePeerAccess));
+      CK(cudaIpcOpenMemHandle(&p2, h2, cudaIpcMemLazyEnablePeerAccess));
+      mem = (int4*)p1;
+      bar = (unsigned long long*)p2;
+      g->p2p_ipc[q] = true;
+    }
+    g->p2p_bufs[q][0] = mem;
+    g->p2p_bufs[q][1] = mem + cap;
+    g->p2p_bars[q] = bar;
+  }
+  long long sync2 = 0;
+  return xp_sum_host(g, &sync2, 1);  // every rank mapped every peer before any kernel runs
 }
 
 igk_status launch_recount(igk_graph* g) {
@@ -563,6 +684,11 @@ igk_status grow_vertex_capacity(igk_graph* g, long long new_cap) {
   d.idbits = ib;
   CK(cudaStreamSynchronize(g->stream));
   g->n_grow++;
+  if (g->sharded) {
+    igk_status st = sort_scratch(g);
+    if (st != IGK_OK) return st;
+  }
+  if (g->p2p) return p2p_setup(g);  // the record buffers hold n_cap entries (collective: growth is)
   return IGK_OK;
 }
 
@@ -812,7 +938,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) && dalloc(g, &d.metav, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) && dalloc(g, &d.delta, N) &&
-            dalloc(g, &g->d_red, 259) && dalloc(g, &g->d_xp, 8);
+            dalloc(g, &g->d_red, 259) && dalloc(g, &g->d_xp, kXpWords);
   if (ok && sharded)  // sharded exchange buffers (bitmap words, restoration keys, round records)
     ok = dalloc(g, &d.bm, N / 64 + 2) && dalloc(g, &d.lossbuf, N) && dalloc(g, &d.recs, N);
   if (!ok) {
@@ -833,6 +959,8 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
       g->nccl = comm;
     }
   }
+  g->p2p = sharded && o.p2p;
+  g->ranks_per_device = o.ranks_per_device > 1 ? o.ranks_per_device : 1;
   if (cudaMallocHost(&g->h_ctl, sizeof(Ctl)) != cudaSuccess ||
       cudaHostAlloc(&g->h_map, sizeof(Ctl), cudaHostAllocMapped) != cudaSuccess ||
       cudaHostAlloc(&g->h_flag, 64, cudaHostAllocMapped) != cudaSuccess ||
@@ -974,6 +1102,21 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   g->split_b = kSplitB;
   if (const char* e = getenv("IGK_SPLIT_B")) g->split_b = atoll(e);
   g->epochA = next_epoch(g);
+  if (sharded && sort_scratch(g) != IGK_OK) {
+    igk_destroy(g);
+    return IGK_ENOMEM;
+  }
+  if (g->p2p) {
+    cudaFuncSetAttribute(k_rounds_p2p, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->smem_refine);
+    const int gp = coop_grid((const void*)k_rounds_p2p, g->smem_refine, 1, dv);
+    g->grid_p2p = std::max(1, gp / g->ranks_per_device);
+    const igk_status ps = p2p_setup(g);
+    if (ps != IGK_OK) {
+      t_create_err = "p2p set-up: " + g->err;
+      igk_destroy(g);
+      return ps;
+    }
+  }
   *out = g;
   return IGK_OK;
 }
@@ -1116,20 +1259,34 @@ static igk_status refine_sharded(igk_graph* g, igk_refine_stats* stats) {
   }
   const long long np = g->h_ctl->sh_np;
   if (np > 0) {  // the canonical pending list: psi[0] sorted by ID into psi[1]
-    size_t need = 0;
-    cub::DeviceRadixSort::SortKeys(nullptr, need, (const uint32_t*)d.psi[0], (uint32_t*)d.psi[1], (int)np, 0,
-                                   d.idbits, g->stream);
-    if (need > g->sort_tmp_cap) {
-      if (g->sort_tmp) cudaFree(g->sort_tmp);
-      g->sort_tmp = nullptr;
-      g->sort_tmp_cap = 0;
-      CK(cudaMalloc(&g->sort_tmp, need));
-      g->sort_tmp_cap = need;
-    }
+    size_t need = g->sort_tmp_cap;  // sized for n_cap keys at create / growth (sort_scratch)
     CK(cub::DeviceRadixSort::SortKeys(g->sort_tmp, need, (const uint32_t*)d.psi[0], (uint32_t*)d.psi[1], (int)np,
                                       0, d.idbits, g->stream));
     g->launches++;
     sh.np = np;
+    if (g->p2p) {  // NEXT-3: every round in one persistent kernel, records through peer memory
+      P2PArgs pa{};
+      pa.n = g->nranks;
+      pa.self = g->rank;
+      for (int q = 0; q < g->nranks; q++) {
+        pa.bufs[q][0] = g->p2p_bufs[q][0];
+        pa.bufs[q][1] = g->p2p_bufs[q][1];
+        pa.bars[q] = g->p2p_bars[q];
+      }
+      pa.bar_base = (unsigned long long)g->nranks * (unsigned long long)g->p2p_rounds;
+      pa.timeout = 4000000000ll;  // ~2 s at 1.9 GHz: a peer that never arrives is an error, not a hang
+      long long npv = np;
+      void* args[] = {(void*)&g->d, (void*)&ra, (void*)&npv, (void*)&pa};
+      CK(cudaLaunchCooperativeKernel((const void*)k_rounds_p2p, g->grid_p2p, kThreads, args, g->smem_refine,
+                                     g->stream));
+      g->launches++;
+      if ((st = sync_ctl(g, -1)) != IGK_OK) return st;
+      if (g->h_ctl->p2p_err) {
+        g->poisoned = true;
+        return fail(g, IGK_ENCCL, "p2p rounds: a peer never reached the device barrier");
+      }
+      g->p2p_rounds += g->h_ctl->rs_rounds_all;  // rounds_all counted from 0 by kShF0
+    } else
     for (long long r = 0; r <= np; r++) {  // <= |Psi| rounds (the minimum-ID pending vertex always moves)
       CK(cudaMemsetAsync(d.recs, 0, (size_t)np * 16, g->stream));
       if ((st = launch(kShGain)) != IGK_OK) return st;
@@ -1835,12 +1992,19 @@ int32_t igk_debug_phase_times(const igk_graph* g, int32_t which, int32_t* ids, i
   return n;
 }
 
-const char* igk_last_error(const igk_graph* g) { return g ? g->err.c_str() : "null handle"; }
+const char* igk_last_error(const igk_graph* g) {
+  return g ? g->err.c_str() : (t_create_err.empty() ? "null handle" : t_create_err.c_str());
+}
 
 void igk_destroy(igk_graph* g) {
   if (!g) return;
   DevGuard dev_guard(g->device);
   cudaStreamSynchronize(g->stream);
+  if (g->p2p) {
+    p2p_teardown(g);
+    if (g->p2p_mem) cudaFree(g->p2p_mem);
+    if (g->p2p_bar) cudaFree(g->p2p_bar);
+  }
   if (g->nccl && nccl_api()) nccl_api()->destroy((ncclComm_t)g->nccl);
   if (g->xp_host) cudaFreeHost(g->xp_host);
   if (g->sort_tmp) cudaFree(g->sort_tmp);

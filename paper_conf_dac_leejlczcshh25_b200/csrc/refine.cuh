@@ -848,8 +848,13 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     auto emit_move = [&](long long j, int u, int best, long long g, long long pwv, bool imbal) {
       int d0 = 255 - (int)min(g, 255ll);
       if (kSh) {  // the record at the vertex's canonical position; installed by every rank in kShFinish
-        d.recs[j] = make_int4(u + 1, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)),
-                              (int)g, (int)pwv);
+        const int4 rec = make_int4(u + 1, (int)(0x80000000u | ((unsigned)d0 << 8) | (unsigned)best | (imbal ? 1u << 30 : 0u)),
+                                   (int)g, (int)pwv);
+        if (d.p2p_n) {  // NEXT-3: straight into every rank's buffer (peer stores over NVLink)
+          for (int q = 0; q < d.p2p_n; q++) d.p2p_recs[q][j] = rec;
+        } else {
+          d.recs[j] = rec;
+        }
         return;
       }
       d.tgt[u] = (uint8_t)best;
@@ -1790,6 +1795,94 @@ __global__ void __launch_bounds__(kThreads) k_refine_sh(Dev d, RefineArgs a, Sha
   cg::grid_group grid = cg::this_grid();
   extern __shared__ __align__(16) unsigned char smem_raw[];
   refine_body<true>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh);
+}
+
+// ---------------------------------------------------------------------------
+// NEXT-3: all rounds of a sharded refine in ONE persistent kernel per rank.
+// Each round the owners store the move records of their selected vertices
+// (16 B each) directly into the round's record buffer of EVERY rank (peer
+// memory: NVLink P2P across GPUs, plain device memory for ranks sharing a
+// GPU), then the ranks meet at a device-side barrier (system-scope atomics
+// on every rank's counter, release / acquire fences) instead of a host
+// round trip + all-reduce; every rank then installs all records, takes the
+// same balanced prefix and applies it (the kShGain / kShFinish
+// logic of run_rounds).  Two buffers alternate by round parity: a rank that
+// zeroed its buffer after installing round r can only receive round r+2's
+// records after everyone passed round r+1's barrier.  A peer that never
+// arrives (bounded spin) sets Ctl::p2p_err and every rank stops.
+// ---------------------------------------------------------------------------
+struct P2PArgs {
+  int n, self;                      // ranks, this rank
+  int4* bufs[8][2];                 // every rank's two record buffers (by round parity)
+  unsigned long long* bars[8];      // every rank's barrier counter
+  unsigned long long bar_base;      // counter value before this refine's first round (n x rounds so far)
+  long long timeout;                // clock64 cycles a rank waits at the barrier before giving up
+};
+
+__global__ void __launch_bounds__(kThreads) k_rounds_p2p(Dev d, RefineArgs a, long long np, P2PArgs pa) {
+  cg::grid_group grid = cg::this_grid();
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  RefSmem& s = *reinterpret_cast<RefSmem*>(smem_raw);
+  Ctl* ctl = d.ctl;
+  const int k = d.k;
+  const long long c = cap_of(ldv(&ctl->W), a.e_ppm, k);
+  const int exact_shift_id = ((d.idbits + 7) / 8) * 8 - 8;
+  for (int p = threadIdx.x; p < 256; p += blockDim.x) {
+    s.acc[p] = 0;
+    s.sel.used[p] = 0;
+    s.sel.active[p] = 0;
+  }
+  for (int t = threadIdx.x; t < kWarps * 256; t += blockDim.x) (&s.wconn[0][0])[t] = 0;
+  __syncthreads();
+  long long scanned = 0, cut_acc = 0;
+  PhaseWork pw_;
+  RoundState rs;
+  rs.cur = 1;
+  rs.rounds = ldv(&ctl->rs_rounds);
+  rs.rounds_all = ldv(&ctl->rs_rounds_all);
+  rs.applied_tot = ldv(&ctl->rs_applied);
+  rs.deferred_tot = ldv(&ctl->rs_deferred);
+  ShardArgs sh{};
+  sh.np = np;
+  for (long long r = 0;; r++) {
+    const int par = (int)(r & 1);
+    Dev dr = d;
+    dr.recs = pa.bufs[pa.self][par];  // installed from here
+    dr.p2p_n = pa.n;
+    for (int q = 0; q < pa.n; q++) dr.p2p_recs[q] = pa.bufs[q][par];
+    sh.mode = kShGain;
+    run_rounds<true>(dr, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh, pw_);
+    __threadfence_system();  // this rank's record stores before its arrival
+    grid.sync();
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      for (int q = 0; q < pa.n; q++) atomicAdd_system(pa.bars[q], 1ull);
+      const unsigned long long target = pa.bar_base + (unsigned long long)pa.n * (unsigned long long)(r + 1);
+      const long long t0 = clock64();
+      int err = 0;
+      while (*(volatile unsigned long long*)pa.bars[pa.self] < target)
+        if (clock64() - t0 > pa.timeout) {
+          err = 1;
+          break;
+        }
+      __threadfence_system();  // the peers' records are visible before anyone installs
+      ctl->p2p_err = err;
+    }
+    grid.sync();
+    if (ldv(&ctl->p2p_err)) break;  // uniform
+    sh.mode = kShFinish;
+    run_rounds<true>(dr, a, s, grid, c, exact_shift_id, rs, scanned, cut_acc, sh, pw_);
+    rr_for(np, [&](long long j) { dr.recs[j] = make_int4(0, 0, 0, 0); });  // free for round r + 2
+    grid.sync();
+    if (ldv(&ctl->rs_pending) == 0) break;
+  }
+  block_atomic_add(&ctl->cut, cut_acc, s.red);
+  block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    ctl->rs_rounds = rs.rounds;
+    ctl->rs_rounds_all = rs.rounds_all;
+    ctl->rs_applied = rs.applied_tot;
+    ctl->rs_deferred = rs.deferred_tot;
+  }
 }
 
 }  // namespace igk

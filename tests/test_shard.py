@@ -254,3 +254,106 @@ def test_sharded_protocol_over_nccl_one_rank():
         assert P.apply(S.next(gi.MODE_MIX, 0.03), f"it{it}") == 0
         P.refine(f"it{it}")
         P.compare_state(f"it{it}", full_csr=(it == 5))
+
+
+# ---------------------------------------------------------------------------
+# NEXT-3: persistent P2P round kernel (records through peer memory, device
+# barrier).  N ranks as N threads of ONE process sharing the test GPU: each
+# rank's persistent kernel takes 1/N of the SMs so all are resident at once;
+# peers are plain device pointers (the same code maps CUDA IPC handles when
+# the ranks are processes on different GPUs).  The host collectives of the
+# pre-round phases go through an in-process transport.
+# ---------------------------------------------------------------------------
+class _ThreadComm:
+    """igk_comm for N threads of one process: all-reduce through a shared
+    numpy buffer and a barrier (test transport; the library calls it from
+    each rank's thread, ctypes holds the GIL only inside the callback)."""
+
+    def __init__(self, n):
+        import threading
+        import paper_conf_dac_leejlczcshh25_b200 as igk
+        self.n = n
+        self.bar = threading.Barrier(n)
+        self.slots = [None] * n
+        self.out = None
+        self.structs = []
+        self.cbs = []
+        for r in range(n):
+            cb = igk.ALLREDUCE_FN(lambda ctx, buf, count, dtype, op, r=r: self._ar(r, buf, count, dtype, op))
+            self.cbs.append(cb)
+            self.structs.append(igk.Comm(None, cb))
+
+    def _ar(self, r, buf, count, dtype, op):
+        try:
+            name, size = {0: ("int64", 8), 1: ("uint32", 4)}[dtype]
+            arr = np.ctypeslib.as_array((C.c_uint8 * (count * size)).from_address(buf)).view(name)
+            self.slots[r] = arr.astype(np.int64)
+            self.bar.wait()
+            if r == 0:
+                st = np.stack(self.slots)
+                self.out = st.sum(0) if op == 0 else (st.min(0) if op == 1 else st.max(0))
+            self.bar.wait()
+            arr[:] = self.out.astype(name)
+            self.bar.wait()
+            return 0
+        except Exception:
+            import traceback
+            traceback.print_exc()
+            return -1
+
+
+class _CommRef:
+    def __init__(self, struct):
+        self.struct = struct
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 3])
+def test_p2p_rounds_match_oracle(world):
+    import threading
+    import igk_inputs as gi
+    import oracle
+    import paper_conf_dac_leejlczcshh25_b200 as igk
+    g = gi.make_graph(10_000, 64, gi.graph_seed(1))
+    part, _ = gi.metis_partition(g, 4)
+    S = gi.Stream(g, 82)
+    batches = [S.next(gi.MODE_MIX, 0.03) for _ in range(8)]
+    O = oracle.Oracle(g.xadj, g.adjncy, 4, 0.03, part)
+    O.refine()
+    expect = []
+    for b in batches:
+        assert O.apply(b)[0] == 0
+        _, so = O.refine()
+        expect.append((O.partition().tobytes(), so["cut"], so["rounds"], so["moves_applied"]))
+    tc = _ThreadComm(world)
+    res = [None] * world
+    err = [None] * world
+
+    def run(r):
+        try:
+            import torch
+            stream = torch.cuda.Stream()  # one non-blocking stream per rank: the persistent kernels run side by side
+            G = igk.IGKGraph(g.xadj, g.adjncy, 4, 0.03, part, nranks=world, rank=r, stream=stream.cuda_stream,
+                             comm=_CommRef(tc.structs[r]), p2p=True, ranks_per_device=world, check=True)
+            G.refine()
+            out = []
+            for b in batches:
+                s, _, bad = G.apply(b)
+                assert s == 0, (s, bad)
+                _, st = G.refine()
+                out.append((G.partition().tobytes(), G.cut(), st["rounds"], st["moves_applied"]))
+            res[r] = (out, G.debug_paths())
+            G.close()
+        except Exception as e:  # reported by the main thread
+            import traceback
+            err[r] = traceback.format_exc()
+
+    ts = [threading.Thread(target=run, args=(r,)) for r in range(world)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout=600)
+    assert not any(err), err
+    for r in range(world):
+        for it, (got, exp) in enumerate(zip(res[r][0], expect)):
+            assert got == exp, (r, it)
