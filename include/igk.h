@@ -107,6 +107,12 @@ typedef struct {
    * SMs so all of them are resident at once. */
   int32_t p2p;
   int32_t ranks_per_device;
+  /* wide_weights = 1: vertex / edge weights up to INT32_MAX with the total
+   * vertex weight and the total edge weight <= INT32_MAX (every per-vertex
+   * sum of the refine then stays exact in 32 bits) -- the coarse graphs of
+   * the full partitioner (igk_fgp_partition).  Such a handle refines but
+   * accepts no modifiers (IGK_EINVAL); single GPU only. */
+  int32_t wide_weights;
 } igk_options;
 
 typedef struct {
@@ -204,6 +210,23 @@ igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t cou
 igk_status igk_stage_batch(igk_graph* g, const igk_modifier* mods, int64_t count);
 igk_status igk_step_begin(igk_graph* g);
 igk_status igk_step_end(igk_graph* g, igk_refine_stats* stats, int64_t* first_new_id, int64_t* bad_index);
+
+/* NEXT-2: full partitioning of a CSR graph on the GPU (IGK-FGP v1, DESIGN.md
+ * 4 readings F1-F6): G-kway-style union-find coarsening with the paper's
+ * constrained grouping (vertices of a subset sorted by their join
+ * iteration and split into groups of group_size, the paper's s = 6), stop
+ * below 35 k vertices or when fewer than 90% of the vertices could be
+ * coarsened, a greedy initial partition of the coarsest graph, and at
+ * every level the projection + global boundary refinement (igk_refine_global
+ * on a wide-weight handle, repeated while it lowers the cut, <= 8 passes).
+ * Inputs as igk_create (host CSR; weights up to INT32_MAX with totals <=
+ * INT32_MAX); opt: device / stream (NULL = defaults).  part_out[n] gets the
+ * partition; level_n (nullable, >= 33 entries) the vertices per level;
+ * *nlevels (nullable) the number of levels.  IGK_EINVAL on invalid input;
+ * the reason of a failure is in igk_last_error(NULL). */
+igk_status igk_fgp_partition(const igk_options* opt, int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                             const int32_t* vwgt, const int32_t* adjwgt, int32_t k, double epsilon,
+                             int32_t group_size, int32_t* part_out, int64_t* level_n, int32_t* nlevels);
 
 /* NCCL unique id for sharded handles (call on ONE rank, share the 128
  * bytes with the others, pass as igk_options.nccl_id).  NCCL is loaded at

@@ -23,9 +23,9 @@ OK, EINVAL, ENOMEM, WIMBALANCED = 0, 1, 2, 6
 
 
 def build(force: bool = False) -> str:
-    src = os.path.join(_HERE, "igk_oracle.c")
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
-        subprocess.check_call(["gcc", "-O2", "-Wall", "-fPIC", "-shared", src, "-o", _SO])
+    srcs = [os.path.join(_HERE, f) for f in ("igk_oracle.c", "igk_fgp.c", "igk_oracle.h")]
+    if force or not os.path.exists(_SO) or any(os.path.getmtime(_SO) < os.path.getmtime(f) for f in srcs):
+        subprocess.check_call(["gcc", "-O2", "-Wall", "-fPIC", "-shared", *srcs[:2], "-o", _SO])
     return _SO
 
 
@@ -78,12 +78,59 @@ def lib():
         L.ora_trace_moves.restype = C.c_int64
         L.ora_trace_moves.argtypes = [P, i64p, C.c_int64]
         L.ora_trace_sets.argtypes = [P, C.c_void_p, C.c_void_p, C.c_void_p]
+        L.ora_fgp.restype = C.c_int
+        L.ora_fgp.argtypes = [C.c_int64, i64p, i32p, i32p, i32p, C.c_int32, C.c_double, C.c_int32, i32p, i64p,
+                              C.c_int64]
+        L.ora_fgp_coarsen_step.restype = C.c_int64
+        L.ora_fgp_coarsen_step.argtypes = [C.c_int64, i64p, i32p, i32p, C.c_int32, i32p, i32p, i32p, i32p,
+                                           C.POINTER(C.c_int64)]
+        L.ora_fgp_set_passes.argtypes = [C.c_int]
+        L.ora_fgp_set_init.argtypes = [C.c_int]
         _lib = L
     return _lib
 
 
 def _p(a, ct):
     return None if a is None else a.ctypes.data_as(C.POINTER(ct))
+
+
+def fgp(xadj, adjncy, k, eps, vwgt=None, adjwgt=None, group_size=6):
+    """IGK-FGP v1 full partition (NEXT-2).  Returns (part, [n per level])."""
+    xadj = np.ascontiguousarray(xadj, dtype=np.int64)
+    adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
+    vwgt = None if vwgt is None else np.ascontiguousarray(vwgt, dtype=np.int32)
+    adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
+    n = len(xadj) - 1
+    part = np.zeros(max(n, 1), np.int32)
+    lv = np.zeros(40, np.int64)
+    r = lib().ora_fgp(n, _p(xadj, C.c_int64), _p(adjncy, C.c_int32), _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32),
+                      k, eps, group_size, _p(part, C.c_int32), _p(lv, C.c_int64), 40)
+    if r < 1:
+        raise ValueError(f"ora_fgp failed ({r})")
+    return part[:n], lv[:r].tolist()
+
+
+def fgp_set_passes(passes: int) -> None:
+    """test-only: refinement passes per FGP level (default 8)"""
+    lib().ora_fgp_set_passes(passes)
+
+
+def fgp_set_init(mode: int) -> None:
+    """test-only: FGP initial partition, 0 = BFS growing (default), 1 = ID blocks"""
+    lib().ora_fgp_set_init(mode)
+
+
+def fgp_coarsen_step(xadj, adjncy, adjwgt=None, group_size=6):
+    """one coarsening step: (sel, root, label, cmap, n_groups, coarsenable)"""
+    xadj = np.ascontiguousarray(xadj, dtype=np.int64)
+    adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
+    adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
+    n = len(xadj) - 1
+    out = [np.zeros(max(n, 1), np.int32) for _ in range(4)]
+    co = C.c_int64(0)
+    ng = lib().ora_fgp_coarsen_step(n, _p(xadj, C.c_int64), _p(adjncy, C.c_int32), _p(adjwgt, C.c_int32),
+                                    group_size, *[_p(a, C.c_int32) for a in out], C.byref(co))
+    return tuple(a[:n] for a in out) + (int(ng), int(co.value))
 
 
 def cap(W: int, eps: float, k: int) -> int:

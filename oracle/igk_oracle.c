@@ -51,6 +51,7 @@ struct ora_graph {
   uint8_t* inF; /* vertices that entered Psi since the last refine (I4) */
   int32_t* prev_part; /* parts at the start of the last refine (I4) */
   int last_imbalanced;
+  int wide;             /* NEXT-2 coarse level: wide weights, no modifiers */
   int64_t last_cap;
   /* trace of the last refine */
   int64_t ntrace, trace_cap;
@@ -169,9 +170,14 @@ static int cmp_pair(const void* a, const void* b) {
 /* ------------------------------------------------------------------ */
 /* create                                                              */
 /* ------------------------------------------------------------------ */
-ora_graph* ora_create(int64_t n, const int64_t* xadj, const int32_t* adjncy,
-                      const int32_t* vwgt, const int32_t* adjwgt, int32_t k,
-                      double epsilon, const int32_t* init_part, int* status) {
+/* wide = 1 (NEXT-2 coarse levels): vertex / edge weights up to INT32_MAX
+ * with the totals bounded by INT32_MAX (so every per-vertex sum of the
+ * method stays exact in 32 bits on the product side); such a graph accepts
+ * no modifiers */
+ora_graph* ora_create_ex(int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                         const int32_t* vwgt, const int32_t* adjwgt, int32_t k,
+                         double epsilon, const int32_t* init_part, int wide, int* status) {
+  const int64_t vw_max = wide ? INT32_MAX : LIM_VW_MAX, ew_max = wide ? INT32_MAX : LIM_EW_MAX;
   *status = ORA_EINVAL;
   if (n < 0 || n > LIM_N_MAX || k < 2 || k > LIM_K_MAX || !(epsilon > 0.0) ||
       !(epsilon <= 1.0) || (n > 0 && (!xadj || !init_part)))
@@ -180,7 +186,7 @@ ora_graph* ora_create(int64_t n, const int64_t* xadj, const int32_t* adjncy,
   for (int64_t u = 0; u < n; u++) {
     if (xadj[u + 1] < xadj[u]) return NULL;
     if (init_part[u] < 0 || init_part[u] >= k) return NULL;
-    if (vwgt && (vwgt[u] < 1 || vwgt[u] > LIM_VW_MAX)) return NULL;
+    if (vwgt && (vwgt[u] < 1 || vwgt[u] > vw_max)) return NULL;
     if (xadj[u + 1] - xadj[u] > LIM_DEG_MAX) return NULL;
   }
   ora_graph* g = (ora_graph*)xcalloc(1, sizeof(ora_graph));
@@ -198,7 +204,7 @@ ora_graph* ora_create(int64_t n, const int64_t* xadj, const int32_t* adjncy,
     for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
       int32_t x = adjncy[j];
       int32_t w = adjwgt ? adjwgt[j] : 1;
-      if (x < 0 || x >= n || x == u || w < 1 || w > LIM_EW_MAX) {
+      if (x < 0 || x >= n || x == u || w < 1 || w > ew_max) {
         ora_destroy(g);
         return NULL;
       }
@@ -245,9 +251,24 @@ ora_graph* ora_create(int64_t n, const int64_t* xadj, const int32_t* adjncy,
     g->W += g->vw[u];
     g->Wp[g->part[u]] += g->vw[u];
   }
+  if (wide) {
+    int64_t ew = 0;
+    for (int64_t j = 0; j < m2; j++) ew += adjwgt ? adjwgt[j] : 1;
+    if (g->W > INT32_MAX || ew / 2 > INT32_MAX) {
+      ora_destroy(g);
+      return NULL;
+    }
+    g->wide = 1;
+  }
   g->last_cap = cap_of(g->W, g->e_ppm, k);
   *status = ORA_OK;
   return g;
+}
+
+ora_graph* ora_create(int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                      const int32_t* vwgt, const int32_t* adjwgt, int32_t k,
+                      double epsilon, const int32_t* init_part, int* status) {
+  return ora_create_ex(n, xadj, adjncy, vwgt, adjwgt, k, epsilon, init_part, 0, status);
 }
 
 void ora_destroy(ora_graph* g) {
@@ -297,7 +318,7 @@ int ora_apply(ora_graph* g, const int32_t* mods, int64_t count, int64_t* first_n
               int64_t* bad_index) {
   if (first_new_id) *first_new_id = g->n;
   if (bad_index) *bad_index = -1;
-  if (count < 0) return ORA_EINVAL;
+  if (count < 0 || g->wide) return ORA_EINVAL;
   if (count == 0) return ORA_OK;
   const int64_t n = g->n;
   int64_t n_ins = 0;

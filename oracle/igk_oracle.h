@@ -98,6 +98,31 @@ void ora_debug_set_frontier(ora_graph* g, int64_t v, int f);
 void ora_debug_add_half_edge(ora_graph* g, int64_t u, int32_t x, int32_t w);
 void ora_debug_set_edge_weight(ora_graph* g, int64_t u, int32_t x, int32_t w);
 
+/* wide = 1: coarse-level graphs of the full partitioner (vertex / edge
+ * weights up to INT32_MAX, totals <= INT32_MAX, no modifiers accepted) */
+ora_graph* ora_create_ex(int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                         const int32_t* vwgt, const int32_t* adjwgt, int32_t k,
+                         double epsilon, const int32_t* init_part, int wide, int* status);
+
+/* NEXT-2: IGK-FGP v1 full partitioning (igk_fgp.c):
+ * constrained coarsening (group size s), greedy initial partition of the
+ * coarsest graph, projection + global boundary refinement per level.
+ * part_out[n]; level_n[l] = vertices of level l (up to maxlev entries).
+ * Returns the number of levels (>= 1) or -ORA_EINVAL. */
+int ora_fgp(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t* vwgt,
+            const int32_t* adjwgt, int32_t k, double epsilon, int32_t group_size,
+            int32_t* part_out, int64_t* level_n, int64_t maxlev);
+/* one coarsening step (selection, join labels, groups) of a CSR graph:
+ * returns the number of groups; sel/root/label/cmap per vertex */
+/* test-only knobs of ora_fgp: refinement passes per level (default 8; 0 =
+ * none, the projected initial partition) and the initial partition (0 = BFS
+ * graph growing, the default; 1 = contiguous ID blocks) */
+void ora_fgp_set_passes(int passes);
+void ora_fgp_set_init(int mode);
+int64_t ora_fgp_coarsen_step(int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                             const int32_t* adjwgt, int32_t group_size, int32_t* sel,
+                             int32_t* root, int32_t* label, int32_t* cmap, int64_t* coarsenable);
+
 /* step-level hooks used by the pinning tests (tests/test_oracle_*.py) */
 int64_t ora_cap(int64_t W, double epsilon, int32_t k);
 /* last refine trace: per round |S_r| and L_r (up to maxr rounds) */

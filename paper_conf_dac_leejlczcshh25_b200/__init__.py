@@ -29,7 +29,7 @@ SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "i
            "igk_step_end",
            "igk_partition", "igk_partition_delta", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
-           "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work",
+           "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work", "igk_fgp_partition",
            "igk_last_error", "igk_destroy"]
 
 
@@ -52,7 +52,8 @@ class Options(C.Structure):
                 ("max_slots", C.c_int64), ("slack_min", C.c_int32), ("validate", C.c_int32),
                 ("check_invariants", C.c_int32), ("blocks_per_sm", C.c_int32),
                 ("nranks", C.c_int32), ("rank", C.c_int32), ("nccl_id", C.c_void_p),
-                ("comm", C.POINTER(Comm)), ("p2p", C.c_int32), ("ranks_per_device", C.c_int32)]
+                ("comm", C.POINTER(Comm)), ("p2p", C.c_int32), ("ranks_per_device", C.c_int32),
+                ("wide_weights", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -170,6 +171,9 @@ def lib():
         L.igk_debug_phase_times.argtypes = [P, C.c_int32, i32p, i64p, C.c_int32]
         L.igk_debug_arrivals.restype = C.c_int32
         L.igk_debug_arrivals.argtypes = [P, C.c_int32, i64p, C.c_int32]
+        L.igk_fgp_partition.restype = C.c_int
+        L.igk_fgp_partition.argtypes = [C.POINTER(Options), i64, i64p, i32p, i32p, i32p, i32, C.c_double, i32,
+                                        i32p, i64p, i32p]
         L.igk_last_error.restype = C.c_char_p
         L.igk_last_error.argtypes = [P]
         L.igk_destroy.restype = None
@@ -191,12 +195,35 @@ def nccl_unique_id() -> bytes:
     return buf.raw
 
 
+def fgp_partition(xadj, adjncy, k, eps, vwgt=None, adjwgt=None, group_size=6, device=0, stream=None):
+    """Full k-way partition on the GPU (igk_fgp_partition, IGK-FGP v1).
+
+    Returns (part int32[n], level sizes list)."""
+    xadj = np.ascontiguousarray(xadj, dtype=np.int64)
+    adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
+    vwgt = None if vwgt is None else np.ascontiguousarray(vwgt, dtype=np.int32)
+    adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
+    n = len(xadj) - 1
+    o = Options()
+    o.device = device
+    o.stream = stream or 0
+    part = np.empty(max(n, 1), np.int32)
+    lv = np.zeros(40, np.int64)
+    nl = C.c_int32(0)
+    s = lib().igk_fgp_partition(C.byref(o), n, _p(xadj, C.c_int64), _p(adjncy, C.c_int32), _p(vwgt, C.c_int32),
+                                _p(adjwgt, C.c_int32), k, eps, group_size, _p(part, C.c_int32),
+                                _p(lv, C.c_int64), C.byref(nl))
+    if s != OK:
+        raise IGKError(s, (lib().igk_last_error(None) or b"").decode())
+    return part[:n], [int(x) for x in lv[:nl.value]]
+
+
 class IGKGraph:
     """One GPU-resident graph + k-way partition (igk_create)."""
 
     def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, device=0, stream=None,
                  max_vertices=0, max_slots=0, slack_min=0, check=False, blocks_per_sm=0,
-                 nranks=1, rank=0, nccl_id: bytes | None = None, comm=None, p2p=False, ranks_per_device=1):
+                 nranks=1, rank=0, nccl_id: bytes | None = None, comm=None, p2p=False, ranks_per_device=1, wide_weights=False):
         """nranks > 1: rank `rank` of a vertex-range sharded graph (collective
         calls; every rank passes the same graph and batches).  Transport: NCCL
         from `nccl_id` (nccl_unique_id() on one rank, shared), else `comm`."""
@@ -210,7 +237,8 @@ class IGKGraph:
         self._comm = comm  # keeps the callback alive as long as the handle
         o = Options(device, stream or None, max_vertices, max_slots, slack_min, 1, int(check), blocks_per_sm,
                     int(nranks), int(rank), None if self._id is None else C.cast(self._id, C.c_void_p),
-                    None if comm is None else C.pointer(comm.struct), int(bool(p2p)), int(ranks_per_device))
+                    None if comm is None else C.pointer(comm.struct), int(bool(p2p)), int(ranks_per_device),
+                    int(bool(wide_weights)))
         h = C.c_void_p()
         s = L.igk_create(C.byref(o), len(xadj) - 1, _p(xadj, C.c_int64), _p(adjncy, C.c_int32),
                          _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(h))

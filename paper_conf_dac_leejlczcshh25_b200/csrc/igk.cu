@@ -22,6 +22,7 @@
 #include "../../include/igk.h"
 #include "apply.cuh"
 #include "common.cuh"
+#include "fgp.cuh"
 #include "recount.cuh"
 #include "refine.cuh"
 #include "step.cuh"
@@ -266,6 +267,7 @@ struct igk_graph {
   long long n_fused = 0;     // igk_step launches as one k_step
   long long n_notice_fallback = 0;  // fast-path steps that fell back to the copy + sync
   // sharding (igk_options.nranks > 1)
+  bool wide = false;           // wide-weight handle (NEXT-2 coarse levels): refine only, no modifiers
   int nranks = 1, rank = 0;
   bool sharded = false;        // the sharded protocol (nranks > 1, or a transport given for one rank)
   igk_comm comm{};             // host-callback transport (when no NCCL communicator)
@@ -776,13 +778,13 @@ igk_status compact_slab(igk_graph* g, long long extra) {
 // range, symmetric with equal weights) and the twin of every entry: the
 // position of u in row x for the entry u -> x
 bool csr_twins(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t* adjwgt,
-               std::vector<int32_t>& twin_pos) {
+               std::vector<int32_t>& twin_pos, long long ew_max = kEwMax) {
   const long long m2 = n > 0 ? xadj[n] : 0;
   std::vector<std::pair<int32_t, int32_t>> rows((size_t)m2);
   for (int64_t u = 0; u < n; u++) {
     for (int64_t j = xadj[u]; j < xadj[u + 1]; j++) {
       int32_t x = adjncy[j], w = adjwgt ? adjwgt[j] : 1;
-      if (x < 0 || x >= n || x == u || w < 1 || w > kEwMax) return false;
+      if (x < 0 || x >= n || x == u || w < 1 || w > ew_max) return false;
       rows[j] = {x, (int32_t)(j - xadj[u])};
     }
     std::sort(rows.begin() + xadj[u], rows.begin() + xadj[u + 1]);
@@ -825,10 +827,17 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   for (int64_t u = 0; u < n; u++) {
     if (xadj[u + 1] < xadj[u] || xadj[u + 1] - xadj[u] > kDegMax) return IGK_EINVAL;
     if (init_part[u] < 0 || init_part[u] >= k) return IGK_EINVAL;
-    if (vwgt && (vwgt[u] < 1 || vwgt[u] > kVwMax)) return IGK_EINVAL;
+    if (vwgt && (vwgt[u] < 1 || (!o.wide_weights && vwgt[u] > kVwMax))) return IGK_EINVAL;
   }
+  const long long ew_max = o.wide_weights ? INT32_MAX : kEwMax;
   std::vector<int32_t> twin_pos;
-  if (!csr_twins(n, xadj, adjncy, adjwgt, twin_pos)) return IGK_EINVAL;
+  if (!csr_twins(n, xadj, adjncy, adjwgt, twin_pos, ew_max)) return IGK_EINVAL;
+  if (o.wide_weights) {  // every per-vertex sum of the refine must stay exact in 32 bits
+    long long tv = 0, te = 0;
+    for (int64_t u = 0; u < n; u++) tv += vwgt ? vwgt[u] : 1;
+    for (int64_t j = 0; j < (n > 0 ? xadj[n] : 0); j++) te += adjwgt ? adjwgt[j] : 1;
+    if (tv > INT32_MAX || te / 2 > INT32_MAX || sharded) return IGK_EINVAL;
+  }
   // sharded: keep the entries u -> x with owner(u) == rank or owner(x) ==
   // rank (own vertices in full + the ghost prefixes pointing at them); the
   // condition is symmetric, so the kept CSR is again symmetric
@@ -849,10 +858,11 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     xadj = fx.data();
     adjncy = fa.data();
     if (adjwgt) adjwgt = fw.data();
-    if (!csr_twins(n, xadj, adjncy, adjwgt, twin_pos)) return IGK_EINVAL;
+    if (!csr_twins(n, xadj, adjncy, adjwgt, twin_pos, ew_max)) return IGK_EINVAL;
   }
   const long long m2 = n > 0 ? xadj[n] : 0;
   igk_graph* g = new igk_graph();
+  g->wide = o.wide_weights != 0;
   g->nranks = nranks;
   g->rank = nranks > 1 ? o.rank : 0;
   g->sharded = sharded;
@@ -1368,6 +1378,7 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   if (count == 0) return IGK_OK;
+  if (g->wide) return fail(g, IGK_EINVAL, "wide-weight handles accept no modifiers");
   if (g->sharded) return apply_dev_sharded(g, dm, count, bad_index);
   for (int attempt = 0;; attempt++) {
     igk_status st = launch_apply(g, dm, count);
@@ -1502,6 +1513,7 @@ static igk_status step_dev(igk_graph* g, const int4* dm, int64_t count, igk_refi
   if (bad_index) *bad_index = -1;
   if (first_new_id) *first_new_id = g->h_ctl->n_total;
   igk_status st;
+  if (g->wide && count > 0) return fail(g, IGK_EINVAL, "wide-weight handles accept no modifiers");
   if (g->sharded) {  // sharded: the collective apply, then the collective refine
     st = apply_dev(g, dm, count, first_new_id, bad_index);
     if (st != IGK_OK) return st;
@@ -1642,6 +1654,277 @@ igk_status igk_step_device(igk_graph* g, const igk_modifier* d_mods, int64_t cou
   ENTRY(g, "igk_step_device");
   if (count < 0 || (count > 0 && !d_mods)) return fail(g, IGK_EINVAL, "bad batch pointer/count");
   return step_dev(g, (const int4*)d_mods, count, stats, first_new_id, bad_index);
+}
+
+// ---------------------------------------------------------------------------
+// NEXT-2: IGK-FGP v1 full partitioning (fgp.cuh; readings F1-F6)
+// ---------------------------------------------------------------------------
+}  // extern "C"
+namespace {
+struct FgpLevel {
+  long long n = 0, m2 = 0;
+  int64_t* xadj = nullptr;
+  int32_t *adj = nullptr, *w = nullptr, *vw = nullptr;
+  int32_t* cmap = nullptr;  // vertex -> coarse vertex of the next level
+};
+struct DevBuf {  // frees its device allocations on scope exit
+  std::vector<void*> ps;
+  template <class T>
+  T* get(size_t n) {
+    void* p = nullptr;
+    if (cudaMalloc(&p, std::max<size_t>(n, 1) * sizeof(T)) != cudaSuccess) return nullptr;
+    ps.push_back(p);
+    return (T*)p;
+  }
+  ~DevBuf() {
+    for (void* p : ps) cudaFree(p);
+  }
+};
+
+// one handle per level (wide weights), the global boundary refinement
+// repeated while it lowers the cut (<= kFgpPasses), the refined labels out
+constexpr int kFgpPasses = 8;
+igk_status fgp_refine_level(const igk_options& o, const FgpLevel& L, int k, double eps, std::vector<int32_t>& part,
+                            std::string& err) {
+  std::vector<int64_t> xa(L.n + 1);
+  std::vector<int32_t> aj(std::max<long long>(L.m2, 1)), ww(std::max<long long>(L.m2, 1)), vw(std::max<long long>(L.n, 1));
+  cudaStream_t s = (cudaStream_t)o.stream;
+  if (cudaMemcpyAsync(xa.data(), L.xadj, (L.n + 1) * 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      (L.m2 && cudaMemcpyAsync(aj.data(), L.adj, L.m2 * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess) ||
+      (L.m2 && cudaMemcpyAsync(ww.data(), L.w, L.m2 * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess) ||
+      cudaMemcpyAsync(vw.data(), L.vw, L.n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess) {
+    err = "fgp: level read-back failed";
+    return IGK_ECUDA;
+  }
+  igk_options lo = o;
+  lo.wide_weights = 1;
+  lo.check_invariants = 0;
+  lo.nranks = 0;
+  lo.nccl_id = nullptr;
+  lo.comm = nullptr;
+  lo.p2p = 0;
+  igk_graph* h = nullptr;
+  igk_status st = igk_create(&lo, L.n, xa.data(), aj.data(), vw.data(), ww.data(), k, eps, part.data(), &h);
+  if (st != IGK_OK) {
+    err = std::string("fgp: level handle: ") + igk_last_error(nullptr);
+    return st;
+  }
+  long long prev = -1;
+  for (int p = 0; p < kFgpPasses; p++) {
+    igk_refine_stats rs{};
+    st = igk_refine_global(h, &rs);
+    if (st != IGK_OK && st != IGK_WIMBALANCED) break;
+    st = IGK_OK;
+    if (prev >= 0 && rs.cut >= prev) break;
+    prev = rs.cut;
+  }
+  if (st == IGK_OK) st = igk_partition(h, part.data(), (int64_t)part.size(), nullptr);
+  if (st != IGK_OK) err = std::string("fgp: level refine: ") + igk_last_error(h);
+  igk_destroy(h);
+  return st;
+}
+}  // namespace
+extern "C" {
+
+igk_status igk_fgp_partition(const igk_options* opt, int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                             const int32_t* vwgt, const int32_t* adjwgt, int32_t k, double epsilon,
+                             int32_t group_size, int32_t* part_out, int64_t* level_n, int32_t* nlevels) {
+  if (n < 1 || !xadj || !part_out || k < 2 || k > kMaxK || group_size < 2 || !(epsilon > 0.0) ||
+      !(epsilon <= 1.0) || n > kNMax)
+    return IGK_EINVAL;
+  igk_options o{};
+  if (opt) o = *opt;
+  DevGuard dev_guard(o.device);
+  NvtxRange nv("igk_fgp_partition");
+  std::vector<int32_t> twin_pos;
+  if (xadj[0] != 0 || !csr_twins(n, xadj, adjncy, adjwgt, twin_pos, INT32_MAX)) return IGK_EINVAL;
+  std::vector<int32_t>().swap(twin_pos);
+  cudaStream_t s = (cudaStream_t)o.stream;
+  DevBuf mem;
+  const int kMaxLv = 32;
+  std::vector<FgpLevel> L(1);
+  const long long m2 = xadj[n];
+  L[0].n = n;
+  L[0].m2 = m2;
+  L[0].xadj = mem.get<int64_t>(n + 1);
+  L[0].adj = mem.get<int32_t>(m2);
+  L[0].w = mem.get<int32_t>(m2);
+  L[0].vw = mem.get<int32_t>(n);
+  if (!L[0].xadj || !L[0].adj || !L[0].w || !L[0].vw) return IGK_ENOMEM;
+  {
+    std::vector<int32_t> w1, v1;
+    if (!adjwgt) w1.assign((size_t)std::max<long long>(m2, 1), 1);
+    if (!vwgt) v1.assign((size_t)n, 1);
+    if (cudaMemcpyAsync(L[0].xadj, xadj, (n + 1) * 8, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        (m2 && cudaMemcpyAsync(L[0].adj, adjncy, m2 * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) ||
+        (m2 && cudaMemcpyAsync(L[0].w, adjwgt ? adjwgt : w1.data(), m2 * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) ||
+        cudaMemcpyAsync(L[0].vw, vwgt ? vwgt : v1.data(), n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return IGK_ECUDA;
+  }
+  int* d_cnt = mem.get<int>(4);
+  unsigned long long* d_ecnt = mem.get<unsigned long long>(1);
+  if (!d_cnt || !d_ecnt) return IGK_ENOMEM;
+  auto fail_cuda = [&]() { return IGK_ECUDA; };
+  const int grid = 1184, blk = 256;
+  // ---- coarsening (readings F1-F4) ----
+  while ((int)L.size() - 1 < kMaxLv && L.back().n >= 35ll * k) {
+    FgpLevel& G = L.back();
+    const long long nl = G.n;
+    int32_t* sel = mem.get<int32_t>(nl);
+    int32_t* P = mem.get<int32_t>(nl);
+    int32_t* Q = mem.get<int32_t>(nl);
+    int32_t* label = mem.get<int32_t>(nl);
+    unsigned long long* key = mem.get<unsigned long long>(nl);
+    unsigned long long* skey = mem.get<unsigned long long>(nl);
+    int32_t* val = mem.get<int32_t>(nl);
+    int32_t* sval = mem.get<int32_t>(nl);
+    long long* mark = mem.get<long long>(nl);
+    long long* segstart = mem.get<long long>(nl);
+    int32_t* flag = mem.get<int32_t>(nl);
+    int32_t* gid = mem.get<int32_t>(nl);
+    int32_t* cmap = mem.get<int32_t>(nl);
+    if (!sel || !P || !Q || !label || !key || !skey || !val || !sval || !mark || !segstart || !flag || !gid || !cmap)
+      return IGK_ENOMEM;
+    k_fgp_select<<<grid, blk, 0, s>>>(nl, G.xadj, G.adj, G.w, sel);
+    cudaMemsetAsync(d_cnt, 0, 16, s);
+    k_fgp_roots<<<grid, blk, 0, s>>>(nl, sel, P, label, d_cnt);
+    int left = 0;
+    if (cudaMemcpyAsync(&left, d_cnt, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_cuda();
+    for (int t = 1; left > 0 && t < 64; t++) {  // synchronous pointer jumping (F2)
+      cudaMemsetAsync(d_cnt, 0, 4, s);
+      k_fgp_jump<<<grid, blk, 0, s>>>(nl, P, Q, label, t, d_cnt);
+      std::swap(P, Q);
+      if (cudaMemcpyAsync(&left, d_cnt, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+          cudaStreamSynchronize(s) != cudaSuccess)
+        return fail_cuda();
+    }
+    // (root, label) stable radix sort of the vertex IDs (F3)
+    k_fgp_keys<<<grid, blk, 0, s>>>(nl, P, label, key, val);
+    int ib = 1;
+    while ((1ll << ib) < nl) ib++;
+    size_t tb = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, tb, key, skey, val, sval, (int)nl, 0, ib + 8, s);
+    void* tmp = mem.get<char>(tb);
+    if (!tmp) return IGK_ENOMEM;
+    cub::DeviceRadixSort::SortPairs(tmp, tb, key, skey, val, sval, (int)nl, 0, ib + 8, s);
+    k_fgp_segmark<<<grid, blk, 0, s>>>(nl, skey, mark);
+    size_t tb2 = 0;
+    cub::DeviceScan::InclusiveScan(nullptr, tb2, mark, segstart, cuda::maximum<>(), (int)nl, s);
+    void* tmp2 = mem.get<char>(tb2);
+    if (!tmp2) return IGK_ENOMEM;
+    cub::DeviceScan::InclusiveScan(tmp2, tb2, mark, segstart, cuda::maximum<>(), (int)nl, s);
+    k_fgp_groups<<<grid, blk, 0, s>>>(nl, segstart, group_size, flag);
+    size_t tb3 = 0;  // gid[i] = the number of group starts up to i (group index + 1)
+    cub::DeviceScan::InclusiveSum(nullptr, tb3, flag, gid, (int)nl, s);
+    void* tmp3 = mem.get<char>(tb3);
+    if (!tmp3) return IGK_ENOMEM;
+    cub::DeviceScan::InclusiveSum(tmp3, tb3, flag, gid, (int)nl, s);
+    k_fgp_cmap<<<grid, blk, 0, s>>>(nl, flag, gid, sval, cmap, d_cnt + 1);
+    int hv[2] = {0, 0};
+    int lastgid = 0;
+    if (cudaMemcpyAsync(hv, d_cnt, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaMemcpyAsync(&lastgid, gid + nl - 1, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_cuda();
+    const long long nc = lastgid, coarsenable = nl - hv[1];
+    if (coarsenable * 10 < nl * 9 || nc >= nl) break;  // F4: fewer than 90% coarsenable / no progress
+    // contraction
+    FgpLevel C;
+    C.n = nc;
+    C.vw = mem.get<int32_t>(nc);
+    C.xadj = mem.get<int64_t>(nc + 1);
+    unsigned long long* ekey = mem.get<unsigned long long>(G.m2);
+    unsigned long long* sekey = mem.get<unsigned long long>(G.m2);
+    int32_t* ew = mem.get<int32_t>(G.m2);
+    int32_t* sew = mem.get<int32_t>(G.m2);
+    unsigned long long* ukey = mem.get<unsigned long long>(G.m2);
+    int32_t* uw = mem.get<int32_t>(G.m2);
+    int* d_nu = mem.get<int>(1);
+    int64_t* rowcnt = mem.get<int64_t>(nc + 1);
+    if (!C.vw || !C.xadj || !ekey || !sekey || !ew || !sew || !ukey || !uw || !d_nu || !rowcnt) return IGK_ENOMEM;
+    cudaMemsetAsync(C.vw, 0, nc * 4, s);
+    k_fgp_cvw<<<grid, blk, 0, s>>>(nl, cmap, G.vw, C.vw);
+    cudaMemsetAsync(d_ecnt, 0, 8, s);
+    k_fgp_edges<<<grid, blk, 0, s>>>(nl, G.xadj, G.adj, G.w, cmap, ekey, ew, d_ecnt);
+    unsigned long long ne = 0;
+    if (cudaMemcpyAsync(&ne, d_ecnt, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_cuda();
+    int cb = 1;
+    while ((1ll << cb) < nc) cb++;
+    size_t tb4 = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, tb4, ekey, sekey, ew, sew, (int)ne, 0, 32 + cb, s);
+    size_t tb5 = 0;
+    cub::DeviceReduce::ReduceByKey(nullptr, tb5, sekey, ukey, sew, uw, d_nu, cuda::std::plus<>(), (int)ne, s);
+    void* tmp4 = mem.get<char>(std::max(tb4, tb5));
+    if (!tmp4) return IGK_ENOMEM;
+    if (ne) {
+      cub::DeviceRadixSort::SortPairs(tmp4, tb4, ekey, sekey, ew, sew, (int)ne, 0, 32 + cb, s);
+      cub::DeviceReduce::ReduceByKey(tmp4, tb5, sekey, ukey, sew, uw, d_nu, cuda::std::plus<>(), (int)ne, s);
+    } else {
+      cudaMemsetAsync(d_nu, 0, 4, s);
+    }
+    int nu = 0;
+    if (cudaMemcpyAsync(&nu, d_nu, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_cuda();
+    C.m2 = nu;
+    C.adj = mem.get<int32_t>(nu);
+    C.w = uw;  // the reduced weights, already in (row, column) order
+    if (!C.adj) return IGK_ENOMEM;
+    cudaMemsetAsync(rowcnt, 0, (nc + 1) * 8, s);
+    k_fgp_rowcount<<<grid, blk, 0, s>>>(nu, ukey, rowcnt + 1);
+    k_fgp_rows<<<grid, blk, 0, s>>>(nu, ukey, C.adj);
+    size_t tb6 = 0;
+    cub::DeviceScan::InclusiveSum(nullptr, tb6, rowcnt, C.xadj, (int)(nc + 1), s);
+    void* tmp6 = mem.get<char>(tb6);
+    if (!tmp6) return IGK_ENOMEM;
+    cub::DeviceScan::InclusiveSum(tmp6, tb6, rowcnt, C.xadj, (int)(nc + 1), s);
+    if (cudaGetLastError() != cudaSuccess) return fail_cuda();
+    G.cmap = cmap;
+    L.push_back(C);
+  }
+  const int nl = (int)L.size() - 1;
+  if (nlevels) *nlevels = nl + 1;
+  if (level_n)
+    for (int l = 0; l <= nl; l++) level_n[l] = L[l].n;
+  // ---- initial partition of the coarsest graph (F5), refine, project + refine down (F6) ----
+  std::vector<int32_t> part((size_t)L[nl].n);
+  {
+    int32_t* dpart = mem.get<int32_t>(L[nl].n);
+    uint8_t* vis = mem.get<uint8_t>(L[nl].n);
+    int32_t* queue = mem.get<int32_t>(L[nl].n);
+    if (!dpart || !vis || !queue) return IGK_ENOMEM;
+    k_fgp_initial<<<1, 1, 0, s>>>(L[nl].n, L[nl].xadj, L[nl].adj, L[nl].vw, k, dpart, vis, queue);
+    if (cudaMemcpyAsync(part.data(), dpart, L[nl].n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_cuda();
+  }
+  std::string err;
+  igk_status st = fgp_refine_level(o, L[nl], k, epsilon, part, err);
+  for (int l = nl - 1; l >= 0 && st == IGK_OK; l--) {
+    int32_t* dc = mem.get<int32_t>(L[l + 1].n);
+    int32_t* df = mem.get<int32_t>(L[l].n);
+    if (!dc || !df) return IGK_ENOMEM;
+    std::vector<int32_t> fine((size_t)L[l].n);
+    if (cudaMemcpyAsync(dc, part.data(), L[l + 1].n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) return fail_cuda();
+    k_fgp_project<<<grid, blk, 0, s>>>(L[l].n, L[l].cmap, dc, df);
+    if (cudaMemcpyAsync(fine.data(), df, L[l].n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_cuda();
+    part.swap(fine);
+    st = fgp_refine_level(o, L[l], k, epsilon, part, err);
+  }
+  if (st != IGK_OK) {
+    t_create_err = err;
+    return st;
+  }
+  std::memcpy(part_out, part.data(), n * 4);
+  return IGK_OK;
 }
 
 igk_status igk_stage_batch(igk_graph* g, const igk_modifier* mods, int64_t count) {
