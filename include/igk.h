@@ -113,6 +113,15 @@ typedef struct {
    * the full partitioner (igk_fgp_partition).  Such a handle refines but
    * accepts no modifiers (IGK_EINVAL); single GPU only. */
   int32_t wide_weights;
+  /* NEXT-2 fallback policy ("applications can resort to FGP ...
+   * especially when the number of graph modifiers reaches 50% of the
+   * graph's size"; reading F9): fgp_fallback_ppm > 0 makes
+   * every successful refine / step check the modifiers accepted since the
+   * last full partition (create or repartition); once they reach
+   * fgp_fallback_ppm / 1e6 of the active vertices counted then, the call
+   * ends with igk_repartition(g, 6) and stats->repartitioned = 1.
+   * 0 = off (default).  Single-GPU handles only. */
+  int64_t fgp_fallback_ppm;
 } igk_options;
 
 typedef struct {
@@ -130,6 +139,9 @@ typedef struct {
   int64_t max_part_weight;
   int64_t imbalanced;      /* 1 iff the weighted fallback fired (IGK_WIMBALANCED)             */
   int64_t adj_entries_scanned; /* adjacency entries read by the refine kernels               */
+  int64_t repartitioned;   /* 1 iff the fallback policy (igk_options.fgp_fallback_ppm) ran a full
+                              repartition at the end of this call; cut / max_part_weight are
+                              then those of the new partition                                 */
 } igk_refine_stats;
 
 /* Create a handle from a symmetric CSR graph.  n vertices with IDs
@@ -227,6 +239,18 @@ igk_status igk_step_end(igk_graph* g, igk_refine_stats* stats, int64_t* first_ne
 igk_status igk_fgp_partition(const igk_options* opt, int64_t n, const int64_t* xadj, const int32_t* adjncy,
                              const int32_t* vwgt, const int32_t* adjwgt, int32_t k, double epsilon,
                              int32_t group_size, int32_t* part_out, int64_t* level_n, int32_t* nlevels);
+
+/* NEXT-2: full repartition of a handle's current graph in place (
+ * reading F8): the active vertices are relabelled densely in ID
+ * order, their induced graph (rows ascending) goes through the same device
+ * pipeline as igk_fgp_partition with the handle's k and epsilon, and the
+ * parts are written back (deleted vertices stay deleted); the maintained cut
+ * and W_p are recounted.  Everything runs on the device (no host copy of the
+ * graph).  IGK_ESTATE if a batch was applied and not yet refined, or after
+ * a CUDA error; IGK_EINVAL for sharded / wide handles or group_size < 2.
+ * *out_cut (nullable) = the new cut.  Afterwards igk_partition_delta
+ * returns IGK_ESTATE until the next refine (read igk_partition). */
+igk_status igk_repartition(igk_graph* g, int32_t group_size, int64_t* out_cut);
 
 /* NCCL unique id for sharded handles (call on ONE rank, share the 128
  * bytes with the others, pass as igk_options.nccl_id).  NCCL is loaded at

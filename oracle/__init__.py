@@ -86,6 +86,12 @@ def lib():
                                            C.POINTER(C.c_int64)]
         L.ora_fgp_set_passes.argtypes = [C.c_int]
         L.ora_fgp_set_init.argtypes = [C.c_int]
+        L.ora_fgp_set_lp_passes.argtypes = [C.c_int]
+        L.ora_repartition.restype = C.c_int
+        L.ora_repartition.argtypes = [P, C.c_int32]
+        L.ora_fgp_lp_pass.restype = C.c_int64
+        L.ora_fgp_lp_pass.argtypes = [C.c_int64, i64p, i32p, i32p, i32p, C.c_int32, C.c_double, i32p,
+                                      C.POINTER(C.c_int64)]
         _lib = L
     return _lib
 
@@ -118,6 +124,24 @@ def fgp_set_passes(passes: int) -> None:
 def fgp_set_init(mode: int) -> None:
     """test-only: FGP initial partition, 0 = BFS growing (default), 1 = ID blocks"""
     lib().ora_fgp_set_init(mode)
+
+
+def fgp_set_lp_passes(passes: int) -> None:
+    """test-only: label-propagation passes per finer FGP level (default 16)"""
+    lib().ora_fgp_set_lp_passes(passes)
+
+
+def fgp_lp_pass(xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None):
+    """one label-propagation pass (reading F7): (new part, moved, cut reduction)"""
+    xadj = np.ascontiguousarray(xadj, dtype=np.int64)
+    adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
+    vwgt = None if vwgt is None else np.ascontiguousarray(vwgt, dtype=np.int32)
+    adjwgt = None if adjwgt is None else np.ascontiguousarray(adjwgt, dtype=np.int32)
+    part = np.array(part, dtype=np.int32)
+    dc = C.c_int64(0)
+    mv = lib().ora_fgp_lp_pass(len(xadj) - 1, _p(xadj, C.c_int64), _p(adjncy, C.c_int32), _p(vwgt, C.c_int32),
+                               _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(dc))
+    return part, int(mv), int(dc.value)
 
 
 def fgp_coarsen_step(xadj, adjncy, adjwgt=None, group_size=6):
@@ -180,6 +204,10 @@ class Oracle:
         st = np.zeros(len(STATS), dtype=np.int64)
         s = lib().ora_refine_global(self.h, _p(st, C.c_int64))
         return int(s), dict(zip(STATS, (int(x) for x in st)))
+
+    def repartition(self, group_size: int = 6) -> int:
+        """NEXT-2 reading F8: full FGP repartition of the current graph in place (status)."""
+        return int(lib().ora_repartition(self.h, group_size))
 
     @property
     def n_total(self):

@@ -33,10 +33,14 @@
  *      on the coarsest graph -- BFS from the smallest unvisited ID,
  *      neighbours in ID order, the current part advances once the running
  *      weight reaches (p + 1) W / k.
- *  uncoarsening (F6): at every level from the coarsest down, the partition
- *      is projected (each vertex takes its group's part) and refined with
- *      the global boundary refinement of NEXT-1 (ora_refine_global: R1-R4,
- *      incl. R3 restoration of any overweight part) on that level's graph.
+ *  coarsest refinement (F6): the initial partition is refined with the
+ *      global boundary refinement of NEXT-1 (ora_refine_global: R1-R4, incl.
+ *      R3 restoration of any overweight part), repeated while a pass lowers
+ *      the cut (at most 8 passes).
+ *  uncoarsening (F7): at every finer level the partition is projected (each
+ *      vertex takes its group's part) and refined by synchronous
+ *      label-propagation passes (fgp_lp_pass below), until a pass moves
+ *      nothing (at most 16 passes).
  */
 #include <stdio.h>
 #include <stdlib.h>
@@ -268,6 +272,129 @@ static int fgp_refine(const fcsr* G, int32_t k, double eps, int32_t* part) {
   return rs == ORA_OK || rs == ORA_WIMBALANCED ? 0 : -1;
 }
 
+/* F7: one synchronous label-propagation pass on a snapshot of part / W_p.
+ *  a. every vertex v in part a: conn_p = sum of w(v, x) over neighbours x
+ *     in part p; b = the part p != a of maximal conn_p, smallest p on ties,
+ *     over the parts of v's neighbours; gain g_v = conn_b - conn_a; v is a
+ *     candidate iff g_v > 0.
+ *  b. a candidate moves only if it beats every candidate neighbour u in
+ *     (g desc, ID asc) -- the movers are pairwise non-adjacent, so the cut
+ *     falls by exactly the sum of their gains.
+ *  c. balance: the movers into part b, in (g desc, ID asc) order, are
+ *     admitted while W_b + (their running weight) <= cap (a prefix).
+ * Returns the number of vertices moved; *dcut gets the cut reduction. */
+static int g_lp_passes = 16;
+
+void ora_fgp_set_lp_passes(int p) { g_lp_passes = p; }
+typedef struct {
+  int32_t b;
+  int64_t g;
+  int32_t id;
+} lpmove;
+static int cmp_lpmove(const void* x, const void* y) {
+  const lpmove* p = (const lpmove*)x;
+  const lpmove* q = (const lpmove*)y;
+  if (p->b != q->b) return p->b < q->b ? -1 : 1;
+  if (p->g != q->g) return p->g > q->g ? -1 : 1;
+  return p->id < q->id ? -1 : (p->id > q->id);
+}
+static int64_t fgp_lp_pass(const fcsr* G, int32_t k, int64_t cap, int32_t* part, int64_t* W, int64_t* dcut) {
+  const int64_t n = G->n;
+  int64_t* conn = (int64_t*)fxalloc(k, sizeof(int64_t));
+  int32_t* tgt = (int32_t*)fxalloc(n, sizeof(int32_t));
+  int64_t* gain = (int64_t*)fxalloc(n, sizeof(int64_t));
+  for (int64_t v = 0; v < n; v++) { /* a */
+    const int32_t a = part[v];
+    for (int32_t p = 0; p < k; p++) conn[p] = 0;
+    for (int64_t j = G->xadj[v]; j < G->xadj[v + 1]; j++) conn[part[G->adj[j]]] += G->w[j];
+    int32_t b = -1;
+    for (int64_t j = G->xadj[v]; j < G->xadj[v + 1]; j++) {
+      const int32_t p = part[G->adj[j]];
+      if (p != a && (b < 0 || conn[p] > conn[b] || (conn[p] == conn[b] && p < b))) b = p;
+    }
+    tgt[v] = -1;
+    if (b >= 0 && conn[b] - conn[a] > 0) {
+      tgt[v] = b;
+      gain[v] = conn[b] - conn[a];
+    }
+  }
+  lpmove* mv = (lpmove*)fxalloc(n, sizeof(lpmove));
+  int64_t nm = 0;
+  for (int64_t v = 0; v < n; v++) { /* b */
+    if (tgt[v] < 0) continue;
+    int beaten = 0;
+    for (int64_t j = G->xadj[v]; j < G->xadj[v + 1] && !beaten; j++) {
+      const int32_t u = G->adj[j];
+      if (tgt[u] >= 0 && (gain[u] > gain[v] || (gain[u] == gain[v] && u < v))) beaten = 1;
+    }
+    if (!beaten) {
+      mv[nm].b = tgt[v];
+      mv[nm].g = gain[v];
+      mv[nm].id = (int32_t)v;
+      nm++;
+    }
+  }
+  qsort(mv, nm, sizeof(lpmove), cmp_lpmove);
+  int64_t moved = 0, red = 0, run = 0;
+  for (int64_t i = 0; i < nm; i++) { /* c: the admission uses the W_b of the snapshot */
+    if (i == 0 || mv[i].b != mv[i - 1].b) run = 0;
+    run += G->vw[mv[i].id];
+    if (W[mv[i].b] + run > cap) continue;
+    tgt[mv[i].id] = -2 - mv[i].b; /* admitted (applied below) */
+  }
+  for (int64_t v = 0; v < n; v++)
+    if (tgt[v] <= -2) {
+      const int32_t b = -2 - tgt[v];
+      W[part[v]] -= G->vw[v];
+      W[b] += G->vw[v];
+      part[v] = b;
+      red += gain[v];
+      moved++;
+    }
+  free(conn);
+  free(tgt);
+  free(gain);
+  free(mv);
+  *dcut = red;
+  return moved;
+}
+
+static void fgp_lp(const fcsr* G, int32_t k, double eps, int32_t* part) {
+  int64_t Wt = 0;
+  int64_t* W = (int64_t*)fxalloc(k, sizeof(int64_t));
+  for (int64_t v = 0; v < G->n; v++) {
+    Wt += G->vw[v];
+    W[part[v]] += G->vw[v];
+  }
+  const int64_t cap = ora_cap(Wt, eps, k);
+  for (int pass = 0; pass < g_lp_passes; pass++) {
+    int64_t dc = 0;
+    if (fgp_lp_pass(G, k, cap, part, W, &dc) == 0) break;
+  }
+  free(W);
+}
+
+int64_t ora_fgp_lp_pass(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t* vwgt,
+                        const int32_t* adjwgt, int32_t k, double epsilon, int32_t* part, int64_t* dcut) {
+  fcsr G;
+  G.n = n;
+  G.xadj = (int64_t*)xadj;
+  G.adj = (int32_t*)adjncy;
+  const int64_t m2 = xadj[n];
+  G.w = (int32_t*)fxalloc(m2, sizeof(int32_t));
+  G.vw = (int32_t*)fxalloc(n, sizeof(int32_t));
+  for (int64_t j = 0; j < m2; j++) G.w[j] = adjwgt ? adjwgt[j] : 1;
+  int64_t Wt = 0;
+  for (int64_t v = 0; v < n; v++) Wt += (G.vw[v] = vwgt ? vwgt[v] : 1);
+  int64_t* W = (int64_t*)fxalloc(k, sizeof(int64_t));
+  for (int64_t v = 0; v < n; v++) W[part[v]] += G.vw[v];
+  const int64_t moved = fgp_lp_pass(&G, k, ora_cap(Wt, epsilon, k), part, W, dcut);
+  free(W);
+  free(G.w);
+  free(G.vw);
+  return moved;
+}
+
 int ora_fgp(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t* vwgt, const int32_t* adjwgt,
             int32_t k, double epsilon, int32_t group_size, int32_t* part_out, int64_t* level_n, int64_t maxlev) {
   if (n < 1 || k < 2 || group_size < 2) return -ORA_EINVAL;
@@ -318,7 +445,7 @@ int ora_fgp(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t
     for (int64_t v = 0; v < L[l].n; v++) fine[v] = part[cmaps[l][v]];
     free(part);
     part = fine;
-    bad = fgp_refine(&L[l], k, epsilon, part);
+    fgp_lp(&L[l], k, epsilon, part);
   }
   if (!bad) memcpy(part_out, part, n * sizeof(int32_t));
   free(part);

@@ -936,3 +936,64 @@ int64_t ora_trace_moves(const ora_graph* g, int64_t* out, int64_t cap3) {
   for (int64_t i = 0; i < g->ntm && i < cap3; i++) out[i] = g->trM[i];
   return g->ntm / 3;
 }
+
+/* NEXT-2 full repartition, reading F8 (see igk_oracle.h) */
+int ora_repartition(ora_graph* g, int32_t group_size) {
+  const int64_t n = g->n;
+  for (int64_t v = 0; v < n; v++)
+    if (g->active[v] && (g->inA[v] || g->part[v] == PSI)) return ORA_ESTATE;
+  int32_t* did = (int32_t*)xcalloc((size_t)n, sizeof(int32_t));
+  int64_t na = 0, m2 = 0;
+  for (int64_t v = 0; v < n; v++)
+    if (g->active[v]) {
+      did[v] = (int32_t)na++;
+      m2 += g->adj[v].cnt;
+    }
+  if (na == 0) {
+    free(did);
+    return ORA_EINVAL;
+  }
+  int64_t* xadj = (int64_t*)xcalloc((size_t)na + 1, sizeof(int64_t));
+  int32_t* adj = (int32_t*)xcalloc((size_t)m2, sizeof(int32_t));
+  int32_t* w = (int32_t*)xcalloc((size_t)m2, sizeof(int32_t));
+  int32_t* vw = (int32_t*)xcalloc((size_t)na, sizeof(int32_t));
+  int32_t* part = (int32_t*)xcalloc((size_t)na, sizeof(int32_t));
+  int64_t pos = 0;
+  for (int64_t v = 0; v < n; v++) {
+    if (!g->active[v]) continue;
+    const ora_adj* L = &g->adj[v];
+    int32_t* tmp = (int32_t*)xcalloc(2 * (size_t)L->cnt, sizeof(int32_t));
+    for (int32_t i = 0; i < L->cnt; i++) {
+      tmp[2 * i] = did[L->nb[i]]; /* dense IDs keep the ID order */
+      tmp[2 * i + 1] = L->w[i];
+    }
+    qsort(tmp, L->cnt, 2 * sizeof(int32_t), cmp_pair);
+    for (int32_t i = 0; i < L->cnt; i++) {
+      adj[pos] = tmp[2 * i];
+      w[pos] = tmp[2 * i + 1];
+      pos++;
+    }
+    free(tmp);
+    vw[did[v]] = g->vw[v];
+    xadj[did[v] + 1] = pos;
+  }
+  int64_t lv[40];
+  const int r = ora_fgp(na, xadj, adj, vw, w, g->k, g->eps, group_size, part, lv, 40);
+  if (r >= 1) {
+    for (int32_t p = 0; p < g->k; p++) g->Wp[p] = 0;
+    for (int64_t v = 0; v < n; v++) {
+      if (!g->active[v]) continue;
+      g->part[v] = part[did[v]];
+      g->Wp[g->part[v]] += g->vw[v];
+      g->prev_part[v] = g->part[v];
+      g->inF[v] = 0;
+    }
+  }
+  free(did);
+  free(xadj);
+  free(adj);
+  free(w);
+  free(vw);
+  free(part);
+  return r >= 1 ? ORA_OK : ORA_EINVAL;
+}

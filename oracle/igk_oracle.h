@@ -38,6 +38,7 @@ typedef struct ora_graph ora_graph;
 #define ORA_OK 0
 #define ORA_EINVAL 1
 #define ORA_ENOMEM 2
+#define ORA_ESTATE 5
 #define ORA_WIMBALANCED 6
 
 /* stats vector layout (ORA_NSTATS int64 entries) */
@@ -69,6 +70,14 @@ int ora_apply(ora_graph* g, const int32_t* mods, int64_t count,
 int ora_refine(ora_graph* g, int64_t* stats /* ORA_NSTATS, nullable */);
 /* NEXT-1: A |= every boundary vertex (adj_ext != 0), then refine */
 int ora_refine_global(ora_graph* g, int64_t* stats /* ORA_NSTATS, nullable */);
+/* NEXT-2 full repartition of the current graph ("applications can
+ * resort to FGP ... when the number of graph modifiers reaches 50% of the
+ * graph's size"), reading F8: the active vertices relabelled
+ * densely in ID order, their induced graph (rows ascending) partitioned by
+ * ora_fgp with the handle's k and epsilon, the parts written back; deleted
+ * vertices stay deleted.  ORA_ESTATE if a batch is applied but not refined
+ * (pending affected or pseudo vertices); the I4 baseline restarts. */
+int ora_repartition(ora_graph* g, int32_t group_size);
 
 int64_t ora_n_total(const ora_graph* g);
 int64_t ora_n_active(const ora_graph* g);
@@ -119,6 +128,12 @@ int ora_fgp(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t
  * graph growing, the default; 1 = contiguous ID blocks) */
 void ora_fgp_set_passes(int passes);
 void ora_fgp_set_init(int mode);
+/* test-only: label-propagation passes per finer level (default 16) */
+void ora_fgp_set_lp_passes(int passes);
+/* one label-propagation pass (reading F7) on a CSR graph: part updated in
+ * place, returns the number of vertices moved, *dcut = the cut reduction */
+int64_t ora_fgp_lp_pass(int64_t n, const int64_t* xadj, const int32_t* adjncy, const int32_t* vwgt,
+                        const int32_t* adjwgt, int32_t k, double epsilon, int32_t* part, int64_t* dcut);
 int64_t ora_fgp_coarsen_step(int64_t n, const int64_t* xadj, const int32_t* adjncy,
                              const int32_t* adjwgt, int32_t group_size, int32_t* sel,
                              int32_t* root, int32_t* label, int32_t* cmap, int64_t* coarsenable);

@@ -21,7 +21,7 @@ EDGE_DELETE, VERTEX_DELETE, VERTEX_INSERT, EDGE_INSERT = 0, 1, 2, 3
 
 STATS = ["affected", "inserted", "expanded", "filtered_in", "expanded_in", "evicted", "rounds",
          "moves_applied", "moves_deferred", "cut", "cap", "max_part_weight", "imbalanced",
-         "adj_entries_scanned"]
+         "adj_entries_scanned", "repartitioned"]
 
 # every symbol include/igk.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "igk_refine", "igk_refine_global",
@@ -29,7 +29,7 @@ SYMBOLS = ["igk_create", "igk_apply_modifiers", "igk_apply_modifiers_device", "i
            "igk_step_end",
            "igk_partition", "igk_partition_delta", "igk_cut_size", "igk_part_weights", "igk_num_vertices", "igk_recount",
            "igk_export_csr", "igk_store_stats", "igk_compact", "igk_kernel_launches", "igk_last_kernel_ms", "igk_debug_phase_times", "igk_debug_arrivals",
-           "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work", "igk_fgp_partition",
+           "igk_debug_paths", "igk_debug_set_profile", "igk_debug_phase_work", "igk_fgp_partition", "igk_repartition",
            "igk_last_error", "igk_destroy"]
 
 
@@ -53,7 +53,7 @@ class Options(C.Structure):
                 ("check_invariants", C.c_int32), ("blocks_per_sm", C.c_int32),
                 ("nranks", C.c_int32), ("rank", C.c_int32), ("nccl_id", C.c_void_p),
                 ("comm", C.POINTER(Comm)), ("p2p", C.c_int32), ("ranks_per_device", C.c_int32),
-                ("wide_weights", C.c_int32)]
+                ("wide_weights", C.c_int32), ("fgp_fallback_ppm", C.c_int64)]
 
 
 class Stats(C.Structure):
@@ -174,6 +174,8 @@ def lib():
         L.igk_fgp_partition.restype = C.c_int
         L.igk_fgp_partition.argtypes = [C.POINTER(Options), i64, i64p, i32p, i32p, i32p, i32, C.c_double, i32,
                                         i32p, i64p, i32p]
+        L.igk_repartition.restype = C.c_int
+        L.igk_repartition.argtypes = [P, C.c_int32, i64p]
         L.igk_last_error.restype = C.c_char_p
         L.igk_last_error.argtypes = [P]
         L.igk_destroy.restype = None
@@ -223,10 +225,13 @@ class IGKGraph:
 
     def __init__(self, xadj, adjncy, k, eps, part, vwgt=None, adjwgt=None, device=0, stream=None,
                  max_vertices=0, max_slots=0, slack_min=0, check=False, blocks_per_sm=0,
-                 nranks=1, rank=0, nccl_id: bytes | None = None, comm=None, p2p=False, ranks_per_device=1, wide_weights=False):
+                 nranks=1, rank=0, nccl_id: bytes | None = None, comm=None, p2p=False, ranks_per_device=1, wide_weights=False,
+                 fgp_fallback: float = 0.0):
         """nranks > 1: rank `rank` of a vertex-range sharded graph (collective
         calls; every rank passes the same graph and batches).  Transport: NCCL
-        from `nccl_id` (nccl_unique_id() on one rank, shared), else `comm`."""
+        from `nccl_id` (nccl_unique_id() on one rank, shared), else `comm`.
+        fgp_fallback > 0: full repartition once the accepted modifiers reach
+        that fraction of |V| (e.g. 0.5)."""
         L = lib()
         xadj = np.ascontiguousarray(xadj, dtype=np.int64)
         adjncy = np.ascontiguousarray(adjncy, dtype=np.int32)
@@ -238,7 +243,7 @@ class IGKGraph:
         o = Options(device, stream or None, max_vertices, max_slots, slack_min, 1, int(check), blocks_per_sm,
                     int(nranks), int(rank), None if self._id is None else C.cast(self._id, C.c_void_p),
                     None if comm is None else C.pointer(comm.struct), int(bool(p2p)), int(ranks_per_device),
-                    int(bool(wide_weights)))
+                    int(bool(wide_weights)), int(round(fgp_fallback * 1e6)))
         h = C.c_void_p()
         s = L.igk_create(C.byref(o), len(xadj) - 1, _p(xadj, C.c_int64), _p(adjncy, C.c_int32),
                          _p(vwgt, C.c_int32), _p(adjwgt, C.c_int32), k, eps, _p(part, C.c_int32), C.byref(h))
@@ -276,6 +281,14 @@ class IGKGraph:
         if s not in (OK, WIMBALANCED):
             raise IGKError(s, self._err())
         return s, {f: int(getattr(st, f)) for f in STATS}
+
+    def repartition(self, group_size: int = 6) -> int:
+        """igk_repartition: full FGP repartition of the current graph in place; returns the new cut."""
+        cut = C.c_int64(0)
+        s = lib().igk_repartition(self.h, group_size, C.byref(cut))
+        if s != OK:
+            raise IGKError(s, self._err())
+        return int(cut.value)
 
     def refine_global(self):
         """igk_refine_global: the partition boundary (adj_ext != 0) joins A, then refine."""

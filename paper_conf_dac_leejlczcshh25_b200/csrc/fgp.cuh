@@ -19,6 +19,15 @@
 //   k_fgp_initial  greedy graph growing on the coarsest graph (one thread:
 //                  a few thousand vertices)
 //   k_fgp_project  fine part = part of the vertex's group
+// and per finer level the label-propagation passes of reading F7:
+//   k_lp_gain      warp per vertex: per-part connectivity in shared memory,
+//                  best other part (conn desc, part asc), gain
+//   k_lp_filter    a candidate survives iff it beats every candidate
+//                  neighbour in (gain desc, ID asc)
+//   k_lp_keys / k_lp_segs / k_lp_admit   (target, gain desc, ID asc) order
+//                  by a stable radix sort of the survivors (listed in ID
+//                  order), running weight per target, admitted while
+//                  W_b + running weight <= cap
 #pragma once
 #include "common.cuh"
 
@@ -181,6 +190,127 @@ __global__ void k_fgp_initial(long long n, const int64_t* xadj, const int32_t* a
 __global__ void k_fgp_project(long long n, const int32_t* cmap, const int32_t* cpart, int32_t* part) {
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
     part[v] = cpart[cmap[v]];
+}
+
+// ---- F7 label propagation --------------------------------------------------
+constexpr int kLpThreads = 256;
+__global__ void k_lp_pw(long long n, const int32_t* part, const int32_t* vw, unsigned long long* W) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    atomicAdd(W + part[v], (unsigned long long)vw[v]);
+}
+
+__global__ void __launch_bounds__(kLpThreads) k_lp_gain(long long n, const int64_t* xadj, const int32_t* adj,
+                                                        const int32_t* w, const int32_t* part, int k, int32_t* tgt,
+                                                        int32_t* gain) {
+  __shared__ int conn_s[kLpThreads / 32][kMaxK + 2];
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  int* conn = conn_s[wi];
+  for (int p = lane; p < k; p += 32) conn[p] = 0;
+  __syncwarp();
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long v = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n; v += nw) {
+    const long long b0 = xadj[v], b1 = xadj[v + 1];
+    for (long long j = b0 + lane; j < b1; j += 32) atomicAdd(conn + part[adj[j]], w[j]);
+    __syncwarp();
+    const int a = part[v];
+    unsigned long long best = 0;  // (conn << 8) | (255 - p): max = (conn desc, p asc)
+    for (int p = lane; p < k; p += 32) {
+      const unsigned long long key = ((unsigned long long)(unsigned)conn[p] << 8) | (unsigned)(255 - p);
+      if (p != a && key > best) best = key;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      const unsigned long long x = __shfl_xor_sync(0xffffffffu, best, o);
+      best = x > best ? x : best;
+    }
+    const long long cb = (long long)(best >> 8), ca = conn[a];
+    __syncwarp();
+    for (int p = lane; p < k; p += 32) conn[p] = 0;
+    __syncwarp();
+    if (lane == 0) {
+      const bool cand = cb - ca > 0;
+      tgt[v] = cand ? 255 - (int)(best & 0xff) : -1;
+      gain[v] = cand ? (int32_t)(cb - ca) : 0;
+    }
+  }
+}
+
+__global__ void k_lp_filter(long long n, const int64_t* xadj, const int32_t* adj, const int32_t* tgt,
+                            const int32_t* gain, int32_t* flag) {
+  const int lane = threadIdx.x & 31;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long v = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n; v += nw) {
+    if (tgt[v] < 0) {
+      if (lane == 0) flag[v] = 0;
+      continue;
+    }
+    const int32_t gv = gain[v];
+    bool beaten = false;
+    for (long long j = xadj[v] + lane; j < xadj[v + 1] && !beaten; j += 32) {
+      const int32_t u = adj[j];
+      if (tgt[u] >= 0) {
+        const int32_t gu = gain[u];
+        beaten = gu > gv || (gu == gv && u < v);
+      }
+    }
+    beaten = __any_sync(0xffffffffu, beaten);
+    if (lane == 0) flag[v] = !beaten;
+  }
+}
+
+__global__ void k_lp_iota(long long n, int32_t* ids) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    ids[v] = (int32_t)v;
+}
+
+// key = target << 31 | (INT32_MAX - gain): ascending = (target, gain desc)
+__global__ void k_lp_keys(const int* nm, const int32_t* sel, const int32_t* tgt, const int32_t* gain,
+                          unsigned long long* key) {
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < *nm; i += (long long)gridDim.x * blockDim.x) {
+    const int32_t v = sel[i];
+    key[i] = ((unsigned long long)tgt[v] << 31) | (unsigned)(0x7fffffff - gain[v]);
+  }
+}
+
+__global__ void k_lp_segs(const int* nm, const unsigned long long* skey, const int32_t* sid, const int32_t* vw,
+                          long long* wts, long long* mark) {
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < *nm; i += (long long)gridDim.x * blockDim.x) {
+    wts[i] = vw[sid[i]];
+    mark[i] = (i == 0 || (skey[i] >> 31) != (skey[i - 1] >> 31)) ? i : 0;
+  }
+}
+
+// admission against the snapshot W; part and the weight deltas written here,
+// W itself updated by k_lp_applyw after the launch
+__global__ void k_lp_admit(const int* nm, const unsigned long long* skey, const int32_t* sid, const long long* incl,
+                           const long long* segstart, const unsigned long long* W, long long cap, const int32_t* vw,
+                           const int32_t* gain, int32_t* part, long long* dW, unsigned long long* cnt) {
+  unsigned long long moved = 0, red = 0;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < *nm; i += (long long)gridDim.x * blockDim.x) {
+    const int b = (int)(skey[i] >> 31);
+    const long long s0 = segstart[i];
+    const long long run = incl[i] - (s0 > 0 ? incl[s0 - 1] : 0);
+    if ((long long)W[b] + run <= cap) {
+      const int32_t v = sid[i];
+      const int a = part[v];
+      atomicAdd((unsigned long long*)(dW + a), (unsigned long long)(-(long long)vw[v]));
+      atomicAdd((unsigned long long*)(dW + b), (unsigned long long)vw[v]);
+      part[v] = b;
+      moved++;
+      red += (unsigned long long)gain[v];
+    }
+  }
+  if (moved) {
+    atomicAdd(cnt, moved);
+    atomicAdd(cnt + 1, red);
+  }
+}
+
+__global__ void k_lp_applyw(int k, unsigned long long* W, long long* dW) {
+  for (int p = threadIdx.x; p < k; p += blockDim.x) {
+    W[p] += (unsigned long long)dW[p];
+    dW[p] = 0;
+  }
 }
 
 }  // namespace igk

@@ -27,6 +27,7 @@
 #include "refine.cuh"
 #include "step.cuh"
 #include <cub/cub.cuh>
+#include <chrono>
 
 using namespace igk;
 
@@ -247,6 +248,52 @@ __global__ void k_export_rows(Dev d, long long n, const long long* xoff, int32_t
   }
 }
 
+// igk_repartition: the active vertices relabelled densely in ID order (act =
+// 0/1 flags, did = their exclusive prefix sum), live rows gathered with
+// dense neighbour IDs (then row-sorted), the FGP partition installed back
+__global__ void k_rp_flag(Dev d, long long n, int32_t* act, int* npsi) {
+  int c = 0;
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
+    const bool a = d.active[v] != 0;
+    act[v] = a;
+    c += a && d.part[v] == kPsi;
+  }
+  if (c) atomicAdd(npsi, c);
+}
+__global__ void k_rp_deg(Dev d, long long n, const int32_t* act, const int32_t* did, long long* cdeg, int32_t* cvw) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    if (act[v]) {
+      cdeg[did[v]] = d.vr[v].ldeg;
+      cvw[did[v]] = d.vw ? d.vw[v] : 1;
+    }
+}
+__global__ void k_rp_rows(Dev d, long long n, const int32_t* act, const int32_t* did, const long long* cx,
+                          int32_t* cadj, int32_t* cw) {
+  const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+  for (long long v = gw; v < n; v += nw) {
+    if (!act[v]) continue;
+    const long long o = d.vr[v].off, base = cx[did[v]];
+    const int dg = d.vr[v].deg;
+    int wr = 0;
+    for (int b = 0; b < dg; b += 32) {
+      const int j = b + lane_id();
+      const int y = j < dg ? d.adj[o + j] : -1;
+      const unsigned keep = __ballot_sync(0xffffffffu, y >= 0);
+      if (y >= 0) {
+        const long long pos = base + wr + __popc(keep & ((1u << lane_id()) - 1u));
+        cadj[pos] = did[y];
+        cw[pos] = d.adjw ? d.adjw[o + j] : 1;
+      }
+      wr += __popc(keep);
+    }
+  }
+}
+__global__ void k_rp_install(Dev d, long long n, const int32_t* act, const int32_t* did, const int32_t* dpart) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    if (act[v]) d.part[v] = (uint8_t)dpart[did[v]];
+}
+
 __global__ void k_export_part(Dev d, long long n, int32_t* out) {
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
     uint8_t p = d.part[v];
@@ -268,6 +315,10 @@ struct igk_graph {
   long long n_notice_fallback = 0;  // fast-path steps that fell back to the copy + sync
   // sharding (igk_options.nranks > 1)
   bool wide = false;           // wide-weight handle (NEXT-2 coarse levels): refine only, no modifiers
+  bool refine_due = false;     // a batch was applied and not yet refined (igk_repartition refuses)
+  long long fallback_ppm = 0;  // igk_options.fgp_fallback_ppm (0 = off)
+  long long mods_since_full = 0, n_at_full = 0;  // the fallback policy's counters
+  bool delta_replaced = false; // igk_repartition replaced the partition: no delta until the next refine
   int nranks = 1, rank = 0;
   bool sharded = false;        // the sharded protocol (nranks > 1, or a transport given for one rank)
   igk_comm comm{};             // host-callback transport (when no NCCL communicator)
@@ -970,6 +1021,8 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     }
   }
   g->p2p = sharded && o.p2p;
+  g->fallback_ppm = sharded || g->wide ? 0 : std::max<long long>(0, o.fgp_fallback_ppm);
+  g->n_at_full = n;
   g->ranks_per_device = o.ranks_per_device > 1 ? o.ranks_per_device : 1;
   if (cudaMallocHost(&g->h_ctl, sizeof(Ctl)) != cudaSuccess ||
       cudaHostAlloc(&g->h_map, sizeof(Ctl), cudaHostAllocMapped) != cudaSuccess ||
@@ -1185,6 +1238,7 @@ static igk_status finish_apply(igk_graph* g, int64_t* bad_index) {
     return fail(g, IGK_EINVAL, buf);
   }
   if (g->h_ctl->err_nomem) return fail(g, IGK_ENOMEM, "vertex or slot capacity exhausted");
+  g->refine_due = true;
   return IGK_OK;
 }
 
@@ -1391,7 +1445,9 @@ static igk_status apply_dev(igk_graph* g, const int4* dm, int64_t count, int64_t
       if (st != IGK_OK) return st;
       continue;
     }
-    return finish_apply(g, bad_index);
+    st = finish_apply(g, bad_index);
+    if (st == IGK_OK) g->mods_since_full += count;
+    return st;
   }
 }
 
@@ -1504,6 +1560,7 @@ static igk_status step_complete(igk_graph* g, const int4* dm, int64_t count, boo
       return fail(g, IGK_EINVAL, buf);  // the kernel ended before the refine: state unchanged
     }
     if (g->h_ctl->err_nomem) return fail(g, IGK_ENOMEM, "vertex or slot capacity exhausted");
+    g->mods_since_full += count;
   }
   return finish_refine(g, stats);
 }
@@ -1580,6 +1637,8 @@ igk_status igk_apply_modifiers_device(igk_graph* g, const igk_modifier* d_mods, 
 
 static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
   if (!g->ms_pending) cudaEventElapsedTime(&g->ms_refine, g->ev[0], g->ev[1]);
+  g->refine_due = false;
+  g->delta_replaced = false;
   g->epochA = next_epoch(g);
   const long long* so = g->h_ctl->st_out;
   if (stats) {
@@ -1610,6 +1669,23 @@ static igk_status finish_refine(igk_graph* g, igk_refine_stats* stats) {
       g->poisoned = true;
       return fail(g, IGK_ESTATE, "invariant check failed: maintained cut/W_p differ from the recount");
     }
+  }
+  if (stats) stats->repartitioned = 0;
+  // the FGP fallback policy (reading F9): modifiers since the last full
+  // partition >= fgp_fallback_ppm / 1e6 of the active vertices counted then
+  if (g->fallback_ppm > 0 && g->mods_since_full * 1000000ll >= g->fallback_ppm * g->n_at_full) {
+    int64_t cut = 0;
+    igk_status st = igk_repartition(g, 6, &cut);
+    if (st != IGK_OK) return st;
+    long long mx = 0;
+    for (int p = 0; p < g->d.k; p++) mx = std::max(mx, g->h_ctl->Wp[p]);
+    if (stats) {
+      stats->repartitioned = 1;
+      stats->cut = cut;
+      stats->max_part_weight = mx;
+      stats->imbalanced = mx > so[ST_CAP];
+    }
+    return mx > so[ST_CAP] ? IGK_WIMBALANCED : IGK_OK;
   }
   return imbal ? IGK_WIMBALANCED : IGK_OK;
 }
@@ -1683,7 +1759,8 @@ struct DevBuf {  // frees its device allocations on scope exit
 
 // one handle per level (wide weights), the global boundary refinement
 // repeated while it lowers the cut (<= kFgpPasses), the refined labels out
-constexpr int kFgpPasses = 8;
+constexpr int kFgpPasses = 8;     // F6: global refinement passes on the coarsest level
+constexpr int kFgpLpPasses = 16;  // F7: label-propagation passes per finer level
 igk_status fgp_refine_level(const igk_options& o, const FgpLevel& L, int k, double eps, std::vector<int32_t>& part,
                             std::string& err) {
   std::vector<int64_t> xa(L.n + 1);
@@ -1705,7 +1782,12 @@ igk_status fgp_refine_level(const igk_options& o, const FgpLevel& L, int k, doub
   lo.comm = nullptr;
   lo.p2p = 0;
   igk_graph* h = nullptr;
+  const bool trace = getenv("IGK_FGP_TRACE") != nullptr;
+  auto now = [] { return std::chrono::steady_clock::now(); };
+  auto ms = [](auto a, auto b) { return std::chrono::duration<double, std::milli>(b - a).count(); };
+  auto t0 = now();
   igk_status st = igk_create(&lo, L.n, xa.data(), aj.data(), vw.data(), ww.data(), k, eps, part.data(), &h);
+  auto t1 = now();
   if (st != IGK_OK) {
     err = std::string("fgp: level handle: ") + igk_last_error(nullptr);
     return st;
@@ -1716,9 +1798,12 @@ igk_status fgp_refine_level(const igk_options& o, const FgpLevel& L, int k, doub
     st = igk_refine_global(h, &rs);
     if (st != IGK_OK && st != IGK_WIMBALANCED) break;
     st = IGK_OK;
+    if (trace) fprintf(stderr, "fgp n=%lld pass %d cut %lld rounds %lld moves %lld t=%.2f ms\n", L.n, p, (long long)rs.cut,
+                       (long long)rs.rounds, (long long)rs.moves_applied, ms(t1, now()));
     if (prev >= 0 && rs.cut >= prev) break;
     prev = rs.cut;
   }
+  if (trace) fprintf(stderr, "fgp n=%lld m2=%lld create %.2f ms refine %.2f ms\n", L.n, L.m2, ms(t0, t1), ms(t1, now()));
   if (st == IGK_OK) st = igk_partition(h, part.data(), (int64_t)part.size(), nullptr);
   if (st != IGK_OK) err = std::string("fgp: level refine: ") + igk_last_error(h);
   igk_destroy(h);
@@ -1727,42 +1812,14 @@ igk_status fgp_refine_level(const igk_options& o, const FgpLevel& L, int k, doub
 }  // namespace
 extern "C" {
 
-igk_status igk_fgp_partition(const igk_options* opt, int64_t n, const int64_t* xadj, const int32_t* adjncy,
-                             const int32_t* vwgt, const int32_t* adjwgt, int32_t k, double epsilon,
-                             int32_t group_size, int32_t* part_out, int64_t* level_n, int32_t* nlevels) {
-  if (n < 1 || !xadj || !part_out || k < 2 || k > kMaxK || group_size < 2 || !(epsilon > 0.0) ||
-      !(epsilon <= 1.0) || n > kNMax)
-    return IGK_EINVAL;
-  igk_options o{};
-  if (opt) o = *opt;
-  DevGuard dev_guard(o.device);
-  NvtxRange nv("igk_fgp_partition");
-  std::vector<int32_t> twin_pos;
-  if (xadj[0] != 0 || !csr_twins(n, xadj, adjncy, adjwgt, twin_pos, INT32_MAX)) return IGK_EINVAL;
-  std::vector<int32_t>().swap(twin_pos);
+// the multilevel core on a device CSR (L[0]; weights explicit): coarsening
+// F1-F4, initial partition F5, coarsest refinement F6, label propagation F7.
+// *d_part_out (from mem) gets the partition of L[0].
+static igk_status fgp_core(const igk_options& o, DevBuf& mem, std::vector<FgpLevel>& L, long long Wt, int k,
+                           double epsilon, int group_size, int32_t** d_part_out, std::string& err) {
   cudaStream_t s = (cudaStream_t)o.stream;
-  DevBuf mem;
+  const long long n = L[0].n;
   const int kMaxLv = 32;
-  std::vector<FgpLevel> L(1);
-  const long long m2 = xadj[n];
-  L[0].n = n;
-  L[0].m2 = m2;
-  L[0].xadj = mem.get<int64_t>(n + 1);
-  L[0].adj = mem.get<int32_t>(m2);
-  L[0].w = mem.get<int32_t>(m2);
-  L[0].vw = mem.get<int32_t>(n);
-  if (!L[0].xadj || !L[0].adj || !L[0].w || !L[0].vw) return IGK_ENOMEM;
-  {
-    std::vector<int32_t> w1, v1;
-    if (!adjwgt) w1.assign((size_t)std::max<long long>(m2, 1), 1);
-    if (!vwgt) v1.assign((size_t)n, 1);
-    if (cudaMemcpyAsync(L[0].xadj, xadj, (n + 1) * 8, cudaMemcpyHostToDevice, s) != cudaSuccess ||
-        (m2 && cudaMemcpyAsync(L[0].adj, adjncy, m2 * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) ||
-        (m2 && cudaMemcpyAsync(L[0].w, adjwgt ? adjwgt : w1.data(), m2 * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) ||
-        cudaMemcpyAsync(L[0].vw, vwgt ? vwgt : v1.data(), n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess ||
-        cudaStreamSynchronize(s) != cudaSuccess)
-      return IGK_ECUDA;
-  }
   int* d_cnt = mem.get<int>(4);
   unsigned long long* d_ecnt = mem.get<unsigned long long>(1);
   if (!d_cnt || !d_ecnt) return IGK_ENOMEM;
@@ -1889,41 +1946,254 @@ igk_status igk_fgp_partition(const igk_options* opt, int64_t n, const int64_t* x
     L.push_back(C);
   }
   const int nl = (int)L.size() - 1;
-  if (nlevels) *nlevels = nl + 1;
-  if (level_n)
-    for (int l = 0; l <= nl; l++) level_n[l] = L[l].n;
-  // ---- initial partition of the coarsest graph (F5), refine, project + refine down (F6) ----
+  // ---- initial partition of the coarsest graph (F5) + global refinement (F6) ----
   std::vector<int32_t> part((size_t)L[nl].n);
+  int32_t* dpart = mem.get<int32_t>(n);  // n = L[0].n  // the partition of the current level (n_l <= n)
+  int32_t* dtmp = mem.get<int32_t>(n);
   {
-    int32_t* dpart = mem.get<int32_t>(L[nl].n);
     uint8_t* vis = mem.get<uint8_t>(L[nl].n);
     int32_t* queue = mem.get<int32_t>(L[nl].n);
-    if (!dpart || !vis || !queue) return IGK_ENOMEM;
+    if (!dpart || !dtmp || !vis || !queue) return IGK_ENOMEM;
     k_fgp_initial<<<1, 1, 0, s>>>(L[nl].n, L[nl].xadj, L[nl].adj, L[nl].vw, k, dpart, vis, queue);
     if (cudaMemcpyAsync(part.data(), dpart, L[nl].n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
         cudaStreamSynchronize(s) != cudaSuccess)
       return fail_cuda();
   }
-  std::string err;
   igk_status st = fgp_refine_level(o, L[nl], k, epsilon, part, err);
-  for (int l = nl - 1; l >= 0 && st == IGK_OK; l--) {
-    int32_t* dc = mem.get<int32_t>(L[l + 1].n);
-    int32_t* df = mem.get<int32_t>(L[l].n);
-    if (!dc || !df) return IGK_ENOMEM;
-    std::vector<int32_t> fine((size_t)L[l].n);
-    if (cudaMemcpyAsync(dc, part.data(), L[l + 1].n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) return fail_cuda();
-    k_fgp_project<<<grid, blk, 0, s>>>(L[l].n, L[l].cmap, dc, df);
-    if (cudaMemcpyAsync(fine.data(), df, L[l].n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
-        cudaStreamSynchronize(s) != cudaSuccess)
-      return fail_cuda();
-    part.swap(fine);
-    st = fgp_refine_level(o, L[l], k, epsilon, part, err);
+  if (st != IGK_OK) return st;
+  if (cudaMemcpyAsync(dpart, part.data(), L[nl].n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) return fail_cuda();
+  // ---- projection + label propagation at every finer level (F7) ----
+  if (nl > 0) {
+    const long long cap = cap_of(Wt, llround(epsilon * 1e6), k);
+    const long long nmax = L[0].n;
+    int32_t* tgt = mem.get<int32_t>(nmax);
+    int32_t* gain = mem.get<int32_t>(nmax);
+    int32_t* flag = mem.get<int32_t>(nmax);
+    int32_t* ids = mem.get<int32_t>(nmax);
+    int32_t* sel = mem.get<int32_t>(nmax);
+    int32_t* sid = mem.get<int32_t>(nmax);
+    unsigned long long* key = mem.get<unsigned long long>(nmax);
+    unsigned long long* skey = mem.get<unsigned long long>(nmax);
+    long long* wts = mem.get<long long>(nmax);
+    long long* incl = mem.get<long long>(nmax);
+    long long* mark = mem.get<long long>(nmax);
+    long long* segs = mem.get<long long>(nmax);
+    unsigned long long* W = mem.get<unsigned long long>(k);
+    long long* dW = mem.get<long long>(k);
+    int* d_nm = mem.get<int>(1);
+    unsigned long long* d_mv = mem.get<unsigned long long>(2);
+    if (!tgt || !gain || !flag || !ids || !sel || !sid || !key || !skey || !wts || !incl || !mark || !segs || !W ||
+        !dW || !d_nm || !d_mv)
+      return IGK_ENOMEM;
+    // CUB scratch sized for the finest level
+    size_t t1 = 0, t2 = 0, t3 = 0, t4 = 0;
+    cub::DeviceSelect::Flagged(nullptr, t1, ids, flag, sel, d_nm, (int)nmax, s);
+    cub::DeviceRadixSort::SortPairs(nullptr, t2, key, skey, sel, sid, (int)nmax, 0, 39, s);
+    cub::DeviceScan::InclusiveSum(nullptr, t3, wts, incl, (int)nmax, s);
+    cub::DeviceScan::InclusiveScan(nullptr, t4, mark, segs, cuda::maximum<>(), (int)nmax, s);
+    size_t tb = std::max(std::max(t1, t2), std::max(t3, t4));
+    void* tmp = mem.get<char>(tb);
+    if (!tmp) return IGK_ENOMEM;
+    k_lp_iota<<<grid, blk, 0, s>>>(nmax, ids);
+    for (int l = nl - 1; l >= 0; l--) {
+      const FgpLevel& F = L[l];
+      const int nlv = (int)F.n;
+      k_fgp_project<<<grid, blk, 0, s>>>(F.n, F.cmap, dpart, dtmp);
+      std::swap(dpart, dtmp);
+      cudaMemsetAsync(W, 0, k * 8, s);
+      cudaMemsetAsync(dW, 0, k * 8, s);
+      k_lp_pw<<<grid, blk, 0, s>>>(F.n, dpart, F.vw, W);
+      for (int pass = 0; pass < kFgpLpPasses; pass++) {
+        cudaMemsetAsync(d_mv, 0, 16, s);
+        k_lp_gain<<<grid, kLpThreads, 0, s>>>(F.n, F.xadj, F.adj, F.w, dpart, k, tgt, gain);
+        k_lp_filter<<<grid, blk, 0, s>>>(F.n, F.xadj, F.adj, tgt, gain, flag);
+        size_t tb1 = tb;
+        cub::DeviceSelect::Flagged(tmp, tb1, ids, flag, sel, d_nm, nlv, s);
+        int nm = 0;
+        if (cudaMemcpyAsync(&nm, d_nm, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+            cudaStreamSynchronize(s) != cudaSuccess)
+          return fail_cuda();
+        if (nm == 0) break;
+        k_lp_keys<<<grid, blk, 0, s>>>(d_nm, sel, tgt, gain, key);
+        size_t tb2 = tb;
+        cub::DeviceRadixSort::SortPairs(tmp, tb2, key, skey, sel, sid, nm, 0, 39, s);
+        k_lp_segs<<<grid, blk, 0, s>>>(d_nm, skey, sid, F.vw, wts, mark);
+        size_t tb3 = tb;
+        cub::DeviceScan::InclusiveSum(tmp, tb3, wts, incl, nm, s);
+        size_t tb4 = tb;
+        cub::DeviceScan::InclusiveScan(tmp, tb4, mark, segs, cuda::maximum<>(), nm, s);
+        k_lp_admit<<<grid, blk, 0, s>>>(d_nm, skey, sid, incl, segs, W, cap, F.vw, gain, dpart, dW, d_mv);
+        k_lp_applyw<<<1, 256, 0, s>>>(k, W, dW);
+        unsigned long long mv[2] = {0, 0};
+        if (cudaMemcpyAsync(mv, d_mv, 16, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+            cudaStreamSynchronize(s) != cudaSuccess)
+          return fail_cuda();
+        if (getenv("IGK_FGP_TRACE"))
+          fprintf(stderr, "fgp lp n=%lld pass %d survivors %d moved %llu dcut %llu\n", F.n, pass, nm, mv[0], mv[1]);
+        if (mv[0] == 0) break;
+      }
+    }
+    if (cudaGetLastError() != cudaSuccess) return fail_cuda();
   }
+  *d_part_out = dpart;
+  return IGK_OK;
+}
+
+
+igk_status igk_fgp_partition(const igk_options* opt, int64_t n, const int64_t* xadj, const int32_t* adjncy,
+                             const int32_t* vwgt, const int32_t* adjwgt, int32_t k, double epsilon,
+                             int32_t group_size, int32_t* part_out, int64_t* level_n, int32_t* nlevels) {
+  if (n < 1 || !xadj || !part_out || k < 2 || k > kMaxK || group_size < 2 || !(epsilon > 0.0) ||
+      !(epsilon <= 1.0) || n > kNMax)
+    return IGK_EINVAL;
+  igk_options o{};
+  if (opt) o = *opt;
+  DevGuard dev_guard(o.device);
+  NvtxRange nv("igk_fgp_partition");
+  std::vector<int32_t> twin_pos;
+  if (xadj[0] != 0 || !csr_twins(n, xadj, adjncy, adjwgt, twin_pos, INT32_MAX)) return IGK_EINVAL;
+  std::vector<int32_t>().swap(twin_pos);
+  {  // coarse weights are int32: both totals must fit (F4)
+    long long tv = 0, te = 0;
+    for (int64_t v = 0; v < n; v++) tv += vwgt ? vwgt[v] : 1;
+    for (int64_t j = 0; j < xadj[n]; j++) te += adjwgt ? adjwgt[j] : 1;
+    if (tv > INT32_MAX || te > INT32_MAX) return IGK_EINVAL;
+    if (vwgt)
+      for (int64_t v = 0; v < n; v++)
+        if (vwgt[v] < 0) return IGK_EINVAL;
+  }
+  cudaStream_t s = (cudaStream_t)o.stream;
+  DevBuf mem;
+  std::vector<FgpLevel> L(1);
+  const long long m2 = xadj[n];
+  L[0].n = n;
+  L[0].m2 = m2;
+  L[0].xadj = mem.get<int64_t>(n + 1);
+  L[0].adj = mem.get<int32_t>(m2);
+  L[0].w = mem.get<int32_t>(m2);
+  L[0].vw = mem.get<int32_t>(n);
+  if (!L[0].xadj || !L[0].adj || !L[0].w || !L[0].vw) return IGK_ENOMEM;
+  {
+    std::vector<int32_t> w1, v1;
+    if (!adjwgt) w1.assign((size_t)std::max<long long>(m2, 1), 1);
+    if (!vwgt) v1.assign((size_t)n, 1);
+    if (cudaMemcpyAsync(L[0].xadj, xadj, (n + 1) * 8, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        (m2 && cudaMemcpyAsync(L[0].adj, adjncy, m2 * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) ||
+        (m2 && cudaMemcpyAsync(L[0].w, adjwgt ? adjwgt : w1.data(), m2 * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) ||
+        cudaMemcpyAsync(L[0].vw, vwgt ? vwgt : v1.data(), n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return IGK_ECUDA;
+  }
+  long long Wt = 0;
+  for (int64_t v = 0; v < n; v++) Wt += vwgt ? vwgt[v] : 1;
+  int32_t* dpart = nullptr;
+  std::string err;
+  igk_status st = fgp_core(o, mem, L, Wt, k, epsilon, group_size, &dpart, err);
   if (st != IGK_OK) {
-    t_create_err = err;
+    t_create_err = err.empty() ? "igk_fgp_partition: device failure" : err;
     return st;
   }
-  std::memcpy(part_out, part.data(), n * 4);
+  if (nlevels) *nlevels = (int32_t)L.size();
+  if (level_n)
+    for (size_t l = 0; l < L.size(); l++) level_n[l] = L[l].n;
+  if (cudaMemcpyAsync(part_out, dpart, n * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return IGK_ECUDA;
+  return IGK_OK;
+}
+
+igk_status igk_repartition(igk_graph* g, int32_t group_size, int64_t* out_cut) {
+  if (!g || g->poisoned) return IGK_ESTATE;
+  ENTRY(g, "igk_repartition");
+  if (g->sharded || g->wide) return fail(g, IGK_EINVAL, "igk_repartition: single-GPU, narrow-weight handles only");
+  if (group_size < 2) return fail(g, IGK_EINVAL, "igk_repartition: group_size < 2");
+  if (g->refine_due) return fail(g, IGK_ESTATE, "igk_repartition: a batch was applied and not yet refined");
+  cudaStream_t s = g->stream;
+  Dev& d = g->d;
+  const long long n = g->h_ctl->n_total;
+  DevBuf mem;
+  int32_t* act = mem.get<int32_t>(n + 1);
+  int32_t* did = mem.get<int32_t>(n + 1);
+  int* d_cnt = mem.get<int>(1);
+  if (!act || !did || !d_cnt) return fail(g, IGK_ENOMEM, "igk_repartition: allocation failed");
+  cudaMemsetAsync(d_cnt, 0, 4, s);
+  cudaMemsetAsync(act + n, 0, 4, s);
+  k_rp_flag<<<1184, 256, 0, s>>>(d, n, act, d_cnt);
+  size_t tb = 0;
+  cub::DeviceScan::ExclusiveSum(nullptr, tb, act, did, (int)(n + 1), s);
+  void* tmp = mem.get<char>(tb);
+  if (!tmp) return fail(g, IGK_ENOMEM, "igk_repartition: allocation failed");
+  cub::DeviceScan::ExclusiveSum(tmp, tb, act, did, (int)(n + 1), s);
+  int hv[2] = {0, 0};
+  CK(cudaMemcpyAsync(&hv[0], d_cnt, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&hv[1], did + n, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (hv[0]) return fail(g, IGK_ESTATE, "igk_repartition: pending (pseudo-partition) vertices");
+  const long long na = hv[1];
+  if (na < 1) return fail(g, IGK_EINVAL, "igk_repartition: no active vertex");
+  std::vector<FgpLevel> L(1);
+  FgpLevel& L0 = L[0];
+  L0.n = na;
+  long long* cdeg = mem.get<long long>(na + 1);
+  L0.xadj = mem.get<int64_t>(na + 1);
+  L0.vw = mem.get<int32_t>(na);
+  if (!cdeg || !L0.xadj || !L0.vw) return fail(g, IGK_ENOMEM, "igk_repartition: allocation failed");
+  cudaMemsetAsync(cdeg, 0, (na + 1) * 8, s);
+  k_rp_deg<<<1184, 256, 0, s>>>(d, n, act, did, cdeg, L0.vw);
+  size_t tb2 = 0;
+  cub::DeviceScan::ExclusiveSum(nullptr, tb2, cdeg, (long long*)L0.xadj, (int)(na + 1), s);
+  void* tmp2 = mem.get<char>(tb2);
+  if (!tmp2) return fail(g, IGK_ENOMEM, "igk_repartition: allocation failed");
+  cub::DeviceScan::ExclusiveSum(tmp2, tb2, cdeg, (long long*)L0.xadj, (int)(na + 1), s);
+  long long m2 = 0;
+  CK(cudaMemcpyAsync(&m2, L0.xadj + na, 8, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  L0.m2 = m2;
+  int32_t* radj = mem.get<int32_t>(m2);
+  int32_t* rw = mem.get<int32_t>(m2);
+  L0.adj = mem.get<int32_t>(m2);
+  L0.w = mem.get<int32_t>(m2);
+  if (!radj || !rw || !L0.adj || !L0.w) return fail(g, IGK_ENOMEM, "igk_repartition: allocation failed");
+  k_rp_rows<<<1184, 256, 0, s>>>(d, n, act, did, (const long long*)L0.xadj, radj, rw);
+  if (m2 > 0) {  // rows in ascending neighbour order (the BFS of F5 walks rows in order)
+    size_t tb3 = 0;
+    cub::DeviceSegmentedSort::SortPairs(nullptr, tb3, radj, L0.adj, rw, L0.w, (int)m2, (int)na, L0.xadj, L0.xadj + 1, s);
+    void* tmp3 = mem.get<char>(tb3);
+    if (!tmp3) return fail(g, IGK_ENOMEM, "igk_repartition: allocation failed");
+    cub::DeviceSegmentedSort::SortPairs(tmp3, tb3, radj, L0.adj, rw, L0.w, (int)m2, (int)na, L0.xadj, L0.xadj + 1, s);
+  }
+  g->launches += 5;
+  CK(cudaGetLastError());
+  // both totals must fit the int32 coarse weights (F4); W is maintained
+  const long long Wt = g->h_ctl->W;
+  if (Wt > INT32_MAX || (long long)m2 * (g->ew_unit ? 1 : 255) > INT32_MAX)
+    return fail(g, IGK_EINVAL, "igk_repartition: total weights exceed the FGP's int32 range");
+  igk_options o{};
+  o.device = g->device;
+  o.stream = (void*)s;
+  int32_t* dpart = nullptr;
+  std::string err;
+  igk_status st = fgp_core(o, mem, L, Wt, d.k, (double)g->e_ppm / 1e6, group_size, &dpart, err);
+  if (st != IGK_OK) return fail(g, st, err.empty() ? "igk_repartition: FGP failed" : err.c_str());
+  k_rp_install<<<1184, 256, 0, s>>>(d, n, act, did, dpart);
+  g->launches++;
+  // maintained cut and W_p from the reduction kernel
+  st = launch_recount(g);
+  if (st != IGK_OK) return st;
+  long long red[259];
+  CK(cudaMemcpyAsync(red, g->d_red, sizeof(red), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  g->h_ctl->cut = red[0];
+  for (int p = 0; p < d.k; p++) g->h_ctl->Wp[p] = red[1 + p];
+  g->h_ctl->n_delta = 0;
+  CK(cudaMemcpyAsync(&d.ctl->cut, &g->h_ctl->cut, 8, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(&d.ctl->Wp[0], &g->h_ctl->Wp[0], 8 * d.k, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(&d.ctl->n_delta, &g->h_ctl->n_delta, 4, cudaMemcpyHostToDevice, s));
+  CK(cudaStreamSynchronize(s));
+  g->delta_replaced = true;
+  g->mods_since_full = 0;
+  g->n_at_full = na;
+  if (out_cut) *out_cut = red[0];
   return IGK_OK;
 }
 
@@ -2020,6 +2290,8 @@ igk_status igk_partition_delta(const igk_graph* gc, int32_t* pairs, int64_t cap,
   igk_graph* g = const_cast<igk_graph*>(gc);
   if (!g || g->poisoned) return IGK_ESTATE;
   ENTRY(g, "igk_partition_delta");
+  if (g->delta_replaced)
+    return fail(g, IGK_ESTATE, "igk_partition_delta: the partition was replaced by igk_repartition (read igk_partition)");
   const long long nd = g->h_ctl->n_delta;  // in the output head read back by the last refine / step
   if (count) *count = nd;
   if (nd == 0) return IGK_OK;

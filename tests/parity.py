@@ -96,6 +96,17 @@ class Pair:
         return sto, stg
 
 
+    def repartition(self, where=""):
+        """NEXT-2 F8 on both sides: partitions, cut and W_p equal afterwards."""
+        assert self.O.repartition() == 0, where
+        cut = self.G.repartition()
+        assert cut == self.O.cut(), f"{where}: repartition cut gpu {cut} oracle {self.O.cut()}"
+        msg = self.O.check_invariants(cut)
+        assert msg is None, f"{where}: invariant violated after repartition: {msg}"
+        self.compare_state(where)
+        return cut
+
+
 def run_stream(pair: Pair, batches, full_csr_every=0, tag=""):
     stats = []
     for it, b in enumerate(batches):

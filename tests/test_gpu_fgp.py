@@ -105,3 +105,67 @@ def test_invalid_host_side():
     for k, s, eps in ((1, 6, 0.03), (2, 1, 0.03), (2, 6, 0.0), (2, 6, 2.0)):
         with pytest.raises(igk.IGKError):
             igk.fgp_partition(xadj, adj, k, eps, group_size=s)
+
+
+# ---- F8 / F9: repartition of a live handle, fallback policy -----------------------
+from tests.parity import Pair  # noqa: E402
+
+
+def _c1_pair(k=4, **kw):
+    cfg = gi.CONFIGS["C1"]
+    g = gi.make_graph(cfg["n"], cfg["fmax"], gi.graph_seed(0))
+    part, _ = gi.metis_partition(g, k)
+    P = Pair(g.xadj, g.adjncy, k, cfg["eps"], part, **kw)
+    P.refine("settle")
+    S = gi.Stream(g, gi.stream_seed(gi.graph_seed(0)))
+    return cfg, P, S
+
+
+@pytest.mark.gpu
+def test_repartition_parity_mid_stream():
+    cfg, P, S = _c1_pair()
+    for it in range(cfg["iters"]):
+        assert P.apply(gi.next_batch(S, cfg), f"it{it}") == 0
+        P.refine(f"it{it}")
+        if it in (4, 12):
+            P.repartition(f"repartition after it{it}")
+            with pytest.raises(igk.IGKError):
+                P.G.partition_delta()
+    P.compare_state("end", full_csr=True)
+
+
+@pytest.mark.gpu
+def test_repartition_refuses_pending():
+    cfg, P, S = _c1_pair()
+    assert P.apply(gi.next_batch(S, cfg)) == 0
+    with pytest.raises(igk.IGKError) as e:
+        P.G.repartition()
+    assert e.value.status == 5
+    P.refine()
+    P.repartition()
+
+
+@pytest.mark.gpu
+def test_fallback_policy():
+    """fgp_fallback = 15%: the handle repartitions by itself once the accepted
+    modifiers (600 per C1 batch) reach 15% of |V| at the last full partition;
+    the oracle side applies the same rule here (reading F9)"""
+    cfg, P, S = _c1_pair(fgp_fallback=0.15)
+    n_full, since, fired = P.O.n_active, 0, 0
+    for it in range(cfg["iters"]):
+        b = gi.next_batch(S, cfg)
+        so = P.O.apply(b)
+        assert so[0] == 0
+        since += len(b)
+        so_st, sto = P.O.refine()
+        due = since * 1_000_000 >= 150_000 * n_full
+        if due:
+            assert P.O.repartition() == 0
+            n_full, since = P.O.n_active, 0
+            fired += 1
+        sg, stg, bad = P.G.step(b)
+        assert stg["repartitioned"] == int(due), it
+        if not due:
+            assert stg["cut"] == sto["cut"]
+        P.compare_state(f"it{it}")
+    assert 4 <= fired <= 8
