@@ -281,10 +281,18 @@ def full_repartition(G, k, igk_cut, ms_per_step):
     e1.record()
     torch.cuda.synchronize()
     gcut = G.cut()
+    # NEXT-2: the GPU full partitioner (IGK-FGP v1) on the same graph, in
+    # place (igk_repartition: device export + coarsening + LP uncoarsening)
+    t = time.perf_counter()
+    fcut = G.repartition()
+    torch.cuda.synchronize()
+    t_fgp = time.perf_counter() - t
     return {"igk_cut": int(igk_cut), "metis_cut": int(mcut), "cut_ratio": igk_cut / max(mcut, 1),
             "metis_s": t_metis, "metis_vs_step": 1e3 * t_metis / ms_per_step,
             "global_refine": {"cut": int(gcut), "cut_ratio": gcut / max(mcut, 1), "ms": e0.elapsed_time(e1),
                               "boundary_affected": gst["affected"], "rounds": gst["rounds"]},
+            "gpu_fgp": {"cut": int(fcut), "cut_ratio": fcut / max(mcut, 1), "ms": 1e3 * t_fgp,
+                        "vs_step": 1e3 * t_fgp / ms_per_step, "how": "igk_repartition (group size 6), wall clock"},
             "n_active": int(act.sum()), "how": "METIS_PartGraphKway default options (ufactor 30), 1 host core, "
                                                "on the graph as it stands after the timed iterations"}
 
