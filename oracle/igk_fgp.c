@@ -13,8 +13,10 @@
  *  per level l, on G_l (vertex weights, edge weights):
  *   1. selection (F1): every vertex points at the neighbour across its
  *      heaviest incident edge, edges totally ordered by (w desc, min ID asc,
- *      max ID asc); an isolated vertex points at itself.  In that order the
- *      pointer graph's only cycles are mutual pairs.
+ *      max ID asc); an isolated vertex points at the smallest isolated
+ *      vertex (that one at itself), so isolated vertices form one subset and
+ *      merge in groups like any other (merging them cuts no edge).  In that
+ *      order the pointer graph's only cycles are mutual pairs.
  *   2. union-find with join labels (F2; "labeling each vertex with the
  *      iteration in which it joins a subset"): roots = self-pointers
  *      and the smaller vertex of each mutual pair; synchronous pointer
@@ -88,6 +90,12 @@ static void fgp_select(const fcsr* G, int32_t* sel) {
     }
     sel[v] = (int32_t)best;
   }
+  int64_t iso0 = -1; /* the smallest isolated vertex */
+  for (int64_t v = 0; v < G->n; v++)
+    if (G->xadj[v] == G->xadj[v + 1]) {
+      if (iso0 < 0) iso0 = v;
+      sel[v] = (int32_t)iso0;
+    }
 }
 
 /* 2. roots, synchronous pointer jumping, join labels */

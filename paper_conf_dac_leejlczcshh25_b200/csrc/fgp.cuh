@@ -52,10 +52,18 @@ __global__ void k_fgp_select(long long n, const int64_t* xadj, const int32_t* ad
   }
 }
 
-__global__ void k_fgp_roots(long long n, const int32_t* sel, int32_t* P, int32_t* label, int* left) {
+// the smallest isolated vertex (it selected itself): every isolated vertex
+// points at it (reading F1), so they merge in groups like any other subset
+__global__ void k_fgp_iso(long long n, const int32_t* sel, int* iso0) {
+  for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    if (sel[v] == v) atomicMin(iso0, (int)v);
+}
+__global__ void k_fgp_roots(long long n, int32_t* sel, const int* iso0p, int32_t* P, int32_t* label, int* left) {
+  const int iso0 = *iso0p;
   int c = 0;
   for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
-    const int32_t s = sel[v];
+    int32_t s = sel[v];
+    if (s == v) s = iso0;  // isolated (a vertex with an edge never selects itself)
     const bool root = s == v || (sel[s] == v && v < s);
     P[v] = root ? (int32_t)v : s;
     label[v] = root ? 0 : -1;

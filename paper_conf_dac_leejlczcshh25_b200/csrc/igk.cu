@@ -1845,8 +1845,10 @@ static igk_status fgp_core(const igk_options& o, DevBuf& mem, std::vector<FgpLev
     if (!sel || !P || !Q || !label || !key || !skey || !val || !sval || !mark || !segstart || !flag || !gid || !cmap)
       return IGK_ENOMEM;
     k_fgp_select<<<grid, blk, 0, s>>>(nl, G.xadj, G.adj, G.w, sel);
-    cudaMemsetAsync(d_cnt, 0, 16, s);
-    k_fgp_roots<<<grid, blk, 0, s>>>(nl, sel, P, label, d_cnt);
+    cudaMemsetAsync(d_cnt, 0, 12, s);
+    cudaMemsetAsync(d_cnt + 3, 0x7f, 4, s);  // iso0 = "none" (0x7f7f7f7f > any ID)
+    k_fgp_iso<<<grid, blk, 0, s>>>(nl, sel, d_cnt + 3);
+    k_fgp_roots<<<grid, blk, 0, s>>>(nl, sel, d_cnt + 3, P, label, d_cnt);
     int left = 0;
     if (cudaMemcpyAsync(&left, d_cnt, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
         cudaStreamSynchronize(s) != cudaSuccess)

@@ -101,6 +101,9 @@ def test_select_is_first_edge_in_global_order(name):
                 edges.append((-int(w[j]), v, x))
     edges.sort()
     want = list(range(n))
+    iso = [v for v in range(n) if xadj[v] == xadj[v + 1]]
+    for v in iso:  # isolated vertices point at the smallest isolated vertex
+        want[v] = iso[0]
     done = [False] * n
     for _, a, b in edges:
         if not done[a]:
@@ -262,15 +265,26 @@ def test_contraction_conserves_weights_and_cuts():
 
 
 def test_stop_rule_90_percent():
-    # a star: the centre selects its smallest leaf, every leaf selects the
-    # centre -> one subset, groups of 6: all coarsenable; a matching of
-    # isolated pairs + many isolated vertices: < 90% coarsenable -> stop
+    # disjoint 7-stars: one subset of 7 each -> a group of 6 + a singleton:
+    # 6/7 = 85.7% coarsenable < 90% -> G_0 is the coarsest graph
     k = 2
-    n = 200
-    edges = {(2 * i, 2 * i + 1): 1 for i in range(40)}  # 80 of 200 vertices paired
+    n = 7 * 30
+    edges = {(7 * i, 7 * i + j): 1 for i in range(30) for j in range(1, 7)}
     xadj, adj, aw = csr_from_edges(n, edges)
+    sel, root, label, cmap, ng, co = oracle.fgp_coarsen_step(xadj, adj, aw, 6)
+    assert ng == 60 and co == 180
     part, lv = oracle.fgp(xadj, adj, k, 0.03, adjwgt=aw)
     assert lv == [n]
+    # 6-stars: 100% coarsenable -> one level down
+    edges = {(6 * i, 6 * i + j): 1 for i in range(40) for j in range(1, 6)}
+    xadj, adj, aw = csr_from_edges(240, edges)
+    part, lv = oracle.fgp(xadj, adj, k, 0.03, adjwgt=aw)
+    assert lv == [240, 40]
+    # isolated vertices form one subset and merge in groups of s (reading F1)
+    xadj, adj, aw = csr_from_edges(240, {})
+    sel, root, label, cmap, ng, co = oracle.fgp_coarsen_step(xadj, adj, aw, 6)
+    assert (sel == 0).all() and (root == 0).all() and ng == 40 and co == 240
+    assert label[0] == 0 and (label[1:] == 1).all()
     star = {(0, i): 1 for i in range(1, 200)}
     xadj, adj, aw = csr_from_edges(200, star)
     sel, root, label, cmap, ng, co = oracle.fgp_coarsen_step(xadj, adj, aw, 6)
