@@ -26,7 +26,10 @@ constexpr int64_t kNMax = int64_t(1) << 30;
 constexpr int kThreads = IGK_THREADS;  // persistent-kernel block size (A/B builds: -DIGK_THREADS=...)
 constexpr int kWarps = kThreads / 32;
 constexpr int kThreadDeg = 16;      // degree <= this: one thread per vertex; above: one warp
-constexpr int kBlockDeg = 1024;     // degree > this (hubs): one whole CTA per vertex
+#ifndef IGK_BLOCKDEG
+#define IGK_BLOCKDEG 1024
+#endif
+constexpr int kBlockDeg = IGK_BLOCKDEG;  // degree > this (hubs): one whole CTA per vertex (A/B: -DIGK_BLOCKDEG)
 constexpr int kVdC = 8;            // vertex deletion: prefix entries per work item (one thread each)
 constexpr int kDigits = 256;        // radix digit bins (8-bit digits)
 constexpr long long kNoErr = 0x7fffffffffffffffLL;

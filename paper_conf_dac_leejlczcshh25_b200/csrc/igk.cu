@@ -24,6 +24,7 @@
 #include "common.cuh"
 #include "fgp.cuh"
 #include "recount.cuh"
+#include "recount3.cuh"
 #include "refine.cuh"
 #include "step.cuh"
 #include <cub/cub.cuh>
@@ -308,7 +309,9 @@ struct igk_graph {
   int device = 0;
   int recount_blocks = 0;    // k_recount grid (occupancy-derived at create)
   int recount_tma_blocks = 0;  // k_recount_tma grid (unit edge weights)
-  int recount_tma = 0;       // S9 kernel: direct gathers (0) or the TMA-pipelined variant (1; IGK_RECOUNT=tma)
+  int recount_tma = 0;       // S9 kernel: k_recount3 (0), the round-1 gathers (2; IGK_RECOUNT=gather) or the TMA variant (1; IGK_RECOUNT=tma)
+  int recount3_blocks = 0;   // k_recount3 grid (cooperative: co-resident CTAs), unit edge weights
+  int recount3w_blocks = 0;  // the same, weighted handles
   long long n_grow = 0;      // vertex-array growths (host path counter)
   long long n_split = 0;     // igk_step launches as k_apply + k_refine (batch >= split_b)
   long long n_fused = 0;     // igk_step launches as one k_step
@@ -349,6 +352,7 @@ struct igk_graph {
   uint32_t epoch = 1;   // last stamp value handed out
   uint32_t epochA = 0;  // stamp of the current affected set
   int grid_apply = 0, grid_refine = 0;
+  int grid_refine_k = 0;     // k_refine alone (igk_refine, split step): its own occupancy
   int grid_apply_wide = 0;   // k_apply at full occupancy (split step of large batches)
   long long split_b = 0;     // igk_step: batches of >= split_b modifiers run k_apply + k_refine
   size_t smem_refine = 0, smem_step = 0;
@@ -375,7 +379,7 @@ struct igk_graph {
   long long inflight_n0 = 0;
   long long hash_cap = 0;
   int32_t* d_out = nullptr;  // export buffer
-  long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active
+  long long* d_red = nullptr;  // recount outputs: [0] cut, [1..256] Wp, [257] entries, [258] active, [259..261] k_recount3 counters
   long long last_entries = 0, last_active = 0;
   Ctl* h_ctl = nullptr;        // pinned mirror of the control block
   Ctl* h_map = nullptr;        // host-mapped output head written by the kernel (igk_step fast path)
@@ -657,14 +661,29 @@ igk_status p2p_setup(igk_graph* g) {
 }
 
 igk_status launch_recount(igk_graph* g) {
-  CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 259, g->stream));
+  CK(cudaMemsetAsync(g->d_red, 0, sizeof(long long) * 262, g->stream));
   long long n = g->h_ctl->n_total;
   CK(cudaEventRecord(g->ev[4], g->stream));
-  if (g->recount_tma && !g->d.adjw)
+  if (g->recount_tma == 1 && !g->d.adjw) {
     k_recount_tma<<<g->recount_tma_blocks, kRcT, sizeof(RcSmem), g->stream>>>(g->d, n, g->d_red, g->d_red + 1,
                                                                              g->d_red + 257);
-  else
+  } else if (g->recount_tma == 2) {
     k_recount<<<g->recount_blocks, 256, 0, g->stream>>>(g->d, n, g->d_red, g->d_red + 1, g->d_red + 257);
+  } else {
+    // pieces of the heavy vertices go to the vertex-deletion scratch (idle
+    // outside k_apply): (n_cap + slot_cap / 8) int2 >= slot_cap / 16 int4,
+    // more than the <= slot_cap / 205 pieces a store can need
+    Dev dd = g->d;
+    long long* out_cut = g->d_red;
+    long long* out_wp = g->d_red + 1;
+    long long* out_cnt = g->d_red + 257;
+    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(g->d_red + 259);
+    int4* pieces = reinterpret_cast<int4*>(g->d.vdch);
+    void* args[] = {&dd, &n, &out_cut, &out_wp, &out_cnt, &ctr, &pieces};
+    const void* fn = g->d.adjw ? (const void*)k_recount3<true> : (const void*)k_recount3<false>;
+    CK(cudaLaunchCooperativeKernel(fn, g->d.adjw ? g->recount3w_blocks : g->recount3_blocks, kR3Threads, args, 0,
+                                   g->stream));
+  }
   g->launches++;
   CK(cudaGetLastError());
   CK(cudaEventRecord(g->ev[5], g->stream));
@@ -946,7 +965,12 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
     // the TMA-pipelined variant is opt-in: measured 2-4x slower than the
     // direct gathers on C2 / C4 / C5 (profiles/r02_s9_recount_ab.txt)
     const char* rc = getenv("IGK_RECOUNT");
-    g->recount_tma = rc && std::strcmp(rc, "tma") == 0;
+    g->recount_tma = !rc ? 0 : std::strcmp(rc, "tma") == 0 ? 1 : std::strcmp(rc, "gather") == 0 ? 2 : 0;
+    int o3 = 0, o3w = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o3, k_recount3<false>, kR3Threads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o3w, k_recount3<true>, kR3Threads, 0);
+    g->recount3_blocks = sms * std::max(1, o3);
+    g->recount3w_blocks = sms * std::max(1, o3w);
   }
   Dev& d = g->d;
   d.k = k;
@@ -999,7 +1023,7 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
             dalloc(g, &d.tgt, N) && dalloc(g, &d.gain, N) && dalloc(g, &d.pw, N) && dalloc(g, &d.meta, N) && dalloc(g, &d.metav, N) &&
             dalloc(g, &d.hist0, 256 * kDigits) && dalloc(g, &d.histR, 3 * 256 * kDigits) &&
             dalloc(g, &d.blkcnt, 4096) && dalloc(g, &d.ctl, 1) && dalloc(g, &g->d_out, N) && dalloc(g, &d.delta, N) &&
-            dalloc(g, &g->d_red, 259) && dalloc(g, &g->d_xp, kXpWords);
+            dalloc(g, &g->d_red, 262) && dalloc(g, &g->d_xp, kXpWords);
   if (ok && sharded)  // sharded exchange buffers (bitmap words, restoration keys, round records)
     ok = dalloc(g, &d.bm, N / 64 + 2) && dalloc(g, &d.lossbuf, N) && dalloc(g, &d.recs, N);
   if (!ok) {
@@ -1160,6 +1184,11 @@ igk_status igk_create(const igk_options* opt, int64_t n, const int64_t* xadj, co
   g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_step, g->smem_step, o.blocks_per_sm, dv));
   g->grid_refine = std::min(g->grid_refine, coop_grid((const void*)k_refine_sh, g->smem_refine, o.blocks_per_sm, dv));
   if (g->grid_apply > 4096) g->grid_apply = 4096;
+  {  // k_refine may run wider than the fused k_step (A/B: IGK_REFINE_BPS)
+    const char* e = getenv("IGK_REFINE_BPS");
+    const int bps = e ? atoi(e) : o.blocks_per_sm;
+    g->grid_refine_k = std::min(4096, coop_grid((const void*)k_refine, g->smem_refine, bps, dv));
+  }
   g->grid_apply_wide = std::min(4096, coop_grid((const void*)k_apply, 0, 64, dv));
 
   g->split_b = kSplitB;
@@ -1285,7 +1314,8 @@ static igk_status launch_refine(igk_graph* g, int after_apply, int global = 0) {
   RefineArgs a = make_refine_args(g, after_apply, global);
   void* args[] = {(void*)&g->d, (void*)&a};
   CK(cudaEventRecord(g->ev[0], g->stream));
-  CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, args, g->smem_refine, g->stream));
+  CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine_k, kThreads, args, g->smem_refine,
+                                 g->stream));
   g->launches++;
   CK(cudaEventRecord(g->ev[1], g->stream));
   return IGK_OK;
@@ -1510,7 +1540,7 @@ static igk_status step_launch(igk_graph* g, const int4* dm, int64_t count, bool*
     CK(cudaEventRecord(g->ev[0], g->stream));
     CK(cudaLaunchCooperativeKernel((const void*)k_apply, g->grid_apply_wide, kThreads, fast ? a1n : a1, 0,
                                    g->stream));
-    CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine, kThreads, a2, g->smem_refine, g->stream));
+    CK(cudaLaunchCooperativeKernel((const void*)k_refine, g->grid_refine_k, kThreads, a2, g->smem_refine, g->stream));
     g->d.seq = 0;
     g->launches += 2;
     g->n_split++;

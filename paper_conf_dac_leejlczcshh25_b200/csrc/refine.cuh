@@ -103,15 +103,17 @@ __device__ __forceinline__ void nbrs_thread(const Dev& d, long long o, int dg, F
 // R2 expansion marks for the neighbours of u: the placed ones join N once
 // (stamp epN).  All stamp probes / exchanges of a chunk are in flight
 // together and N is appended with one atomic per lane and chunk.
+// mk0 / dg0: the neighbours' stamps and prefix lengths when the caller
+// already loaded them in its own gather round trip (the commit), else null
 template <int C>
 __device__ __forceinline__ void mark_chunk(const Dev& d, const int* x, const uint8_t* q, uint32_t epN,
-                                           uint32_t epC) {
+                                           uint32_t epC, const unsigned* mk0 = nullptr, const int* dg0 = nullptr) {
   bool want[C];
   int dgx[C];
 #pragma unroll
   for (int t = 0; t < C; t++) {
-    unsigned mk = x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN;
-    dgx[t] = x[t] >= 0 ? ldro(&d.vr[x[t]].deg) : 0;
+    unsigned mk = mk0 ? mk0[t] : (x[t] >= 0 ? __ldcg(d.markT + x[t]) : epN);
+    dgx[t] = dg0 ? dg0[t] : (x[t] >= 0 ? ldro(&d.vr[x[t]].deg) : 0);
     // C1 members are pseudo on sigma2; sharded: each rank lists its own vertices
     want[t] = x[t] >= 0 && q[t] != kPsi && mk != epN && mk != epC && own(d, x[t]);
   }
@@ -677,11 +679,13 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
         w[t] = (i + t < dg && d.adjw) ? ldro(d.adjw + o + i + t) : 1;
       }
       uint8_t op[kTCc];
+      int dgx[kTCc];
 #pragma unroll
-      for (int t = 0; t < kTCc; t++) {  // label, stamp and saved label in one round trip
+      for (int t = 0; t < kTCc; t++) {  // label, stamp, saved label (+ expansion: prefix length) in one round trip
         q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
         mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
         op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+        dgx[t] = (expand && x[t] >= 0) ? ldro(&d.vr[x[t]].deg) : 0;
       }
 #pragma unroll
       for (int t = 0; t < kTCc; t++) {
@@ -690,7 +694,7 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
         const uint8_t qx = xc ? op[t] : q[t];
         if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
       }
-      if (expand) mark_chunk<kTCc>(d, x, q, a.epN, ep);
+      if (expand) mark_chunk<kTCc>(d, x, q, a.epN, ep, mk, dgx);
     }
     if (own(d, u)) cut_acc -= del;  // sharded: the owner (full prefix) keeps the cut delta
     finish(u, pu);
@@ -710,11 +714,13 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
         w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
       }
       uint8_t op[8];
+      int dgx[8];
 #pragma unroll
       for (int t = 0; t < 8; t++) {
         q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
         mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
         op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
+        dgx[t] = (expand && x[t] >= 0) ? ldro(&d.vr[x[t]].deg) : 0;
       }
 #pragma unroll
       for (int t = 0; t < 8; t++) {
@@ -723,7 +729,7 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
         const uint8_t qx = xc ? op[t] : q[t];
         if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
       }
-      if (expand) mark_chunk<8>(d, x, q, a.epN, ep);
+      if (expand) mark_chunk<8>(d, x, q, a.epN, ep, mk, dgx);
     }
     del = warp_sum(del);
     if (lane_id() == 0) {
@@ -1781,7 +1787,10 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   }
 }
 
-__global__ void __launch_bounds__(kThreads) k_refine(Dev d, RefineArgs a) {
+#ifndef IGK_REFINE_MINB
+#define IGK_REFINE_MINB 1
+#endif
+__global__ void __launch_bounds__(kThreads, IGK_REFINE_MINB) k_refine(Dev d, RefineArgs a) {
   cg::grid_group grid = cg::this_grid();
   extern __shared__ __align__(16) unsigned char smem_raw[];
   ShardArgs sh{};

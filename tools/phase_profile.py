@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """Average per-phase durations inside k_apply / k_refine (globaltimer stamps)
-over C2 iterations.  Usage: python tools/phase_profile.py [iters]"""
+over C2 iterations.  Usage: python tools/phase_profile.py [iters] [config] [k] [frac]
+(IGK_FLUSH=1: L2 flushed before every iteration; IGK_DEBUG_ARRIVALS=1: per-CTA barrier arrivals)"""
 import os
 import sys
 from collections import defaultdict
@@ -35,7 +36,14 @@ def main():
     S = gi.Stream(g, gi.stream_seed(gi.graph_seed(idx)), region0=region0)
     acc = [defaultdict(list), defaultdict(list)]
     tot = [[], []]
+    flush = None
+    if os.environ.get("IGK_FLUSH"):  # L2 flushed before every iteration, as in bench.py
+        import torch
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     for it in range(iters):
+        if flush is not None:
+            flush.zero_()
+            torch.cuda.synchronize()
         G.apply(gi.next_batch(S, cfg, cfg.get("frac") if cfg["mode"] == gi.MODE_MIX else None))
         pa = G.phase_times(0)
         _, st = G.refine()

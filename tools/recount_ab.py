@@ -1,9 +1,10 @@
 #!/usr/bin/env python
-"""A/B of the S9 cut / W_p reduction kernels on one store: the TMA-pipelined
-k_recount_tma (IGK_RECOUNT=tma, read at igk_create) and the direct-gather
-k_recount (the default).  Prints median kernel ms (L2 flushed before each launch)
-and the algorithmic-bytes bandwidth of bench.py's S9 line.
-Usage: python tools/recount_ab.py C4 [reps]"""
+"""A/B of the S9 cut / W_p reduction kernels on one store: k_recount3 (the
+default, "v3"), the round-1 direct-gather k_recount (IGK_RECOUNT=gather) and
+the TMA-pipelined k_recount_tma (IGK_RECOUNT=tma); the variant is read at
+igk_create.  Prints median kernel ms (L2 flushed before each launch) and the
+algorithmic-bytes bandwidth of bench.py's S9 line.
+Usage: python tools/recount_ab.py C4 [reps] [variants, comma-separated]"""
 import json
 import os
 import sys
@@ -26,7 +27,8 @@ part, _ = gi.metis_partition(g, k)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
 out = {}
-for variant in ("tma", "gather"):
+variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["v3", "gather", "tma"]
+for variant in variants:
     os.environ["IGK_RECOUNT"] = variant
     G = igk.IGKGraph(g.xadj, g.adjncy, k, cfg["eps"], part)
     G.refine()
@@ -44,5 +46,6 @@ for variant in ("tma", "gather"):
     out[variant] = {"ms": ms, "cut": cut, "bytes": by, "gbs": by / ms / 1e6, "frac": by / ms / 1e6 / peak}
     print(name, variant, json.dumps(out[variant]), flush=True)
     G.close()
-assert out["tma"]["cut"] == out["gather"]["cut"]
-print(name, "speedup", out["gather"]["ms"] / out["tma"]["ms"])
+assert len({o["cut"] for o in out.values()}) == 1, out
+if "v3" in out and "gather" in out:
+    print(name, "speedup v3 vs gather", out["gather"]["ms"] / out["v3"]["ms"])
