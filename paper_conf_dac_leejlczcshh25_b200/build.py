@@ -8,7 +8,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SO = os.path.join(HERE, "libigk.so")
 SRCS = ["csrc/igk.cu"]
-DEPS = ["csrc/igk.cu", "csrc/common.cuh", "csrc/apply.cuh", "csrc/refine.cuh", "csrc/step.cuh", "csrc/recount.cuh", "csrc/fgp.cuh", "../include/igk.h"]
+DEPS = ["csrc/igk.cu", "csrc/common.cuh", "csrc/apply.cuh", "csrc/refine.cuh", "csrc/step.cuh", "csrc/recount.cuh", "csrc/recount3.cuh", "csrc/fgp.cuh", "../include/igk.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-v"]

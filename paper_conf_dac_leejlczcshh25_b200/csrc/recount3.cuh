@@ -38,13 +38,20 @@ namespace igk {
 #endif
 constexpr int kR3V = IGK_R3V;     // vertices per lane per tile (A/B builds: -DIGK_R3V=...)
 constexpr int kR3T = 32 * kR3V;   // vertices per warp tile (consecutive IDs)
-constexpr int kR3In = 8;          // entries counted in-thread per vertex (two int4 chunks)
+#ifndef IGK_R3IN
+#define IGK_R3IN 4
+#endif
+constexpr int kR3In = IGK_R3IN;   // entries counted in-thread per vertex (int4 chunks of 4; A/B: -DIGK_R3IN)
+constexpr int kR3InC = kR3In / 4;
 constexpr int kR3Big = 256;       // more entries: the vertex is split into global pieces
 constexpr int kR3Piece = 1024;    // entries per piece
-constexpr int kR3U = 2;           // residual chunks per lane per trip
+#ifndef IGK_R3U
+#define IGK_R3U 2
+#endif
+constexpr int kR3U = IGK_R3U;     // residual chunks per lane per trip
 constexpr int kR3PU = 4;          // piece chunks per lane per trip
 #ifndef IGK_R3MINB
-#define IGK_R3MINB 1
+#define IGK_R3MINB 4
 #endif
 constexpr int kR3Threads = 256;
 constexpr int kR3Warps = kR3Threads / 32;
@@ -105,7 +112,7 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
   // the next tile's index is fetched while the current tile is counted (the
   // counter atomic is a full L2 round trip)
 #ifndef IGK_R3PF
-#define IGK_R3PF 1
+#define IGK_R3PF 0
 #endif
   unsigned long long t_next = 0;
   if (IGK_R3PF && lane == 0) t_next = atomicAdd(ctr, 1ull);
@@ -155,7 +162,7 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
       din[j] = big ? 0 : min(dgo, kR3In);
       const int res = big ? 0 : dgo - din[j];
       const unsigned mr = __ballot_sync(0xffffffffu, res > 0);
-      if (res > 0) S.hv[w][nh + __popc(mr & lt)] = make_int4((int)(c0 + 2), v, res, pv[j]);
+      if (res > 0) S.hv[w][nh + __popc(mr & lt)] = make_int4((int)(c0 + kR3InC), v, res, pv[j]);
       nh += __popc(mr);
       if (big) {  // rare: pieces of kR3Piece entries for the phase after the grid barrier
         const int np = (dgo + kR3Piece - 1) / kR3Piece;
@@ -166,11 +173,11 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
       r[j].x = (long long)c0;
     }
     // ---- trip 2: in-thread chunks (entries 0..7 of every vertex)
-    int4 xa[kR3V][2], wa[kR3V][2];
+    int4 xa[kR3V][kR3InC], wa[kR3V][kR3InC];
 #pragma unroll
     for (int j = 0; j < kR3V; j++)
 #pragma unroll
-      for (int c = 0; c < 2; c++) {
+      for (int c = 0; c < kR3InC; c++) {
         const bool ld = din[j] > 4 * c;
         xa[j][c] = ld ? __ldg(a4 + (unsigned)r[j].x + c) : none;
         wa[j][c] = (kW && ld) ? __ldg(w4 + (unsigned)r[j].x + c) : ones;
@@ -179,10 +186,10 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
     int R = 0;
     if (nh) {
       __syncwarp();
-      int cs[4], s = 0;
+      int cs[kR3V], s = 0;
 #pragma unroll
-      for (int i = 0; i < 4; i++) {
-        const int h = 4 * lane + i;
+      for (int i = 0; i < kR3V; i++) {
+        const int h = kR3V * lane + i;
         cs[i] = h < nh ? (S.hv[w][h].z + 3) >> 2 : 0;
         s += cs[i];
       }
@@ -194,22 +201,17 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
       }
       int run = inc - s;
 #pragma unroll
-      for (int i = 0; i < 4; i++) {
+      for (int i = 0; i < kR3V; i++) {
         run += cs[i];
-        if (4 * lane + i < nh) S.incl[w][4 * lane + i] = run;
+        if (kR3V * lane + i < nh) S.incl[w][kR3V * lane + i] = run;
       }
       R = __shfl_sync(0xffffffffu, inc, 31);
       __syncwarp();
     }
-    // ---- trip 3: labels of the in-thread entries
-#pragma unroll
-    for (int j = 0; j < kR3V; j++)
-#pragma unroll
-      for (int c = 0; c < 2; c++) count_chunk(xa[j][c], wa[j][c], (int)(base + 32 * j + lane), pv[j]);
-    // ---- residual entries, kR3U chunks per lane per trip
-    for (int e0 = 0; e0 < R; e0 += 32 * kR3U) {
-      int4 xr[kR3U], wr[kR3U];
-      int vr[kR3U], pr[kR3U];
+    // residual chunks e0 + 32 u + lane (u < kR3U), owner by binary search
+    int4 xr[kR3U], wr[kR3U];
+    int vr[kR3U], pr[kR3U];
+    auto load_res = [&](int e0) {
 #pragma unroll
       for (int u = 0; u < kR3U; u++) {
         const int e = e0 + 32 * u + lane;
@@ -230,6 +232,21 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
           pr[u] = H.w;
         }
       }
+    };
+    // the first residual batch is issued before the in-thread label gathers:
+    // both depend only on the records, so their trips overlap
+#ifndef IGK_R3PEEL
+#define IGK_R3PEEL 1
+#endif
+    if (IGK_R3PEEL && R > 0) load_res(0);
+    // ---- trip 3: labels of the in-thread entries
+#pragma unroll
+    for (int j = 0; j < kR3V; j++)
+#pragma unroll
+      for (int c = 0; c < kR3InC; c++) count_chunk(xa[j][c], wa[j][c], (int)(base + 32 * j + lane), pv[j]);
+    // ---- residual entries, kR3U chunks per lane per trip
+    for (int e0 = 0; e0 < R; e0 += 32 * kR3U) {
+      if (!IGK_R3PEEL || e0 > 0) load_res(e0);
 #pragma unroll
       for (int u = 0; u < kR3U; u++) count_chunk(xr[u], wr[u], vr[u], pr[u]);
     }

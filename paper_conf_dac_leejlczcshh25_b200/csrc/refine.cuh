@@ -1559,7 +1559,9 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   });
   filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
               counted, a.epA);  // hubs of A: CTA-cooperative below
+  arrive_stamp(d.dbg, 113);
   hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
+  arrive_stamp(d.dbg, 114);
   if (kSh && d.rank != 0) cnt_ins = 0;  // replicated count: summed over the ranks, so rank 0 adds it
   block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
   block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
@@ -1590,7 +1592,9 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     const int nc = ldv(&ctl->ncand), nhC = ldv(&ctl->nhubC);
     if (tid == 0) ctl->st[ST_FILTERED_IN] = nc + nhC;
     commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
+    arrive_stamp(d.dbg, 110);  // diagnostics only (IGK_DEBUG_ARRIVALS): sub-phase ends per CTA
     hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
+    arrive_stamp(d.dbg, 111);
     // neighbours of the pseudo vertices pending since apply
     auto get = [&](long long i) { return __ldcg(d.psi[0] + i); };  // C1 joins beyond np0
     auto pre = [&](int u, long long) -> int { return ld_part(d.part, u) == kPsi ? (int)kPsi : -1; };
@@ -1603,6 +1607,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       mark_nbrs_warp(d, o, dg, a.epN, a.epC1);
     };
     foreach_vertex(d, np0, get, pre, mt, mw);
+    arrive_stamp(d.dbg, 112);
     flush_acc(s, ctl->Wp, k);
     PHASE_FLUSH(PH_F1, nc + nhC + np0);
   }

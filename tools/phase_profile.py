@@ -48,6 +48,9 @@ def main():
         pa = G.phase_times(0)
         _, st = G.refine()
         pr = G.phase_times(1)
+        if os.environ.get("IGK_DEBUG_ARRIVALS") and it >= iters - 3:
+            print(f"k_refine arrivals, iteration {it}:")
+            arrivals_report(G, 1)
         if it < 3:
             continue
         for w, ph in enumerate((pa, pr)):
@@ -55,10 +58,6 @@ def main():
                 acc[w][(i1, NAMES.get(i1, f"phase {i1}"))].append((t1 - t0) / 1e3)
             tot[w].append((ph[-1][1] - ph[0][1]) / 1e3)
     ms = G.last_ms()
-    if os.environ.get("IGK_DEBUG_ARRIVALS"):
-        for w in (0, 1):
-            print(["k_apply", "k_refine"][w], "arrivals (last launch):")
-            arrivals_report(G, w)
     for w, name in enumerate(("k_apply", "k_refine")):
         print(f"{name}: stamped span {np.mean(tot[w]):.1f} us (event-timed last launch {ms['apply' if w == 0 else 'refine'] * 1e3:.1f} us)")
         for key, v in sorted(acc[w].items(), key=lambda kv: kv[0][0]):
@@ -74,13 +73,21 @@ def arrivals_report(G, which):
         return
     ph = dict(G.phase_times(which))
     t0 = min(v for v in A.flatten() if v > 0)
+    slow = {}
     for s in range(128):
         row = A[s]
         if not row.any():
             continue
         r = (row - t0) / 1e3
+        slow[s] = int(np.argmax(row))
         print(f"   slot {s:3d}: arrivals min {r.min():8.2f} med {np.median(r):8.2f} max {r.max():8.2f} us, "
-              f"slowest CTA {int(np.argmax(row))}")
+              f"slowest CTA {slow[s]}")
+    # sub-phase stamps (slots 110-114) of the CTAs that closed F0 (slot 1) and F1 (slot 2) last
+    for bar, subs in ((1, (113, 114)), (2, (110, 111, 112))):
+        if bar in slow and all(x in slow for x in subs):
+            c = slow[bar]
+            print(f"   slowest CTA {c} at barrier slot {bar}: " +
+                  ", ".join(f"slot {x} at {(A[x][c] - t0) / 1e3:.2f} us" for x in subs))
 
 
 if __name__ == "__main__":
