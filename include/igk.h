@@ -357,7 +357,10 @@ igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply
 int32_t igk_debug_phase_times(const igk_graph* g, int32_t which, int32_t* ids, int64_t* t_ns, int32_t cap);
 /* instrumentation (only if the environment had IGK_DEBUG_ARRIVALS set at
  * igk_create): per-CTA %globaltimer arrival stamps at barrier slot s of the
- * last kernel, out[s * grid + cta], 128 slots; returns the grid size. */
+ * last kernel, out[s * grid + cta], 128 slots; returns the grid size.
+ * which = 2: per-warp diagnostics of the last F1 commit pass (out[0, 4096):
+ * end times, out[4096, 8192): heaviest prefix handled, + 2^20 if it was a
+ * commit on the warp path); returns the number of warps. */
 int32_t igk_debug_arrivals(const igk_graph* g, int32_t which, int64_t* out, int32_t cap);
 /* the last failure of g; with g == NULL: why this thread's last igk_create failed */
 const char* igk_last_error(const igk_graph* g);

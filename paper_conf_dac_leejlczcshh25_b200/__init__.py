@@ -458,9 +458,12 @@ class IGKGraph:
         return list(zip(ids[:n].tolist(), ts[:n].tolist()))
 
     def arrivals(self, which):
-        """(128, grid) per-CTA barrier arrival stamps (needs IGK_DEBUG_ARRIVALS at create)."""
+        """(128, grid) per-CTA barrier arrival stamps (needs IGK_DEBUG_ARRIVALS at create);
+        which = 2: (2, warps) per-warp end times / heaviest prefix of the last F1 commit pass."""
         out = np.zeros(128 * 4096, np.int64)
         gsz = lib().igk_debug_arrivals(self.h, which, _p(out, C.c_int64), len(out))
+        if which == 2:
+            return np.stack([out[:gsz], out[4096:4096 + gsz]]) if gsz else None
         return out[: 128 * gsz].reshape(128, gsz) if gsz else None
 
     def last_ms(self):

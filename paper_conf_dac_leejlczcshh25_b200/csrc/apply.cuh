@@ -133,6 +133,25 @@ __device__ __forceinline__ void mark_affected_pre(const Dev& d, int x, uint32_t 
   }
 }
 
+// both endpoints of an edge modifier join A: stamps preloaded, both
+// exchanges in flight together, one warp-aggregated list reservation
+__device__ __forceinline__ void mark_affected_pair(const Dev& d, int x0, int x1, uint32_t epA, int dg0, int dg1,
+                                                   uint32_t st0, uint32_t st1) {
+  const bool na0 = st0 != epA && atomicExch(d.markA + x0, epA) != epA;
+  const bool na1 = st1 != epA && atomicExch(d.markA + x1, epA) != epA;  // (x0 == x1: sees the first)
+  int s2 = agg_alloc(&d.ctl->nA, (int)na0 + (int)na1);
+  if (na0) d.Alist[s2++] = x0;
+  if (na1) d.Alist[s2] = x1;
+  if (na0 && dg0 > kBlockDeg) {
+    d.markH[x0] = epA;
+    d.hubA[atomicAdd(&d.ctl->nhubA, 1)] = x0;
+  }
+  if (na1 && dg1 > kBlockDeg) {
+    d.markH[x1] = epA;
+    d.hubA[atomicAdd(&d.ctl->nhubA, 1)] = x1;
+  }
+}
+
 // mark_affected for C candidates of one thread: every stamp probe and
 // exchange in flight together, one list reservation per thread
 template <int C>
@@ -293,6 +312,16 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       icz = zr ? __ldcg(d.icnt + m.z) : 0;
     }
     const int vcy = (m.x == kVertDel && yo) ? __ldcg(d.vcnt + m.y) : 0;
+    // first-touch stamps and capacities of an insertion's endpoints (the grow
+    // reservations below), in the same round trip as the other words
+    uint32_t mgy = a.epG, mgz = a.epG;
+    int capy = 0, capz = 0;
+    if (m.x == kEdgeIns) {
+      if (yr) mgy = __ldcg(d.markG + m.y);
+      if (zr) mgz = __ldcg(d.markG + m.z);
+      if (yo) capy = __ldcg(d.capv + m.y);
+      if (zo) capz = __ldcg(d.capv + m.z);
+    }
     unsigned long long hkey = 0, hk0 = 0;
     long long hs = 0;
     int hc0 = 0;
@@ -340,36 +369,49 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       ok = false;
     }
     if (!ok) atomicMin((long long*)&ctl->err_idx, i);
-    if (m.x == kEdgeIns && rel) {  // slots for every endpoint an insertion touches (first touch)
-      int ends[2] = {m.y, m.z};
-      for (int e = 0; e < 2; e++) {
-        int x = ends[e];
-        if (x < 0 || x >= d.n_cap) continue;
-        bool first = stamp_insert(d.markG, x, a.epG);
-        int slot = agg_append(&ctl->ngrow, first);
-        if (!first) continue;
-        d.glist[slot] = x;
-        long long need = (x < n0 ? __ldcg(&d.vr[x].deg) : 0) + __ldcg(d.icnt + x);
-        long long have = x < n0 ? __ldcg(d.capv + x) : 0;
-        long long pk = -1;
-        const bool mv = need > have;
-        unsigned long long nc = 0;
-        if (mv) {
-          nc = (unsigned long long)(need + max((long long)d.slack_min, need / 4));
-          nc = (nc + 3) & ~3ull;
-        }
-        // one slab reservation and one relocation-list slot per warp, not per
-        // vertex (C4: ~10^5 relocations per batch on one counter)
-        const long long no = (long long)agg_alloc((unsigned long long*)&ctl->slab_top, nc);
-        const int rs = agg_append(&ctl->nreloc, mv);
-        if (mv) {
-          if (no + (long long)nc > d.slot_cap) atomicOr(&ctl->err_nomem, 2);  // 2: adjacency slab exhausted
-          pk = (no << 24) | (long long)nc;
-          d.rlist[rs] = x;  // M3 / M4 walk only the moving prefixes
-        }
-        d.reloc[x] = pk;
-      }
+    // slots for every endpoint an insertion touches (first touch): both stamp
+    // exchanges in flight together, then ONE warp-aggregated reservation
+    // round for the grow list, the slab and the relocation list (one
+    // dependent atomic trip each instead of three per endpoint)
+    bool fy = false, fz = false;
+    if (m.x == kEdgeIns && rel) {
+      const uint32_t oy = (yr && mgy != a.epG) ? atomicExch(d.markG + m.y, a.epG) : a.epG;
+      const uint32_t oz = (zr && mgz != a.epG) ? atomicExch(d.markG + m.z, a.epG) : a.epG;
+      fy = oy != a.epG;
+      fz = oz != a.epG;  // (m.y == m.z: the second exchange sees the first)
     }
+    auto grow_nc = [&](bool f, int x, int dg, int ic, int cap, bool& mv) -> unsigned long long {
+      mv = false;
+      if (!f) return 0ull;
+      const long long need = (x < n0 ? dg : 0) + ic;  // prefix length (incl. tombstones) + insertions
+      const long long have = x < n0 ? cap : 0;
+      mv = need > have;
+      if (!mv) return 0ull;
+      const unsigned long long nc = (unsigned long long)(need + max((long long)d.slack_min, need / 4));
+      return (nc + 3) & ~3ull;
+    };
+    bool mvy, mvz;
+    const unsigned long long ncy = grow_nc(fy, m.y, dgy, icy, capy, mvy);
+    const unsigned long long ncz = grow_nc(fz, m.z, dgz, icz, capz, mvz);
+    int bg, br;
+    unsigned long long bs;
+    agg_alloc3(&ctl->ngrow, (int)fy + (int)fz, (unsigned long long*)&ctl->slab_top, ncy + ncz, &ctl->nreloc,
+               (int)mvy + (int)mvz, bg, bs, br);
+    auto place = [&](bool f, int x, bool mv, unsigned long long nc) {
+      if (!f) return;
+      d.glist[bg++] = x;
+      long long pk = -1;
+      if (mv) {
+        const long long no = (long long)bs;
+        bs += nc;
+        if (no + (long long)nc > d.slot_cap) atomicOr(&ctl->err_nomem, 2);  // 2: adjacency slab exhausted
+        pk = (no << 24) | (long long)nc;
+        d.rlist[br++] = x;  // M3 / M4 walk only the moving prefixes
+      }
+      d.reloc[x] = pk;
+    };
+    place(fy, m.y, mvy, ncy);
+    place(fz, m.z, mvz, ncz);
   });
   GRID_SYNC_STAMPED(ctl, 102);
   if (tid == 0 && d.sharded) {  // this rank's verdict, all-reduced (MIN, MAX) before the mutation launch
@@ -416,14 +458,22 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     int a0 = m.y, b0 = m.z;
     long long oa = 0;
     int da = 0, du = 0, dv = 0;
-    if (ed) {
-      du = __ldcg(&d.vr[m.y].deg);
-      dv = __ldcg(&d.vr[m.z].deg);
+    uint8_t pu = 0, pv = 0;
+    uint32_t sty = 0, stz = 0;
+    if (ed) {  // both records, labels and A stamps in one round trip
+      long long ou, ov;
+      vr_ldcg(d, m.y, ou, du);
+      vr_ldcg(d, m.z, ov, dv);
+      pu = ld_part(d.part, m.y);
+      pv = ld_part(d.part, m.z);
+      sty = __ldcg(d.markA + m.y);
+      stz = __ldcg(d.markA + m.z);
+      oa = ou;
       if (dv < du) {
         a0 = m.z;
         b0 = m.y;
+        oa = ov;
       }
-      oa = __ldcg(&d.vr[a0].off);
       da = min(du, dv);
     }
     long long sa = (ed && da <= 32) ? thread_find(d.adj, oa, da, b0) : -1;
@@ -442,11 +492,9 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       d.adj[sb] = -1;
       atomicSub(&d.vr[m.y].ldeg, 1);
       atomicSub(&d.vr[m.z].ldeg, 1);
-      uint8_t pu = ld_part(d.part, m.y), pv = ld_part(d.part, m.z);
       if (pu != kPsi && pv != kPsi && pu != pv && own(d, m.y)) cut_acc -= w;
-      mark_affected(d, m.y, a.epA, du);
-      mark_affected(d, m.z, a.epA, dv);
     }
+    if (ed) mark_affected_pair(d, m.y, m.z, a.epA, du, dv, sty, stz);
   });
   // vertex deletions, in kVdC-entry work items (most deleted vertices have
   // degree <= 8: one item each; a hub's items spread over the grid).
@@ -469,15 +517,16 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       const int w = (x >= 0 && d.adjw) ? __ldcg(d.adjw + o + j) : 1;
       const bool xdel = x >= 0 && __ldcg(d.markD + x) == a.epD;
       const int dx = x >= 0 ? __ldcg(&d.vr[x].deg) : 0;
+      const uint32_t stx = x >= 0 ? __ldcg(d.markA + x) : a.epA;  // same round trip as the words above
+      const uint8_t px = x >= 0 ? ld_part(d.part, x) : kPsi;
       if (x >= 0 && !xdel) {  // the twin is u's entry in x's prefix
         d.adj[__ldcg(d.twin + o + j)] = -1;
         atomicSub(&d.vr[x].ldeg, 1);
       }
       if (x >= 0) {
-        const uint8_t px = ld_part(d.part, x);
         if (pu != kPsi && px != kPsi && pu != px && (!xdel || u < x) && own(d, u)) cut_acc -= w;
       }
-      if (x >= 0 && !xdel) mark_affected(d, x, a.epA, dx);
+      if (x >= 0 && !xdel) mark_affected_pre(d, x, a.epA, dx, stx);
       if (ch.y == 0 && lane_id() == 0) {
         int vwu = d.vw ? __ldcg(d.vw + u) : 1;
         if (pu != kPsi) atomic_add_ll(&ctl->Wp[pu], -(long long)vwu);

@@ -300,6 +300,9 @@ __device__ __forceinline__ void stamp_phase(Ctl* ctl, int id) {
   }
 }
 
+// per-warp diagnostics region of the arrival buffer (past every slot row of
+// grids up to 2048 CTAs): [kDbgWarp, +4096) times, [+4096, +8192) values
+constexpr long long kDbgWarp = 64ll * 4096;
 // opt-in instrumentation: every CTA stamps its arrival at barrier `slot`
 __device__ __forceinline__ void arrive_stamp(unsigned long long* dbg, int slot) {
   if (dbg && slot < 128) {
@@ -390,6 +393,42 @@ __device__ __forceinline__ T agg_alloc(T* ctr, T v) {
   if (lane == leader && total) base = atomicAdd(ctr, total);
   base = __shfl_sync(act, base, leader);
   return base + excl;
+}
+
+// three warp-aggregated bump allocations in ONE round of leader atomics (the
+// three counters are independent, so their round trips overlap): per lane
+// amounts (g, s, r) -> this lane's exclusive bases (bg, bs, br)
+__device__ __forceinline__ void agg_alloc3(int* cg, int g, unsigned long long* cs, unsigned long long s, int* cr,
+                                           int r, int& bg, unsigned long long& bs, int& br) {
+  const unsigned act = __activemask();
+  const int lane = lane_id();
+  int tg = 0, eg = 0, tr = 0, er = 0;
+  unsigned long long ts = 0, es = 0;
+  for (unsigned m = act; m; m &= m - 1) {
+    const int src = __ffs(m) - 1;
+    const int vg = __shfl_sync(act, g, src);
+    const unsigned long long vs = __shfl_sync(act, s, src);
+    const int vr = __shfl_sync(act, r, src);
+    if (src < lane) {
+      eg += vg;
+      es += vs;
+      er += vr;
+    }
+    tg += vg;
+    ts += vs;
+    tr += vr;
+  }
+  const int leader = __ffs(act) - 1;
+  int b1 = 0, b3 = 0;
+  unsigned long long b2 = 0;
+  if (lane == leader) {
+    if (tg) b1 = atomicAdd(cg, tg);
+    if (ts) b2 = atomicAdd(cs, ts);
+    if (tr) b3 = atomicAdd(cr, tr);
+  }
+  bg = __shfl_sync(act, b1, leader) + eg;
+  bs = __shfl_sync(act, b2, leader) + es;
+  br = __shfl_sync(act, b3, leader) + er;
 }
 
 template <typename T>

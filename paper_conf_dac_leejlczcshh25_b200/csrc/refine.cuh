@@ -602,13 +602,21 @@ __device__ void hub_filter(const Dev& d, RefSmem& s, const int32_t* hubs, int nh
 // filter (Alg. 3 L8-24): candidates = listed placed vertices with ext > int;
 // pseudo neighbours count as external (Q13); strict > (Q2)
 // (vertices stamped markH == hub_ep are left to the CTA-cooperative hub pass)
+// nx > 0 (F0): items n .. n + nx of the same pass are xlist[0, nx) (the
+// vertices pending since the apply); each one still pending adds 1 to *xcnt
+// and is not filtered -- one pass instead of a separate counting loop
 template <class Get>
 __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int32_t* cand, uint32_t ep,
-                            long long& scanned, long long& counted, uint32_t hub_ep = 0) {
+                            long long& scanned, long long& counted, uint32_t hub_ep = 0, int nx = 0,
+                            const int32_t* xlist = nullptr, long long* xcnt = nullptr) {
   // the label doubles as the active flag; hubs of A go to the CTA pass;
   // sharded: the owner filters
-  auto pre = [&](int u, long long) -> int {
+  auto pre = [&](int u, long long i) -> int {
     const uint8_t pu = ld_part(d.part, u);
+    if (i >= n) {
+      *xcnt += pu == kPsi;
+      return -1;
+    }
     const bool hub = hub_ep && __ldcg(d.markH + u) == hub_ep;
     return (pu == kDel || hub || pu == kPsi || !own(d, u)) ? -1 : (int)pu;
   };
@@ -647,7 +655,8 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
       }
     }
   };
-  foreach_vertex(d, n, get, pre, tf, wf);
+  foreach_vertex(
+      d, n + nx, [&](long long i) { return i < n ? get(i) : __ldcg(xlist + (i - n)); }, pre, tf, wf);
 }
 
 // deferred commit to the pseudo-partition (Alg. 3 L25-26) of the candidates
@@ -655,8 +664,15 @@ __device__ void filter_pass(const Dev& d, long long n, Get get, int* ncand, int3
 // neighbour's snapshot label is its saved label if it is a candidate (its
 // current label may already be psi), else its current label.  With `expand`,
 // the placed-on-sigma2 neighbours are marked for R2.
+//
+// np0 > 0 (F1): the same pass also marks the placed neighbours of the np0
+// vertices pending since the apply (plist0[0, np0): items nc .. nc + np0 of
+// the pass), so the commit chains and the marking chains run side by side on
+// different warps instead of one after the other (C2: the marking pass
+// alone held the slowest CTA ~10 us past the commit).
 __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, const int32_t* cand, uint32_t ep,
-                       bool expand, long long& scanned, long long& cut_acc) {
+                       bool expand, long long& scanned, long long& cut_acc, int np0 = 0,
+                       const int32_t* plist0 = nullptr) {
   Ctl* ctl = d.ctl;
   auto finish = [&](int u, uint8_t pu) {
     acc_add(s.acc, pu, -(long long)vert_w(d.vw, u));
@@ -664,10 +680,19 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     int slot = agg_append(&ctl->npsi[0], true);
     d.psi[0][slot] = u;
   };
-  auto pre = [&](int u, long long) -> int { return __ldcg(d.oldp + u); };
-  auto tf = [&](int u, long long, long long o, int dg, int pvv) {
-    const uint8_t pu = (uint8_t)pvv;
+  auto pre = [&](int u, long long i) -> int {
+    if (i >= nc) return ld_part(d.part, u) == kPsi ? (int)kPsi : -1;  // pending since the apply: mark only
+    return __ldcg(d.oldp + u);
+  };
+  int dmax = 0;  // diagnostics (IGK_DEBUG_ARRIVALS): the heaviest prefix this warp handled
+  auto tf = [&](int u, long long i, long long o, int dg, int pvv) {
     scanned += dg;
+    dmax = max(dmax, dg);
+    if (i >= nc) {
+      mark_nbrs_thread(d, o, dg, a.epN, ep);
+      return;
+    }
+    const uint8_t pu = (uint8_t)pvv;
     long long del = 0;
     for (int i = 0; i < dg; i += kTCc) {
       int x[kTCc], w[kTCc];
@@ -699,9 +724,14 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     if (own(d, u)) cut_acc -= del;  // sharded: the owner (full prefix) keeps the cut delta
     finish(u, pu);
   };
-  auto wf = [&](int u, long long, long long o, int dg, int pvv) {
-    const uint8_t pu = (uint8_t)pvv;
+  auto wf = [&](int u, long long i, long long o, int dg, int pvv) {
     if (lane_id() == 0) scanned += dg;
+    dmax = max(dmax, dg + (i >= nc ? 0 : 1 << 20));  // + 2^20: a commit (not a mark) on the warp path
+    if (i >= nc) {
+      mark_nbrs_warp(d, o, dg, a.epN, ep);
+      return;
+    }
+    const uint8_t pu = (uint8_t)pvv;
     long long del = 0;
     for (int b = 0; b < dg; b += 256) {
       int x[8], w[8];
@@ -737,7 +767,18 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
       finish(u, pu);
     }
   };
-  foreach_vertex(d, nc, [&](long long i) { return __ldcg(cand + i); }, pre, tf, wf);
+  foreach_vertex(
+      d, (long long)nc + np0, [&](long long i) { return i < nc ? __ldcg(cand + i) : __ldcg(plist0 + (i - nc)); },
+      pre, tf, wf);
+  if (d.dbg && expand) {  // per warp: end time, heaviest prefix (igk_debug_arrivals which = 2)
+#pragma unroll
+    for (int o2 = 16; o2; o2 >>= 1) dmax = max(dmax, __shfl_xor_sync(0xffffffffu, dmax, o2));
+    const long long wi = (long long)blockIdx.x * (blockDim.x >> 5) + warp_id();
+    if (lane_id() == 0 && wi < 4096) {
+      d.dbg[kDbgWarp + wi] = gtimer();
+      d.dbg[kDbgWarp + 4096 + wi] = (unsigned long long)dmax;
+    }
+  }
 }
 
 // commit of hub candidates by a whole CTA each (same arithmetic as commit());
@@ -1553,12 +1594,10 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   const int nA = ldv(&ctl->nA);
   const int np0 = ldv(&ctl->npsi[0]);
   const int nhA = ldv(&ctl->nhubA);
-  rr_for(np0, [&](long long i) {
-    int u = __ldcg(d.psi[0] + i);
-    if (ld_part(d.part, u) == kPsi) cnt_ins++;
-  });
+  // R1 filter over A; the pending-since-apply vertices (psi[0]) are counted
+  // in the same pass (stat `inserted`)
   filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
-              counted, a.epA);  // hubs of A: CTA-cooperative below
+              counted, a.epA, np0, d.psi[0], &cnt_ins);  // hubs of A: CTA-cooperative below
   arrive_stamp(d.dbg, 113);
   hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
   arrive_stamp(d.dbg, 114);
@@ -1591,23 +1630,12 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     const int np0 = ldv(&ctl->npsi[0]);  // pending since apply (C1 joins beyond)
     const int nc = ldv(&ctl->ncand), nhC = ldv(&ctl->nhubC);
     if (tid == 0) ctl->st[ST_FILTERED_IN] = nc + nhC;
-    commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc);
+    // commit C1 and, in the same pass, mark the neighbours of the pseudo
+    // vertices pending since apply (psi[0][0, np0); C1 joins beyond np0)
+    commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc, np0, d.psi[0]);
     arrive_stamp(d.dbg, 110);  // diagnostics only (IGK_DEBUG_ARRIVALS): sub-phase ends per CTA
     hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
     arrive_stamp(d.dbg, 111);
-    // neighbours of the pseudo vertices pending since apply
-    auto get = [&](long long i) { return __ldcg(d.psi[0] + i); };  // C1 joins beyond np0
-    auto pre = [&](int u, long long) -> int { return ld_part(d.part, u) == kPsi ? (int)kPsi : -1; };
-    auto mt = [&](int u, long long, long long o, int dg, int) {
-      scanned += dg;
-      mark_nbrs_thread(d, o, dg, a.epN, a.epC1);
-    };
-    auto mw = [&](int u, long long, long long o, int dg, int) {
-      if (lane_id() == 0) scanned += dg;
-      mark_nbrs_warp(d, o, dg, a.epN, a.epC1);
-    };
-    foreach_vertex(d, np0, get, pre, mt, mw);
-    arrive_stamp(d.dbg, 112);
     flush_acc(s, ctl->Wp, k);
     PHASE_FLUSH(PH_F1, nc + nhC + np0);
   }

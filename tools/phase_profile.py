@@ -82,6 +82,13 @@ def arrivals_report(G, which):
         slow[s] = int(np.argmax(row))
         print(f"   slot {s:3d}: arrivals min {r.min():8.2f} med {np.median(r):8.2f} max {r.max():8.2f} us, "
               f"slowest CTA {slow[s]}")
+    W = G.arrivals(2)  # per warp: F1 commit-pass end time, heaviest prefix
+    if W is not None and W[0].any():
+        t = (W[0] - t0) / 1e3
+        order = np.argsort(-t)[:5]
+        print("   F1 commit pass, latest warps (cta.warp: end us, heaviest prefix, warp-path commit):",
+              "; ".join(f"{i // 16}.{i % 16}: {t[i]:.2f}, {W[1][i] & 0xfffff}, {bool(W[1][i] >> 20)}" for i in order))
+        print(f"   F1 commit pass warp ends: median {np.median(t):.2f} us, p90 {np.percentile(t, 90):.2f} us")
     # sub-phase stamps (slots 110-114) of the CTAs that closed F0 (slot 1) and F1 (slot 2) last
     for bar, subs in ((1, (113, 114)), (2, (110, 111, 112))):
         if bar in slow and all(x in slow for x in subs):
