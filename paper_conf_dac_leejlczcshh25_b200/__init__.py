@@ -463,7 +463,7 @@ class IGKGraph:
         out = np.zeros(128 * 4096, np.int64)
         gsz = lib().igk_debug_arrivals(self.h, which, _p(out, C.c_int64), len(out))
         if which == 2:
-            return np.stack([out[:gsz], out[4096:4096 + gsz]]) if gsz else None
+            return np.stack([out[j * 4096:j * 4096 + gsz] for j in range(4)]) if gsz else None
         return out[: 128 * gsz].reshape(128, gsz) if gsz else None
 
     def last_ms(self):

@@ -25,7 +25,10 @@ constexpr int64_t kNMax = int64_t(1) << 30;
 #endif
 constexpr int kThreads = IGK_THREADS;  // persistent-kernel block size (A/B builds: -DIGK_THREADS=...)
 constexpr int kWarps = kThreads / 32;
-constexpr int kThreadDeg = 16;      // degree <= this: one thread per vertex; above: one warp
+#ifndef IGK_THREADDEG
+#define IGK_THREADDEG 8
+#endif
+constexpr int kThreadDeg = IGK_THREADDEG;  // degree <= this: one thread per vertex; above: one warp (A/B: -DIGK_THREADDEG)
 #ifndef IGK_BLOCKDEG
 #define IGK_BLOCKDEG 1024
 #endif

@@ -2562,7 +2562,7 @@ igk_status igk_last_kernel_ms(const igk_graph* g, float* refine_ms, float* apply
 int32_t igk_debug_arrivals(const igk_graph* g, int32_t which, int64_t* out, int32_t cap) {
   if (!g || !g->d.dbg || !out) return 0;
   if (which == 2) {  // per-warp diagnostics of the last F1 commit pass: 4096 times, then 4096 values
-    std::vector<unsigned long long> h(8192);
+    std::vector<unsigned long long> h(16384);
     if (cudaMemcpy(h.data(), g->d.dbg + kDbgWarp, h.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return 0;
     for (size_t i = 0; i < h.size() && (int64_t)i < cap; i++) out[i] = (int64_t)h[i];
     return g->grid_refine_k * (kThreads / 32);

@@ -78,7 +78,7 @@ struct ShardArgs {
 // ---------------------------------------------------------------------------
 // thread: f(x, w, q) for each neighbour; a chunk issues all its ID/weight
 // loads, then all its label loads, before f runs; f returns false to stop
-constexpr int kTC = 16;  // thread chunk (== kThreadDeg: one round trip per vertex)
+constexpr int kTC = kThreadDeg;  // thread chunk (one round trip per thread-bucket vertex)
 // the commit's thread chunk: five values per slot (ID, weight, label, stamp,
 // saved label) plus the expansion marks -- 8 slots keep it off the local stack
 constexpr int kTCc = 8;
@@ -216,8 +216,12 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
   const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
   const long long gw = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long per_round = nw * 32;
+  // (packing a short list into the lanes of one warp per CTA -- item
+  // r0 + cta + G (lane + 32 warp), warp-aggregated appends -- measured
+  // slower: C2 0.201 vs 0.185 ms per step, profiles/r02_z_*)
+  auto item = [&](int ln) -> long long { return (long long)ln * nw + gw; };
   for (long long r0 = 0; r0 < n; r0 += per_round) {
-    long long i = r0 + (long long)lane_id() * nw + gw;
+    long long i = r0 + item(lane_id());
     int u = i < n ? get(i) : -1;
     long long o = 0;
     int dg = 0, pv = -1;
@@ -236,7 +240,7 @@ __device__ __forceinline__ void foreach_vertex(const Dev& d, long long n, Get ge
       long long oo = __shfl_sync(0xffffffffu, o, src);
       int dd = __shfl_sync(0xffffffffu, dg, src);
       int pp = __shfl_sync(0xffffffffu, pv, src);
-      wf(uu, r0 + (long long)src * nw + gw, oo, dd, pp);
+      wf(uu, r0 + item(src), oo, dd, pp);
     }
   }
 }
@@ -687,7 +691,7 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
   int dmax = 0;  // diagnostics (IGK_DEBUG_ARRIVALS): the heaviest prefix this warp handled
   auto tf = [&](int u, long long i, long long o, int dg, int pvv) {
     scanned += dg;
-    dmax = max(dmax, dg);
+    dmax = max(dmax, dg | (i >= nc ? 1 << 21 : 0));
     if (i >= nc) {
       mark_nbrs_thread(d, o, dg, a.epN, ep);
       return;

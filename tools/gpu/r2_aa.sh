@@ -1,0 +1,11 @@
+# round 2, session AA: same-box A/B of the warp-aggregated N reservation in mark_chunk (aggN) vs per-lane (main)
+set -x
+mkdir -p gpurun_out
+AB=$PWD/paper_conf_dac_leejlczcshh25_b200/ab
+for rep in 1 2 3; do
+for v in main aggN; do
+  if [ $v = main ]; then L=""; else L="IGK_LIB=$AB/libigk_$v.so"; fi
+  env $L timeout 400 python bench.py --steps 40 --no-cpu-baseline --no-repartition > gpurun_out/aa_bench_c2_${v}_$rep.json 2> gpurun_out/aa_bench_c2_${v}_$rep.err
+done
+done
+for f in gpurun_out/aa_bench_*.json; do echo $f; python -c "import json,sys; d=json.loads(open('$f').read().strip().split(chr(10))[-1]); print(d['ms_per_step'], d['iteration']['ms_p50'], d['e2e']['ms_per_step'])"; done

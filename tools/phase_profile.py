@@ -86,8 +86,17 @@ def arrivals_report(G, which):
     if W is not None and W[0].any():
         t = (W[0] - t0) / 1e3
         order = np.argsort(-t)[:5]
-        print("   F1 commit pass, latest warps (cta.warp: end us, heaviest prefix, warp-path commit):",
-              "; ".join(f"{i // 16}.{i % 16}: {t[i]:.2f}, {W[1][i] & 0xfffff}, {bool(W[1][i] >> 20)}" for i in order))
+        tin = np.where(W[2] > 0, (W[2] - t0) / 1e3, np.nan)
+        tout = np.where(W[3] > 0, (W[3] - t0) / 1e3, np.nan)
+        print("   F1 commit pass, latest warps (cta.warp: end us, heaviest prefix, warp-path commit, mark item,"
+              " lane-0 item enter/exit us):",
+              "; ".join(f"{i // 16}.{i % 16}: {t[i]:.2f}, {W[1][i] & 0xfffff}, {bool(W[1][i] >> 20 & 1)}, "
+                        f"{bool(W[1][i] >> 21 & 1)}, {tin[i]:.2f}/{tout[i]:.2f}" for i in order))
+        ok = ~np.isnan(tin)
+        if ok.any():
+            print(f"   lane-0 thread items: enter median {np.nanmedian(tin):.2f} p90 {np.nanpercentile(tin, 90):.2f}; "
+                  f"body median {np.nanmedian(tout - tin):.2f} p90 {np.nanpercentile(tout - tin, 90):.2f} max "
+                  f"{np.nanmax(tout - tin):.2f} us")
         print(f"   F1 commit pass warp ends: median {np.median(t):.2f} us, p90 {np.percentile(t, 90):.2f} us")
     # sub-phase stamps (slots 110-114) of the CTAs that closed F0 (slot 1) and F1 (slot 2) last
     for bar, subs in ((1, (113, 114)), (2, (110, 111, 112))):
