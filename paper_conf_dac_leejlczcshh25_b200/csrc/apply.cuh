@@ -455,7 +455,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
     int4 m = valid ? a.mods[i] : make_int4(-1, 0, 0, 0);
     const bool ed = m.x == kEdgeDel && rel_edge(d, m);
     // search the shorter prefix; the twin gives the reverse slot
-    int a0 = m.y, b0 = m.z;
+    int b0 = m.z;  // the endpoint searched for (in the other's, shorter prefix)
     long long oa = 0;
     int da = 0, du = 0, dv = 0;
     uint8_t pu = 0, pv = 0;
@@ -470,7 +470,6 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       stz = __ldcg(d.markA + m.z);
       oa = ou;
       if (dv < du) {
-        a0 = m.z;
         b0 = m.y;
         oa = ov;
       }

@@ -1588,6 +1588,55 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     }
     return;
   }
+  if constexpr (!kSh) {
+    if (a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
+      boundary_mark(d, a.epA);
+      PHASE_FLUSH(PH_BOUNDARY, ldv(&ctl->n_total));
+      GRID_SYNC_STAMPED(ctl, 220);
+    }
+    const int np0 = ldv(&ctl->npsi[0]);  // pending since apply (C1 joins psi[0] beyond np0)
+    // F0 + F1 and F2 + F3 are the same two passes (a filter, then the deferred
+    // commit of its candidates) over different lists and snapshots, so they
+    // run from ONE copy of the code: the second pair executes instructions
+    // the first already brought into the instruction caches (the step after
+    // a flushed L2 stalls on instruction fetch)
+    for (int pass = 0; pass < 2; pass++) {
+      const bool p0 = pass == 0;
+      {  // ---- F0: R1 filter over A on sigma1 (+ the pending-since-apply count)
+         //      F2: R2 filter over N on sigma2
+        const int n = ldv(p0 ? &ctl->nA : &ctl->nN);
+        const int nh = ldv(p0 ? &ctl->nhubA : &ctl->nhubN);
+        const int32_t* list = p0 ? d.Alist : d.Nlist;
+        const uint32_t ep = p0 ? a.epC1 : a.epC2;
+        long long cnt = 0;
+        filter_pass(d, n, [&](long long i) { return __ldcg(list + i); }, p0 ? &ctl->ncand : &ctl->ncand2,
+                    p0 ? d.cand : d.cand2, ep, scanned, cnt, p0 ? a.epA : 0u, p0 ? np0 : 0, d.psi[0], &cnt_ins);
+        hub_filter(d, s, p0 ? d.hubA : d.hubN, nh, ep, p0 ? &ctl->nhubC : &ctl->nhubC2, p0 ? d.hubC : d.hubC2,
+                   scanned, cnt);  // hubs: CTA-cooperative
+        if (p0) {
+          block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
+          block_atomic_add(&ctl->st[ST_AFFECTED], cnt + cnt_ins, s.red);
+          PHASE_FLUSH(PH_F0, n + nh + np0);
+        } else {
+          block_atomic_add(&ctl->st[ST_EXPANDED], cnt, s.red);
+          if (tid == 0) ctl->ncand = 0;  // read by every CTA before the last barrier
+          PHASE_FLUSH(PH_F2, n + nh);
+        }
+        GRID_SYNC_STAMPED(ctl, p0 ? 201 : 203);
+      }
+      {  // ---- F1: commit C1 + R2 expansion marks (+ marks of the pending-since-
+         //      apply vertices' neighbours, same pass) | F3: commit C2
+        const int nc = ldv(p0 ? &ctl->ncand : &ctl->ncand2), nhC = ldv(p0 ? &ctl->nhubC : &ctl->nhubC2);
+        const uint32_t ep = p0 ? a.epC1 : a.epC2;
+        if (tid == 0) ctl->st[p0 ? ST_FILTERED_IN : ST_EXPANDED_IN] = nc + nhC;
+        commit(d, s, a, nc, p0 ? d.cand : d.cand2, ep, p0, scanned, cut_acc, p0 ? np0 : 0, d.psi[0]);
+        hub_commit(d, s, a, p0 ? d.hubC : d.hubC2, nhC, ep, p0, scanned, cut_acc);
+        flush_acc(s, ctl->Wp, k);
+        PHASE_FLUSH(p0 ? PH_F1 : PH_F3, nc + nhC + (p0 ? np0 : 0));
+        GRID_SYNC_STAMPED(ctl, p0 ? 202 : 204);
+      }
+    }
+  } else {  // sharded: the same phases as staged launches (RefineMode)
   if (mode == kModeFull || mode == kShF0) {
   if (!kSh && a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
     boundary_mark(d, a.epA);
@@ -1602,9 +1651,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   // in the same pass (stat `inserted`)
   filter_pass(d, nA, [&](long long i) { return __ldcg(d.Alist + i); }, &ctl->ncand, d.cand, a.epC1, scanned,
               counted, a.epA, np0, d.psi[0], &cnt_ins);  // hubs of A: CTA-cooperative below
-  arrive_stamp(d.dbg, 113);
   hub_filter(d, s, d.hubA, nhA, a.epC1, &ctl->nhubC, d.hubC, scanned, counted);
-  arrive_stamp(d.dbg, 114);
   if (kSh && d.rank != 0) cnt_ins = 0;  // replicated count: summed over the ranks, so rank 0 adds it
   block_atomic_add(&ctl->st[ST_INSERTED], cnt_ins, s.red);
   block_atomic_add(&ctl->st[ST_AFFECTED], counted + cnt_ins, s.red);
@@ -1637,9 +1684,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     // commit C1 and, in the same pass, mark the neighbours of the pseudo
     // vertices pending since apply (psi[0][0, np0); C1 joins beyond np0)
     commit(d, s, a, nc, d.cand, a.epC1, true, scanned, cut_acc, np0, d.psi[0]);
-    arrive_stamp(d.dbg, 110);  // diagnostics only (IGK_DEBUG_ARRIVALS): sub-phase ends per CTA
     hub_commit(d, s, a, d.hubC, nhC, a.epC1, true, scanned, cut_acc);
-    arrive_stamp(d.dbg, 111);
     flush_acc(s, ctl->Wp, k);
     PHASE_FLUSH(PH_F1, nc + nhC + np0);
   }
@@ -1686,6 +1731,8 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     PHASE_FLUSH(PH_F3, nc + nhC2);
   }
   GRID_SYNC_STAMPED(ctl, 204);
+  }  // F3 (sharded)
+  }  // sharded F0-F3
 
   // ---- R3: balance restoration (reading Q9), helpers above -------------------------
   if (mode == kModeFull || mode == kShF3) {
@@ -1746,7 +1793,6 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       flush_partial();
       return;
     }
-  }
   }
   if (kSh && mode == kShR3) {  // every rank: the all-reduced keys -> the replicated select + commit
     r3_setup();

@@ -39,10 +39,19 @@ for it in range(4):
         P.refine_global("global")
     P.compare_state(f"it{it}", full_csr=(it == 3))
     P.G.partition_delta()
-os.environ["IGK_RECOUNT"] = "tma"
 from paper_conf_dac_leejlczcshh25_b200 import IGKGraph  # noqa: E402
-G2 = IGKGraph(g.xadj, g.adjncy, 4, cfg["eps"], part)
-assert G2.recount()[0] == G2.cut()
+for variant in ("tma", "gather"):  # the A/B S9 kernels (the default k_recount3 ran in check mode above)
+    os.environ["IGK_RECOUNT"] = variant
+    G2 = IGKGraph(g.xadj, g.adjncy, 4, cfg["eps"], part)
+    assert G2.recount()[0] == G2.cut()
+    G2.close()
+os.environ.pop("IGK_RECOUNT")
+# weighted handle: k_recount3<true> (edge weights 2, vertex weights 3)
+G3 = IGKGraph(g.xadj, g.adjncy, 4, cfg["eps"], part, vwgt=np.full(g.n, 3, np.int32),
+              adjwgt=np.full(len(g.adjncy), 2, np.int32))
+c3, w3 = G3.recount()
+assert c3 == G3.cut() and c3 == 2 * G2.cut(), (c3, G3.cut())
+G3.close()
 P.G.compact()
 P.compare_state("compacted", full_csr=True)
 print("sanitize run ok, cut", P.G.cut())
