@@ -676,8 +676,7 @@ __device__ __forceinline__ bool apply_body(const Dev& d, const ApplyArgs& a, cg:
       d.adjw[sv] = m.w;
     }
     if (pu != kPsi && pv != kPsi && pu != pv && own(d, m.y)) cut_acc += m.w;
-    mark_affected_pre(d, m.y, a.epA, pu_pos + 1, sy);
-    mark_affected_pre(d, m.z, a.epA, pv_pos + 1, sz);
+    mark_affected_pair(d, m.y, m.z, a.epA, pu_pos + 1, pv_pos + 1, sy, sz);
   });
   // twin fix-ups of moved entries: resolve forward marks of moved partners,
   // then point the partner back at the new slot (idempotent when both moved)

@@ -1298,22 +1298,26 @@ __device__ void run_rounds(const Dev& d, const RefineArgs& a, RefSmem& s, cg::gr
     // -- apply the prefix (moves with key < K*); the rest stay pseudo
     long long app = 0;
     rr_for(np, [&](long long j) {
-      int u = __ldcg(plist + j);
-      if (u < 0) return;
+      // the list entry and its move record in one round trip, then the
+      // vertex's words (placed-neighbour weight, gain) in the next
+      const int u = __ldcg(plist + j);
       unsigned m = __ldcg(d.meta + j);
+      if (u < 0) return;
       if (m == kMetaHub) m = __ldcg(d.metav + u);
+      const bool sel = (m & 0x80000000u) != 0;
+      const int pwu = sel ? __ldcg(d.pw + u) : 0;
+      const int gu = sel ? __ldcg(d.gain + u) : 0;
       bool keep = true;
-      if (m & 0x80000000u) {
-        int p, d0;
-        unsigned long long R;
-        long long w;
-        items(j, p, d0, R, w);
+      if (sel) {
+        const int p = (int)(m & 255u), d0 = (int)((m >> 8) & 255u);
+        const unsigned long long R =
+            d0 ? (unsigned long long)u : (((unsigned long long)(0x7fffffffu - (unsigned)gu)) << 32) | (unsigned)u;
         if (key_less(d0, R, kd, kr)) {
           keep = false;
           d.part[u] = (uint8_t)p;
-          acc_add(s.acc, p, w);
+          acc_add(s.acc, p, vert_w(d.vw, u));
           if (!kSh || own(d, u))  // sharded: the owner keeps this delta in its partial cut
-            cut_acc += (long long)__ldcg(d.pw + u) - __ldcg(d.gain + u);  // independent set: exact
+            cut_acc += (long long)pwu - gu;  // independent set: exact
           app++;
         }
       } else if (ld_part(d.part, u) != kPsi) {
@@ -1837,16 +1841,24 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
   GRID_SYNC_STAMPED(ctl, 211);
   if (tid == 0) {
-    ctl->st[ST_ROUNDS] = rounds;
-    ctl->st[ST_MOVES_APPLIED] = applied_tot;
-    ctl->st[ST_MOVES_DEFERRED] = deferred_tot;
-    ctl->st[ST_CUT] = ctl->cut;
-    ctl->st[ST_CAP] = c;
+    // every word read first (one round trip: no store in between to order
+    // them behind), then the stores
+    long long v[ST_N];
+#pragma unroll
+    for (int i = 0; i < ST_N; i++) v[i] = __ldcg(&ctl->st[i]);
+    const long long cut_now = __ldcg(&ctl->cut);
     long long mx = 0;
-    for (int p = 0; p < k; p++) mx = max(mx, ctl->Wp[p]);
-    ctl->st[ST_MAXW] = mx;
+#pragma unroll 8
+    for (int p = 0; p < k; p++) mx = max(mx, __ldcg(&ctl->Wp[p]));
+    v[ST_ROUNDS] = rounds;
+    v[ST_MOVES_APPLIED] = applied_tot;
+    v[ST_MOVES_DEFERRED] = deferred_tot;
+    v[ST_CUT] = cut_now;
+    v[ST_CAP] = c;
+    v[ST_MAXW] = mx;
+#pragma unroll
     for (int i = 0; i < ST_N; i++) {
-      ctl->st_out[i] = ctl->st[i];
+      ctl->st_out[i] = v[i];
       ctl->st[i] = 0;
     }
     for (int r = 0; r < 3; r++) {
