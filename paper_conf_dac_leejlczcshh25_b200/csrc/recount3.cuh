@@ -12,10 +12,11 @@
 //  * Dynamic tiles: a warp takes the next tile of kR3T = 128 consecutive IDs
 //    from a global counter (one atomic per 128 vertices).  Lane l holds the
 //    vertices base + 32 j + l (j < 4): four coalesced 16-byte record loads.
-//  * In-thread prefixes: a vertex's first 8 entries (two int4 chunks -- 96%
-//    of the vertices, 81% of the entries of the circuit graphs)
-//    are read and counted by its own lane with no shuffles at all.
-//  * Residual: the entries beyond 8 of vertices with degree <= kR3Big are
+//  * In-thread prefixes: a vertex's first 4 entries (one int4 chunk -- 75%
+//    of the vertices of the circuit graphs have degree <= 4)
+//    are read and counted by its own lane with no shuffles at all (two
+//    chunks in-thread measured slower: 0.140 vs 0.130 ms at C4).
+//  * Residual: the entries beyond 4 of vertices with degree <= kR3Big are
 //    listed in shared memory (warp-private) with an inclusive chunk prefix;
 //    the warp deals them lane-strided, owner found by a 7-step binary search
 //    in shared memory.
@@ -109,18 +110,15 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
   };
   const int4 none = make_int4(-1, -1, -1, -1), ones = make_int4(1, 1, 1, 1);
 
-  // the next tile's index is fetched while the current tile is counted (the
-  // counter atomic is a full L2 round trip)
-#ifndef IGK_R3PF
-#define IGK_R3PF 0
-#endif
-  unsigned long long t_next = 0;
-  if (IGK_R3PF && lane == 0) t_next = atomicAdd(ctr, 1ull);
+  // (tried and measured slower at C4, profiles/r02_{t,aj}_*: fetching the
+  // next tile's index one tile ahead, 0.142 vs 0.139 ms; pairs of adjacent
+  // tiles with the second one's records, labels and slab lines prefetched
+  // into L2 while the first is counted, 0.137 vs 0.129 ms)
   while (true) {
-    if (!IGK_R3PF && lane == 0) t_next = atomicAdd(ctr, 1ull);
-    const unsigned long long t = __shfl_sync(0xffffffffu, t_next, 0);
+    unsigned long long t = 0;
+    if (lane == 0) t = atomicAdd(ctr, 1ull);
+    t = __shfl_sync(0xffffffffu, t, 0);
     if (t >= ntiles) break;
-    if (IGK_R3PF && lane == 0) t_next = atomicAdd(ctr, 1ull);
     const long long base = (long long)t * kR3T;
     // ---- trip 1: the tile's vertex records and labels (coalesced)
     longlong2 r[kR3V];
@@ -136,7 +134,7 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
         r[j] = make_longlong2(0, 0);
       }
     }
-    int din[kR3V];  // entries counted in-thread (<= 8)
+    int din[kR3V];  // entries counted in-thread (<= kR3In)
     int nh = 0;     // residual vertices listed (warp-uniform)
 #pragma unroll
     for (int j = 0; j < kR3V; j++) {
@@ -172,7 +170,7 @@ __global__ void __launch_bounds__(kR3Threads, IGK_R3MINB) k_recount3(Dev d, long
       }
       r[j].x = (long long)c0;
     }
-    // ---- trip 2: in-thread chunks (entries 0..7 of every vertex)
+    // ---- trip 2: in-thread chunk (entries 0..3 of every vertex)
     int4 xa[kR3V][kR3InC], wa[kR3V][kR3InC];
 #pragma unroll
     for (int j = 0; j < kR3V; j++)
