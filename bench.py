@@ -499,7 +499,7 @@ def main():
         # 16-byte record + 1-byte label
         b9 = ss["adj_entries"] * 4 + ss["adj_entries"] // 2 + ss["n_active"] * 17
         a9 = b9 / (float(np.median(t9)) / 1e3) / 1e9
-        s9 = {"kernel": "k_recount", "bound": "hbm", "achieved": a9, "unit": "GB/s", "bytes_per_launch": b9,
+        s9 = {"kernel": "k_recount3", "bound": "hbm", "achieved": a9, "unit": "GB/s", "bytes_per_launch": b9,
               "launch_ms": float(np.median(t9)), "adj_entries": ss["adj_entries"], "n_active": ss["n_active"]}
 
     if rank != 0:

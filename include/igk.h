@@ -286,7 +286,14 @@ igk_status igk_part_weights(const igk_graph* g, int64_t* out_k);
  * reduction over the labels, one 8-byte read back).  Either may be NULL. */
 igk_status igk_num_vertices(const igk_graph* g, int64_t* n_total, int64_t* n_active);
 /* Recount cut and W_p from scratch with the cut/weight reduction kernel
- * (S9, HBM-bound full store scan).  out_wp may be NULL. */
+ * (S9: cut = sum of W_e over edges whose endpoints lie in different parts,
+ * W_p = sum of vertex weights per part; pending vertices count for no
+ * part).  One cooperative launch of k_recount3 (HBM-bound full store scan,
+ * DESIGN.md 6); the environment variable IGK_RECOUNT=gather|tma read at
+ * igk_create selects the round-1 gather kernel or the TMA variant instead
+ * (A/B only).  Synchronises the handle's stream.  out_cut: 1 value, out_wp:
+ * k values (may be NULL), host memory owned by the caller.  Errors:
+ * IGK_ESTATE on a poisoned handle, IGK_ECUDA if a CUDA call fails. */
 igk_status igk_recount(igk_graph* g, int64_t* out_cut, int64_t* out_wp);
 /* Debug/test: current graph as a symmetric CSR over all IDs (deleted rows
  * empty; order inside a row unspecified).  Size query: call with xadj ==
