@@ -115,6 +115,7 @@ struct Ctl {
   unsigned long long tph[128];  // %globaltimer after each phase (CTA 0)
   int idph[128];                // phase ids
   int ndone;                    // CTAs finished (publish: the last one posts the notice)
+  int ndone_ref;                // CTAs past the refine epilogue (the last one finalises the stats)
   long long paths[PA_N_DEV];    // device path counters (cumulative)
   long long phscan[8];          // profile mode: adjacency entries scanned per refine phase (PH_*)
   long long phitems[8];         // profile mode: list items (vertices) processed per refine phase
@@ -267,6 +268,8 @@ __device__ __forceinline__ unsigned long long gtimer() {
 // system scope and raises the flag to this launch's sequence number.  The
 // host polls the flag instead of a D2H copy + stream synchronisation.  Every
 // CTA of the grid must call it exactly once, at its exit.
+// the copy + flag half of publish(), for a CTA already known to be the last
+__device__ __forceinline__ void publish_copy(const Dev& d);
 __device__ __forceinline__ void publish(const Dev& d) {
   if (d.seq == 0) return;
   __shared__ int s_last;
@@ -277,6 +280,10 @@ __device__ __forceinline__ void publish(const Dev& d) {
   }
   __syncthreads();
   if (!s_last) return;
+  publish_copy(d);
+}
+__device__ __forceinline__ void publish_copy(const Dev& d) {
+  if (d.seq == 0) return;
   __threadfence();
   const int nw = (int)(offsetof(Ctl, Wp) / 8);
   const long long* src = reinterpret_cast<const long long*>(d.ctl);

@@ -1472,8 +1472,11 @@ __device__ void sh_clear_bm(const Dev& d, long long nwords) {
   rr_for(nwords, [&](long long w) { d.bm[w] = 0; });
 }
 
+// Returns true (on every CTA) iff the epilogue ran; the unsharded epilogue
+// then also posted the completion notice (publish_copy), so the kernel must
+// not call publish() again.
 template <bool kSh>
-__device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s,
+__device__ __forceinline__ bool refine_body(const Dev& d, const RefineArgs& a, cg::grid_group& grid, RefSmem& s,
                                             const ShardArgs& sh) {
   Ctl* ctl = d.ctl;
   const int k = d.k;
@@ -1481,7 +1484,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
   const int mode = kSh ? sh.mode : (int)kModeFull;
   if (!kSh && a.after_apply && (ldv(&ctl->err_idx) != kNoErr || ldv(&ctl->err_nomem) != 0)) {
     if (tid == 0) ctl->refine_skipped = 1;  // uniform exit: nothing was modified
-    return;
+    return false;
   }
   if (tid == 0 && (mode == kModeFull || mode == kShF0)) {
     ctl->refine_skipped = 0;
@@ -1590,7 +1593,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
       ctl->rs_applied = rs.applied_tot;
       ctl->rs_deferred = rs.deferred_tot;
     }
-    return;
+    return false;
   }
   if constexpr (!kSh) {
     if (a.global) {  // NEXT-1: A |= partition boundary, then the ordinary refine
@@ -1664,7 +1667,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     grid.sync();
     sh_publish(d, ldv(&ctl->ncand), d.cand, ldv(&ctl->nhubC), d.hubC);
     flush_partial();
-    return;
+    return false;
   }
   GRID_SYNC_STAMPED(ctl, 201);
   }
@@ -1709,7 +1712,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     grid.sync();
     sh_publish(d, ldv(&ctl->ncand2), d.cand2, ldv(&ctl->nhubC2), d.hubC2);
     flush_partial();
-    return;
+    return false;
   }
   GRID_SYNC_STAMPED(ctl, 203);
   }
@@ -1795,7 +1798,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     if (kSh) {
       if (tid == 0) ctl->sh_np = ldv(&ctl->npsi[0]);  // every commit is behind barrier 204
       flush_partial();
-      return;
+      return false;
     }
   }
   if (kSh && mode == kShR3) {  // every rank: the all-reduced keys -> the replicated select + commit
@@ -1809,7 +1812,7 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     r3_select_evict_commit();
     if (tid == 0) ctl->sh_np = ldv(&ctl->npsi[0]);  // the eviction commit is behind barrier 207
     flush_partial();
-    return;
+    return false;
   }
 
   // ---- R4: rounds (Alg. 4), grid-wide (a CTA-local variant for small tails
@@ -1839,8 +1842,26 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
 
   block_atomic_add(&ctl->cut, cut_acc, s.red);
   block_atomic_add(&ctl->st[ST_SCANNED], scanned, s.red);
-  GRID_SYNC_STAMPED(ctl, 211);
-  if (tid == 0) {
+  // no grid barrier: the LAST CTA past this point (every CTA's atomics and
+  // delta entries are fenced before its arrival) finalises the stats and
+  // posts the completion notice -- one grid-wide wait less per step
+  __shared__ int s_fin;
+  arrive_stamp(d.dbg, 11);
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_fin = atomicAdd(&ctl->ndone_ref, 1) == (int)gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_fin) return true;
+  if (threadIdx.x == 0) {
+    __threadfence();
+    ctl->ndone_ref = 0;
+    const int ip = ctl->nph;  // the epilogue's phase stamp (CTA 0 wrote its earlier ones before arriving)
+    if (ip < 128) {
+      ctl->tph[ip] = gtimer();
+      ctl->idph[ip] = 211;
+      ctl->nph = ip + 1;
+    }
     // every word read first (one round trip: no store in between to order
     // them behind), then the stores
     long long v[ST_N];
@@ -1880,6 +1901,9 @@ __device__ __forceinline__ void refine_body(const Dev& d, const RefineArgs& a, c
     ctl->npsi[1] = 0;
     ctl->npsi[2] = 0;
   }
+  __syncthreads();
+  if (!kSh) publish_copy(d);
+  return true;
 }
 
 #ifndef IGK_REFINE_MINB
@@ -1890,8 +1914,7 @@ __global__ void __launch_bounds__(kThreads, IGK_REFINE_MINB) k_refine(Dev d, Ref
   extern __shared__ __align__(16) unsigned char smem_raw[];
   ShardArgs sh{};
   sh.mode = kModeFull;
-  refine_body<false>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh);
-  publish(d);
+  if (!refine_body<false>(d, a, grid, *reinterpret_cast<RefSmem*>(smem_raw), sh)) publish(d);
 }
 
 // sharded refine: one launch per mode (RefineMode kSh*), driven by igk.cu refine_sharded

@@ -24,8 +24,7 @@ __global__ void __launch_bounds__(kThreads) k_step(Dev d, ApplyArgs aa, RefineAr
   grid.sync();  // the refine starts from the complete applied state
   ShardArgs sh{};
   sh.mode = kModeFull;
-  refine_body<false>(d, ra, grid, sm.rf, sh);
-  publish(d);
+  if (!refine_body<false>(d, ra, grid, sm.rf, sh)) publish(d);  // (the epilogue posts the notice itself)
 }
 
 }  // namespace igk
