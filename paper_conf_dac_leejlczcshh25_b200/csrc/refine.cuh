@@ -78,6 +78,11 @@ struct ShardArgs {
 // ---------------------------------------------------------------------------
 // thread: f(x, w, q) for each neighbour; a chunk issues all its ID/weight
 // loads, then all its label loads, before f runs; f returns false to stop
+#ifndef IGK_WARPU
+#define IGK_WARPU 8
+#endif
+constexpr int kWU = IGK_WARPU;  // warp bucket: entries per lane per round trip (A/B: -DIGK_WARPU)
+constexpr int kWB = 32 * kWU;   // entries per warp per round trip
 constexpr int kTC = kThreadDeg;  // thread chunk (one round trip per thread-bucket vertex)
 // the commit's thread chunk: five values per slot (ID, weight, label, stamp,
 // saved label) plus the expansion marks -- 8 slots keep it off the local stack
@@ -147,35 +152,35 @@ __device__ __forceinline__ void mark_nbrs_thread(const Dev& d, long long o, int 
   }
 }
 __device__ __forceinline__ void mark_nbrs_warp(const Dev& d, long long o, int dg, uint32_t epN, uint32_t epC) {
-  for (int b = 0; b < dg; b += 256) {
-    int x[8];
-    uint8_t q[8];
+  for (int b = 0; b < dg; b += kWB) {
+    int x[kWU];
+    uint8_t q[kWU];
 #pragma unroll
-    for (int t = 0; t < 8; t++) {
+    for (int t = 0; t < kWU; t++) {
       int i = b + t * 32 + lane_id();
       x[t] = i < dg ? ldro(d.adj + o + i) : -1;
     }
 #pragma unroll
-    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
-    mark_chunk<8>(d, x, q, epN, epC);
+    for (int t = 0; t < kWU; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    mark_chunk<kWU>(d, x, q, epN, epC);
   }
 }
 // warp: lane-strided, 8 entries per lane per round trip (256 per warp)
 template <class F>
 __device__ __forceinline__ void nbrs_warp(const Dev& d, long long o, int dg, F f) {
-  for (int b = 0; b < dg; b += 256) {
-    int x[8], w[8];
-    uint8_t q[8];
+  for (int b = 0; b < dg; b += kWB) {
+    int x[kWU], w[kWU];
+    uint8_t q[kWU];
 #pragma unroll
-    for (int t = 0; t < 8; t++) {
+    for (int t = 0; t < kWU; t++) {
       int i = b + t * 32 + lane_id();
       x[t] = i < dg ? ldro(d.adj + o + i) : -1;
       w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
     }
 #pragma unroll
-    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    for (int t = 0; t < kWU; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
 #pragma unroll
-    for (int t = 0; t < 8; t++)
+    for (int t = 0; t < kWU; t++)
       if (x[t] >= 0) f(x[t], w[t], q[t]);
   }
 }
@@ -184,19 +189,19 @@ __device__ __forceinline__ void nbrs_warp(const Dev& d, long long o, int dg, F f
 // stop() holds (the round gain of a blocked vertex)
 template <class F, class S>
 __device__ __forceinline__ void nbrs_warp_until(const Dev& d, long long o, int dg, F f, S stop) {
-  for (int b = 0; b < dg; b += 256) {
-    int x[8], w[8];
-    uint8_t q[8];
+  for (int b = 0; b < dg; b += kWB) {
+    int x[kWU], w[kWU];
+    uint8_t q[kWU];
 #pragma unroll
-    for (int t = 0; t < 8; t++) {
+    for (int t = 0; t < kWU; t++) {
       int i = b + t * 32 + lane_id();
       x[t] = i < dg ? ldro(d.adj + o + i) : -1;
       w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
     }
 #pragma unroll
-    for (int t = 0; t < 8; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
+    for (int t = 0; t < kWU; t++) q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
 #pragma unroll
-    for (int t = 0; t < 8; t++)
+    for (int t = 0; t < kWU; t++)
       if (x[t] >= 0) f(x[t], w[t], q[t]);
     if (__any_sync(0xffffffffu, stop())) return;
   }
@@ -737,33 +742,33 @@ __device__ void commit(const Dev& d, RefSmem& s, const RefineArgs& a, int nc, co
     }
     const uint8_t pu = (uint8_t)pvv;
     long long del = 0;
-    for (int b = 0; b < dg; b += 256) {
-      int x[8], w[8];
-      uint8_t q[8];
-      unsigned mk[8];
+    for (int b = 0; b < dg; b += kWB) {
+      int x[kWU], w[kWU];
+      uint8_t q[kWU];
+      unsigned mk[kWU];
 #pragma unroll
-      for (int t = 0; t < 8; t++) {
+      for (int t = 0; t < kWU; t++) {
         int i = b + t * 32 + lane_id();
         x[t] = i < dg ? ldro(d.adj + o + i) : -1;
         w[t] = (i < dg && d.adjw) ? ldro(d.adjw + o + i) : 1;
       }
-      uint8_t op[8];
-      int dgx[8];
+      uint8_t op[kWU];
+      int dgx[kWU];
 #pragma unroll
-      for (int t = 0; t < 8; t++) {
+      for (int t = 0; t < kWU; t++) {
         q[t] = x[t] >= 0 ? ld_part(d.part, x[t]) : (uint8_t)0;
         mk[t] = x[t] >= 0 ? __ldcg(d.markT + x[t]) : 0u;
         op[t] = x[t] >= 0 ? __ldcg(d.oldp + x[t]) : (uint8_t)0;
         dgx[t] = (expand && x[t] >= 0) ? ldro(&d.vr[x[t]].deg) : 0;
       }
 #pragma unroll
-      for (int t = 0; t < 8; t++) {
+      for (int t = 0; t < kWU; t++) {
         if (x[t] < 0) continue;
         const bool xc = mk[t] == ep;
         const uint8_t qx = xc ? op[t] : q[t];
         if (qx != kPsi && qx != pu && !(xc && x[t] < u)) del += w[t];
       }
-      if (expand) mark_chunk<8>(d, x, q, a.epN, ep, mk, dgx);
+      if (expand) mark_chunk<kWU>(d, x, q, a.epN, ep, mk, dgx);
     }
     del = warp_sum(del);
     if (lane_id() == 0) {
